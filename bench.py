@@ -1,0 +1,400 @@
+#!/usr/bin/env python
+"""Benchmark of the star-image render path (BASELINE.json metric) -- one JSON line on rank 0.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config T] [--method tiled|atomic]
+
+A step is one frame: the whole hot path (per-star prep + binning + radix sort + CSR + tile accumulation) over one
+synthetic catalogue resident in HBM, written to a device-resident fp32 image.  N=1 renders the north-star frame T
+(4096x4096, 1M uniform stars, R=15, sigma=2.5).  Under torchrun (N>1) the job is weak-scaled: the frame is
+4096 wide and 4096*N tall with N*1M stars, every rank renders its own 4096-row band and the
+bands are assembled with one NCCL all-gather, included in the step.
+
+Timing: W untimed warm-up steps; the L2 (126 MB) is flushed by writing a 256 MiB buffer before every step (the frame's
+79 MB of inputs+image would otherwise stay L2-resident); each step is bracketed by CUDA events on the render stream;
+barrier + synchronize on both sides of the timed region; max over ranks.  `e2e` repeats the step through the same
+C-ABI call with the catalogue copied in from pinned host memory and the image copied back, inside the timed region.
+`roofline` is for the dominant kernel (k_tile), timed live with the library's per-kernel CUDA events.
+`cpu_baseline` / --impl reference time the fp64 oracle on the host cores (bounded sample).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "star-pixel updates/s and frames/s at 1/2/4/8 B200; % of FP32/SFU roofline"
+UNIT = "star-pixel updates/s"
+FLUSH_BYTES = 256 << 20
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="T")
+    ap.add_argument("--method", default="tiled", choices=["tiled", "atomic"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------------------------------------ roofline model
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured (MEASURED_PEAKS.json)"
+    return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback (B200_PROFILING.md)"
+
+
+def fp32_sfu_peak_updates(sm_mhz, U, E, sms=148):
+    """Roofline rate of the separable-PSF work: per SM per clock 128 FP32 FMA (measured
+    126-128, bench_micro) and 16 MUFU.EX2 (measured 16.0).  T* = max(U / P_fma, E / P_mufu); peak = U / T*."""
+    f = sm_mhz * 1e6
+    p_fma = sms * 128 * f
+    p_mufu = sms * 16 * f
+    t_star = max(U / p_fma, E / p_mufu)
+    return U / t_star, t_star
+
+
+# ------------------------------------------------------------------------------------------------ clocks (NVML)
+class ClockSampler:
+    def __init__(self, index=0, period=0.005):
+        self.samples, self.reasons, self.period, self.index = [], set(), period, index
+        self._stop = threading.Event()
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover
+            self.err = str(e)
+
+    def _run(self):
+        nv = self.nv
+        names = {getattr(nv, k): k for k in dir(nv) if k.startswith("nvmlClocksEventReason") or
+                 k.startswith("nvmlClocksThrottleReason")}
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h) if hasattr(
+                    nv, "nvmlDeviceGetCurrentClocksEventReasons") else nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+                for bit, name in names.items():
+                    if isinstance(bit, int) and bit and (r & bit) == bit and bit not in (0xFFFFFFFFFFFFFFFF,):
+                        if "None" in name or "All" in name or "Unknown" in name:
+                            continue
+                        self.reasons.add(name.replace("nvmlClocksEventReason", "").replace(
+                            "nvmlClocksThrottleReason", ""))
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "note": "nvml unavailable"}
+        hi = [s for s in self.samples if s > 0.5 * max(self.samples)]
+        return {"sm_mhz": statistics.median(hi), "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------------------------------------ workload
+def workload(cfg_name, world, rank):
+    import synth
+    cfg = synth.CONFIGS[cfg_name]
+    if world == 1:
+        return cfg, cfg.field(), cfg.H, (0, cfg.H)
+    # weak scaling: frame W x (H*world), world*n stars; every rank holds the full catalogue (replicated)
+    H = cfg.H * world
+    big = synth.Config(f"{cfg.name}x{world}", cfg.W, H, cfg.n * world, cfg.R, cfg.sigma, cfg.kind, cfg.seed)
+    return big, big.field(), H, None
+
+
+def units_of(f, W, H, R):
+    """U, E over the frame with the exact per-star clipping of the method (numpy, same rules as the oracle)."""
+    import numpy as np
+    x, y, m = (a.astype(np.float64) for a in (f.x, f.y, f.mag))
+    ok = np.isfinite(x) & np.isfinite(y) & np.isfinite(m)
+    fx = np.floor(x)
+    if R % 2:
+        lx = fx + (x >= fx + 0.5) - (R - 1) // 2
+        fy = np.floor(y)
+        ly = fy + (y >= fy + 0.5) - (R - 1) // 2
+    else:
+        lx = fx + 1 - R // 2
+        ly = np.floor(y) + 1 - R // 2
+    w = np.minimum(lx + R - 1, W - 1) - np.maximum(lx, 0) + 1
+    h = np.minimum(ly + R - 1, H - 1) - np.maximum(ly, 0) + 1
+    ok &= (w > 0) & (h > 0)
+    return int((w * h)[ok].sum()), int((w + h)[ok].sum())
+
+
+# ------------------------------------------------------------------------------------------------ CPU baseline
+def cpu_baseline(cfg, f, W, H, budget_s=12.0):
+    """The fp64 oracle as it stands on all host cores, on a prefix of the catalogue sized for ~budget_s."""
+    import numpy as np
+    import oracle
+    import synth
+    threads = os.cpu_count() or 1
+    A = synth.bench_gain(cfg.sigma)
+    n_cal = max(1000, f.n // 200)
+    t0 = time.perf_counter()
+    oracle.render(f.x[:n_cal], f.y[:n_cal], f.mag[:n_cal], W, H, cfg.sigma, cfg.R, A, threads=threads)
+    dt = time.perf_counter() - t0
+    n_s = int(min(f.n, max(n_cal, n_cal * budget_s / max(dt, 1e-6))))
+    t0 = time.perf_counter()
+    oracle.render(f.x[:n_s], f.y[:n_s], f.mag[:n_s], W, H, cfg.sigma, cfg.R, A, threads=threads)
+    dt = time.perf_counter() - t0
+    sub = synth.Field(f.x[:n_s], f.y[:n_s], f.mag[:n_s])
+    U, _ = units_of(sub, W, H, cfg.R)
+    return {"value": U / dt, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": f"first {n_s} of {f.n} stars of the same frame ({W}x{H}, R={cfg.R}), fp64 oracle, "
+                      f"{threads} pthreads over row bands, {dt:.2f} s wall (includes zeroing the fp64 image)",
+            "seconds": dt}
+
+
+# ------------------------------------------------------------------------------------------------ reference arm
+def run_reference(args, world, rank):
+    if rank != 0:
+        return
+    import oracle
+    import synth
+    cfg, f, H, _ = workload(args.config, 1, 0)
+    W = cfg.W
+    A = synth.bench_gain(cfg.sigma)
+    threads = os.cpu_count() or 1
+    total_budget = 150.0
+    per_step = total_budget / max(1, args.steps + args.warmup)
+    n_cal = max(1000, f.n // 500)
+    t0 = time.perf_counter()
+    oracle.render(f.x[:n_cal], f.y[:n_cal], f.mag[:n_cal], W, H, cfg.sigma, cfg.R, A, threads=threads)
+    dt = time.perf_counter() - t0
+    n_s = int(min(f.n, max(n_cal, n_cal * per_step / max(dt, 1e-6))))
+    sub = synth.Field(f.x[:n_s], f.y[:n_s], f.mag[:n_s])
+    U, _ = units_of(sub, W, H, cfg.R)
+    for _ in range(args.warmup):
+        oracle.render(sub.x, sub.y, sub.mag, W, H, cfg.sigma, cfg.R, A, threads=threads)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.render(sub.x, sub.y, sub.mag, W, H, cfg.sigma, cfg.R, A, threads=threads)
+        times.append(time.perf_counter() - t0)
+    ms = 1e3 * sum(times) / len(times)
+    value = U / (ms * 1e-3)
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": f"{cfg.name}: {W}x{H}, {cfg.n} uniform stars, R={cfg.R}, sigma={cfg.sigma:g}",
+                       "sample_stars": n_s, "frames_per_s_equiv": value / max(1, units_of(f, W, H, cfg.R)[0])},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+                             "sample": f"first {n_s} of {f.n} stars per step, fp64 oracle, {threads} pthreads"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------------------------ our arm
+def run_ours(args, world, rank, local_rank):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    import synth
+    from paper_conf_ipps_lizzh12_b200 import Context, dist as sdist
+
+    dev = torch.device(f"cuda:{local_rank}")
+    torch.cuda.set_device(dev)
+    cfg, f, H, _ = workload(args.config, world, rank)
+    W, R, sigma = cfg.W, cfg.R, cfg.sigma
+    A = synth.bench_gain(sigma)
+    U_frame, E_frame = units_of(f, W, H, R)
+    ctx = Context(local_rank)
+    stream = torch.cuda.Stream(dev)
+    x, y, m = (torch.from_numpy(a).to(dev) for a in (f.x, f.y, f.mag))
+    prow = sdist.padded_band_rows(H, world)
+    band = torch.zeros((prow, W), dtype=torch.float32, device=dev)
+    full = torch.empty((world * prow, W), dtype=torch.float32, device=dev) if world > 1 else None
+    row0, rows = sdist.band_rows(H, world, rank)
+    flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
+
+    def step(xx, yy, mm):
+        with torch.cuda.stream(stream):
+            if args.method == "atomic":
+                ctx.render_atomic(xx, yy, mm, W, H, sigma, R, A, out=band[:H], stream=stream)
+            else:
+                ctx.render_band(xx, yy, mm, W, H, row0, rows, sigma, R, A, out=band[:rows], stream=stream)
+            if world > 1:
+                dist.all_gather_into_tensor(full, band)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(max(3, args.warmup)):
+        step(x, y, m)
+    barrier()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    ctx.profile(True)
+    with ClockSampler(local_rank) as clk:
+        barrier()
+        for i in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.fill_(float(i))                  # evict L2 (256 MiB > 126 MB), untimed
+                ev[i][0].record(stream)
+            step(x, y, m)
+            ev[i][1].record(stream)
+        barrier()
+        kt = ctx.kernel_times()
+        ctx.profile(False)
+        # keep sampling clocks over >= 0.3 s of the same step so a short timed region still gets samples
+        t_end = time.time() + 0.3
+        while time.time() < t_end:
+            step(x, y, m)
+        torch.cuda.synchronize()
+    ms_steps = [a.elapsed_time(b) for a, b in ev]
+    ms = sum(ms_steps) / len(ms_steps)
+    t = torch.tensor([ms], device=dev, dtype=torch.float64)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    value = U_frame / (ms * 1e-3)      # updates of the whole frame (all ranks) per second
+
+    # per-kernel live timings (this rank); launches of our own kernels per step
+    launches = sum(v[1] for k, v in kt.items() if k not in ("memset",)) / args.steps
+    tile_ms = kt["tile"][0] / max(1, kt["tile"][1])
+    clocks = clk.summary()
+    sm_mhz = clocks["sm_mhz"] or 1965.0
+    # roofline of the dominant kernel (k_tile) on this rank's band
+    band_f_units = units_of(synth.Field(f.x, f.y, f.mag), W, H, R) if world == 1 else None
+    U_band, E_band = (U_frame, E_frame) if world == 1 else (U_frame / world, E_frame / world)
+    peak_rate, t_star = fp32_sfu_peak_updates(sm_mhz, U_band, E_band)
+    peak_max, _ = fp32_sfu_peak_updates(1965.0, U_band, E_band)
+    achieved = U_band / (tile_ms * 1e-3) if args.method == "tiled" else None
+    peaks, peak_src = load_peaks()
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "ncu_tile_traffic.json")
+    if os.path.exists(prof):
+        try:
+            traffic = json.load(open(prof)).get(cfg.name, {}).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    roofline = {"bound": "alu", "kernel": "k_tile", "achieved": achieved / 1e9 if achieved else None,
+                "peak": peak_rate / 1e9, "unit": "Gupdates/s", "frac": (achieved / peak_rate) if achieved else None,
+                "traffic": traffic,
+                "peak_basis": f"FP32/SFU roofline max(U/(148*128*f), E/(148*16*f)) at the measured SM clock "
+                              f"f={sm_mhz:.0f} MHz; U={U_band}, E={E_band}; frac at 1965 MHz = "
+                              f"{(achieved / peak_max) if achieved else 0:.3f}",
+                "kernel_ms": tile_ms,
+                "hbm": {"bytes": 4 * W * (rows if world > 1 else H) + 16 * f.n,
+                        "achieved_GBps": (4 * W * (rows if world > 1 else H) + 16 * f.n) / (tile_ms * 1e-3) / 1e9,
+                        "peak_GBps": peaks.get("hbm_gbs"), "peak_source": peak_src}}
+    kernels = {k: {"ms_per_step": v[0] / args.steps, "launches_per_step": v[1] / args.steps} for k, v in kt.items()
+               if v[1]}
+
+    # e2e: the same C-ABI call with host (pinned) catalogue in and image out, copies inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        hx, hy, hm = (torch.from_numpy(a).pin_memory() for a in (f.x, f.y, f.mag))
+        himg = torch.empty((rows if world > 1 else H, W), dtype=torch.float32).pin_memory()
+        dx, dy, dm = (torch.empty_like(x) for _ in range(3))
+
+        def e2e_step():
+            with torch.cuda.stream(stream):
+                dx.copy_(hx, non_blocking=True)
+                dy.copy_(hy, non_blocking=True)
+                dm.copy_(hm, non_blocking=True)
+            step(dx, dy, dm)
+            with torch.cuda.stream(stream):
+                himg.copy_(band[:himg.shape[0]], non_blocking=True)
+
+        for _ in range(2):
+            e2e_step()
+        barrier()
+        e_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                for _ in range(args.steps)]
+        for i in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.fill_(float(i))
+                e_ev[i][0].record(stream)
+            e2e_step()
+            e_ev[i][1].record(stream)
+        barrier()
+        e_ms = sum(a.elapsed_time(b) for a, b in e_ev) / args.steps
+        te = torch.tensor([e_ms], device=dev, dtype=torch.float64)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e_ms = float(te.item())
+        e2e = {"value": U_frame / (e_ms * 1e-3), "unit": UNIT, "ms_per_step": e_ms,
+               "h2d_bytes_per_step": int(3 * 4 * f.n), "d2h_bytes_per_step": int(himg.numel() * 4),
+               "note": "pinned host catalogue -> device, render, image -> pinned host, per step"}
+
+    if rank != 0:
+        ctx.close()
+        return
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        cpu = cpu_baseline(cfg, f, W, H)
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"{cfg.name}: {W}x{H}, {cfg.n} uniform stars, R={R}, sigma={sigma:g}"
+                                   + (f"; {world} bands of {prow} rows + NCCL all-gather" if world > 1 else ""),
+                       "W": W, "H": H, "stars": f.n, "R": R, "sigma": sigma, "gain": A, "method": args.method,
+                       "frames_per_s": 1e3 / ms, "updates_per_frame": U_frame, "exps_per_frame": E_frame,
+                       "parallelism": f"bands{world}" if world > 1 else "single",
+                       "l2": "flushed before every step (256 MiB write, untimed)"},
+            "clocks": clocks, "gpu_launches": int(round(launches * args.steps)),
+            "gpu_launches_per_step": launches, "kernels": kernels, "roofline": roofline, "e2e": e2e,
+            "cpu_baseline": cpu}
+    print(json.dumps(line), flush=True)
+    ctx.close()
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, world, rank)
+        return
+    import __graft_entry__
+    if rank == 0 or world == 1:
+        __graft_entry__.build()
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local_rank}"))
+        dist.barrier()
+        __graft_entry__.build()
+    run_ours(args, world, rank, local_rank)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

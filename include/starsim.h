@@ -1,0 +1,129 @@
+/*
+ * include/starsim.h -- C ABI of libstarsim.so, the B200-native (sm_100a) star-image renderer.
+ *
+ * What it computes (C. Li et al., IPDPS-W 2012, Sec. II):
+ *   Eq. 1  g(m) = A * 2.512^(-m)                       -- brightness from magnitude, A = `gain`
+ *   Eq. 2  mu(x,y) = 1/(2 pi s^2) exp(-((x-X)^2+(y-Y)^2)/(2 s^2))   -- Gaussian PSF, s = `sigma`
+ *   Eq. 3  phi(m,x,y) = g(m) * mu(x,y) for pixels (x,y) inside the star's ROI, summed over stars
+ *   ROI: a square of side R = `roi` (Fig. 1, Fig. 5 loops PAPER.md:94-112): the R columns nearest to the
+ *   star's x (ties at k+1/2 round up) times the R rows nearest to its y; pixels outside the image are dropped
+ *   (PAPER.md:106, 134), nothing is renormalised.  Pixel (px,py) is sampled at integer (px,py); the image is
+ *   row-major with y = row: out[py*width + px].  DESIGN.md "Readings" lists every such choice.
+ *
+ * Conventions for every entry point:
+ *   - Array pointers marked (device) are CUDA device pointers on the ctx's device; (host) are host pointers.
+ *   - The caller owns every input and output buffer.  The ctx owns its scratch (star records, tile pairs, sort
+ *     buffers, offsets); scratch grows geometrically, is reused across calls and is freed by starsim_destroy.
+ *   - Calls are stream-ordered and asynchronous on `stream` (0 = legacy default stream); host-side validation is
+ *     synchronous and happens before anything is enqueued.
+ *   - A ctx is bound to one device and is not thread-safe: use one ctx per host thread / stream.
+ *   - Return codes: STARSIM_OK, or a negative code.  On STARSIM_EINVAL nothing is enqueued and `out` is untouched.
+ *     starsim_last_error() describes the most recent failure.
+ *   - Per-star bad data is not an error: stars with a non-finite x, y or mag, or whose ROI misses the image (or the
+ *     band), contribute nothing -- exactly as the oracle does.
+ */
+#ifndef STARSIM_H
+#define STARSIM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct starsim_ctx starsim_ctx;
+typedef struct CUstream_st* starsim_stream_t; /* == cudaStream_t */
+
+enum {
+  STARSIM_OK = 0,
+  STARSIM_EINVAL = -1, /* an argument is out of range (list at each call)            */
+  STARSIM_ENOMEM = -2, /* scratch growth failed (cudaMalloc)                          */
+  STARSIM_ECUDA = -3,  /* a CUDA runtime error; text in starsim_last_error            */
+  STARSIM_ENODEV = -4  /* the device is not an sm_100 (B200-class) GPU                */
+};
+
+/* Limits checked by every render call (EINVAL otherwise). */
+#define STARSIM_MAX_DIM 32767      /* width, height in [1, 32767], width*height < 2^31 */
+#define STARSIM_MAX_ROI 255        /* roi (R, the ROI side) in [1, 255]                 */
+
+/* Create a context on CUDA device `cuda_device`.  Fails with ENODEV unless its compute capability is 10.x
+ * (this library carries sm_100a code only).  *out is set to NULL on failure. */
+int starsim_create(starsim_ctx** out, int cuda_device);
+
+/* Destroy a context and free its scratch.  NULL-safe.  Synchronises the ctx's device first. */
+void starsim_destroy(starsim_ctx* ctx);
+
+/* Text of the last error on this ctx ("" if none).  Owned by the ctx, valid until its next call.  ctx may be NULL
+ * (then a static description of the last create failure). */
+const char* starsim_last_error(const starsim_ctx* ctx);
+
+/* Render a full frame with the tiled, atomic-free path: per-star prep + binning of (tile, star)
+ * pairs + stable radix sort + CSR, then one register-accumulating tile kernel that writes every pixel once.
+ *   x, y, mag  (device) float[n]: the star catalogue as SoA -- sub-pixel centre (image coordinates) and magnitude.
+ *   n          number of stars, >= 0 (0 -> an all-zero image).  x, y, mag may be NULL iff n == 0.
+ *   width, height   image size in pixels, each in [1, 32767], width*height < 2^31.
+ *   sigma      PSF standard deviation delta of Eq. 2, finite and > 0.
+ *   roi        ROI side R in pixels, [1, 255].
+ *   gain       A of Eq. 1, finite and >= 0.
+ *   out        (device) float[height*width], fully overwritten (0 where no star contributes); must not alias inputs.
+ * Per-pixel accumulation is fp32 in star-index order, so the image is bitwise reproducible run to run.
+ * Errors: EINVAL (ctx NULL, n < 0, n > 0 with a NULL x/y/mag, out NULL, sizes/sigma/roi/gain out of range),
+ *         ENOMEM, ECUDA. */
+int starsim_render(starsim_ctx* ctx, const float* x, const float* y, const float* mag, int64_t n,
+                   int32_t width, int32_t height, float sigma, int32_t roi, float gain,
+                   float* out, starsim_stream_t stream);
+
+/* Render rows [row0, row0+rows) of the width x height frame into out_band (device) float[rows*width]: the
+ * multi-GPU band decomposition.  Stars are routed to the band iff their clipped ROI rows
+ * intersect it.  When row0 and rows are multiples of the tile height the band is bitwise equal to the same rows of
+ * starsim_render.  Extra EINVAL: row0 < 0, rows < 1, row0 + rows > height. */
+int starsim_render_band(starsim_ctx* ctx, const float* x, const float* y, const float* mag, int64_t n,
+                        int32_t width, int32_t height, int32_t row0, int32_t rows,
+                        float sigma, int32_t roi, float gain, float* out_band, starsim_stream_t stream);
+
+/* The paper's own design, kept as the measured comparison (Fig. 6): zero the image, then one
+ * warp per star adds g*mu into every ROI pixel with global fp32 reductions (red.global.add.f32).  Same arguments
+ * and EINVAL cases as starsim_render.  The summation order is nondeterministic. */
+int starsim_render_atomic(starsim_ctx* ctx, const float* x, const float* y, const float* mag, int64_t n,
+                          int32_t width, int32_t height, float sigma, int32_t roi, float gain,
+                          float* out, starsim_stream_t stream);
+
+/* Upload the paper's AoS star records {float mag, posX, posY}[n] (Fig. 6 step 4) from host memory
+ * `host_aos` (host, any alignment) and split them into the device SoA arrays x, y, mag (device, float[n] each).
+ * The host->device copy goes through a ctx-owned staging buffer on `stream`; the call returns once the host
+ * buffer may be reused.  EINVAL: n < 0, or n > 0 with a NULL pointer. */
+int starsim_upload_aos(starsim_ctx* ctx, const void* host_aos, int64_t n,
+                       float* x, float* y, float* mag, starsim_stream_t stream);
+
+/* Output stage: q = min(2^bits - 1, floor(v + 1/2)) computed exactly, v <= 0 or NaN -> 0.
+ *   img (device) float[npix]; out (device) uint8_t[npix] if bits == 8, uint16_t[npix] if bits == 16.
+ * EINVAL: npix < 0, NULL pointers with npix > 0, bits not 8 or 16. */
+int starsim_quantize(starsim_ctx* ctx, const float* img, int64_t npix, int32_t bits, void* out,
+                     starsim_stream_t stream);
+
+/* Introspection of the last starsim_render / starsim_render_band on this ctx (for the bit-exact binning tests):
+ * synchronises that call's stream, then copies the CSR to host memory.
+ *   *tile_w, *tile_h   tile size in pixels; tiles are numbered key = ty*ceil(width/tile_w) + tx over the frame
+ *                      (over the band's rows for render_band, ty counted from row0).
+ *   tile_off_host (host) uint32[off_cap]: CSR offsets, ntiles+1 entries are written if off_cap allows.
+ *   ids_host      (host) uint32[ids_cap]: star indices, tile-major, star order inside a tile; P entries written.
+ *   *n_pairs      P, the number of (tile, star) pairs.
+ * EINVAL if no render happened yet or a capacity is too small (*n_pairs is still set). */
+int starsim_get_bins(starsim_ctx* ctx, int32_t* tile_w, int32_t* tile_h,
+                     uint32_t* tile_off_host, int64_t off_cap, uint32_t* ids_host, int64_t ids_cap,
+                     int64_t* n_pairs);
+
+/* Per-kernel device timing for roofline reporting.  When enabled, every launch of the library records CUDA events
+ * on the launching stream around it; starsim_kernel_times() synchronises and returns, per kernel class, the summed
+ * elapsed milliseconds and launch counts since the last reset.  Classes (index into the arrays):
+ *   0 prep+scan+emit, 1 radix passes, 2 tile offsets, 3 tile accumulate, 4 atomic scatter, 5 memsets/zero,
+ *   6 quantise, 7 aos upload split.
+ * `ms` and `launches` must hold STARSIM_NUM_KCLASS entries.  enable != 0 turns recording on and resets. */
+#define STARSIM_NUM_KCLASS 8
+int starsim_profile(starsim_ctx* ctx, int enable);
+int starsim_kernel_times(starsim_ctx* ctx, double* ms, int64_t* launches);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* STARSIM_H */

@@ -1,0 +1,418 @@
+// The C ABI of libstarsim.so (include/starsim.h): handle lifecycle, argument validation, scratch arena,
+// stream-ordered orchestration of the sm_100a kernels, per-kernel CUDA-event timing, error strings.
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/starsim.h"
+#include "common.cuh"
+#include "launch.h"
+
+using namespace starsim;
+
+namespace {
+
+thread_local std::string g_create_error;
+
+struct Buf {
+  void* p = nullptr;
+  size_t cap = 0;
+};
+
+struct Launch {
+  int kclass;
+  cudaEvent_t a, b;
+};
+
+}  // namespace
+
+struct starsim_ctx {
+  int dev = 0;
+  int num_sms = 148;
+  std::string err;
+  Buf rec, pairs[2], tile_off, st_bin, st_rad, hdr, stage;
+  uint32_t epoch = 0;
+  // last tiled render, for starsim_get_bins
+  bool have_bins = false;
+  cudaStream_t last_stream = nullptr;
+  int last_sorted = 0;
+  int64_t last_ntiles = 0;
+  // profiling
+  bool prof = false;
+  std::vector<cudaEvent_t> ev_pool;
+  std::vector<Launch> pending;
+  double ms[STARSIM_NUM_KCLASS] = {};
+  int64_t launches[STARSIM_NUM_KCLASS] = {};
+};
+
+namespace {
+
+struct DevGuard {
+  int prev = -1;
+  explicit DevGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DevGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+int fail(starsim_ctx* c, int code, const std::string& msg) {
+  if (c) c->err = msg;
+  return code;
+}
+
+int cuda_fail(starsim_ctx* c, cudaError_t e, const char* where) {
+  return fail(c, e == cudaErrorMemoryAllocation ? STARSIM_ENOMEM : STARSIM_ECUDA,
+              std::string(where) + ": " + cudaGetErrorString(e));
+}
+
+// Grow a scratch buffer geometrically (x1.5); contents are not preserved.
+int grow(starsim_ctx* c, Buf& b, size_t bytes, const char* what) {
+  if (bytes <= b.cap) return STARSIM_OK;
+  size_t want = b.cap + b.cap / 2;
+  if (want < bytes) want = bytes;
+  if (want < 4096) want = 4096;
+  if (b.p) {
+    cudaFree(b.p);  // implicitly synchronises the device: earlier calls that used b are done
+    b.p = nullptr;
+    b.cap = 0;
+  }
+  cudaError_t e = cudaMalloc(&b.p, want);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    e = cudaMalloc(&b.p, bytes);  // retry without headroom
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      b.p = nullptr;
+      return fail(c, STARSIM_ENOMEM, std::string("cudaMalloc(") + what + ", " + std::to_string(bytes) + " B) failed");
+    }
+    want = bytes;
+  }
+  b.cap = want;
+  return STARSIM_OK;
+}
+
+cudaEvent_t get_event(starsim_ctx* c) {
+  if (!c->ev_pool.empty()) {
+    cudaEvent_t e = c->ev_pool.back();
+    c->ev_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+
+// Run `launch` on stream st, bracketed by CUDA events on the same stream when profiling is on.
+template <typename F>
+void timed(starsim_ctx* c, int kclass, cudaStream_t st, F&& launch) {
+  if (!c->prof) {
+    launch();
+    return;
+  }
+  Launch l{kclass, get_event(c), get_event(c)};
+  cudaEventRecord(l.a, st);
+  launch();
+  cudaEventRecord(l.b, st);
+  c->pending.push_back(l);
+}
+
+int check_launch(starsim_ctx* c, const char* where) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, where);
+  return STARSIM_OK;
+}
+
+int validate_frame(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
+                   float sigma, int32_t R, float gain, const void* out) {
+  if (n < 0) return fail(c, STARSIM_EINVAL, "n < 0");
+  if (n > 0 && (!x || !y || !mag)) return fail(c, STARSIM_EINVAL, "n > 0 with a NULL x, y or mag");
+  if (n > 0xFFFFFFFFll) return fail(c, STARSIM_EINVAL, "n >= 2^32 (star indices are 32-bit)");
+  if (!out) return fail(c, STARSIM_EINVAL, "out is NULL");
+  if (W < 1 || W > STARSIM_MAX_DIM || H < 1 || H > STARSIM_MAX_DIM)
+    return fail(c, STARSIM_EINVAL, "width/height outside [1, 32767]");
+  if ((int64_t)W * H >= (1ll << 31)) return fail(c, STARSIM_EINVAL, "width*height >= 2^31");
+  if (!std::isfinite(sigma) || !(sigma > 0.f)) return fail(c, STARSIM_EINVAL, "sigma not finite or <= 0");
+  if (R < 1 || R > STARSIM_MAX_ROI) return fail(c, STARSIM_EINVAL, "roi outside [1, 255]");
+  if (!std::isfinite(gain) || gain < 0.f) return fail(c, STARSIM_EINVAL, "gain not finite or < 0");
+  return STARSIM_OK;
+}
+
+FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float sigma, int32_t R, float gain) {
+  FrameParams fp;
+  fp.W = W;
+  fp.H = H;
+  fp.row0 = row0;
+  fp.rows = rows;
+  fp.R = R;
+  fp.ntx = (W + TILE_W - 1) / TILE_W;
+  fp.nty = (rows + TILE_H - 1) / TILE_H;
+  const double s = (double)sigma;
+  fp.kexp = (float)(-1.0 / (2.0 * s * s * std::log(2.0)));   // exp(-d^2/(2 s^2)) = 2^(kexp d^2)
+  fp.s_scale = (double)gain / (2.0 * M_PI * s * s);          // Eq. 1 gain with Eq. 2's 1/(2 pi s^2)
+  return fp;
+}
+
+int tiles_per_axis(int R, int tile, int ntiles_axis) {
+  int t = (R - 1 + tile - 1) / tile + 1;
+  return t < ntiles_axis ? t : ntiles_axis;
+}
+
+int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
+                 int32_t row0, int32_t rows, float sigma, int32_t R, float gain, float* out, cudaStream_t st) {
+  DevGuard g(c->dev);
+  const FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain);
+  const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
+  const int64_t pmax = n * tiles_per_axis(R, TILE_W, fp.ntx) * (int64_t)tiles_per_axis(R, TILE_H, fp.nty);
+  if (pmax >= 0xFFFFFFFFll) return fail(c, STARSIM_EINVAL, "n * tiles-per-star >= 2^32 (pair counts are 32-bit)");
+  int keybits = 0;
+  while (keybits < 32 && ((int64_t)1 << keybits) < ntiles) ++keybits;
+  const int passes = (keybits + RADIX_BITS - 1) / RADIX_BITS;
+  const int64_t nbin_blk = (n + BIN_TILE - 1) / BIN_TILE;
+  const int64_t nrad_blk = (pmax + RAD_TILE - 1) / RAD_TILE;
+  int rc;
+  if ((rc = grow(c, c->rec, sizeof(StarRec) * (size_t)(n > 0 ? n : 1), "records"))) return rc;
+  if ((rc = grow(c, c->pairs[0], sizeof(uint64_t) * (size_t)(pmax > 0 ? pmax : 1), "pairs"))) return rc;
+  if ((rc = grow(c, c->pairs[1], sizeof(uint64_t) * (size_t)(pmax > 0 ? pmax : 1), "pairs"))) return rc;
+  if ((rc = grow(c, c->tile_off, sizeof(uint32_t) * (size_t)(ntiles + 1), "tile offsets"))) return rc;
+  if ((rc = grow(c, c->st_bin, sizeof(uint64_t) * (size_t)(nbin_blk > 0 ? nbin_blk : 1), "scan status"))) return rc;
+  if ((rc = grow(c, c->st_rad, sizeof(uint64_t) * RADIX * (size_t)(nrad_blk > 0 ? nrad_blk : 1), "radix status")))
+    return rc;
+  if ((rc = grow(c, c->hdr, sizeof(Header), "header"))) return rc;
+
+  c->epoch = (c->epoch + 1) & 0x07FFFFFFu;
+  const uint32_t tag0 = c->epoch * 8u;
+  Header* hdr = (Header*)c->hdr.p;
+  uint64_t* pairs[2] = {(uint64_t*)c->pairs[0].p, (uint64_t*)c->pairs[1].p};
+
+  timed(c, 5, st, [&] { cudaMemsetAsync(hdr, 0, sizeof(Header), st); });
+  if (n > 0)
+    timed(c, 0, st, [&] {
+      launch_bin(x, y, mag, n, fp, (StarRec*)c->rec.p, pairs[0], hdr, (uint64_t*)c->st_bin.p, tag0, passes, st);
+    });
+  if ((rc = check_launch(c, "k_bin"))) return rc;
+  int cur = 0;
+  if (n > 0)
+    for (int p = 0; p < passes; ++p) {
+      timed(c, 1, st, [&] {
+        launch_radix(pairs[cur], pairs[cur ^ 1], hdr, p, (uint64_t*)c->st_rad.p, tag0 + 1u + (uint32_t)p, pmax, st);
+      });
+      cur ^= 1;
+    }
+  if ((rc = check_launch(c, "k_radix"))) return rc;
+  timed(c, 2, st, [&] {
+    launch_offsets(pairs[cur], hdr, (uint32_t)ntiles, (uint32_t*)c->tile_off.p, pmax, c->num_sms, st);
+  });
+  if ((rc = check_launch(c, "k_offsets"))) return rc;
+  timed(c, 3, st, [&] {
+    launch_tile(pairs[cur], (const uint32_t*)c->tile_off.p, (const StarRec*)c->rec.p, fp, out, st);
+  });
+  if ((rc = check_launch(c, "k_tile"))) return rc;
+  c->have_bins = true;
+  c->last_stream = st;
+  c->last_sorted = cur;
+  c->last_ntiles = ntiles;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int starsim_create(starsim_ctx** out, int cuda_device) {
+  if (!out) {
+    g_create_error = "out is NULL";
+    return STARSIM_EINVAL;
+  }
+  *out = nullptr;
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    g_create_error = std::string("no CUDA device: ") + cudaGetErrorString(e);
+    return STARSIM_ENODEV;
+  }
+  if (cuda_device < 0 || cuda_device >= ndev) {
+    g_create_error = "cuda_device out of range";
+    return STARSIM_EINVAL;
+  }
+  cudaDeviceProp prop;
+  if ((e = cudaGetDeviceProperties(&prop, cuda_device)) != cudaSuccess) {
+    g_create_error = std::string("cudaGetDeviceProperties: ") + cudaGetErrorString(e);
+    return STARSIM_ECUDA;
+  }
+  if (!(prop.major == 10 && prop.minor == 0)) {
+    g_create_error = std::string("device ") + prop.name + " is sm_" + std::to_string(prop.major) +
+                     std::to_string(prop.minor) + "; libstarsim.so carries sm_100a code only";
+    return STARSIM_ENODEV;
+  }
+  starsim_ctx* c = new starsim_ctx();
+  c->dev = cuda_device;
+  c->num_sms = prop.multiProcessorCount;
+  *out = c;
+  g_create_error.clear();
+  return STARSIM_OK;
+}
+
+void starsim_destroy(starsim_ctx* c) {
+  if (!c) return;
+  {
+    DevGuard g(c->dev);
+    cudaDeviceSynchronize();
+    Buf* bufs[] = {&c->rec, &c->pairs[0], &c->pairs[1], &c->tile_off, &c->st_bin, &c->st_rad, &c->hdr, &c->stage};
+    for (Buf* b : bufs)
+      if (b->p) cudaFree(b->p);
+    for (auto& l : c->pending) {
+      cudaEventDestroy(l.a);
+      cudaEventDestroy(l.b);
+    }
+    for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
+  }
+  delete c;
+}
+
+const char* starsim_last_error(const starsim_ctx* c) { return c ? c->err.c_str() : g_create_error.c_str(); }
+
+int starsim_render(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
+                   float sigma, int32_t R, float gain, float* out, starsim_stream_t stream) {
+  if (!c) return STARSIM_EINVAL;
+  int rc = validate_frame(c, x, y, mag, n, W, H, sigma, R, gain, out);
+  if (rc) return rc;
+  return render_tiled(c, x, y, mag, n, W, H, 0, H, sigma, R, gain, out, (cudaStream_t)stream);
+}
+
+int starsim_render_band(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W,
+                        int32_t H, int32_t row0, int32_t rows, float sigma, int32_t R, float gain, float* out_band,
+                        starsim_stream_t stream) {
+  if (!c) return STARSIM_EINVAL;
+  int rc = validate_frame(c, x, y, mag, n, W, H, sigma, R, gain, out_band);
+  if (rc) return rc;
+  if (row0 < 0 || rows < 1 || (int64_t)row0 + rows > H) return fail(c, STARSIM_EINVAL, "band not inside the image");
+  return render_tiled(c, x, y, mag, n, W, H, row0, rows, sigma, R, gain, out_band, (cudaStream_t)stream);
+}
+
+int starsim_render_atomic(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W,
+                          int32_t H, float sigma, int32_t R, float gain, float* out, starsim_stream_t stream) {
+  if (!c) return STARSIM_EINVAL;
+  int rc = validate_frame(c, x, y, mag, n, W, H, sigma, R, gain, out);
+  if (rc) return rc;
+  DevGuard g(c->dev);
+  cudaStream_t st = (cudaStream_t)stream;
+  const FrameParams fp = make_params(W, H, 0, H, sigma, R, gain);
+  timed(c, 5, st, [&] { cudaMemsetAsync(out, 0, sizeof(float) * (size_t)W * H, st); });
+  timed(c, 4, st, [&] { launch_atomic(x, y, mag, n, fp, out, st); });
+  if ((rc = check_launch(c, "k_atomic"))) return rc;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
+int starsim_upload_aos(starsim_ctx* c, const void* host_aos, int64_t n, float* x, float* y, float* mag,
+                       starsim_stream_t stream) {
+  if (!c) return STARSIM_EINVAL;
+  if (n < 0) return fail(c, STARSIM_EINVAL, "n < 0");
+  if (n == 0) return STARSIM_OK;
+  if (!host_aos || !x || !y || !mag) return fail(c, STARSIM_EINVAL, "NULL pointer with n > 0");
+  DevGuard g(c->dev);
+  cudaStream_t st = (cudaStream_t)stream;
+  int rc = grow(c, c->stage, sizeof(float) * 3 * (size_t)n, "aos staging");
+  if (rc) return rc;
+  cudaError_t e = cudaMemcpyAsync(c->stage.p, host_aos, sizeof(float) * 3 * (size_t)n, cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) return cuda_fail(c, e, "cudaMemcpyAsync(aos)");
+  timed(c, 7, st, [&] { launch_split_aos((const float*)c->stage.p, n, x, y, mag, c->num_sms, st); });
+  if ((rc = check_launch(c, "k_split_aos"))) return rc;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
+int starsim_quantize(starsim_ctx* c, const float* img, int64_t npix, int32_t bits, void* out,
+                     starsim_stream_t stream) {
+  if (!c) return STARSIM_EINVAL;
+  if (npix < 0) return fail(c, STARSIM_EINVAL, "npix < 0");
+  if (bits != 8 && bits != 16) return fail(c, STARSIM_EINVAL, "bits must be 8 or 16");
+  if (npix > 0 && (!img || !out)) return fail(c, STARSIM_EINVAL, "NULL pointer with npix > 0");
+  if (npix == 0) return STARSIM_OK;
+  DevGuard g(c->dev);
+  cudaStream_t st = (cudaStream_t)stream;
+  timed(c, 6, st, [&] { launch_quantize(img, npix, bits, out, c->num_sms, st); });
+  int rc = check_launch(c, "k_quantize");
+  if (rc) return rc;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
+int starsim_get_bins(starsim_ctx* c, int32_t* tile_w, int32_t* tile_h, uint32_t* tile_off_host, int64_t off_cap,
+                     uint32_t* ids_host, int64_t ids_cap, int64_t* n_pairs) {
+  if (!c) return STARSIM_EINVAL;
+  if (!c->have_bins) return fail(c, STARSIM_EINVAL, "no tiled render on this ctx yet");
+  DevGuard g(c->dev);
+  cudaError_t e = cudaStreamSynchronize(c->last_stream);
+  if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamSynchronize");
+  Header h;
+  if ((e = cudaMemcpy(&h, c->hdr.p, sizeof(Header), cudaMemcpyDeviceToHost)) != cudaSuccess)
+    return cuda_fail(c, e, "cudaMemcpy(header)");
+  if (tile_w) *tile_w = TILE_W;
+  if (tile_h) *tile_h = TILE_H;
+  if (n_pairs) *n_pairs = h.P;
+  if (off_cap < c->last_ntiles + 1 || ids_cap < (int64_t)h.P || !tile_off_host || (!ids_host && h.P))
+    return fail(c, STARSIM_EINVAL, "capacity too small (need ntiles+1 offsets and P ids)");
+  if ((e = cudaMemcpy(tile_off_host, c->tile_off.p, sizeof(uint32_t) * (size_t)(c->last_ntiles + 1),
+                      cudaMemcpyDeviceToHost)) != cudaSuccess)
+    return cuda_fail(c, e, "cudaMemcpy(tile_off)");
+  if (h.P) {
+    std::vector<uint64_t> tmp(h.P);
+    if ((e = cudaMemcpy(tmp.data(), c->pairs[c->last_sorted].p, sizeof(uint64_t) * h.P, cudaMemcpyDeviceToHost)) !=
+        cudaSuccess)
+      return cuda_fail(c, e, "cudaMemcpy(pairs)");
+    for (uint32_t i = 0; i < h.P; ++i) ids_host[i] = (uint32_t)tmp[i];
+  }
+  c->err.clear();
+  return STARSIM_OK;
+}
+
+int starsim_profile(starsim_ctx* c, int enable) {
+  if (!c) return STARSIM_EINVAL;
+  DevGuard g(c->dev);
+  for (auto& l : c->pending) {
+    cudaEventSynchronize(l.b);
+    c->ev_pool.push_back(l.a);
+    c->ev_pool.push_back(l.b);
+  }
+  c->pending.clear();
+  for (int k = 0; k < STARSIM_NUM_KCLASS; ++k) {
+    c->ms[k] = 0;
+    c->launches[k] = 0;
+  }
+  c->prof = enable != 0;
+  return STARSIM_OK;
+}
+
+int starsim_kernel_times(starsim_ctx* c, double* ms, int64_t* launches) {
+  if (!c) return STARSIM_EINVAL;
+  if (!ms || !launches) return fail(c, STARSIM_EINVAL, "NULL output array");
+  DevGuard g(c->dev);
+  for (auto& l : c->pending) {
+    cudaError_t e = cudaEventSynchronize(l.b);
+    if (e != cudaSuccess) return cuda_fail(c, e, "cudaEventSynchronize");
+    float t = 0;
+    cudaEventElapsedTime(&t, l.a, l.b);
+    c->ms[l.kclass] += t;
+    c->launches[l.kclass] += 1;
+    c->ev_pool.push_back(l.a);
+    c->ev_pool.push_back(l.b);
+  }
+  c->pending.clear();
+  for (int k = 0; k < STARSIM_NUM_KCLASS; ++k) {
+    ms[k] = c->ms[k];
+    launches[k] = c->launches[k];
+  }
+  return STARSIM_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,64 @@
+"""Multi-GPU frames: horizontal bands, one per rank, assembled with one all-gather.
+
+The paper is single-GPU and names multi-GPU scaling as future work (Sec. V).  Here the image is split
+into G horizontal bands of whole 32-row tiles; every rank holds the full catalogue, renders its band with
+``starsim_render_band`` (stars are routed to a band iff their clipped ROI rows intersect it -- done inside the
+library's binning pass), and ``torch.distributed.all_gather_into_tensor`` concatenates the bands: row-major band
+concatenation *is* the frame, so there is no re-layout.  With tile-aligned band edges the assembled frame is bitwise
+equal to the single-GPU render (same per-pixel star order).
+
+torch.distributed (NCCL on GPUs, gloo in the CPU tests) is plumbing only; the render runs in libstarsim.so.
+"""
+from __future__ import annotations
+
+TILE_H = 32
+
+
+def band_rows(height: int, world: int, rank: int, align: int = TILE_H) -> tuple[int, int]:
+    """Rows [row0, row0 + rows) of rank's band: equal bands of whole `align`-row tiles when height allows, the last
+    band taking the remainder.  Every row is in exactly one band."""
+    if world < 1 or not (0 <= rank < world):
+        raise ValueError("bad world/rank")
+    tiles = -(-height // align)
+    per = -(-tiles // world)                      # tiles per band (ceil); trailing ranks may get fewer / none
+    t0 = min(tiles, rank * per)
+    t1 = min(tiles, (rank + 1) * per)
+    row0 = min(height, t0 * align)
+    row1 = min(height, t1 * align)
+    return row0, row1 - row0
+
+
+def padded_band_rows(height: int, world: int, align: int = TILE_H) -> int:
+    """Rows of the equal-size band buffers used by the all-gather (all_gather_into_tensor needs equal chunks)."""
+    tiles = -(-height // align)
+    return -(-tiles // world) * align
+
+
+def render_frame(render_band, x, y, mag, width: int, height: int, sigma: float, roi: int, gain: float,
+                 group=None, full_out=None, band_out=None):
+    """Render this rank's band and all-gather the frame.
+
+    ``render_band(x, y, mag, width, height, row0, rows, sigma, roi, gain, out)`` renders rows [row0, row0+rows) into
+    ``out`` (rows x width); for the product it is ``Context.render_band``.  Returns (full_frame, band_view).
+    The gathered tensor has world * padded rows; the frame is its first ``height`` rows.
+    """
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    rank = dist.get_rank(group) if dist.is_initialized() else 0
+    prow = padded_band_rows(height, world)
+    dev = x.device
+    if band_out is None:
+        band_out = torch.zeros((prow, width), dtype=torch.float32, device=dev)
+    row0, rows = band_rows(height, world, rank)
+    if rows > 0:
+        render_band(x, y, mag, width, height, row0, rows, sigma, roi, gain, band_out[:rows])
+    if rows < prow:
+        band_out[rows:].zero_()
+    if world == 1:
+        return band_out[:height], band_out
+    if full_out is None:
+        full_out = torch.empty((world * prow, width), dtype=torch.float32, device=dev)
+    dist.all_gather_into_tensor(full_out, band_out, group=group)
+    return full_out[:height], band_out

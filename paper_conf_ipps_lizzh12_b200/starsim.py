@@ -1,0 +1,257 @@
+"""Thin ctypes binding of libstarsim.so (include/starsim.h) -- argument marshalling only.
+
+Every step of the render runs in the library's sm_100a kernels; this module only converts torch CUDA tensors to
+device pointers and the current torch stream to a ``cudaStream_t``.  There is no CPU fallback: if the library is not
+built, or the device is not an sm_100 GPU, the calls raise.  torch is used for device memory and streams only.
+
+Names mirror the C ABI: ``starsim_create``, ``starsim_render``, ``starsim_render_band``, ``starsim_render_atomic``,
+``starsim_upload_aos``, ``starsim_quantize``, ``starsim_get_bins``, ``starsim_profile``, ``starsim_kernel_times``,
+``starsim_destroy``; :class:`Context` wraps a handle with the same methods.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import threading
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libstarsim.so")
+
+STARSIM_OK, STARSIM_EINVAL, STARSIM_ENOMEM, STARSIM_ECUDA, STARSIM_ENODEV = 0, -1, -2, -3, -4
+KCLASSES = ("bin", "radix", "offsets", "tile", "atomic", "memset", "quantize", "aos")
+NUM_KCLASS = len(KCLASSES)
+
+_lock = threading.Lock()
+_lib = None
+
+
+class StarsimError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"starsim error {code}: {msg}")
+        self.code = code
+
+
+def lib():
+    """Load libstarsim.so (fails loudly if it has not been built)."""
+    global _lib
+    with _lock:
+        if _lib is not None:
+            return _lib
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is not built; run `python -c 'import __graft_entry__ as g; g.build()'`")
+        L = ctypes.CDLL(LIB_PATH)
+        vp, i32, i64, f32 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_float
+        L.starsim_create.argtypes = [ctypes.POINTER(vp), ctypes.c_int]
+        L.starsim_create.restype = ctypes.c_int
+        L.starsim_destroy.argtypes = [vp]
+        L.starsim_destroy.restype = None
+        L.starsim_last_error.argtypes = [vp]
+        L.starsim_last_error.restype = ctypes.c_char_p
+        L.starsim_render.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
+        L.starsim_render.restype = ctypes.c_int
+        L.starsim_render_band.argtypes = [vp, vp, vp, vp, i64, i32, i32, i32, i32, f32, i32, f32, vp, vp]
+        L.starsim_render_band.restype = ctypes.c_int
+        L.starsim_render_atomic.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
+        L.starsim_render_atomic.restype = ctypes.c_int
+        L.starsim_upload_aos.argtypes = [vp, vp, i64, vp, vp, vp, vp]
+        L.starsim_upload_aos.restype = ctypes.c_int
+        L.starsim_quantize.argtypes = [vp, vp, i64, i32, vp, vp]
+        L.starsim_quantize.restype = ctypes.c_int
+        L.starsim_get_bins.argtypes = [vp, ctypes.POINTER(i32), ctypes.POINTER(i32), vp, i64, vp, i64,
+                                       ctypes.POINTER(i64)]
+        L.starsim_get_bins.restype = ctypes.c_int
+        L.starsim_profile.argtypes = [vp, ctypes.c_int]
+        L.starsim_profile.restype = ctypes.c_int
+        L.starsim_kernel_times.argtypes = [vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(i64)]
+        L.starsim_kernel_times.restype = ctypes.c_int
+        _lib = L
+        return L
+
+
+def _check(ctx, rc: int):
+    if rc != STARSIM_OK:
+        raise StarsimError(rc, lib().starsim_last_error(ctx).decode(errors="replace"))
+
+
+def _stream(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
+
+
+def _ptr(t, dtype=None, name="tensor"):
+    if t is None:
+        return None
+    if not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA tensor")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    if dtype is not None and t.dtype != dtype:
+        raise ValueError(f"{name} must be {dtype}, got {t.dtype}")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+# ------------------------------------------------------------------ C-named functions
+
+def starsim_create(device: int = 0):
+    h = ctypes.c_void_p()
+    rc = lib().starsim_create(ctypes.byref(h), int(device))
+    if rc != STARSIM_OK:
+        raise StarsimError(rc, lib().starsim_last_error(None).decode(errors="replace"))
+    return h
+
+
+def starsim_destroy(h) -> None:
+    if h:
+        lib().starsim_destroy(h)
+
+
+def starsim_render(h, x, y, mag, width, height, sigma, roi, gain, out, stream=None) -> None:
+    import torch
+    n = int(x.numel()) if x is not None else 0
+    _check(h, lib().starsim_render(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
+                                   _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
+                                   int(roi), float(gain), _ptr(out, torch.float32, "out"), _stream(stream)))
+
+
+def starsim_render_band(h, x, y, mag, width, height, row0, rows, sigma, roi, gain, out_band, stream=None) -> None:
+    import torch
+    n = int(x.numel()) if x is not None else 0
+    _check(h, lib().starsim_render_band(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
+                                        _ptr(mag, torch.float32, "mag"), n, int(width), int(height), int(row0),
+                                        int(rows), float(sigma), int(roi), float(gain),
+                                        _ptr(out_band, torch.float32, "out_band"), _stream(stream)))
+
+
+def starsim_render_atomic(h, x, y, mag, width, height, sigma, roi, gain, out, stream=None) -> None:
+    import torch
+    n = int(x.numel()) if x is not None else 0
+    _check(h, lib().starsim_render_atomic(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
+                                          _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
+                                          int(roi), float(gain), _ptr(out, torch.float32, "out"), _stream(stream)))
+
+
+def starsim_upload_aos(h, host_aos: np.ndarray, x, y, mag, stream=None) -> None:
+    import torch
+    a = np.ascontiguousarray(host_aos, dtype=np.float32)
+    if a.ndim != 2 or a.shape[1] != 3:
+        raise ValueError("host_aos must be (n, 3) float32 {mag, posX, posY}")
+    _check(h, lib().starsim_upload_aos(h, a.ctypes.data_as(ctypes.c_void_p), a.shape[0],
+                                       _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
+                                       _ptr(mag, torch.float32, "mag"), _stream(stream)))
+
+
+def starsim_quantize(h, img, bits, out, stream=None) -> None:
+    import torch
+    want = torch.uint8 if bits == 8 else torch.uint16 if bits == 16 else None
+    _check(h, lib().starsim_quantize(h, _ptr(img, torch.float32, "img"), int(img.numel()), int(bits),
+                                     _ptr(out, want, "out") if want is not None else ctypes.c_void_p(out.data_ptr()),
+                                     _stream(stream)))
+
+
+def starsim_get_bins(h, max_pairs: int | None = None):
+    """(tile_w, tile_h, tile_off uint32[ntiles+1], ids uint32[P]) of the last tiled render (synchronises)."""
+    tw, th, P = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int64()
+    rc = lib().starsim_get_bins(h, ctypes.byref(tw), ctypes.byref(th), None, 0, None, 0, ctypes.byref(P))
+    if rc not in (STARSIM_OK, STARSIM_EINVAL) or P.value < 0:
+        _check(h, rc)
+    # ask again with buffers sized from the reply; ntiles is unknown here so grow until accepted
+    cap_off = 1 << 12
+    while True:
+        off = np.zeros(cap_off, dtype=np.uint32)
+        ids = np.zeros(max(1, P.value), dtype=np.uint32)
+        rc = lib().starsim_get_bins(h, ctypes.byref(tw), ctypes.byref(th), off.ctypes.data_as(ctypes.c_void_p),
+                                    cap_off, ids.ctypes.data_as(ctypes.c_void_p), ids.size, ctypes.byref(P))
+        if rc == STARSIM_OK:
+            break
+        if rc != STARSIM_EINVAL or cap_off > (1 << 26):
+            _check(h, rc)
+        cap_off *= 4
+    return tw.value, th.value, off, ids[:P.value]
+
+
+def starsim_profile(h, enable: bool) -> None:
+    _check(h, lib().starsim_profile(h, 1 if enable else 0))
+
+
+def starsim_kernel_times(h) -> dict:
+    ms = (ctypes.c_double * NUM_KCLASS)()
+    ln = (ctypes.c_int64 * NUM_KCLASS)()
+    _check(h, lib().starsim_kernel_times(h, ms, ln))
+    return {k: (ms[i], ln[i]) for i, k in enumerate(KCLASSES)}
+
+
+# ------------------------------------------------------------------ convenience handle
+
+class Context:
+    """One libstarsim context bound to one CUDA device (not thread-safe)."""
+
+    def __init__(self, device: int | None = None):
+        import torch
+        self.device = torch.cuda.current_device() if device is None else int(device)
+        self.h = starsim_create(self.device)
+
+    def close(self):
+        if self.h:
+            starsim_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def _out(self, rows, width, out):
+        import torch
+        if out is None:
+            out = torch.empty((rows, width), dtype=torch.float32, device=f"cuda:{self.device}")
+        return out
+
+    def render(self, x, y, mag, width, height, sigma, roi, gain, out=None, stream=None):
+        out = self._out(height, width, out)
+        starsim_render(self.h, x, y, mag, width, height, sigma, roi, gain, out, stream)
+        return out
+
+    def render_band(self, x, y, mag, width, height, row0, rows, sigma, roi, gain, out=None, stream=None):
+        out = self._out(rows, width, out)
+        starsim_render_band(self.h, x, y, mag, width, height, row0, rows, sigma, roi, gain, out, stream)
+        return out
+
+    def render_atomic(self, x, y, mag, width, height, sigma, roi, gain, out=None, stream=None):
+        out = self._out(height, width, out)
+        starsim_render_atomic(self.h, x, y, mag, width, height, sigma, roi, gain, out, stream)
+        return out
+
+    def upload_aos(self, host_aos, stream=None):
+        import torch
+        n = int(np.asarray(host_aos).shape[0])
+        dev = f"cuda:{self.device}"
+        x, y, m = (torch.empty(n, dtype=torch.float32, device=dev) for _ in range(3))
+        starsim_upload_aos(self.h, host_aos, x, y, m, stream)
+        return x, y, m
+
+    def quantize(self, img, bits=8, out=None, stream=None):
+        import torch
+        if out is None:
+            out = torch.empty(img.shape, dtype=torch.uint8 if bits == 8 else torch.uint16, device=img.device)
+        starsim_quantize(self.h, img, bits, out, stream)
+        return out
+
+    def get_bins(self):
+        return starsim_get_bins(self.h)
+
+    def profile(self, enable=True):
+        starsim_profile(self.h, enable)
+
+    def kernel_times(self):
+        return starsim_kernel_times(self.h)

@@ -1,0 +1,290 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle on the same seeded inputs.
+
+Tolerances (BASELINE.json north_star): float image max-abs error <= 1e-5 * peak and relative L2 error <= 1e-6;
+quantised gray within +-1 LSB (bit-exact on identical fp32 input); binning (CSR) bit-exact.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+MAX_ABS = 1e-5
+REL_L2 = 1e-6
+
+
+@pytest.fixture(scope="module")
+def torch_dev():
+    import torch
+    if not torch.cuda.is_available():
+        raise RuntimeError("GPU tests need a CUDA device")
+    import __graft_entry__
+    __graft_entry__.build()
+    return torch, torch.device("cuda:0")
+
+
+@pytest.fixture(scope="module")
+def ctx(torch_dev):
+    from paper_conf_ipps_lizzh12_b200 import Context
+    c = Context(0)
+    yield c
+    c.close()
+
+
+def to_dev(torch_dev, f):
+    torch, dev = torch_dev
+    return tuple(torch.from_numpy(np.ascontiguousarray(a)).to(dev) for a in (f.x, f.y, f.mag))
+
+
+def errors(got, ref):
+    peak = float(np.abs(ref).max()) if ref.size else 0.0
+    if peak == 0.0:
+        return float(np.abs(got).max()) if got.size else 0.0, 0.0
+    return float(np.abs(got - ref).max()) / peak, float(np.linalg.norm(got - ref) / np.linalg.norm(ref))
+
+
+def assert_parity(got, ref, what=""):
+    ma, rl = errors(got.astype(np.float64), ref)
+    assert ma <= MAX_ABS and rl <= REL_L2, f"{what}: max_abs/peak={ma:.3e} rel_l2={rl:.3e}"
+
+
+# ---------------------------------------------------------------- C1 (BASELINE configs[0]) and fig2
+
+@pytest.mark.parametrize("mags", [(0.0, 15.0), (0.0, 2.0)])
+@pytest.mark.parametrize("method", ["render", "render_atomic"])
+def test_c1_parity(torch_dev, ctx, mags, method):
+    cfg = synth.CONFIGS["C1"]
+    f = cfg.field(mag_lo=mags[0], mag_hi=mags[1])
+    ref = oracle.render(f.x, f.y, f.mag, cfg.W, cfg.H, cfg.sigma, cfg.R, 1.0)
+    img = getattr(ctx, method)(*to_dev(torch_dev, f), cfg.W, cfg.H, cfg.sigma, cfg.R, 1.0)
+    assert_parity(img.cpu().numpy(), ref, f"C1 {method} {mags}")
+
+
+@pytest.mark.parametrize("R", [10, 11])
+def test_fig2_parity(torch_dev, ctx, R):
+    cfg = synth.CONFIGS["fig2"]
+    f = cfg.field(mag_lo=0.0, mag_hi=2.0)
+    ref = oracle.render(f.x, f.y, f.mag, cfg.W, cfg.H, 1.0, R, 1.0)
+    for method in ("render", "render_atomic"):
+        img = getattr(ctx, method)(*to_dev(torch_dev, f), cfg.W, cfg.H, 1.0, R, 1.0)
+        assert_parity(img.cpu().numpy(), ref, f"fig2 R={R} {method}")
+
+
+# ---------------------------------------------------------------- randomized edge cases
+
+def fuzz_cases(count=40):
+    rng = np.random.default_rng(2024)
+    cases = []
+    for k in range(count):
+        W, H = int(rng.integers(1, 300)), int(rng.integers(1, 300))
+        n = int(rng.integers(0, 2000))
+        R = int(rng.integers(1, 64))
+        sigma = float(np.exp(rng.uniform(math.log(0.3), math.log(20.0))))
+        cases.append((k, W, H, n, R, sigma))
+    # explicit extremes: 1x1 image, empty catalogue, R = 1, largest R, R = 16 (window switch), tile-multiple sizes
+    cases += [(100, 1, 1, 10, 1, 1.0), (101, 64, 64, 0, 5, 1.0), (102, 65, 33, 500, 16, 2.0),
+              (103, 300, 200, 300, 255, 40.0), (104, 256, 256, 2000, 15, 2.5), (105, 33, 1, 50, 7, 1.0)]
+    return cases
+
+
+@pytest.mark.parametrize("case", fuzz_cases(), ids=lambda c: f"k{c[0]}-{c[1]}x{c[2]}-n{c[3]}-R{c[4]}")
+def test_fuzz_parity(torch_dev, ctx, case):
+    k, W, H, n, R, sigma = case
+    f = synth.adversarial_field(n, W, H, R, seed=k + 7) if k % 2 else synth.uniform_field(n, W, H, seed=k, mag_hi=2.0)
+    ref = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0)
+    img = ctx.render(*to_dev(torch_dev, f), W, H, sigma, R, 1.0).cpu().numpy()
+    if not np.any(ref):
+        assert not np.any(img)
+    else:
+        assert_parity(img, ref, f"fuzz {case}")
+    img_a = ctx.render_atomic(*to_dev(torch_dev, f), W, H, sigma, R, 1.0).cpu().numpy()
+    if np.any(ref):
+        assert_parity(img_a, ref, f"fuzz atomic {case}")
+
+
+# ---------------------------------------------------------------- binning bit-exact (CSR)
+
+@pytest.mark.parametrize("name,n,R,kind", [("small", 3000, 15, "uniform"), ("adv", 2000, 9, "adversarial"),
+                                            ("wide", 500, 63, "uniform"), ("clustered", 20000, 15, "clustered"),
+                                            ("r1", 5000, 1, "uniform")])
+def test_bins_bit_exact(torch_dev, ctx, name, n, R, kind):
+    W, H = 700, 530
+    if kind == "adversarial":
+        f = synth.adversarial_field(n, W, H, R, seed=5)
+    elif kind == "clustered":
+        f = synth.clustered_field(n, W, H, seed=6)
+    else:
+        f = synth.uniform_field(n, W, H, seed=7)
+    ctx.render(*to_dev(torch_dev, f), W, H, R / 6, R, 1.0)
+    tw, th, off, ids = ctx.get_bins()
+    ntiles = (-(-W // tw)) * (-(-H // th))
+    ref_off, ref_ids = oracle.bins(f.x, f.y, f.mag, W, H, R, tw, th)
+    assert np.array_equal(off[:ntiles + 1], ref_off)
+    assert np.array_equal(ids, ref_ids)
+
+
+# ---------------------------------------------------------------- determinism and translation
+
+def test_deterministic_and_tile_translation(torch_dev, ctx):
+    torch, dev = torch_dev
+    W, H = 512, 384
+    f = synth.uniform_field(20000, W - 64, H - 64, seed=3, mag_hi=2.0)
+    # positions on a 1/256 grid so that x + 32 and y + 64 are exact in fp32
+    f = synth.Field(np.round(f.x * 256).astype(np.float32) / np.float32(256),
+                    np.round(f.y * 256).astype(np.float32) / np.float32(256), f.mag)
+    x, y, m = to_dev(torch_dev, f)
+    a = ctx.render(x, y, m, W, H, 2.5, 15, 7.0)
+    b = ctx.render(x, y, m, W, H, 2.5, 15, 7.0)
+    assert torch.equal(a, b)
+    # shift by whole tiles: every per-pixel sum sees the same stars in the same order
+    c = ctx.render(x + 32, y + 64, m, W, H, 2.5, 15, 7.0)
+    assert torch.equal(a[:H - 64, :W - 32], c[64:, 32:])
+
+
+# ---------------------------------------------------------------- bands (multi-GPU decomposition, one device)
+
+@pytest.mark.parametrize("G", [2, 4, 8])
+def test_bands_concatenate_to_frame(torch_dev, ctx, G):
+    torch, dev = torch_dev
+    W, H = 640, 512
+    f = synth.uniform_field(15000, W, H, seed=G, mag_hi=2.0)
+    x, y, m = to_dev(torch_dev, f)
+    full = ctx.render(x, y, m, W, H, 2.5, 15, 1.0)
+    rows = H // G
+    bands = [ctx.render_band(x, y, m, W, H, g * rows, rows, 2.5, 15, 1.0) for g in range(G)]
+    assert torch.equal(torch.cat(bands, 0), full)
+
+
+def test_unaligned_band_matches_oracle(torch_dev, ctx):
+    W, H = 200, 150
+    f = synth.adversarial_field(800, W, H, 11, seed=9)
+    ref = oracle.render_band(f.x, f.y, f.mag, W, H, 37, 61, 1.8, 11, 1.0)
+    got = ctx.render_band(*to_dev(torch_dev, f), W, H, 37, 61, 1.8, 11, 1.0).cpu().numpy()
+    assert_parity(got, ref, "band 37+61")
+
+
+# ---------------------------------------------------------------- quantiser
+
+@pytest.mark.parametrize("bits", [8, 16])
+def test_quantize(torch_dev, ctx, bits):
+    torch, dev = torch_dev
+    cfg = synth.CONFIGS["C1"]
+    f = cfg.field(mag_lo=0.0, mag_hi=4.0)
+    A = synth.bench_gain(cfg.sigma, bits)
+    img = ctx.render(*to_dev(torch_dev, f), cfg.W, cfg.H, cfg.sigma, cfg.R, A)
+    q = ctx.quantize(img, bits).cpu().numpy()
+    # bit-exact on the same fp32 input
+    q_same = oracle.quantize(img.cpu().numpy().astype(np.float64), bits)
+    assert np.array_equal(q, q_same)
+    # within +-1 LSB of quantising the fp64 oracle image
+    ref = oracle.render(f.x, f.y, f.mag, cfg.W, cfg.H, cfg.sigma, cfg.R, A)
+    q_ref = oracle.quantize(ref, bits)
+    d = np.abs(q.astype(np.int64) - q_ref.astype(np.int64))
+    assert d.max() <= 1
+
+
+def test_quantize_edge_values(torch_dev, ctx):
+    torch, dev = torch_dev
+    vals = np.array([0.0, -0.0, -3.0, 0.49999997, 0.5, 0.50000006, 1.5, 2.5, 254.5, 254.49998, 255.49998, 255.5,
+                     1e30, np.inf, -np.inf, np.nan, 65534.5, 65535.5, 7.0], dtype=np.float32)
+    for off in range(4):   # misaligned heads exercise the scalar path
+        v = np.concatenate([np.zeros(off, np.float32), vals, np.full(5, 3.7, np.float32)])
+        t = torch.from_numpy(v).to(dev)
+        for bits in (8, 16):
+            got = ctx.quantize(t, bits).cpu().numpy()
+            assert np.array_equal(got, oracle.quantize(v.astype(np.float64), bits))
+
+
+# ---------------------------------------------------------------- boundary contract (T1)
+
+def test_einval_leaves_out_untouched(torch_dev, ctx):
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import StarsimError, starsim as S
+    f = synth.uniform_field(10, 32, 32, seed=1)
+    x, y, m = to_dev(torch_dev, f)
+    out = torch.full((32, 32), 7.0, device=dev)
+    bad = [dict(width=0), dict(height=40000), dict(sigma=0.0), dict(sigma=float("nan")), dict(roi=0),
+           dict(roi=256), dict(gain=-1.0), dict(gain=float("inf"))]
+    for b in bad:
+        kw = dict(width=32, height=32, sigma=1.0, roi=5, gain=1.0)
+        kw.update(b)
+        with pytest.raises(StarsimError) as e:
+            S.starsim_render(ctx.h, x, y, m, kw["width"], kw["height"], kw["sigma"], kw["roi"], kw["gain"], out)
+        assert e.value.code == -1
+    with pytest.raises(StarsimError):
+        S.starsim_render_band(ctx.h, x, y, m, 32, 32, 20, 13, 1.0, 5, 1.0, out)
+    with pytest.raises(StarsimError):
+        S.starsim_quantize(ctx.h, out, 7, torch.empty(32, 32, dtype=torch.uint8, device=dev))
+    torch.cuda.synchronize()
+    assert bool((out == 7.0).all())
+
+
+def test_empty_catalogue_gives_zero_image(torch_dev, ctx):
+    torch, dev = torch_dev
+    e = torch.empty(0, dtype=torch.float32, device=dev)
+    out = torch.full((70, 90), 5.0, device=dev)
+    ctx.render(e, e, e, 90, 70, 1.0, 5, 1.0, out=out)
+    assert bool((out == 0).all())
+    out.fill_(5.0)
+    ctx.render_atomic(e, e, e, 90, 70, 1.0, 5, 1.0, out=out)
+    assert bool((out == 0).all())
+
+
+def test_upload_aos_splits_the_paper_record(torch_dev, ctx):
+    f = synth.uniform_field(12345, 1000, 800, seed=2)
+    x, y, m = ctx.upload_aos(f.aos())
+    assert np.array_equal(x.cpu().numpy(), f.x) and np.array_equal(y.cpu().numpy(), f.y)
+    assert np.array_equal(m.cpu().numpy(), f.mag)
+
+
+def test_kernel_times_recorded(torch_dev, ctx):
+    cfg = synth.CONFIGS["C1"]
+    f = cfg.field()
+    args = to_dev(torch_dev, f)
+    ctx.profile(True)
+    ctx.render(*args, cfg.W, cfg.H, cfg.sigma, cfg.R, 1.0)
+    t = ctx.kernel_times()
+    ctx.profile(False)
+    assert t["tile"][1] == 1 and t["tile"][0] > 0 and t["bin"][1] == 1
+
+
+# ---------------------------------------------------------------- B200-scale frames (full images, threaded oracle)
+
+def _threads():
+    import os
+    return max(1, os.cpu_count() or 1)
+
+
+@pytest.mark.parametrize("name", ["C2", "T"])
+def test_full_frame_parity(torch_dev, ctx, name):
+    cfg = synth.CONFIGS[name]
+    f = cfg.field(mag_lo=0.0, mag_hi=15.0)
+    A = synth.bench_gain(cfg.sigma)
+    ref = oracle.render(f.x, f.y, f.mag, cfg.W, cfg.H, cfg.sigma, cfg.R, A, threads=_threads())
+    img = ctx.render(*to_dev(torch_dev, f), cfg.W, cfg.H, cfg.sigma, cfg.R, A).cpu().numpy()
+    assert_parity(img, ref, name)
+
+
+@pytest.mark.parametrize("R", [3, 15, 63])
+def test_c4_clustered_parity(torch_dev, ctx, R):
+    cfg = synth.with_R(synth.CONFIGS["C4"], R)
+    f = cfg.field()
+    A = synth.bench_gain(cfg.sigma)
+    ref = oracle.render(f.x, f.y, f.mag, cfg.W, cfg.H, cfg.sigma, cfg.R, A, threads=_threads())
+    img = ctx.render(*to_dev(torch_dev, f), cfg.W, cfg.H, cfg.sigma, cfg.R, A).cpu().numpy()
+    assert_parity(img, ref, cfg.name)
+
+
+def test_c5_sampled_rows(torch_dev, ctx):
+    """16384^2, 10M stars, R=15 in the bench's launch configuration: rows sampled and computed by the oracle."""
+    cfg = synth.CONFIGS["C5"]
+    f = cfg.field()
+    A = synth.bench_gain(cfg.sigma)
+    img = ctx.render(*to_dev(torch_dev, f), cfg.W, cfg.H, cfg.sigma, cfg.R, A)
+    for row in [0, 1, 4095, 8191, 8192, 16383]:
+        ref = oracle.render_band(f.x, f.y, f.mag, cfg.W, cfg.H, row, 1, cfg.sigma, cfg.R, A)
+        assert_parity(img[row:row + 1].cpu().numpy(), ref, f"C5 row {row}")
