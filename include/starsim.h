@@ -12,8 +12,8 @@
  *
  * Conventions for every entry point:
  *   - Array pointers marked (device) are CUDA device pointers on the ctx's device; (host) are host pointers.
- *   - The caller owns every input and output buffer.  The ctx owns its scratch (star records, tile pairs, sort
- *     buffers, offsets); scratch grows geometrically, is reused across calls and is freed by starsim_destroy.
+ *   - The caller owns every input and output buffer.  The ctx owns its scratch (star records, tile lists, sort
+ *     scratch, offsets); scratch grows geometrically, is reused across calls and is freed by starsim_destroy.
  *   - Calls are stream-ordered and asynchronous on `stream` (0 = legacy default stream); host-side validation is
  *     synchronous and happens before anything is enqueued.
  *   - A ctx is bound to one device and is not thread-safe: use one ctx per host thread / stream.
@@ -57,8 +57,9 @@ void starsim_destroy(starsim_ctx* ctx);
  * (then a static description of the last create failure). */
 const char* starsim_last_error(const starsim_ctx* ctx);
 
-/* Render a full frame with the tiled, atomic-free path: per-star prep + binning of (tile, star)
- * pairs + stable radix sort + CSR, then one register-accumulating tile kernel that writes every pixel once.
+/* Render a full frame with the tiled path: per-star prep + binning of the (tile, star) pairs by a
+ * one-digit counting (radix) sort on the tile key + per-tile sort into star order (CSR), then one register-
+ * accumulating tile kernel, free of atomics on the image, that writes every pixel once.
  *   x, y, mag  (device) float[n]: the star catalogue as SoA -- sub-pixel centre (image coordinates) and magnitude.
  *   n          number of stars, >= 0 (0 -> an all-zero image).  x, y, mag may be NULL iff n == 0.
  *   width, height   image size in pixels, each in [1, 32767], width*height < 2^31.
@@ -116,8 +117,8 @@ int starsim_get_bins(starsim_ctx* ctx, int32_t* tile_w, int32_t* tile_h,
 /* Per-kernel device timing for roofline reporting.  When enabled, every launch of the library records CUDA events
  * on the launching stream around it; starsim_kernel_times() synchronises and returns, per kernel class, the summed
  * elapsed milliseconds and launch counts since the last reset.  Classes (index into the arrays):
- *   0 prep+scan+emit, 1 radix passes, 2 tile offsets, 3 tile accumulate, 4 atomic scatter, 5 memsets/zero,
- *   6 quantise, 7 aos upload split.
+ *   0 prep + tile counting + CSR scan (k_count), 1 counting-sort scatter (k_scatter), 2 per-tile star-order sort
+ *   (k_segsort), 3 tile accumulate (k_tile), 4 atomic scatter (k_atomic), 5 memsets, 6 quantise, 7 aos split.
  * `ms` and `launches` must hold STARSIM_NUM_KCLASS entries.  enable != 0 turns recording on and resets. */
 #define STARSIM_NUM_KCLASS 8
 int starsim_profile(starsim_ctx* ctx, int enable);

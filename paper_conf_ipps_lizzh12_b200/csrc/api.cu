@@ -32,12 +32,11 @@ struct starsim_ctx {
   int dev = 0;
   int num_sms = 148;
   std::string err;
-  Buf rec, pairs[2], tile_off, st_bin, st_rad, hdr, stage;
+  Buf rec, ids, scratch, tile_off, hdr, stage;
   uint32_t epoch = 0;
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
   cudaStream_t last_stream = nullptr;
-  int last_sorted = 0;
   int64_t last_ntiles = 0;
   // profiling
   bool prof = false;
@@ -171,52 +170,33 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   const int64_t pmax = n * tiles_per_axis(R, TILE_W, fp.ntx) * (int64_t)tiles_per_axis(R, TILE_H, fp.nty);
   if (pmax >= 0xFFFFFFFFll) return fail(c, STARSIM_EINVAL, "n * tiles-per-star >= 2^32 (pair counts are 32-bit)");
-  int keybits = 0;
-  while (keybits < 32 && ((int64_t)1 << keybits) < ntiles) ++keybits;
-  const int passes = (keybits + RADIX_BITS - 1) / RADIX_BITS;
-  const int64_t nbin_blk = (n + BIN_TILE - 1) / BIN_TILE;
-  const int64_t nrad_blk = (pmax + RAD_TILE - 1) / RAD_TILE;
   int rc;
   if ((rc = grow(c, c->rec, sizeof(StarRec) * (size_t)(n > 0 ? n : 1), "records"))) return rc;
-  if ((rc = grow(c, c->pairs[0], sizeof(uint64_t) * (size_t)(pmax > 0 ? pmax : 1), "pairs"))) return rc;
-  if ((rc = grow(c, c->pairs[1], sizeof(uint64_t) * (size_t)(pmax > 0 ? pmax : 1), "pairs"))) return rc;
+  if ((rc = grow(c, c->ids, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "tile lists"))) return rc;
+  if ((rc = grow(c, c->scratch, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "sort scratch"))) return rc;
   if ((rc = grow(c, c->tile_off, sizeof(uint32_t) * (size_t)(ntiles + 1), "tile offsets"))) return rc;
-  if ((rc = grow(c, c->st_bin, sizeof(uint64_t) * (size_t)(nbin_blk > 0 ? nbin_blk : 1), "scan status"))) return rc;
-  if ((rc = grow(c, c->st_rad, sizeof(uint64_t) * RADIX * (size_t)(nrad_blk > 0 ? nrad_blk : 1), "radix status")))
-    return rc;
-  if ((rc = grow(c, c->hdr, sizeof(Header), "header"))) return rc;
+  const size_t hdr_bytes = sizeof(Header) + sizeof(uint32_t) * (size_t)ntiles;
+  if ((rc = grow(c, c->hdr, hdr_bytes, "header+counters"))) return rc;
 
-  c->epoch = (c->epoch + 1) & 0x07FFFFFFu;
-  const uint32_t tag0 = c->epoch * 8u;
   Header* hdr = (Header*)c->hdr.p;
-  uint64_t* pairs[2] = {(uint64_t*)c->pairs[0].p, (uint64_t*)c->pairs[1].p};
+  uint32_t* cnt = (uint32_t*)(hdr + 1);
+  uint32_t* ids = (uint32_t*)c->ids.p;
+  uint32_t* tile_off = (uint32_t*)c->tile_off.p;
+  StarRec* rec = (StarRec*)c->rec.p;
 
-  timed(c, 5, st, [&] { cudaMemsetAsync(hdr, 0, sizeof(Header), st); });
-  if (n > 0)
-    timed(c, 0, st, [&] {
-      launch_bin(x, y, mag, n, fp, (StarRec*)c->rec.p, pairs[0], hdr, (uint64_t*)c->st_bin.p, tag0, passes, st);
-    });
-  if ((rc = check_launch(c, "k_bin"))) return rc;
-  int cur = 0;
-  if (n > 0)
-    for (int p = 0; p < passes; ++p) {
-      timed(c, 1, st, [&] {
-        launch_radix(pairs[cur], pairs[cur ^ 1], hdr, p, (uint64_t*)c->st_rad.p, tag0 + 1u + (uint32_t)p, pmax, st);
-      });
-      cur ^= 1;
-    }
-  if ((rc = check_launch(c, "k_radix"))) return rc;
-  timed(c, 2, st, [&] {
-    launch_offsets(pairs[cur], hdr, (uint32_t)ntiles, (uint32_t*)c->tile_off.p, pmax, c->num_sms, st);
-  });
-  if ((rc = check_launch(c, "k_offsets"))) return rc;
-  timed(c, 3, st, [&] {
-    launch_tile(pairs[cur], (const uint32_t*)c->tile_off.p, (const StarRec*)c->rec.p, fp, out, st);
-  });
+  timed(c, 5, st, [&] { cudaMemsetAsync(hdr, 0, hdr_bytes, st); });
+  timed(c, 0, st, [&] { launch_count(x, y, mag, n, fp, rec, cnt, hdr, tile_off, (uint32_t)ntiles, st); });
+  if ((rc = check_launch(c, "k_count"))) return rc;
+  if (n > 0) {
+    timed(c, 1, st, [&] { launch_scatter(rec, n, fp, cnt, ids, st); });
+    if ((rc = check_launch(c, "k_scatter"))) return rc;
+    timed(c, 2, st, [&] { launch_segsort(ids, (uint32_t*)c->scratch.p, tile_off, (uint32_t)ntiles, st); });
+    if ((rc = check_launch(c, "k_segsort"))) return rc;
+  }
+  timed(c, 3, st, [&] { launch_tile(ids, tile_off, rec, fp, out, st); });
   if ((rc = check_launch(c, "k_tile"))) return rc;
   c->have_bins = true;
   c->last_stream = st;
-  c->last_sorted = cur;
   c->last_ntiles = ntiles;
   c->err.clear();
   return STARSIM_OK;
@@ -266,7 +246,7 @@ void starsim_destroy(starsim_ctx* c) {
   {
     DevGuard g(c->dev);
     cudaDeviceSynchronize();
-    Buf* bufs[] = {&c->rec, &c->pairs[0], &c->pairs[1], &c->tile_off, &c->st_bin, &c->st_rad, &c->hdr, &c->stage};
+    Buf* bufs[] = {&c->rec, &c->ids, &c->scratch, &c->tile_off, &c->hdr, &c->stage};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {
@@ -365,13 +345,8 @@ int starsim_get_bins(starsim_ctx* c, int32_t* tile_w, int32_t* tile_h, uint32_t*
   if ((e = cudaMemcpy(tile_off_host, c->tile_off.p, sizeof(uint32_t) * (size_t)(c->last_ntiles + 1),
                       cudaMemcpyDeviceToHost)) != cudaSuccess)
     return cuda_fail(c, e, "cudaMemcpy(tile_off)");
-  if (h.P) {
-    std::vector<uint64_t> tmp(h.P);
-    if ((e = cudaMemcpy(tmp.data(), c->pairs[c->last_sorted].p, sizeof(uint64_t) * h.P, cudaMemcpyDeviceToHost)) !=
-        cudaSuccess)
-      return cuda_fail(c, e, "cudaMemcpy(pairs)");
-    for (uint32_t i = 0; i < h.P; ++i) ids_host[i] = (uint32_t)tmp[i];
-  }
+  if (h.P && (e = cudaMemcpy(ids_host, c->ids.p, sizeof(uint32_t) * h.P, cudaMemcpyDeviceToHost)) != cudaSuccess)
+    return cuda_fail(c, e, "cudaMemcpy(ids)");
   c->err.clear();
   return STARSIM_OK;
 }

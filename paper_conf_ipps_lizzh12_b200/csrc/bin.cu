@@ -1,5 +1,12 @@
-// Binning: per-star prep + scan + emit of (tile, star) pairs (k_bin), stable LSD radix sort (k_radix), CSR tile
-// offsets (k_offsets).  DESIGN.md §Path steps a1-a4.  All sm_100a CUDA, no library calls.
+// Binning of the catalogue into 32x32 image tiles (DESIGN.md §Path steps a1-a4):
+//   k_count   a1: per-star prep (validity, s' in fp64, exact ROI origin, clip) + counting of the (tile, star) pairs
+//             per tile key with global atomics; the last block to finish scans the counts into the CSR offsets.
+//   k_scatter a3: every star writes its index into each overlapped tile's segment (slot from an atomic cursor) --
+//             a one-digit (radix 2^keybits) counting sort by tile key.
+//   k_segsort a4: restores star-index order inside every tile segment (bitonic in shared memory; heavy segments by
+//             a warp merge sort through global scratch), so the CSR is unique and the per-pixel summation order of
+//             k_tile is the paper's star order -- bitwise reproducible and identical across band decompositions.
+// All sm_100a CUDA, no library calls.
 #include <algorithm>
 
 #include "common.cuh"
@@ -7,238 +14,217 @@
 
 namespace starsim {
 
-// ---------------------------------------------------------------------------------------------------------------
-// k_bin -- one pass over the catalogue (step a1 + a2 + a3 + the radix histograms):
-//   per star: reject non-finite x, y, mag (reading R11); s' = A 2.512^-m / (2 pi sigma^2) in fp64 (Eq. 1 with the
-//   1/(2 pi sigma^2) of Eq. 2 folded in); exact ROI origin (reading R7); clip to the image columns and the band rows;
-//   count the 32x32 tiles the clipped ROI overlaps; single-pass exclusive scan of the counts over stars (decoupled
-//   look-back across blocks); emit the star's pairs (key = ty*ntx + tx, value = star index) in star order, tiles
-//   row-major; histogram the radix digits of every key.
-// Layout: 256 threads x 8 stars, striped loads (coalesced), blocked scan through shared memory.
-// ---------------------------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(BIN_THREADS) k_bin(const float* __restrict__ X, const float* __restrict__ Y,
-                                                     const float* __restrict__ M, int64_t n, FrameParams fp,
-                                                     StarRec* __restrict__ rec, uint64_t* __restrict__ pairs,
-                                                     Header* hdr, uint64_t* status, uint32_t tag, int passes) {
-  __shared__ uint32_t s_cnt[BIN_TILE];
-  __shared__ uint32_t s_hist[MAX_PASSES][RADIX];
-  __shared__ uint32_t s_warp[BIN_THREADS / 32];
-  __shared__ uint32_t s_base;
-  __shared__ int64_t s_blk;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid == 0) s_blk = atomicAdd(&hdr->ticket[0], 1u);
-  for (int i = tid; i < MAX_PASSES * RADIX; i += BIN_THREADS) (&s_hist[0][0])[i] = 0;
-  __syncthreads();
-  const int64_t blk = s_blk;
-  const int64_t base = blk * BIN_TILE;
+// Clipped ROI of a record against the frame columns and the band rows; false if culled or empty.
+__device__ __forceinline__ bool clip_roi(const FrameParams& fp, uint32_t lo, int& cx0, int& cx1, int& cy0, int& cy1) {
+  if (lo == LO_CULLED) return false;
+  const int lx = lo_x_of(lo), ly = lo_y_of(lo);
+  cx0 = max(lx, 0);
+  cx1 = min(lx + fp.R - 1, fp.W - 1);
+  cy0 = max(ly, fp.row0);
+  cy1 = min(ly + fp.R - 1, fp.row0 + fp.rows - 1);
+  return cx0 <= cx1 && cy0 <= cy1;
+}
 
-  // ---- a1: per-star prep (striped: star base + k*256 + tid)
-  uint32_t cnts[BIN_ITEMS];      // tiles per star
-  uint16_t tr[BIN_ITEMS][4];     // its tile range tx0, tx1, ty0, ty1
-#pragma unroll
-  for (int k = 0; k < BIN_ITEMS; ++k) {
-    const int64_t i = base + k * BIN_THREADS + tid;
-    uint32_t cnt = 0;
-    if (i < n) {
-      const float x = X[i], y = Y[i], m = M[i];
-      const float R = (float)fp.R;
-      bool ok = isfinite(x) && isfinite(y) && isfinite(m);
-      // pre-filter far-off stars (keeps the int conversions exact); the exact test is the clip below
-      ok = ok && x > -R - 2.f && x < (float)fp.W + R + 2.f && y > (float)fp.row0 - R - 2.f &&
-           y < (float)(fp.row0 + fp.rows) + R + 2.f;
-      int lx = 0, ly = 0, cx0 = 0, cx1 = -1, cy0 = 0, cy1 = -1;
-      if (ok) {
-        lx = roi_lo_exact(x, fp.R);
-        ly = roi_lo_exact(y, fp.R);
-        cx0 = max(lx, 0);
-        cx1 = min(lx + fp.R - 1, fp.W - 1);
-        cy0 = max(ly, fp.row0);
-        cy1 = min(ly + fp.R - 1, fp.row0 + fp.rows - 1);
-        ok = cx0 <= cx1 && cy0 <= cy1;
-      }
-      StarRec r;
-      r.x = x;
-      r.y = y;
-      r.s = ok ? (float)(fp.s_scale * pow(2.512, -(double)m)) : 0.f;
+// ---------------------------------------------------------------------------------------------------------------
+// k_count -- step a1 + tile counting.  One thread per star.
+//   reject non-finite x, y, mag (reading R11); s' = A 2.512^-m / (2 pi sigma^2) in fp64 (Eq. 1 with the
+//   1/(2 pi sigma^2) of Eq. 2 folded in), rounded once to fp32; exact ROI origin (reading R7); clip to the image
+//   columns and the band rows; count one pair per overlapped tile.  The last block scans the per-tile counts into
+//   tile_off[0..ntiles] and leaves cnt[t] = tile_off[t] as the scatter cursor.
+// ---------------------------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(SCAN_THREADS) k_count(const float* __restrict__ X, const float* __restrict__ Y,
+                                                        const float* __restrict__ M, int64_t n, FrameParams fp,
+                                                        StarRec* __restrict__ rec, uint32_t* cnt, Header* hdr,
+                                                        uint32_t* __restrict__ tile_off, uint32_t ntiles) {
+  __shared__ uint32_t s_warp[SCAN_THREADS / 32];
+  __shared__ uint32_t s_max[SCAN_THREADS / 32];
+  __shared__ bool s_last;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t i = (int64_t)blockIdx.x * SCAN_THREADS + tid;
+  if (i < n) {
+    const float x = X[i], y = Y[i], m = M[i];
+    const float R = (float)fp.R;
+    bool ok = isfinite(x) && isfinite(y) && isfinite(m);
+    // pre-filter far-off stars (keeps the int conversions exact); the exact test is the clip below
+    ok = ok && x > -R - 2.f && x < (float)fp.W + R + 2.f && y > (float)fp.row0 - R - 2.f &&
+         y < (float)(fp.row0 + fp.rows) + R + 2.f;
+    StarRec r;
+    r.x = x;
+    r.y = y;
+    r.s = 0.f;
+    r.lo = LO_CULLED;
+    int cx0, cx1, cy0, cy1;
+    if (ok) {
+      const int lx = roi_lo_exact(x, fp.R), ly = roi_lo_exact(y, fp.R);
       r.lo = ((uint32_t)(uint16_t)(int16_t)lx) | ((uint32_t)(uint16_t)(int16_t)ly << 16);
-      rec[i] = r;
-      if (ok) {
+      if (clip_roi(fp, r.lo, cx0, cx1, cy0, cy1)) {
+        r.s = (float)(fp.s_scale * exp2(-(double)m * 1.3288364642295399628));  // 2.512^-m, Eq. 1
         const int tx0 = cx0 / TILE_W, tx1 = cx1 / TILE_W;
         const int ty0 = (cy0 - fp.row0) / TILE_H, ty1 = (cy1 - fp.row0) / TILE_H;
-        tr[k][0] = (uint16_t)tx0; tr[k][1] = (uint16_t)tx1; tr[k][2] = (uint16_t)ty0; tr[k][3] = (uint16_t)ty1;
-        cnt = (uint32_t)((tx1 - tx0 + 1) * (ty1 - ty0 + 1));
+        for (int ty = ty0; ty <= ty1; ++ty)
+          for (int tx = tx0; tx <= tx1; ++tx) atomicAdd(&cnt[ty * fp.ntx + tx], 1u);
+      } else {
+        r.lo = LO_CULLED;
       }
     }
-    cnts[k] = cnt;
-    s_cnt[k * BIN_THREADS + tid] = cnt;
+    rec[i] = r;
   }
-  __syncthreads();
 
-  // ---- a2: block-wide exclusive scan in star order (thread t owns stars t*8 .. t*8+7 of the block)
-  uint32_t v[BIN_ITEMS], tsum = 0;
-#pragma unroll
-  for (int j = 0; j < BIN_ITEMS; ++j) { v[j] = s_cnt[tid * BIN_ITEMS + j]; tsum += v[j]; }
-  uint32_t incl = tsum;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
-    if (lane >= o) incl += t;
-  }
-  if (lane == 31) s_warp[warp] = incl;
+  // ---- the last block to finish turns counts into CSR offsets (threadFenceReduction pattern)
   __syncthreads();
   if (tid == 0) {
-    uint32_t run = 0;
-    for (int w = 0; w < BIN_THREADS / 32; ++w) { uint32_t t = s_warp[w]; s_warp[w] = run; run += t; }
-    // cross-block decoupled look-back: exclusive prefix of this block
-    const uint32_t excl = lookback(status, blk, 1, tag, run);
-    s_base = excl;
-    const int64_t nblk = (n + BIN_TILE - 1) / BIN_TILE;
-    if (blk == nblk - 1) hdr->P = excl + run;
+    __threadfence();
+    s_last = atomicAdd(&hdr->done, 1u) == gridDim.x - 1;
   }
   __syncthreads();
-  {
-    uint32_t off = s_base + s_warp[warp] + incl - tsum;
-#pragma unroll
-    for (int j = 0; j < BIN_ITEMS; ++j) { s_cnt[tid * BIN_ITEMS + j] = off; off += v[j]; }
+  if (!s_last) return;
+  __threadfence();
+  const uint32_t per = (ntiles + SCAN_THREADS - 1) / SCAN_THREADS;
+  const uint32_t b0 = min(ntiles, tid * per), b1 = min(ntiles, b0 + per);
+  uint32_t sum = 0, mx = 0;
+  for (uint32_t t = b0; t < b1; ++t) {
+    const uint32_t c = __ldcg(&cnt[t]);
+    sum += c;
+    mx = max(mx, c);
   }
-  __syncthreads();
-
-  // ---- a3: emit pairs in star order; histogram every pass's digit
-#pragma unroll
-  for (int k = 0; k < BIN_ITEMS; ++k) {
-    if (cnts[k] == 0) continue;
-    const int64_t i = base + k * BIN_THREADS + tid;
-    uint32_t o = s_cnt[k * BIN_THREADS + tid];
-    for (int ty = tr[k][2]; ty <= tr[k][3]; ++ty)
-      for (int tx = tr[k][0]; tx <= tr[k][1]; ++tx) {
-        const uint32_t key = (uint32_t)ty * (uint32_t)fp.ntx + (uint32_t)tx;
-        pairs[o++] = ((uint64_t)key << 32) | (uint64_t)(uint32_t)i;
-        for (int p = 0; p < passes; ++p) atomicAdd(&s_hist[p][(key >> (p * RADIX_BITS)) & (RADIX - 1)], 1u);
-      }
-  }
-  __syncthreads();
-  for (int p = 0; p < passes; ++p) {
-    const uint32_t c = s_hist[p][tid];
-    if (c) atomicAdd(&hdr->hist[p][tid], c);
-  }
-}
-
-// ---------------------------------------------------------------------------------------------------------------
-// k_radix -- one stable LSD pass on digit (key >> shift) & 255 (step a4).  Onesweep structure: the digit
-// histogram over all keys comes from k_bin; each block ranks its 4096 pairs stably (warp match_any + per-warp digit
-// counters in shared memory), looks back across blocks per digit, and scatters.
-// ---------------------------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(RAD_THREADS) k_radix(const uint64_t* __restrict__ in, uint64_t* __restrict__ out,
-                                                       Header* hdr, int pass, uint64_t* status, uint32_t tag) {
-  __shared__ uint32_t s_wcnt[RAD_THREADS / 32][RADIX];
-  __shared__ uint32_t s_base[RADIX];
-  __shared__ uint32_t s_warp[RAD_THREADS / 32];
-  __shared__ int64_t s_blk;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint32_t P = hdr->P;
-  const int64_t nblk = ((int64_t)P + RAD_TILE - 1) / RAD_TILE;
-  if (tid == 0) s_blk = atomicAdd(&hdr->ticket[1 + pass], 1u);
-  for (int i = tid; i < (RAD_THREADS / 32) * RADIX; i += RAD_THREADS) (&s_wcnt[0][0])[i] = 0;
-  __syncthreads();
-  const int64_t blk = s_blk;
-  if (blk >= nblk) return;
-  const int shift = pass * RADIX_BITS;
-  const int64_t wbase = blk * RAD_TILE + (int64_t)warp * (RAD_CHUNKS * 32);
-  const uint32_t lt = (1u << lane) - 1u;
-
-  uint64_t item[RAD_CHUNKS];
-  uint32_t rank[RAD_CHUNKS];
-#pragma unroll
-  for (int c = 0; c < RAD_CHUNKS; ++c) {
-    const int64_t j = wbase + c * 32 + lane;
-    const bool valid = j < (int64_t)P;
-    item[c] = valid ? in[j] : ~0ull;
-    const uint32_t d = valid ? (uint32_t)(item[c] >> (32 + shift)) & (RADIX - 1) : 0x100u;
-    const uint32_t peers = __match_any_sync(0xffffffffu, d);
-    uint32_t before = 0;
-    if (valid) before = s_wcnt[warp][d];
-    __syncwarp();
-    rank[c] = before + __popc(peers & lt);
-    if (valid && (__ffs(peers) - 1) == lane) s_wcnt[warp][d] = before + __popc(peers);
-    __syncwarp();
-  }
-  __syncthreads();
-
-  // thread tid = digit d: exclusive scan over warps, block count, global digit start, look-back
-  const int d = tid;
-  uint32_t run = 0;
-#pragma unroll
-  for (int w = 0; w < RAD_THREADS / 32; ++w) { const uint32_t t = s_wcnt[w][d]; s_wcnt[w][d] = run; run += t; }
-  // exclusive scan of the global histogram -> start of digit d
-  const uint32_t h = hdr->hist[pass][d];
-  uint32_t incl = h;
+  uint32_t incl = sum;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
-    if (lane >= o) incl += t;
+    const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += v;
   }
-  if (lane == 31) s_warp[warp] = incl;
-  __syncthreads();
-  uint32_t wpre = 0;
-  for (int w = 0; w < warp; ++w) wpre += s_warp[w];
-  const uint32_t gstart = wpre + incl - h;
-  const uint32_t excl = lookback(status + d, blk, RADIX, tag, run);
-  s_base[d] = gstart + excl;
-  __syncthreads();
-
 #pragma unroll
-  for (int c = 0; c < RAD_CHUNKS; ++c) {
-    const int64_t j = wbase + c * 32 + lane;
-    if (j < (int64_t)P) {
-      const uint32_t dd = (uint32_t)(item[c] >> (32 + shift)) & (RADIX - 1);
-      out[s_base[dd] + s_wcnt[warp][dd] + rank[c]] = item[c];
+  for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  if (lane == 31) s_warp[warp] = incl;
+  if (lane == 0) s_max[warp] = mx;
+  __syncthreads();
+  if (tid == 0) {
+    uint32_t run = 0, m2 = 0;
+    for (int w = 0; w < SCAN_THREADS / 32; ++w) {
+      const uint32_t v = s_warp[w];
+      s_warp[w] = run;
+      run += v;
+      m2 = max(m2, s_max[w]);
     }
+    hdr->P = run;
+    hdr->max_seg = m2;
+    tile_off[ntiles] = run;
+  }
+  __syncthreads();
+  uint32_t off = s_warp[warp] + incl - sum;
+  for (uint32_t t = b0; t < b1; ++t) {
+    const uint32_t c = __ldcg(&cnt[t]);
+    tile_off[t] = off;
+    cnt[t] = off;  // scatter cursor
+    off += c;
   }
 }
 
 // ---------------------------------------------------------------------------------------------------------------
-// k_offsets -- CSR: tile_off[t] = first sorted position with key >= t (t in [0, ntiles]).
+// k_scatter -- step a3: one thread per star, its index into every overlapped tile's segment.
 // ---------------------------------------------------------------------------------------------------------------
-__global__ void k_offsets(const uint64_t* __restrict__ sorted, const Header* __restrict__ hdr, uint32_t ntiles,
-                          uint32_t* __restrict__ tile_off) {
-  const uint32_t P = hdr->P;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (P == 0) {
-    for (int64_t t = t0; t <= ntiles; t += stride) tile_off[t] = 0;
-    return;
-  }
-  for (int64_t p = t0; p < P; p += stride) {
-    const int64_t k = (int64_t)(sorted[p] >> 32);
-    const int64_t kp = p ? (int64_t)(sorted[p - 1] >> 32) : -1;
-    for (int64_t t = kp + 1; t <= k; ++t) tile_off[t] = (uint32_t)p;
-    if (p == (int64_t)P - 1)
-      for (int64_t t = k + 1; t <= ntiles; ++t) tile_off[t] = P;
-  }
+__global__ void __launch_bounds__(256) k_scatter(const StarRec* __restrict__ rec, int64_t n, FrameParams fp,
+                                                 uint32_t* cursor, uint32_t* __restrict__ ids) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  int cx0, cx1, cy0, cy1;
+  if (!clip_roi(fp, rec[i].lo, cx0, cx1, cy0, cy1)) return;
+  const int tx0 = cx0 / TILE_W, tx1 = cx1 / TILE_W;
+  const int ty0 = (cy0 - fp.row0) / TILE_H, ty1 = (cy1 - fp.row0) / TILE_H;
+  for (int ty = ty0; ty <= ty1; ++ty)
+    for (int tx = tx0; tx <= tx1; ++tx) ids[atomicAdd(&cursor[ty * fp.ntx + tx], 1u)] = (uint32_t)i;
 }
 
 // ---------------------------------------------------------------------------------------------------------------
-void launch_bin(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
-                uint64_t* pairs, Header* hdr, uint64_t* status, uint32_t tag, int passes, cudaStream_t st) {
-  const int64_t nblk = (n + BIN_TILE - 1) / BIN_TILE;
-  if (nblk == 0) return;
-  k_bin<<<(unsigned)nblk, BIN_THREADS, 0, st>>>(x, y, m, n, fp, rec, pairs, hdr, status, tag, passes);
+// k_segsort -- step a4: sort every tile segment by star index.  One warp per tile.
+// ---------------------------------------------------------------------------------------------------------------
+__device__ void warp_bitonic_smem(uint32_t* s, int p2, int lane) {
+  for (int k = 2; k <= p2; k <<= 1)
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      for (int i = lane; i < p2; i += 32) {
+        const int ixj = i ^ j;
+        if (ixj > i) {
+          const uint32_t a = s[i], b = s[ixj];
+          const bool up = (i & k) == 0;
+          if ((a > b) == up) {
+            s[i] = b;
+            s[ixj] = a;
+          }
+        }
+      }
+      __syncwarp();
+    }
 }
 
-void launch_radix(const uint64_t* in, uint64_t* out, Header* hdr, int pass, uint64_t* status, uint32_t tag,
-                  int64_t pmax, cudaStream_t st) {
-  const int64_t nblk = (pmax + RAD_TILE - 1) / RAD_TILE;
-  if (nblk == 0) return;
-  k_radix<<<(unsigned)nblk, RAD_THREADS, 0, st>>>(in, out, hdr, pass, status, tag);
+__device__ __forceinline__ uint32_t lower_bound_g(const uint32_t* a, uint32_t len, uint32_t v) {
+  uint32_t lo = 0, hi = len;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (a[mid] < v) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
 }
 
-void launch_offsets(const uint64_t* sorted, const Header* hdr, uint32_t ntiles, uint32_t* tile_off, int64_t pmax,
-                    int num_sms, cudaStream_t st) {
-  int64_t want = (std::max<int64_t>(pmax, (int64_t)ntiles + 1) + 255) / 256;
-  const int64_t cap = (int64_t)num_sms * 8;
-  if (want > cap) want = cap;
-  if (want < 1) want = 1;
-  k_offsets<<<(unsigned)want, 256, 0, st>>>(sorted, hdr, ntiles, tile_off);
+__global__ void __launch_bounds__(SORT_WARPS * 32) k_segsort(uint32_t* __restrict__ ids, uint32_t* __restrict__ scratch,
+                                                            const uint32_t* __restrict__ tile_off, uint32_t ntiles) {
+  __shared__ uint32_t s_buf[SORT_WARPS][SORT_MAX];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t t = (int64_t)blockIdx.x * SORT_WARPS + warp;
+  if (t >= ntiles) return;
+  const uint32_t a = tile_off[t], L = tile_off[t + 1] - a;
+  if (L <= 1) return;
+  uint32_t* s = s_buf[warp];
+  uint32_t* seg = ids + a;
+  // runs of SORT_MAX sorted in shared memory (one run unless the tile is heavy)
+  for (uint32_t r0 = 0; r0 < L; r0 += SORT_MAX) {
+    const uint32_t len = min((uint32_t)SORT_MAX, L - r0);
+    int p2 = 32;
+    while ((uint32_t)p2 < len) p2 <<= 1;
+    for (int i = lane; i < p2; i += 32) s[i] = (uint32_t)i < len ? seg[r0 + i] : 0xFFFFFFFFu;
+    __syncwarp();
+    warp_bitonic_smem(s, p2, lane);
+    for (uint32_t i = lane; i < len; i += 32) seg[r0 + i] = s[i];
+    __syncwarp();
+  }
+  if (L <= SORT_MAX) return;
+  // heavy tile: bottom-up merge of the sorted runs through global scratch (ids are unique: rank = lower bound)
+  uint32_t* src = seg;
+  uint32_t* dst = scratch + a;
+  for (uint32_t w = SORT_MAX; w < L; w <<= 1) {
+    for (uint32_t lo = 0; lo < L; lo += 2 * w) {
+      const uint32_t mid = min(lo + w, L), hi = min(lo + 2 * w, L);
+      for (uint32_t i = lo + lane; i < mid; i += 32)
+        dst[i + lower_bound_g(src + mid, hi - mid, src[i])] = src[i];
+      for (uint32_t j = mid + lane; j < hi; j += 32)
+        dst[lo + (j - mid) + lower_bound_g(src + lo, mid - lo, src[j])] = src[j];
+    }
+    __syncwarp();
+    uint32_t* tmp = src;
+    src = dst;
+    dst = tmp;
+  }
+  if (src != seg) {
+    for (uint32_t i = lane; i < L; i += 32) seg[i] = src[i];
+    __syncwarp();
+  }
+}
+
+// ---------------------------------------------------------------------------------------------------------------
+void launch_count(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
+                  uint32_t* cnt, Header* hdr, uint32_t* tile_off, uint32_t ntiles, cudaStream_t st) {
+  const int64_t nblk = std::max<int64_t>(1, (n + SCAN_THREADS - 1) / SCAN_THREADS);
+  k_count<<<(unsigned)nblk, SCAN_THREADS, 0, st>>>(x, y, m, n, fp, rec, cnt, hdr, tile_off, ntiles);
+}
+
+void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, uint32_t* cursor, uint32_t* ids,
+                    cudaStream_t st) {
+  if (n <= 0) return;
+  k_scatter<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(rec, n, fp, cursor, ids);
+}
+
+void launch_segsort(uint32_t* ids, uint32_t* scratch, const uint32_t* tile_off, uint32_t ntiles, cudaStream_t st) {
+  k_segsort<<<(ntiles + SORT_WARPS - 1) / SORT_WARPS, SORT_WARPS * 32, 0, st>>>(ids, scratch, tile_off, ntiles);
 }
 
 }  // namespace starsim
