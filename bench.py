@@ -283,7 +283,7 @@ def run_ours(args, world, rank, local_rank):
 
     # per-kernel live timings (this rank); launches of our own kernels per step
     launches = sum(v[1] for k, v in kt.items() if k not in ("memset",)) / args.steps
-    tile_ms = kt["tile"][0] / max(1, kt["tile"][1])
+    tile_ms = kt["tile"][0] / max(1, kt["tile"][1]) if kt["tile"][1] else kt["atomic"][0] / max(1, kt["atomic"][1])
     clocks = clk.summary()
     sm_mhz = clocks["sm_mhz"] or 1965.0
     # roofline of the dominant kernel (k_tile) on this rank's band

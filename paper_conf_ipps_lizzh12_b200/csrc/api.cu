@@ -154,6 +154,7 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   fp.nty = (rows + TILE_H - 1) / TILE_H;
   const double s = (double)sigma;
   fp.kexp = (float)(-1.0 / (2.0 * s * s * std::log(2.0)));   // exp(-d^2/(2 s^2)) = 2^(kexp d^2)
+  fp.sk = (float)std::sqrt(1.0 / (2.0 * s * s * std::log(2.0)));  // exp(-d^2/(2 s^2)) = 2^(-(d sk)^2)
   fp.s_scale = (double)gain / (2.0 * M_PI * s * s);          // Eq. 1 gain with Eq. 2's 1/(2 pi s^2)
   return fp;
 }
@@ -168,7 +169,10 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   DevGuard g(c->dev);
   const FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain);
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
-  const int64_t pmax = n * tiles_per_axis(R, TILE_W, fp.ntx) * (int64_t)tiles_per_axis(R, TILE_H, fp.nty);
+  // tiles per star at most tpx x tpy; tps = 4 whenever R <= 33 (the fast 2 x 2 path of k_count / k_scatter)
+  const int tpx = tiles_per_axis(R, TILE_W, fp.ntx), tpy = tiles_per_axis(R, TILE_H, fp.nty);
+  const int tps = (tpx <= 2 && tpy <= 2) ? 4 : tpx * tpy;
+  const int64_t pmax = n * (int64_t)tps;
   if (pmax >= 0xFFFFFFFFll) return fail(c, STARSIM_EINVAL, "n * tiles-per-star >= 2^32 (pair counts are 32-bit)");
   int rc;
   if ((rc = grow(c, c->rec, sizeof(StarRec) * (size_t)(n > 0 ? n : 1), "records"))) return rc;
@@ -185,10 +189,14 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   StarRec* rec = (StarRec*)c->rec.p;
 
   timed(c, 5, st, [&] { cudaMemsetAsync(hdr, 0, hdr_bytes, st); });
-  timed(c, 0, st, [&] { launch_count(x, y, mag, n, fp, rec, cnt, hdr, tile_off, (uint32_t)ntiles, st); });
+  // slots of the pairs (k_count -> k_scatter) live in the sort scratch, free again before k_segsort needs it
+  uint32_t* slots = (uint32_t*)c->scratch.p;
+  timed(c, 0, st, [&] {
+    launch_count(x, y, mag, n, fp, rec, cnt, slots, tps, hdr, tile_off, (uint32_t)ntiles, st);
+  });
   if ((rc = check_launch(c, "k_count"))) return rc;
   if (n > 0) {
-    timed(c, 1, st, [&] { launch_scatter(rec, n, fp, cnt, ids, st); });
+    timed(c, 1, st, [&] { launch_scatter(rec, n, fp, slots, tps, tile_off, ids, st); });
     if ((rc = check_launch(c, "k_scatter"))) return rc;
     timed(c, 2, st, [&] { launch_segsort(ids, (uint32_t*)c->scratch.p, tile_off, (uint32_t)ntiles, st); });
     if ((rc = check_launch(c, "k_segsort"))) return rc;

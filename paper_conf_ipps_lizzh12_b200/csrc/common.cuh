@@ -8,14 +8,14 @@ namespace starsim {
 
 // ---------------------------------------------------------------- tile geometry (DESIGN.md §Data layout)
 constexpr int TILE_W = 32;   // tile width: one warp, 16 columns x 2 halves per lane
-constexpr int TILE_H = 32;   // tile height: 16 rows of one parity per lane, in fp32 registers
+constexpr int TILE_H = 64;   // tile height: 32 rows of one parity per lane, in fp32 registers
 
-// k_count: one thread per star
+// k_count: one thread per star (the last block also scans the tile counts)
 constexpr int CNT_THREADS = 256;
-constexpr int SCAN_THREADS = 1024;
+constexpr int SCAN_V = 32;          // tile counts per thread per pass of the last block's scan
 // k_segsort: one warp per tile, segments up to SORT_MAX sorted in shared memory
-constexpr int SORT_WARPS = 4;
-constexpr int SORT_MAX = 2048;
+constexpr int SORT_WARPS = 8;
+constexpr int SORT_MAX = 1024;
 // k_tile: 4 warps per block, one 32x32 tile per warp
 constexpr int TILE_WARPS = 4;
 
@@ -43,6 +43,7 @@ struct FrameParams {
   int32_t R;
   int32_t ntx, nty;      // tiles over the band
   float kexp;            // -log2(e) / (2 sigma^2): exp(-d^2/(2 sigma^2)) = ex2(kexp * d^2)
+  float sk;              // sqrt(log2(e) / (2 sigma^2)):  exp(-d^2/(2 sigma^2)) = ex2(-(d * sk)^2)
   double s_scale;        // A / (2 pi sigma^2), applied in fp64 before rounding s' to fp32
 };
 

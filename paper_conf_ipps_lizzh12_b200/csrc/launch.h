@@ -8,9 +8,10 @@
 namespace starsim {
 
 void launch_count(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
-                  uint32_t* cnt, Header* hdr, uint32_t* tile_off, uint32_t ntiles, cudaStream_t st);
-void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, uint32_t* cursor, uint32_t* ids,
-                    cudaStream_t st);
+                  uint32_t* cnt, uint32_t* slots, int tps, Header* hdr, uint32_t* tile_off, uint32_t ntiles,
+                  cudaStream_t st);
+void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* slots, int tps,
+                    const uint32_t* tile_off, uint32_t* ids, cudaStream_t st);
 void launch_segsort(uint32_t* ids, uint32_t* scratch, const uint32_t* tile_off, uint32_t ntiles, cudaStream_t st);
 void launch_tile(const uint32_t* ids, const uint32_t* tile_off, const StarRec* rec, const FrameParams& fp,
                  float* out, cudaStream_t st);

@@ -11,7 +11,7 @@ torch.distributed (NCCL on GPUs, gloo in the CPU tests) is plumbing only; the re
 """
 from __future__ import annotations
 
-TILE_H = 32
+TILE_H = 64   # must equal the library tile height (csrc/common.cuh) for bitwise band equality
 
 
 def band_rows(height: int, world: int, rank: int, align: int = TILE_H) -> tuple[int, int]:
