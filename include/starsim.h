@@ -57,9 +57,10 @@ void starsim_destroy(starsim_ctx* ctx);
  * (then a static description of the last create failure). */
 const char* starsim_last_error(const starsim_ctx* ctx);
 
-/* Render a full frame with the tiled path: per-star prep + binning of the (tile, star) pairs by a
- * one-digit counting (radix) sort on the tile key + per-tile sort into star order (CSR), then one register-
- * accumulating tile kernel, free of atomics on the image, that writes every pixel once.
+/* Render a full frame with the tiled path: per-star prep + binning of the (tile, star) pairs and a
+ * stable hand-written radix sort on the tile key (CSR in star order), then one register-accumulating tile kernel,
+ * free of atomics on the image, that writes every pixel once.  On a non-default stream the launches are captured
+ * once into a CUDA graph and replayed while the arguments repeat (STARSIM_NO_GRAPH=1 disables this).
  *   x, y, mag  (device) float[n]: the star catalogue as SoA -- sub-pixel centre (image coordinates) and magnitude.
  *   n          number of stars, >= 0 (0 -> an all-zero image).  x, y, mag may be NULL iff n == 0.
  *   width, height   image size in pixels, each in [1, 32767], width*height < 2^31.
@@ -117,8 +118,10 @@ int starsim_get_bins(starsim_ctx* ctx, int32_t* tile_w, int32_t* tile_h,
 /* Per-kernel device timing for roofline reporting.  When enabled, every launch of the library records CUDA events
  * on the launching stream around it; starsim_kernel_times() synchronises and returns, per kernel class, the summed
  * elapsed milliseconds and launch counts since the last reset.  Classes (index into the arrays):
- *   0 prep + tile counting + CSR scan (k_count), 1 counting-sort scatter (k_scatter), 2 per-tile star-order sort
- *   (k_segsort), 3 tile accumulate (k_tile), 4 atomic scatter (k_atomic), 5 memsets, 6 quantise, 7 aos split.
+ *   0 k_bin (prep + scan + emit + digit histograms), 1 k_radix passes, 2 k_offsets (CSR), 3 k_tile (accumulate),
+ *   4 k_atomic, 5 memsets, 6 k_quantize, 7 k_split_aos.
+ * While profiling is enabled, renders are launched directly (not through the captured CUDA graph) so that every
+ * kernel can be bracketed; kernel durations are unaffected, only the launch gaps differ.
  * `ms` and `launches` must hold STARSIM_NUM_KCLASS entries.  enable != 0 turns recording on and resets. */
 #define STARSIM_NUM_KCLASS 8
 int starsim_profile(starsim_ctx* ctx, int enable);

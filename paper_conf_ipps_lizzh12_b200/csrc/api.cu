@@ -28,16 +28,36 @@ struct Launch {
 
 }  // namespace
 
+// A captured render (CUDA graph) and the arguments it was captured with: replayed when a call repeats them.
+struct GraphKey {
+  const void *x, *y, *mag, *out;
+  int64_t n;
+  int32_t W, H, row0, rows, R;
+  float sigma, gain;
+  cudaStream_t st;
+  uint64_t scratch_gen;
+  bool operator==(const GraphKey& o) const {
+    return x == o.x && y == o.y && mag == o.mag && out == o.out && n == o.n && W == o.W && H == o.H &&
+           row0 == o.row0 && rows == o.rows && R == o.R && sigma == o.sigma && gain == o.gain && st == o.st &&
+           scratch_gen == o.scratch_gen;
+  }
+};
+
 struct starsim_ctx {
   int dev = 0;
   int num_sms = 148;
   std::string err;
-  Buf rec, ids, scratch, tile_off, hdr, stage;
-  uint32_t epoch = 0;
+  Buf rec, pairs[2], ids, tile_off, zeroed, stage;
+  uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
   cudaStream_t last_stream = nullptr;
   int64_t last_ntiles = 0;
+  // CUDA graph of the last render signature (non-default streams only; STARSIM_NO_GRAPH=1 disables)
+  bool use_graphs = true;
+  bool have_graph = false;
+  GraphKey gkey{};
+  cudaGraphExec_t gexec = nullptr;
   // profiling
   bool prof = false;
   std::vector<cudaEvent_t> ev_pool;
@@ -77,6 +97,7 @@ int grow(starsim_ctx* c, Buf& b, size_t bytes, const char* what) {
   size_t want = b.cap + b.cap / 2;
   if (want < bytes) want = bytes;
   if (want < 4096) want = 4096;
+  c->scratch_gen++;
   if (b.p) {
     cudaFree(b.p);  // implicitly synchronises the device: earlier calls that used b are done
     b.p = nullptr;
@@ -164,45 +185,100 @@ int tiles_per_axis(int R, int tile, int ntiles_axis) {
   return t < ntiles_axis ? t : ntiles_axis;
 }
 
+// Enqueue the tiled render on stream st (memset of the per-render header + look-back status words, k_bin, one or two
+// k_radix passes, k_offsets, k_tile).
+int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, const FrameParams& fp,
+                  int64_t ntiles, int64_t pmax, int bits0, int bits1, float* out, cudaStream_t st) {
+  Header* hdr = (Header*)c->zeroed.p;
+  const int64_t nbin_blk = (n + BIN_TILE - 1) / BIN_TILE;
+  const int64_t nrad_blk = (pmax + RAD_TILE - 1) / RAD_TILE;
+  unsigned long long* st_bin = (unsigned long long*)(hdr + 1);
+  unsigned long long* st_rad0 = st_bin + nbin_blk;
+  unsigned long long* st_rad1 = st_rad0 + nrad_blk * ((int64_t)1 << bits0);
+  const size_t zbytes = sizeof(Header) + sizeof(unsigned long long) *
+                        (size_t)(nbin_blk + nrad_blk * (((int64_t)1 << bits0) + (bits1 ? ((int64_t)1 << bits1) : 0)));
+  uint64_t* pairs[2] = {(uint64_t*)c->pairs[0].p, (uint64_t*)c->pairs[1].p};
+  uint32_t* ids = (uint32_t*)c->ids.p;
+  uint32_t* tile_off = (uint32_t*)c->tile_off.p;
+  StarRec* rec = (StarRec*)c->rec.p;
+  int rc;
+  timed(c, 5, st, [&] { cudaMemsetAsync(hdr, 0, zbytes, st); });
+  int cur = 0;
+  if (n > 0) {
+    timed(c, 0, st, [&] { launch_bin(x, y, mag, n, fp, rec, pairs[0], hdr, st_bin, bits0, bits1, st); });
+    if ((rc = check_launch(c, "k_bin"))) return rc;
+    if (bits0) {
+      timed(c, 1, st, [&] { launch_radix(pairs[0], pairs[1], hdr, 0, 0, bits0, st_rad0, pmax, st); });
+      cur = 1;
+      if (bits1) {
+        timed(c, 1, st, [&] { launch_radix(pairs[1], pairs[0], hdr, 1, bits0, bits1, st_rad1, pmax, st); });
+        cur = 0;
+      }
+      if ((rc = check_launch(c, "k_radix"))) return rc;
+    }
+  }
+  timed(c, 2, st, [&] {
+    launch_offsets(pairs[cur], hdr, (uint32_t)ntiles, tile_off, ids, pmax, c->num_sms, st);
+  });
+  if ((rc = check_launch(c, "k_offsets"))) return rc;
+  timed(c, 3, st, [&] { launch_tile(ids, tile_off, rec, fp, out, st); });
+  if ((rc = check_launch(c, "k_tile"))) return rc;
+  return STARSIM_OK;
+}
+
 int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
                  int32_t row0, int32_t rows, float sigma, int32_t R, float gain, float* out, cudaStream_t st) {
   DevGuard g(c->dev);
   const FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain);
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
-  // tiles per star at most tpx x tpy; tps = 4 whenever R <= 33 (the fast 2 x 2 path of k_count / k_scatter)
   const int tpx = tiles_per_axis(R, TILE_W, fp.ntx), tpy = tiles_per_axis(R, TILE_H, fp.nty);
-  const int tps = (tpx <= 2 && tpy <= 2) ? 4 : tpx * tpy;
-  const int64_t pmax = n * (int64_t)tps;
+  const int64_t pmax = n * (int64_t)tpx * tpy;
   if (pmax >= 0xFFFFFFFFll) return fail(c, STARSIM_EINVAL, "n * tiles-per-star >= 2^32 (pair counts are 32-bit)");
+  // radix digits: the tile key needs keybits bits; one pass if <= 10, else two passes of ceil/floor(keybits/2)
+  int keybits = 0;
+  while (((int64_t)1 << keybits) < ntiles) ++keybits;
+  const int bits0 = keybits <= MAX_RADIX_BITS ? keybits : (keybits + 1) / 2;
+  const int bits1 = keybits <= MAX_RADIX_BITS ? 0 : keybits - bits0;
+  const int64_t nbin_blk = (n + BIN_TILE - 1) / BIN_TILE;
+  const int64_t nrad_blk = (pmax + RAD_TILE - 1) / RAD_TILE;
+  const size_t zbytes = sizeof(Header) + sizeof(unsigned long long) *
+                        (size_t)(nbin_blk + nrad_blk * (((int64_t)1 << bits0) + (bits1 ? ((int64_t)1 << bits1) : 0)));
   int rc;
   if ((rc = grow(c, c->rec, sizeof(StarRec) * (size_t)(n > 0 ? n : 1), "records"))) return rc;
+  if ((rc = grow(c, c->pairs[0], sizeof(uint64_t) * (size_t)(pmax > 0 ? pmax : 1), "pairs"))) return rc;
+  if ((rc = grow(c, c->pairs[1], sizeof(uint64_t) * (size_t)(pmax > 0 ? pmax : 1), "pairs"))) return rc;
   if ((rc = grow(c, c->ids, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "tile lists"))) return rc;
-  if ((rc = grow(c, c->scratch, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "sort scratch"))) return rc;
   if ((rc = grow(c, c->tile_off, sizeof(uint32_t) * (size_t)(ntiles + 1), "tile offsets"))) return rc;
-  const size_t hdr_bytes = sizeof(Header) + sizeof(uint32_t) * (size_t)ntiles;
-  if ((rc = grow(c, c->hdr, hdr_bytes, "header+counters"))) return rc;
+  if ((rc = grow(c, c->zeroed, zbytes, "header+status"))) return rc;
 
-  Header* hdr = (Header*)c->hdr.p;
-  uint32_t* cnt = (uint32_t*)(hdr + 1);
-  uint32_t* ids = (uint32_t*)c->ids.p;
-  uint32_t* tile_off = (uint32_t*)c->tile_off.p;
-  StarRec* rec = (StarRec*)c->rec.p;
-
-  timed(c, 5, st, [&] { cudaMemsetAsync(hdr, 0, hdr_bytes, st); });
-  // slots of the pairs (k_count -> k_scatter) live in the sort scratch, free again before k_segsort needs it
-  uint32_t* slots = (uint32_t*)c->scratch.p;
-  timed(c, 0, st, [&] {
-    launch_count(x, y, mag, n, fp, rec, cnt, slots, tps, hdr, tile_off, (uint32_t)ntiles, st);
-  });
-  if ((rc = check_launch(c, "k_count"))) return rc;
-  if (n > 0) {
-    timed(c, 1, st, [&] { launch_scatter(rec, n, fp, slots, tps, tile_off, ids, st); });
-    if ((rc = check_launch(c, "k_scatter"))) return rc;
-    timed(c, 2, st, [&] { launch_segsort(ids, (uint32_t*)c->scratch.p, tile_off, (uint32_t)ntiles, st); });
-    if ((rc = check_launch(c, "k_segsort"))) return rc;
+  const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, sigma, gain, st, c->scratch_gen};
+  if (st == nullptr || c->prof || !c->use_graphs) {
+    if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, pmax, bits0, bits1, out, st))) return rc;
+  } else {
+    if (!(c->have_graph && c->gkey == key)) {
+      if (c->have_graph) {
+        cudaGraphExecDestroy(c->gexec);
+        c->have_graph = false;
+      }
+      cudaError_t e = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal);
+      if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamBeginCapture");
+      rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, pmax, bits0, bits1, out, st);
+      cudaGraph_t graph = nullptr;
+      e = cudaStreamEndCapture(st, &graph);
+      if (rc) {
+        if (graph) cudaGraphDestroy(graph);
+        return rc;
+      }
+      if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamEndCapture");
+      e = cudaGraphInstantiate(&c->gexec, graph, 0);
+      cudaGraphDestroy(graph);
+      if (e != cudaSuccess) return cuda_fail(c, e, "cudaGraphInstantiate");
+      c->gkey = key;
+      c->have_graph = true;
+    }
+    cudaError_t e = cudaGraphLaunch(c->gexec, st);
+    if (e != cudaSuccess) return cuda_fail(c, e, "cudaGraphLaunch");
   }
-  timed(c, 3, st, [&] { launch_tile(ids, tile_off, rec, fp, out, st); });
-  if ((rc = check_launch(c, "k_tile"))) return rc;
   c->have_bins = true;
   c->last_stream = st;
   c->last_ntiles = ntiles;
@@ -244,6 +320,9 @@ int starsim_create(starsim_ctx** out, int cuda_device) {
   starsim_ctx* c = new starsim_ctx();
   c->dev = cuda_device;
   c->num_sms = prop.multiProcessorCount;
+  init_kernels();
+  const char* ng = getenv("STARSIM_NO_GRAPH");
+  c->use_graphs = !(ng && ng[0] == '1');
   *out = c;
   g_create_error.clear();
   return STARSIM_OK;
@@ -254,7 +333,8 @@ void starsim_destroy(starsim_ctx* c) {
   {
     DevGuard g(c->dev);
     cudaDeviceSynchronize();
-    Buf* bufs[] = {&c->rec, &c->ids, &c->scratch, &c->tile_off, &c->hdr, &c->stage};
+    if (c->have_graph) cudaGraphExecDestroy(c->gexec);
+    Buf* bufs[] = {&c->rec, &c->pairs[0], &c->pairs[1], &c->ids, &c->tile_off, &c->zeroed, &c->stage};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {
@@ -343,7 +423,7 @@ int starsim_get_bins(starsim_ctx* c, int32_t* tile_w, int32_t* tile_h, uint32_t*
   cudaError_t e = cudaStreamSynchronize(c->last_stream);
   if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamSynchronize");
   Header h;
-  if ((e = cudaMemcpy(&h, c->hdr.p, sizeof(Header), cudaMemcpyDeviceToHost)) != cudaSuccess)
+  if ((e = cudaMemcpy(&h, c->zeroed.p, sizeof(Header), cudaMemcpyDeviceToHost)) != cudaSuccess)
     return cuda_fail(c, e, "cudaMemcpy(header)");
   if (tile_w) *tile_w = TILE_W;
   if (tile_h) *tile_h = TILE_H;

@@ -10,21 +10,25 @@ namespace starsim {
 constexpr int TILE_W = 32;   // tile width: one warp, 16 columns x 2 halves per lane
 constexpr int TILE_H = 64;   // tile height: 32 rows of one parity per lane, in fp32 registers
 
-// k_count: one thread per star (the last block also scans the tile counts)
-constexpr int CNT_THREADS = 256;
-constexpr int SCAN_V = 32;          // tile counts per thread per pass of the last block's scan
-// k_segsort: one warp per tile, segments up to SORT_MAX sorted in shared memory
-constexpr int SORT_WARPS = 8;
-constexpr int SORT_MAX = 1024;
-// k_tile: 4 warps per block, one 32x32 tile per warp
+// k_bin: BIN_THREADS threads x BIN_ITEMS stars per block
+constexpr int BIN_THREADS = 256;
+constexpr int BIN_ITEMS = 4;
+constexpr int BIN_TILE = BIN_THREADS * BIN_ITEMS;
+// k_radix: RAD_THREADS threads = 8 warps x RAD_CHUNKS chunks of 32 pairs per block; digits of <= 10 bits
+constexpr int RAD_THREADS = 256;
+constexpr int RAD_CHUNKS = 16;
+constexpr int RAD_TILE = RAD_THREADS * RAD_CHUNKS;
+constexpr int MAX_RADIX_BITS = 10;
+constexpr int MAX_RADIX = 1 << MAX_RADIX_BITS;
+// k_tile: 4 warps per block, one tile per warp
 constexpr int TILE_WARPS = 4;
 
-// Per-render header in device scratch, zeroed by one cudaMemsetAsync per render.
+// Per-render header in device scratch, zeroed (with the look-back status arrays) by one cudaMemsetAsync per render.
 struct Header {
-  uint32_t done;      // k_count blocks finished (last one scans)
-  uint32_t P;         // number of (tile, star) pairs
-  uint32_t max_seg;   // longest tile list
-  uint32_t pad[13];
+  uint32_t ticket[4];                  // dynamic block ids: [0] k_bin, [1], [2] radix passes
+  uint32_t P;                          // number of (tile, star) pairs
+  uint32_t pad[11];
+  uint32_t hist[2][MAX_RADIX];         // digit histograms of all keys for the (at most two) radix passes
 };
 
 // Star record written by k_count, read by k_scatter and k_tile: {x, y, s', lo_x | lo_y << 16}.

@@ -255,7 +255,7 @@ def test_kernel_times_recorded(torch_dev, ctx):
     ctx.render(*args, cfg.W, cfg.H, cfg.sigma, cfg.R, 1.0)
     t = ctx.kernel_times()
     ctx.profile(False)
-    assert t["tile"][1] == 1 and t["tile"][0] > 0 and t["count"][1] == 1 and t["segsort"][1] == 1
+    assert t["tile"][1] == 1 and t["tile"][0] > 0 and t["bin"][1] == 1 and t["offsets"][1] == 1
 
 
 # ---------------------------------------------------------------- B200-scale frames (full images, threaded oracle)
