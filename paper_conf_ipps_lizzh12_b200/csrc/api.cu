@@ -47,7 +47,7 @@ struct starsim_ctx {
   int dev = 0;
   int num_sms = 148;
   std::string err;
-  Buf rec, pairs[2], ids, tile_off, zeroed, stage;
+  Buf rec, slots, ids, tmp, tile_off, zeroed, stage;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
@@ -185,42 +185,30 @@ int tiles_per_axis(int R, int tile, int ntiles_axis) {
   return t < ntiles_axis ? t : ntiles_axis;
 }
 
-// Enqueue the tiled render on stream st (memset of the per-render header + look-back status words, k_bin, one or two
-// k_radix passes, k_offsets, k_tile).
+// Enqueue the tiled render on stream st: memset of the header + tile counters, k_prep, k_scan, k_scatter,
+// k_sortlists, k_tile.
 int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, const FrameParams& fp,
-                  int64_t ntiles, int64_t pmax, int bits0, int bits1, float* out, cudaStream_t st) {
+                  int64_t ntiles, int tps, float* out, cudaStream_t st) {
   Header* hdr = (Header*)c->zeroed.p;
-  const int64_t nbin_blk = (n + BIN_TILE - 1) / BIN_TILE;
-  const int64_t nrad_blk = (pmax + RAD_TILE - 1) / RAD_TILE;
-  unsigned long long* st_bin = (unsigned long long*)(hdr + 1);
-  unsigned long long* st_rad0 = st_bin + nbin_blk;
-  unsigned long long* st_rad1 = st_rad0 + nrad_blk * ((int64_t)1 << bits0);
-  const size_t zbytes = sizeof(Header) + sizeof(unsigned long long) *
-                        (size_t)(nbin_blk + nrad_blk * (((int64_t)1 << bits0) + (bits1 ? ((int64_t)1 << bits1) : 0)));
-  uint64_t* pairs[2] = {(uint64_t*)c->pairs[0].p, (uint64_t*)c->pairs[1].p};
+  uint32_t* cnt = (uint32_t*)(hdr + 1);
+  const size_t zbytes = sizeof(Header) + sizeof(uint32_t) * CNT_STRIDE * (size_t)ntiles;
   uint32_t* ids = (uint32_t*)c->ids.p;
   uint32_t* tile_off = (uint32_t*)c->tile_off.p;
+  uint32_t* slots = (uint32_t*)c->slots.p;
   StarRec* rec = (StarRec*)c->rec.p;
   int rc;
   timed(c, 5, st, [&] { cudaMemsetAsync(hdr, 0, zbytes, st); });
-  int cur = 0;
   if (n > 0) {
-    timed(c, 0, st, [&] { launch_bin(x, y, mag, n, fp, rec, pairs[0], hdr, st_bin, bits0, bits1, st); });
-    if ((rc = check_launch(c, "k_bin"))) return rc;
-    if (bits0) {
-      timed(c, 1, st, [&] { launch_radix(pairs[0], pairs[1], hdr, 0, 0, bits0, st_rad0, pmax, st); });
-      cur = 1;
-      if (bits1) {
-        timed(c, 1, st, [&] { launch_radix(pairs[1], pairs[0], hdr, 1, bits0, bits1, st_rad1, pmax, st); });
-        cur = 0;
-      }
-      if ((rc = check_launch(c, "k_radix"))) return rc;
-    }
+    timed(c, 0, st, [&] { launch_prep(x, y, mag, n, fp, rec, cnt, slots, tps, st); });
+    if ((rc = check_launch(c, "k_prep"))) return rc;
   }
   timed(c, 2, st, [&] {
-    launch_offsets(pairs[cur], hdr, (uint32_t)ntiles, tile_off, ids, pmax, c->num_sms, st);
+    launch_scan(cnt, ntiles, tile_off, hdr, st);
+    launch_scatter(rec, n, fp, slots, tps, tile_off, ids, st);
   });
-  if ((rc = check_launch(c, "k_offsets"))) return rc;
+  if ((rc = check_launch(c, "k_scan/k_scatter"))) return rc;
+  timed(c, 1, st, [&] { launch_sortlists(ids, (uint32_t*)c->tmp.p, tile_off, ntiles, n, st); });
+  if ((rc = check_launch(c, "k_sortlists"))) return rc;
   timed(c, 3, st, [&] { launch_tile(ids, tile_off, rec, fp, out, st); });
   if ((rc = check_launch(c, "k_tile"))) return rc;
   return STARSIM_OK;
@@ -229,31 +217,24 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
 int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
                  int32_t row0, int32_t rows, float sigma, int32_t R, float gain, float* out, cudaStream_t st) {
   DevGuard g(c->dev);
-  const FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain);
+  FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain);
+  fp.vec = (W % 4 == 0 && ((uintptr_t)out & 15) == 0) ? 1 : 0;
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
-  const int tpx = tiles_per_axis(R, TILE_W, fp.ntx), tpy = tiles_per_axis(R, TILE_H, fp.nty);
-  const int64_t pmax = n * (int64_t)tpx * tpy;
+  const int tps = tiles_per_axis(R, TILE_W, fp.ntx) * tiles_per_axis(R, TILE_H, fp.nty);
+  const int64_t pmax = n * (int64_t)tps;
   if (pmax >= 0xFFFFFFFFll) return fail(c, STARSIM_EINVAL, "n * tiles-per-star >= 2^32 (pair counts are 32-bit)");
-  // radix digits: the tile key needs keybits bits; one pass if <= 10, else two passes of ceil/floor(keybits/2)
-  int keybits = 0;
-  while (((int64_t)1 << keybits) < ntiles) ++keybits;
-  const int bits0 = keybits <= MAX_RADIX_BITS ? keybits : (keybits + 1) / 2;
-  const int bits1 = keybits <= MAX_RADIX_BITS ? 0 : keybits - bits0;
-  const int64_t nbin_blk = (n + BIN_TILE - 1) / BIN_TILE;
-  const int64_t nrad_blk = (pmax + RAD_TILE - 1) / RAD_TILE;
-  const size_t zbytes = sizeof(Header) + sizeof(unsigned long long) *
-                        (size_t)(nbin_blk + nrad_blk * (((int64_t)1 << bits0) + (bits1 ? ((int64_t)1 << bits1) : 0)));
+  const size_t zbytes = sizeof(Header) + sizeof(uint32_t) * CNT_STRIDE * (size_t)ntiles;
   int rc;
   if ((rc = grow(c, c->rec, sizeof(StarRec) * (size_t)(n > 0 ? n : 1), "records"))) return rc;
-  if ((rc = grow(c, c->pairs[0], sizeof(uint64_t) * (size_t)(pmax > 0 ? pmax : 1), "pairs"))) return rc;
-  if ((rc = grow(c, c->pairs[1], sizeof(uint64_t) * (size_t)(pmax > 0 ? pmax : 1), "pairs"))) return rc;
+  if ((rc = grow(c, c->slots, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "tile slots"))) return rc;
   if ((rc = grow(c, c->ids, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "tile lists"))) return rc;
+  if ((rc = grow(c, c->tmp, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "sort scratch"))) return rc;
   if ((rc = grow(c, c->tile_off, sizeof(uint32_t) * (size_t)(ntiles + 1), "tile offsets"))) return rc;
-  if ((rc = grow(c, c->zeroed, zbytes, "header+status"))) return rc;
+  if ((rc = grow(c, c->zeroed, zbytes, "header+counters"))) return rc;
 
   const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, sigma, gain, st, c->scratch_gen};
   if (st == nullptr || c->prof || !c->use_graphs) {
-    if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, pmax, bits0, bits1, out, st))) return rc;
+    if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, out, st))) return rc;
   } else {
     if (!(c->have_graph && c->gkey == key)) {
       if (c->have_graph) {
@@ -262,7 +243,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
       }
       cudaError_t e = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal);
       if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamBeginCapture");
-      rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, pmax, bits0, bits1, out, st);
+      rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, out, st);
       cudaGraph_t graph = nullptr;
       e = cudaStreamEndCapture(st, &graph);
       if (rc) {
@@ -334,7 +315,7 @@ void starsim_destroy(starsim_ctx* c) {
     DevGuard g(c->dev);
     cudaDeviceSynchronize();
     if (c->have_graph) cudaGraphExecDestroy(c->gexec);
-    Buf* bufs[] = {&c->rec, &c->pairs[0], &c->pairs[1], &c->ids, &c->tile_off, &c->zeroed, &c->stage};
+    Buf* bufs[] = {&c->rec, &c->slots, &c->ids, &c->tmp, &c->tile_off, &c->zeroed, &c->stage};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {

@@ -7,31 +7,41 @@
 namespace starsim {
 
 // ---------------------------------------------------------------- tile geometry (DESIGN.md §Data layout)
-constexpr int TILE_W = 32;   // tile width: one warp, 16 columns x 2 halves per lane
-constexpr int TILE_H = 64;   // tile height: 32 rows of one parity per lane, in fp32 registers
+// A tile is the unit of binning and of one k_tile CTA: TILE_W x TILE_H pixels.  Inside it, warp (wx, wy) owns the
+// 64 x 16 block at columns 64*wx, rows 16*wy; the block is 8 strips of STRIP_W = 8 columns, one per group of 4 lanes.
+constexpr int TILE_W = 128;
+constexpr int TILE_H = 64;
+constexpr int BAND_H = 16;                       // rows per warp band
+constexpr int STRIP_W = 8;                       // columns per lane-group strip
+constexpr int NBANDS = TILE_H / BAND_H;          // 4
+constexpr int NSTRIPS = TILE_W / STRIP_W;        // 16
+constexpr int TILE_WARPS = 8;                    // 2 (x) x 4 (bands)
+constexpr int TILE_THREADS = TILE_WARPS * 32;
+constexpr int CHUNK = TILE_THREADS;              // stars per chunk of a tile's list (one per thread)
+constexpr int GY_CAP = 384;                      // band slots (16 floats: the row profile on one band) per chunk
+constexpr int RCAP = 56;                         // strip slots (8 floats: the column profile on one strip) per strip
+constexpr int LCAP = 32;                         // entries per (band, strip) list per chunk
+constexpr int GX_PAIRS = 768;                    // (star, strip) pairs per chunk
 
-// k_bin: BIN_THREADS threads x BIN_ITEMS stars per block
-constexpr int BIN_THREADS = 256;
-constexpr int BIN_ITEMS = 4;
-constexpr int BIN_TILE = BIN_THREADS * BIN_ITEMS;
-// k_radix: RAD_THREADS threads = 8 warps x RAD_CHUNKS chunks of 32 pairs per block; digits of <= 10 bits
-constexpr int RAD_THREADS = 256;
-constexpr int RAD_CHUNKS = 16;
-constexpr int RAD_TILE = RAD_THREADS * RAD_CHUNKS;
-constexpr int MAX_RADIX_BITS = 10;
-constexpr int MAX_RADIX = 1 << MAX_RADIX_BITS;
-// k_tile: 4 warps per block, one tile per warp
-constexpr int TILE_WARPS = 4;
+// k_prep: one star per thread; per-tile counters CNT_STRIDE words apart (one 128-B line each, so that the
+// atomics of different tiles never serialise on one L2 line)
+constexpr int CNT_STRIDE = 32;
+constexpr int PREP_THREADS = 256;
+// k_sortlists: one tile list per CTA; lists of up to SORT_CAP ids stay in shared memory
+constexpr int SORT_THREADS = 256;
+constexpr int SORT_CAP = 4096;
+constexpr int SORT_CHUNKS = SORT_CAP / SORT_THREADS;  // 32-item chunks per warp: SORT_CAP / 8 warps / 32 lanes
+constexpr int SORT_BITS = 8;
+constexpr int SORT_RADIX = 1 << SORT_BITS;
+constexpr int SORT_NB = 1024;                    // buckets of the range bucket sort
 
-// Per-render header in device scratch, zeroed (with the look-back status arrays) by one cudaMemsetAsync per render.
+// Per-render header in device scratch, zeroed (with the tile counters) by one cudaMemsetAsync per render.
 struct Header {
-  uint32_t ticket[4];                  // dynamic block ids: [0] k_bin, [1], [2] radix passes
   uint32_t P;                          // number of (tile, star) pairs
-  uint32_t pad[11];
-  uint32_t hist[2][MAX_RADIX];         // digit histograms of all keys for the (at most two) radix passes
+  uint32_t pad[31];
 };
 
-// Star record written by k_count, read by k_scatter and k_tile: {x, y, s', lo_x | lo_y << 16}.
+// Star record written by k_prep, read by k_scatter and k_tile: {x, y, s', lo_x | lo_y << 16}.
 // s' = A * 2.512^-m / (2 pi sigma^2), evaluated in fp64 and rounded once to fp32.
 struct __align__(16) StarRec {
   float x, y, s;
@@ -46,6 +56,7 @@ struct FrameParams {
   int32_t row0, rows;    // band (row0 = 0, rows = H for a full frame)
   int32_t R;
   int32_t ntx, nty;      // tiles over the band
+  int32_t vec;           // 1 if out rows are 16-B aligned (W % 4 == 0 and out 16-B aligned): float4 stores
   float kexp;            // -log2(e) / (2 sigma^2): exp(-d^2/(2 sigma^2)) = ex2(kexp * d^2)
   float sk;              // sqrt(log2(e) / (2 sigma^2)):  exp(-d^2/(2 sigma^2)) = ex2(-(d * sk)^2)
   double s_scale;        // A / (2 pi sigma^2), applied in fp64 before rounding s' to fp32

@@ -8,12 +8,14 @@
 namespace starsim {
 
 void init_kernels();
-void launch_bin(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
-                uint64_t* pairs, Header* hdr, unsigned long long* status, int bits0, int bits1, cudaStream_t st);
-void launch_radix(const uint64_t* in, uint64_t* out, Header* hdr, int pass, int shift, int bits,
-                  unsigned long long* status, int64_t pmax, cudaStream_t st);
-void launch_offsets(const uint64_t* sorted, const Header* hdr, uint32_t ntiles, uint32_t* tile_off, uint32_t* ids,
-                    int64_t pmax, int num_sms, cudaStream_t st);
+void init_tile_kernel();
+void launch_prep(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
+                 uint32_t* cnt, uint32_t* slots, int tps, cudaStream_t st);
+void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, cudaStream_t st);
+void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* slots, int tps,
+                    const uint32_t* tile_off, uint32_t* ids, cudaStream_t st);
+void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, int64_t ntiles, int64_t n,
+                      cudaStream_t st);
 void launch_tile(const uint32_t* ids, const uint32_t* tile_off, const StarRec* rec, const FrameParams& fp,
                  float* out, cudaStream_t st);
 void launch_atomic(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, float* out,

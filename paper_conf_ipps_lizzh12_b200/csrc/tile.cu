@@ -1,143 +1,306 @@
-// Tile accumulation (DESIGN.md §Path step a5).
+// Tile accumulation (DESIGN.md §Path step a5, §The tile kernel).
 //
-// One warp owns one 32-wide x 64-tall tile.  Lane (c, h) = (lane & 15, lane >> 4) owns columns c and c+16 and the
-// 32 rows of parity h (rows 2k+h), as 32 float2 register pairs acc[k] = (pixel(2k+h, c), pixel(2k+h, c+16)).  The
-// tile's star list (CSR from the binning, star-index order) is walked in chunks of 32:
-//   chunk phase (lane = star): load the star's id and record, clip its ROI to the tile, and evaluate its 1-D row
-//     profile s' * exp(-(r-y)^2 / 2 sigma^2) (Eq. 2 is separable: a row factor times a column factor; Eq. 1's
-//     brightness and the 1/(2 pi sigma^2) are in s') on the window of 2*NPAR rows that covers the ROI rows, split
-//     by parity, into shared memory -- one MUFU.EX2 per value, every lane busy.
-//   star phase: the chunk's stars are grouped by window start k0 (one ballot per k0), and each group runs a loop
-//     whose body is specialised for its k0: every lane evaluates the column profile at its two columns (MUFU.EX2,
-//     masked to the ROI columns by a 32-bit column mask), loads the NPAR row-profile values of its parity
-//     (LDS.128) and updates the NPAR register pairs of the window with FFMA2: acc[k] += g[k] * (gx(c), gx(c+16)).
-//     Rows outside the window cost nothing.
-// The per-pixel order of the fp32 additions is (chunk, window start, star index) -- deterministic, and the same for
-// a tile whatever the band decomposition.  The tile is written once, coalesced.  No atomics.
-#include <type_traits>
-
+// One CTA renders one 128 x 64 tile from its star list (CSR from the binning, star-index order), in chunks of up to
+// 256 stars.  Eq. 2 is separable: a star's contribution at pixel (r, c) is [s' gy(r)] * gx(c) with
+// gy(r) = exp(-(r-y)^2 / 2 sigma^2), gx(c) = exp(-(c-x)^2 / 2 sigma^2) and s' = A 2.512^-m / (2 pi sigma^2)
+// (Eq. 1 and the normaliser of Eq. 2, evaluated in fp64 by k_prep).
+//
+// Layout.  Warp (wx, B) owns the 64 x 16 block at tile columns 64 wx, rows 16 B ("band" B); inside it, lane group
+// q = lane/4 owns the 8-column strip Q = 8 wx + q and lane hq = lane%4 the rows 16 B + hq + 4 i (i = 0..3): 4 rows x
+// 8 columns = 32 fp32 accumulators per lane, updated with FFMA2 (gy broadcast x a column pair).
+//
+// Per chunk:
+//   prep (thread = star): clip the star's ROI to the tile; evaluate its row profile s' gy on the ROI rows and its
+//     column profile gx on the ROI columns (one MUFU.EX2 each, the ROI's R + R values, not R^2) into shared-memory
+//     slots: a 16-float "band slot" per (star, band) in the [hq][i] order the lanes read, an 8-float "strip slot"
+//     per (star, strip) placed at index rank * 16 + Q with its two halves XOR-swizzled by bit 2 of Q -- so the 8 lane
+//     groups of a warp always hit 8 distinct bank groups; and one entry (band slot, strip slot) in the list of every
+//     (band, strip) block the ROI overlaps.  Ranks and list positions come from warp ballots + a cross-warp prefix,
+//     so every list is in star order.  A chunk is cut short (deterministically) when a capacity would overflow.
+//   accumulate (warp): lane group q walks the list of its block (B, Q); step t loads entry t (one LDS), the row
+//     profile (one LDS.128: rows hq + 4i), the column profile (two LDS.128: 8 columns) and issues 16 FFMA2.  Groups
+//     whose list is shorter pad with an all-zero strip slot.
+// The per-pixel order of the fp32 additions is star order within the tile's list -- deterministic, and the same for a
+// tile whatever the band decomposition.  The tile is written once, coalesced (each lane stores 2 x 16 B per row).
+// No atomics on the image.
 #include "common.cuh"
 #include "launch.h"
 
 namespace starsim {
 
-constexpr int CHUNK = 32;
-constexpr int PROWS = TILE_H / 2;  // parity rows per lane
+struct TileSmem {
+  float gy[GY_CAP * 16];                 // band slots [slot][hq][i]
+  float gx[(RCAP * NSTRIPS + 1) * 8];    // strip slots [rank*16 + Q][half ^ swz(Q)][4]; last slot = zeros
+  uint32_t ent[LCAP * NBANDS * NSTRIPS]; // entries [t][B][Q] = band slot | strip slot << 16
+  uint32_t bb[TILE_WARPS][NBANDS];       // per-warp ballots: stars overlapping band B
+  uint32_t sb[TILE_WARPS][NSTRIPS];      // per-warp ballots: stars overlapping strip Q
+  uint32_t lpre[NBANDS * NSTRIPS][TILE_WARPS];  // per (B,Q): entries of the warps before
+  uint32_t rpre[NSTRIPS][TILE_WARPS];           // per Q: strip slots of the warps before
+  uint32_t len[NBANDS * NSTRIPS];
+  uint32_t wsum[TILE_WARPS];
+  float4 py[CHUNK];                      // per star: (y - IY0, s', r0 | r1 << 8, -)
+  float2 px[CHUNK];                      // per star: (x - X0, c0 | c1 << 8)
+  uint16_t gyown[GY_CAP];                // band slot -> star | band << 8
+  uint32_t gxown[GX_PAIRS];              // (star, strip) pair j -> strip slot | star << 16
+  int ns, ngy, ngx;
+};
 
-template <int KV, int KMAX, typename F>
-__device__ __forceinline__ void for_each_window(F&& f) {
-  f(std::integral_constant<int, KV>());
-  if constexpr (KV < KMAX) for_each_window<KV + 1, KMAX>(f);
-}
+constexpr uint32_t ZERO_GX = RCAP * NSTRIPS;
+constexpr uint32_t ZERO_ENT = ZERO_GX * 32u << 16;  // gy byte offset 0, all-zero strip slot
 
-// NPAR = parity rows per lane per star (a window of 2*NPAR image rows whose start 2*k0 is clamped so that it stays
-// inside the tile): 8 for R <= 15, 16 for R <= 31, 32 (the whole tile) beyond.
-template <int NPAR>
-__global__ void __launch_bounds__(TILE_WARPS * 32) k_tile(const uint32_t* __restrict__ ids,
+__global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __restrict__ ids,
                                                           const uint32_t* __restrict__ tile_off,
                                                           const StarRec* __restrict__ rec, FrameParams fp,
                                                           float* __restrict__ out) {
-  constexpr int KMAX = PROWS - NPAR;
-  __shared__ __align__(16) float s_gy[TILE_WARPS][CHUNK][2 * NPAR];
-  __shared__ __align__(8) float2 s_par[TILE_WARPS][CHUNK];
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int c = lane & 15, h = lane >> 4;
-  const int64_t t = (int64_t)blockIdx.x * TILE_WARPS + warp;
-  if (t >= (int64_t)fp.ntx * fp.nty) return;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  TileSmem& S = *reinterpret_cast<TileSmem*>(smem_raw);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  const int64_t t = blockIdx.x;
   const int tx = (int)(t % fp.ntx), ty = (int)(t / fp.ntx);
   const int X0 = tx * TILE_W;    // first column of the tile
   const int Y0 = ty * TILE_H;    // first row of the tile, relative to the band
   const int IY0 = fp.row0 + Y0;  // first image row of the tile
-  // exp(-d^2 / 2 sigma^2) = 2^(-(d * sk)^2), sk = sqrt(log2(e) / (2 sigma^2)).  d = col - x is formed exactly
-  // (tile-relative column minus the tile-relative star x, both exact in fp32) before the one scaling rounding.
+  const int TWe = min(TILE_W, fp.W - X0), THe = min(TILE_H, fp.rows - Y0);
+  // exp(-d^2 / 2 sigma^2) = 2^(-(d * sk)^2), sk = sqrt(log2(e) / (2 sigma^2)).  d = pixel - centre is formed exactly
+  // (tile-relative integer minus the tile-relative centre, both exact in fp32) before the one scaling rounding.
   const float sk = fp.sk;
-  const float fcA = (float)c, fcB = (float)(c + 16);
-  const uint32_t mA = 1u << c, mB = 1u << (c + 16);
 
-  float2 acc[PROWS];
+  // accumulate-phase identity of this lane
+  const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
+  const int Q = 8 * wx + q, p = B * NSTRIPS + Q;
+  const int swz = (Q >> 2) & 1;
+  const uint32_t gy_base = (uint32_t)__cvta_generic_to_shared(S.gy) + 16u * hq;
+  const uint32_t gxa_base = (uint32_t)__cvta_generic_to_shared(S.gx) + 16u * swz;
+  const uint32_t gxb_base = (uint32_t)__cvta_generic_to_shared(S.gx) + 16u * (swz ^ 1);
+  float2 acc[4][4];
 #pragma unroll
-  for (int i = 0; i < PROWS; ++i) acc[i] = make_float2(0.f, 0.f);
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
+
+  if (tid < 8) S.gx[ZERO_GX * 8 + tid] = 0.f;
 
   const uint32_t j0 = tile_off[t], j1 = tile_off[t + 1];
-  for (uint32_t base = j0; base < j1; base += CHUNK) {
-    const int cnt = (int)min((uint32_t)CHUNK, j1 - base);
-    // ---------------- chunk phase: lane = star
-    int k0 = -1;
-    if (lane < cnt) {
-      const StarRec r = rec[ids[base + lane]];
+  for (uint32_t base = j0; base < j1;) {
+    // ======================= prep: thread = star (base + tid)
+    const int nvalid = (int)min((uint32_t)CHUNK, j1 - base);
+    const bool valid = tid < nvalid;
+    StarRec r = {};
+    int c0 = 0, c1 = -1, r0 = 0, r1 = -1;
+    if (valid) {
+      r = rec[ids[base + tid]];
       const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
-      const int c0 = max(lx, 0), c1 = min(lx + fp.R - 1, TILE_W - 1);
-      const int r0 = max(ly, 0), r1 = min(ly + fp.R - 1, TILE_H - 1);
-      k0 = min(r0 >> 1, KMAX);
-      float* g = &s_gy[warp][lane][0];
-      const float yr = r.y - (float)IY0;  // star y relative to the tile (exact)
-#pragma unroll
-      for (int hh = 0; hh < 2; ++hh)
-#pragma unroll
-        for (int j = 0; j < NPAR; ++j) {
-          const int row = 2 * (k0 + j) + hh;
-          const float d = ((float)row - yr) * sk;
-          const float e = r.s * ex2_approx(-(d * d));
-          g[hh * NPAR + j] = (row >= r0 && row <= r1) ? e : 0.f;
-        }
-      // the ROI's columns of this tile as a bit mask (c1 - c0 <= 31; 2u << 31 wraps to 0 -> all ones)
-      const uint32_t bm = ((2u << (uint32_t)(c1 - c0)) - 1u) << c0;
-      s_par[warp][lane] = make_float2(r.x - (float)X0, __uint_as_float(bm));
+      c0 = max(lx, 0);
+      c1 = min(lx + fp.R - 1, TWe - 1);
+      r0 = max(ly, 0);
+      r1 = min(ly + fp.R - 1, THe - 1);
     }
-    __syncwarp();
-    // ---------------- star phase
-    auto star = [&](int s, auto KW) {
-      constexpr int K = decltype(KW)::value;
-      const float2 par = s_par[warp][s];
-      const uint32_t bm = __float_as_uint(par.y);
-      const float dA = (fcA - par.x) * sk, dB = (fcB - par.x) * sk;
-      const float eA = ex2_approx(-(dA * dA)), eB = ex2_approx(-(dB * dB));
-      const float2 gx2 = make_float2((bm & mA) ? eA : 0.f, (bm & mB) ? eB : 0.f);
-      const float4* g4 = reinterpret_cast<const float4*>(&s_gy[warp][s][h * NPAR]);
+    const int b0 = r0 >> 4, b1 = r1 >> 4, q0 = c0 >> 3, q1 = c1 >> 3;  // empty ranges when !valid
+    const int ngy = valid ? b1 - b0 + 1 : 0, ngx = valid ? q1 - q0 + 1 : 0;
+    __syncthreads();  // the previous chunk's accumulate phase is done with the shared buffers
+    if (tid == 0) S.ns = CHUNK;
+    {
+      uint32_t bbv = 0, sbv = 0;
 #pragma unroll
-      for (int q = 0; q < NPAR / 4; ++q) {
-        const float4 u = g4[q];
-        acc[K + 4 * q + 0] = __ffma2_rn(make_float2(u.x, u.x), gx2, acc[K + 4 * q + 0]);
-        acc[K + 4 * q + 1] = __ffma2_rn(make_float2(u.y, u.y), gx2, acc[K + 4 * q + 1]);
-        acc[K + 4 * q + 2] = __ffma2_rn(make_float2(u.z, u.z), gx2, acc[K + 4 * q + 2]);
-        acc[K + 4 * q + 3] = __ffma2_rn(make_float2(u.w, u.w), gx2, acc[K + 4 * q + 3]);
+      for (int k = 0; k < NBANDS; ++k) {
+        const uint32_t m = __ballot_sync(0xffffffffu, b0 <= k && k <= b1);
+        if (lane == k) bbv = m;
       }
-    };
-    // group the chunk's stars by window start: one ballot per k0, then a loop over that group's stars
-    for_each_window<0, KMAX>([&](auto KW) {
-      constexpr int K = decltype(KW)::value;
-      uint32_t m = __ballot_sync(0xffffffffu, k0 == K);
-      while (m) {
-        const int s = __ffs(m) - 1;
-        m &= m - 1;
-        star(s, KW);
+#pragma unroll
+      for (int k = 0; k < NSTRIPS; ++k) {
+        const uint32_t m = __ballot_sync(0xffffffffu, q0 <= k && k <= q1);
+        if (lane == k) sbv = m;
       }
-    });
-    __syncwarp();
+      if (lane < NBANDS) S.bb[warp][lane] = bbv;
+      if (lane < NSTRIPS) S.sb[warp][lane] = sbv;
+    }
+    // band-slot and (star, strip)-pair scans in star order (packed: ngy | ngx << 16)
+    const uint32_t pk = (uint32_t)ngy | ((uint32_t)ngx << 16);
+    uint32_t incl = pk;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += v;
+    }
+    if (lane == 31) S.wsum[warp] = incl;
+    __syncthreads();
+    if (tid < NBANDS * NSTRIPS) {
+      const int pb = tid >> 4, pq = tid & 15;
+      uint32_t run = 0;
+#pragma unroll
+      for (int w = 0; w < TILE_WARPS; ++w) {
+        S.lpre[tid][w] = run;
+        run += __popc(S.bb[w][pb] & S.sb[w][pq]);
+      }
+    } else if (tid < NBANDS * NSTRIPS + NSTRIPS) {
+      const int pq = tid - NBANDS * NSTRIPS;
+      uint32_t run = 0;
+#pragma unroll
+      for (int w = 0; w < TILE_WARPS; ++w) {
+        S.rpre[pq][w] = run;
+        run += __popc(S.sb[w][pq]);
+      }
+    }
+    uint32_t excl = incl - pk;
+    for (int w = 0; w < warp; ++w) excl += S.wsum[w];
+    const uint32_t gyb = excl & 0xFFFFu, gxb = excl >> 16;
+    __syncthreads();
+    // slots, list entries and the capacity check in one pass: a star whose slot or list position would overflow
+    // ends the chunk (its own writes land beyond the lengths used below and are ignored / overwritten)
+    if (valid) {
+      bool fits = gyb + (uint32_t)ngy <= (uint32_t)GY_CAP && gxb + (uint32_t)ngx <= (uint32_t)GX_PAIRS;
+      uint32_t j = gxb;
+      for (int k = q0; k <= q1 && fits; ++k, ++j) {
+        const uint32_t sbk = S.sb[warp][k];
+        const uint32_t rk = S.rpre[k][warp] + __popc(sbk & lt);
+        fits = rk < (uint32_t)RCAP;
+        const uint32_t slot = rk * NSTRIPS + k;
+        if (fits) S.gxown[j] = slot | ((uint32_t)tid << 16);
+        for (int b = b0; b <= b1 && fits; ++b) {
+          const uint32_t pos = S.lpre[b * NSTRIPS + k][warp] + __popc(S.bb[warp][b] & sbk & lt);
+          fits = pos < (uint32_t)LCAP;
+          if (fits) S.ent[(pos * NBANDS + b) * NSTRIPS + k] = (gyb + (uint32_t)(b - b0)) * 64u | (slot * 32u << 16);
+        }
+      }
+      if (fits) {
+        for (int b = b0; b <= b1; ++b) S.gyown[gyb + b - b0] = (uint16_t)(tid | (b << 8));
+      } else {
+        atomicMin(&S.ns, tid);
+      }
+      S.py[tid] = make_float4(r.y - (float)IY0, r.s, __int_as_float(r0 | (r1 << 8)), 0.f);
+      S.px[tid] = make_float2(r.x - (float)X0, __int_as_float(c0 | (c1 << 8)));
+    }
+    __syncthreads();
+    const int ns = min(S.ns, nvalid);
+    if (tid == ns - 1) {
+      S.ngy = (int)(gyb + ngy);
+      S.ngx = (int)(gxb + ngx);
+    }
+    if (tid < NBANDS * NSTRIPS) {
+      const int pb = tid >> 4, pq = tid & 15;
+      uint32_t n = 0;
+#pragma unroll
+      for (int w = 0; w < TILE_WARPS; ++w) {
+        const int lo = ns - 32 * w;
+        const uint32_t below = lo >= 32 ? 0xffffffffu : (lo <= 0 ? 0u : ((1u << lo) - 1u));
+        n += __popc(S.bb[w][pb] & S.sb[w][pq] & below);
+      }
+      S.len[tid] = n;
+    }
+    __syncthreads();
+    // profiles: thread = 4 values of one slot.  Band slot (row profile s' gy): rows 16 b + h4 + 4 i, i = 0..3;
+    // strip slot (column profile gx): columns 8 k + 4 half + i.  d = (pixel - centre) is exact before the scaling;
+    // values outside the ROI are 0.  FADD2/FMUL2 pairs, one MUFU.EX2 per value.
+    {
+      const int ngq = S.ngy * 4;
+      for (int gq = tid; gq < ngq; gq += TILE_THREADS) {
+        const int k = gq >> 2, h4 = gq & 3;
+        const uint32_t own = S.gyown[k];
+        const float4 pp = S.py[own & 0xFFu];
+        const int rel = 16 * (int)(own >> 8) + h4;                 // first row of this quad (tile-relative)
+        const int lo = (__float_as_int(pp.z) & 0xFF) - rel, hi = (__float_as_int(pp.z) >> 8) - rel;
+        const float b0f = (float)rel - pp.x;                       // exact
+        const float2 sk2 = make_float2(sk, sk);
+        float2 d01 = __fmul2_rn(__fadd2_rn(make_float2(b0f, b0f), make_float2(0.f, 4.f)), sk2);
+        float2 d23 = __fmul2_rn(__fadd2_rn(make_float2(b0f, b0f), make_float2(8.f, 12.f)), sk2);
+        d01 = __fmul2_rn(d01, make_float2(-d01.x, -d01.y));
+        d23 = __fmul2_rn(d23, make_float2(-d23.x, -d23.y));
+        float2 e01 = make_float2(ex2_approx(d01.x), ex2_approx(d01.y));
+        float2 e23 = make_float2(ex2_approx(d23.x), ex2_approx(d23.y));
+        e01 = __fmul2_rn(e01, make_float2(pp.y, pp.y));
+        e23 = __fmul2_rn(e23, make_float2(pp.y, pp.y));
+        const float4 v = make_float4(lo <= 0 && 0 <= hi ? e01.x : 0.f, lo <= 4 && 4 <= hi ? e01.y : 0.f,
+                                     lo <= 8 && 8 <= hi ? e23.x : 0.f, lo <= 12 && 12 <= hi ? e23.y : 0.f);
+        *reinterpret_cast<float4*>(&S.gy[k * 16 + h4 * 4]) = v;
+      }
+      const int nxq = S.ngx * 2;
+      for (int gq = tid; gq < nxq; gq += TILE_THREADS) {
+        const uint32_t own = S.gxown[gq >> 1];
+        const int half = gq & 1;
+        const uint32_t slot = own & 0xFFFFu;
+        const int k = (int)(slot & 15u);
+        const float2 pp = S.px[own >> 16];
+        const int rel = 8 * k + 4 * half;
+        const int lo = (__float_as_int(pp.y) & 0xFF) - rel, hi = (__float_as_int(pp.y) >> 8) - rel;
+        const float b0f = (float)rel - pp.x;
+        const float2 sk2 = make_float2(sk, sk);
+        float2 d01 = __fmul2_rn(__fadd2_rn(make_float2(b0f, b0f), make_float2(0.f, 1.f)), sk2);
+        float2 d23 = __fmul2_rn(__fadd2_rn(make_float2(b0f, b0f), make_float2(2.f, 3.f)), sk2);
+        d01 = __fmul2_rn(d01, make_float2(-d01.x, -d01.y));
+        d23 = __fmul2_rn(d23, make_float2(-d23.x, -d23.y));
+        const float4 v = make_float4(lo <= 0 && 0 <= hi ? ex2_approx(d01.x) : 0.f,
+                                     lo <= 1 && 1 <= hi ? ex2_approx(d01.y) : 0.f,
+                                     lo <= 2 && 2 <= hi ? ex2_approx(d23.x) : 0.f,
+                                     lo <= 3 && 3 <= hi ? ex2_approx(d23.y) : 0.f);
+        *reinterpret_cast<float4*>(&S.gx[slot * 8 + ((half ^ ((k >> 2) & 1)) * 4)]) = v;
+      }
+      // pad every list with all-zero entries up to the longest list of its warp
+      if (tid < NBANDS * NSTRIPS) {
+        const int pb = tid >> 4, pq = tid & 15, w0 = pq & 8;
+        uint32_t mxl = 0;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) mxl = max(mxl, S.len[pb * NSTRIPS + w0 + k]);
+        for (uint32_t st = S.len[tid]; st < mxl; ++st) S.ent[(st * NBANDS + pb) * NSTRIPS + pq] = ZERO_ENT;
+      }
+    }
+    __syncthreads();
+
+    // ======================= accumulate: lane group q walks the (padded) list of block (B, Q)
+    {
+      const uint32_t steps = __reduce_max_sync(0xffffffffu, S.len[p]);
+      const uint32_t* ent = &S.ent[B * NSTRIPS + Q];
+#pragma unroll 4
+      for (uint32_t st = 0; st < steps; ++st) {
+        const uint32_t e = ent[st * (NBANDS * NSTRIPS)];
+        const uint32_t go = e & 0xFFFFu, xo = e >> 16;
+        float4 g, a, c;
+        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(g.x), "=f"(g.y), "=f"(g.z), "=f"(g.w) : "r"(gy_base + go));
+        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "r"(gxa_base + xo));
+        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(c.x), "=f"(c.y), "=f"(c.z), "=f"(c.w) : "r"(gxb_base + xo));
+        const float gi[4] = {g.x, g.y, g.z, g.w};
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const float2 gg = make_float2(gi[i], gi[i]);
+          acc[i][0] = __ffma2_rn(gg, make_float2(a.x, a.y), acc[i][0]);
+          acc[i][1] = __ffma2_rn(gg, make_float2(a.z, a.w), acc[i][1]);
+          acc[i][2] = __ffma2_rn(gg, make_float2(c.x, c.y), acc[i][2]);
+          acc[i][3] = __ffma2_rn(gg, make_float2(c.z, c.w), acc[i][3]);
+        }
+      }
+    }
+    base += (uint32_t)ns;
   }
 
-  // ---------------- write the tile once: row 2k+h, columns X0+c and X0+c+16
-  float* o = out + (int64_t)(Y0 + h) * fp.W + X0 + c;
-  const bool okA = X0 + c < fp.W, okB = X0 + c + 16 < fp.W;
+  // ======================= write the tile once: row 16 B + hq + 4 i, columns 64 wx + 8 q .. +7
+  const int col0 = X0 + 64 * wx + 8 * q;
 #pragma unroll
-  for (int k = 0; k < PROWS; ++k) {
-    if (Y0 + 2 * k + h < fp.rows) {
-      if (okA) o[(int64_t)(2 * k) * fp.W] = acc[k].x;
-      if (okB) o[(int64_t)(2 * k) * fp.W + 16] = acc[k].y;
+  for (int i = 0; i < 4; ++i) {
+    const int row = Y0 + 16 * B + hq + 4 * i;  // band-relative
+    if (row >= fp.rows || col0 >= fp.W) continue;
+    float* o = out + (int64_t)row * fp.W + col0;
+    if (fp.vec && col0 + 8 <= fp.W) {
+      reinterpret_cast<float4*>(o)[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
+      reinterpret_cast<float4*>(o)[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
+    } else {
+      const float v[8] = {acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y,
+                          acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y};
+#pragma unroll
+      for (int k = 0; k < 8; ++k)
+        if (col0 + k < fp.W) o[k] = v[k];
     }
   }
+}
+
+void init_tile_kernel() {
+  cudaFuncSetAttribute(k_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
 }
 
 void launch_tile(const uint32_t* ids, const uint32_t* tile_off, const StarRec* rec, const FrameParams& fp,
                  float* out, cudaStream_t st) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
-  const unsigned blocks = (unsigned)((ntiles + TILE_WARPS - 1) / TILE_WARPS);
-  if (fp.R <= 15)
-    k_tile<8><<<blocks, TILE_WARPS * 32, 0, st>>>(ids, tile_off, rec, fp, out);
-  else if (fp.R <= 31)
-    k_tile<16><<<blocks, TILE_WARPS * 32, 0, st>>>(ids, tile_off, rec, fp, out);
-  else
-    k_tile<PROWS><<<blocks, TILE_WARPS * 32, 0, st>>>(ids, tile_off, rec, fp, out);
+  if (ntiles <= 0) return;
+  k_tile<<<(unsigned)ntiles, TILE_THREADS, sizeof(TileSmem), st>>>(ids, tile_off, rec, fp, out);
 }
 
 }  // namespace starsim

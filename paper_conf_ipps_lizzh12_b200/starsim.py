@@ -20,7 +20,7 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_PKG, "libstarsim.so")
 
 STARSIM_OK, STARSIM_EINVAL, STARSIM_ENOMEM, STARSIM_ECUDA, STARSIM_ENODEV = 0, -1, -2, -3, -4
-KCLASSES = ("bin", "radix", "offsets", "tile", "atomic", "memset", "quantize", "aos")
+KCLASSES = ("prep", "sort", "csr", "tile", "atomic", "memset", "quantize", "aos")
 NUM_KCLASS = len(KCLASSES)
 
 _lock = threading.Lock()

@@ -138,8 +138,8 @@ def test_bins_bit_exact(torch_dev, ctx, name, n, R, kind):
 def test_deterministic_and_tile_translation(torch_dev, ctx):
     torch, dev = torch_dev
     W, H = 512, 384
-    f = synth.uniform_field(20000, W - 64, H - 64, seed=3, mag_hi=2.0)
-    # positions on a 1/256 grid so that x + 32 and y + 64 are exact in fp32
+    f = synth.uniform_field(20000, W - 128, H - 64, seed=3, mag_hi=2.0)
+    # positions on a 1/256 grid so that x + 128 and y + 64 are exact in fp32
     f = synth.Field(np.round(f.x * 256).astype(np.float32) / np.float32(256),
                     np.round(f.y * 256).astype(np.float32) / np.float32(256), f.mag)
     x, y, m = to_dev(torch_dev, f)
@@ -147,8 +147,8 @@ def test_deterministic_and_tile_translation(torch_dev, ctx):
     b = ctx.render(x, y, m, W, H, 2.5, 15, 7.0)
     assert torch.equal(a, b)
     # shift by whole tiles: every per-pixel sum sees the same stars in the same order
-    c = ctx.render(x + 32, y + 64, m, W, H, 2.5, 15, 7.0)
-    assert torch.equal(a[:H - 64, :W - 32], c[64:, 32:])
+    c = ctx.render(x + 128, y + 64, m, W, H, 2.5, 15, 7.0)
+    assert torch.equal(a[:H - 64, :W - 128], c[64:, 128:])
 
 
 # ---------------------------------------------------------------- bands (multi-GPU decomposition, one device)
@@ -255,7 +255,7 @@ def test_kernel_times_recorded(torch_dev, ctx):
     ctx.render(*args, cfg.W, cfg.H, cfg.sigma, cfg.R, 1.0)
     t = ctx.kernel_times()
     ctx.profile(False)
-    assert t["tile"][1] == 1 and t["tile"][0] > 0 and t["bin"][1] == 1 and t["offsets"][1] == 1
+    assert t["tile"][1] == 1 and t["tile"][0] > 0 and t["prep"][1] == 1 and t["sort"][1] == 1 and t["csr"][1] == 1
 
 
 # ---------------------------------------------------------------- B200-scale frames (full images, threaded oracle)
