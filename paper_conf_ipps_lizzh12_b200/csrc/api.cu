@@ -2,6 +2,7 @@
 // stream-ordered orchestration of the sm_100a kernels, per-kernel CUDA-event timing, error strings.
 #include <cmath>
 #include <cstdio>
+#include <algorithm>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -47,7 +48,7 @@ struct starsim_ctx {
   int dev = 0;
   int num_sms = 148;
   std::string err;
-  Buf rec, slots, ids, tmp, tile_off, zeroed, stage;
+  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, zeroed, stage;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
@@ -188,10 +189,11 @@ int tiles_per_axis(int R, int tile, int ntiles_axis) {
 // Enqueue the tiled render on stream st: memset of the header + tile counters, k_prep, k_scan, k_scatter,
 // k_sortlists, k_tile.
 int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, const FrameParams& fp,
-                  int64_t ntiles, int tps, float* out, cudaStream_t st) {
+                  int64_t ntiles, int tps, int part_cap, float* out, cudaStream_t st) {
   Header* hdr = (Header*)c->zeroed.p;
   uint32_t* cnt = (uint32_t*)(hdr + 1);
-  const size_t zbytes = sizeof(Header) + sizeof(uint32_t) * CNT_STRIDE * (size_t)ntiles;
+  const size_t zbytes = sizeof(Header) + sizeof(uint32_t) * (CNT_STRIDE + 1) * (size_t)ntiles;
+  uint32_t* done = cnt + CNT_STRIDE * ntiles;
   uint32_t* ids = (uint32_t*)c->ids.p;
   uint32_t* tile_off = (uint32_t*)c->tile_off.p;
   uint32_t* slots = (uint32_t*)c->slots.p;
@@ -203,13 +205,16 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
     if ((rc = check_launch(c, "k_prep"))) return rc;
   }
   timed(c, 2, st, [&] {
-    launch_scan(cnt, ntiles, tile_off, hdr, st);
+    launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap, st);
     launch_scatter(rec, n, fp, slots, tps, tile_off, ids, st);
   });
   if ((rc = check_launch(c, "k_scan/k_scatter"))) return rc;
   timed(c, 1, st, [&] { launch_sortlists(ids, (uint32_t*)c->tmp.p, tile_off, ntiles, n, st); });
   if ((rc = check_launch(c, "k_sortlists"))) return rc;
-  timed(c, 3, st, [&] { launch_tile(ids, tile_off, rec, fp, out, st); });
+  timed(c, 3, st, [&] {
+    launch_tile(ids, rec, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p, part_cap, done,
+                hdr, st);
+  });
   if ((rc = check_launch(c, "k_tile"))) return rc;
   return STARSIM_OK;
 }
@@ -223,7 +228,9 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   const int tps = tiles_per_axis(R, TILE_W, fp.ntx) * tiles_per_axis(R, TILE_H, fp.nty);
   const int64_t pmax = n * (int64_t)tps;
   if (pmax >= 0xFFFFFFFFll) return fail(c, STARSIM_EINVAL, "n * tiles-per-star >= 2^32 (pair counts are 32-bit)");
-  const size_t zbytes = sizeof(Header) + sizeof(uint32_t) * CNT_STRIDE * (size_t)ntiles;
+  const size_t zbytes = sizeof(Header) + sizeof(uint32_t) * (CNT_STRIDE + 1) * (size_t)ntiles;
+  // partial-tile buffers for split heavy tiles: at most P / SPLIT_LEN parts exist
+  const int part_cap = (int)std::min<int64_t>(PART_CAP, pmax / SPLIT_LEN + 1);
   int rc;
   if ((rc = grow(c, c->rec, sizeof(StarRec) * (size_t)(n > 0 ? n : 1), "records"))) return rc;
   if ((rc = grow(c, c->slots, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "tile slots"))) return rc;
@@ -231,10 +238,13 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   if ((rc = grow(c, c->tmp, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "sort scratch"))) return rc;
   if ((rc = grow(c, c->tile_off, sizeof(uint32_t) * (size_t)(ntiles + 1), "tile offsets"))) return rc;
   if ((rc = grow(c, c->zeroed, zbytes, "header+counters"))) return rc;
+  if ((rc = grow(c, c->items, sizeof(WorkItem) * (size_t)(ntiles + part_cap), "work items"))) return rc;
+  if ((rc = grow(c, c->split_tab, sizeof(uint2) * (size_t)ntiles, "split table"))) return rc;
+  if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
 
   const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, sigma, gain, st, c->scratch_gen};
   if (st == nullptr || c->prof || !c->use_graphs) {
-    if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, out, st))) return rc;
+    if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st))) return rc;
   } else {
     if (!(c->have_graph && c->gkey == key)) {
       if (c->have_graph) {
@@ -243,7 +253,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
       }
       cudaError_t e = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal);
       if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamBeginCapture");
-      rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, out, st);
+      rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st);
       cudaGraph_t graph = nullptr;
       e = cudaStreamEndCapture(st, &graph);
       if (rc) {
@@ -315,7 +325,8 @@ void starsim_destroy(starsim_ctx* c) {
     DevGuard g(c->dev);
     cudaDeviceSynchronize();
     if (c->have_graph) cudaGraphExecDestroy(c->gexec);
-    Buf* bufs[] = {&c->rec, &c->slots, &c->ids, &c->tmp, &c->tile_off, &c->zeroed, &c->stage};
+    Buf* bufs[] = {&c->rec, &c->slots, &c->ids, &c->tmp, &c->tile_off, &c->items, &c->split_tab, &c->parts,
+                   &c->zeroed, &c->stage};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {

@@ -2,7 +2,8 @@
 //   k_prep       a1: per star -- validity, s' in fp64, exact ROI origin, clip to the frame columns and band rows; the
 //                tiles its clipped ROI overlaps (row-major), and for each one a slot in that tile's list from an
 //                atomic counter (one ATOMG per (tile, star) pair).  Writes the 16-B star record.
-//   k_scan       a2: exclusive scan of the per-tile counts -> tile_off[ntiles+1] (one CTA), P.
+//   k_scan       a2: exclusive scan of the per-tile counts -> tile_off[ntiles+1] (one CTA), P; then k_tile's work
+//                list (heavy tiles split into parts).
 //   k_scatter    a3: ids[tile_off[tile] + slot] = star for every pair.
 //   k_sortlists  a4: sort every tile's list ascending (LSD radix on the star index in shared memory, 8-bit digits,
 //                stable warp-ballot ranking); lists longer than SORT_CAP are sorted in SORT_CAP chunks through a
@@ -66,44 +67,84 @@ __global__ void __launch_bounds__(PREP_THREADS) k_prep(const float* __restrict__
 }
 
 // ---------------------------------------------------------------------------------------------------------------
-// k_scan -- step a2: tile_off[t] = sum of cnt[0..t), tile_off[ntiles] = P; one CTA of 1024 threads, each thread a
-// contiguous run of tiles.
+// k_scan -- step a2 and k_tile's work list, one CTA of 1024 threads, each a contiguous run of tiles:
+//   tile_off[t] = sum of cnt[0..t), tile_off[ntiles] = P;
+//   a tile whose list is longer than SPLIT_LEN becomes ceil(len / SPLIT_LEN) work items over consecutive star ranges
+//   (its parts), every other tile one item; parts come first (the heavy work starts first).  The split depends only
+//   on the tile's own list, so it is the same for any band decomposition.  If the parts would need more than
+//   `part_cap` partial buffers, nothing is split.
 // ---------------------------------------------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t parts_of(uint32_t len) {
+  if (len <= (uint32_t)SPLIT_LEN) return 0u;
+  return min((len + SPLIT_LEN - 1) / SPLIT_LEN, 4095u);
+}
+
 __global__ void __launch_bounds__(1024) k_scan(const uint32_t* __restrict__ cnt, int64_t ntiles,
-                                               uint32_t* __restrict__ tile_off, Header* hdr) {
-  __shared__ uint32_t s_w[32];
+                                               uint32_t* __restrict__ tile_off, Header* hdr,
+                                               WorkItem* __restrict__ items, uint2* __restrict__ split_tab,
+                                               int part_cap) {
+  __shared__ uint3 s_w[32];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t per = (ntiles + 1023) / 1024;
   const int64_t a = min((int64_t)tid * per, ntiles), b = min(a + per, ntiles);
-  uint32_t sum = 0;
-  for (int64_t t = a; t < b; ++t) sum += cnt[t * CNT_STRIDE];
-  uint32_t incl = sum;
+  uint3 sum = make_uint3(0, 0, 0);  // pairs, parts, split tiles
+  for (int64_t t = a; t < b; ++t) {
+    const uint32_t c = cnt[t * CNT_STRIDE], np = parts_of(c);
+    sum.x += c;
+    sum.y += np;
+    sum.z += np ? 1u : 0u;
+  }
+  uint3 incl = sum;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
-    if (lane >= o) incl += v;
+    const uint32_t vx = __shfl_up_sync(0xffffffffu, incl.x, o), vy = __shfl_up_sync(0xffffffffu, incl.y, o),
+                   vz = __shfl_up_sync(0xffffffffu, incl.z, o);
+    if (lane >= o) {
+      incl.x += vx;
+      incl.y += vy;
+      incl.z += vz;
+    }
   }
   if (lane == 31) s_w[warp] = incl;
   __syncthreads();
-  if (warp == 0) {
-    const uint32_t w = s_w[lane];
-    uint32_t wi = w;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t v = __shfl_up_sync(0xffffffffu, wi, o);
-      if (lane >= o) wi += v;
+  uint3 pre = make_uint3(incl.x - sum.x, incl.y - sum.y, incl.z - sum.z), tot = make_uint3(0, 0, 0);
+  for (int w = 0; w < 32; ++w) {
+    const uint3 v = s_w[w];
+    if (w < warp) {
+      pre.x += v.x;
+      pre.y += v.y;
+      pre.z += v.z;
     }
-    s_w[lane] = wi - w;
-    if (lane == 31) {
-      hdr->P = wi;
-      tile_off[ntiles] = wi;
-    }
+    tot.x += v.x;
+    tot.y += v.y;
+    tot.z += v.z;
   }
-  __syncthreads();
-  uint32_t run = s_w[warp] + incl - sum;
+  const bool split_on = tot.y <= (uint32_t)part_cap;
+  const uint32_t nparts = split_on ? tot.y : 0u, nsplit = split_on ? tot.z : 0u;
+  if (tid == 0) {
+    hdr->P = tot.x;
+    tile_off[ntiles] = tot.x;
+    hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
+    hdr->nsplit = nsplit;
+  }
+  uint32_t run = pre.x, pb = pre.y, si = pre.z;
   for (int64_t t = a; t < b; ++t) {
+    const uint32_t c = cnt[t * CNT_STRIDE];
     tile_off[t] = run;
-    run += cnt[t * CNT_STRIDE];
+    const uint32_t np = split_on ? parts_of(c) : 0u;
+    if (np) {
+      split_tab[si] = make_uint2(pb, np);
+      const uint32_t per_part = (c + np - 1) / np;
+      for (uint32_t k = 0; k < np; ++k)
+        items[pb + k] = WorkItem{(uint32_t)t, run + k * per_part, min(run + c, run + (k + 1) * per_part),
+                                 (si << 12) | k};
+      pb += np;
+      ++si;
+    } else {
+      // whole tiles follow the parts, in tile order: index = nparts + (tiles before t that are not split)
+      items[nparts + (uint32_t)t - (split_on ? si : 0u)] = WorkItem{(uint32_t)t, run, run + c, ITEM_WHOLE};
+    }
+    run += c;
   }
 }
 
@@ -376,8 +417,9 @@ void launch_prep(const float* x, const float* y, const float* m, int64_t n, cons
                                                                                      tps);
 }
 
-void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, cudaStream_t st) {
-  k_scan<<<1, 1024, 0, st>>>(cnt, ntiles, tile_off, hdr);
+void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items,
+                 uint2* split_tab, int part_cap, cudaStream_t st) {
+  k_scan<<<1, 1024, 0, st>>>(cnt, ntiles, tile_off, hdr, items, split_tab, part_cap);
 }
 
 void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* slots, int tps,

@@ -23,6 +23,8 @@
 // The per-pixel order of the fp32 additions is star order within the tile's list -- deterministic, and the same for a
 // tile whatever the band decomposition.  The tile is written once, coalesced (each lane stores 2 x 16 B per row).
 // No atomics on the image.
+#include <algorithm>
+
 #include "common.cuh"
 #include "launch.h"
 
@@ -48,20 +50,21 @@ struct TileSmem {
 constexpr uint32_t ZERO_GX = RCAP * NSTRIPS;
 constexpr uint32_t ZERO_ENT = ZERO_GX * 32u << 16;  // gy byte offset 0, all-zero strip slot
 
+// ---------------------------------------------------------------------------------------------------------------
+// k_tile: one CTA per work item (item = blockIdx.x; parts first, so the heavy work starts first).  A whole tile is written to `out`
+// directly; a part writes its 128 x 64 partial to part_buf, and the last part to finish (per-tile counter) sums the
+// parts in part order -- a fixed order, so the image stays deterministic.
+// ---------------------------------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __restrict__ ids,
-                                                          const uint32_t* __restrict__ tile_off,
                                                           const StarRec* __restrict__ rec, FrameParams fp,
-                                                          float* __restrict__ out) {
+                                                          float* __restrict__ out, const WorkItem* __restrict__ items,
+                                                          const uint2* __restrict__ split_tab,
+                                                          float* __restrict__ part_buf, uint32_t* __restrict__ done,
+                                                          Header* hdr) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   TileSmem& S = *reinterpret_cast<TileSmem*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t lt = (1u << lane) - 1u;
-  const int64_t t = blockIdx.x;
-  const int tx = (int)(t % fp.ntx), ty = (int)(t / fp.ntx);
-  const int X0 = tx * TILE_W;    // first column of the tile
-  const int Y0 = ty * TILE_H;    // first row of the tile, relative to the band
-  const int IY0 = fp.row0 + Y0;  // first image row of the tile
-  const int TWe = min(TILE_W, fp.W - X0), THe = min(TILE_H, fp.rows - Y0);
   // exp(-d^2 / 2 sigma^2) = 2^(-(d * sk)^2), sk = sqrt(log2(e) / (2 sigma^2)).  d = pixel - centre is formed exactly
   // (tile-relative integer minus the tile-relative centre, both exact in fp32) before the one scaling rounding.
   const float sk = fp.sk;
@@ -73,16 +76,25 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
   const uint32_t gy_base = (uint32_t)__cvta_generic_to_shared(S.gy) + 16u * hq;
   const uint32_t gxa_base = (uint32_t)__cvta_generic_to_shared(S.gx) + 16u * swz;
   const uint32_t gxb_base = (uint32_t)__cvta_generic_to_shared(S.gx) + 16u * (swz ^ 1);
+  __shared__ int s_last;
+  if (tid < 8) S.gx[ZERO_GX * 8 + tid] = 0.f;
+
+  for (int once = 0; once < 1; ++once) {
+  if (blockIdx.x >= __ldcg(&hdr->nitems)) return;
+  const WorkItem wi = items[blockIdx.x];
+  const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
+  const int X0 = tx * TILE_W;    // first column of the tile
+  const int Y0 = ty * TILE_H;    // first row of the tile, relative to the band
+  const int IY0 = fp.row0 + Y0;  // first image row of the tile
+  const int TWe = min(TILE_W, fp.W - X0), THe = min(TILE_H, fp.rows - Y0);
   float2 acc[4][4];
 #pragma unroll
   for (int i = 0; i < 4; ++i)
 #pragma unroll
     for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
 
-  if (tid < 8) S.gx[ZERO_GX * 8 + tid] = 0.f;
-
-  const uint32_t j0 = tile_off[t], j1 = tile_off[t + 1];
-  for (uint32_t base = j0; base < j1;) {
+  const uint32_t j1 = wi.je;
+  for (uint32_t base = wi.jb; base < j1;) {
     // ======================= prep: thread = star (base + tid)
     const int nvalid = (int)min((uint32_t)CHUNK, j1 - base);
     const bool valid = tid < nvalid;
@@ -272,8 +284,41 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
     base += (uint32_t)ns;
   }
 
-  // ======================= write the tile once: row 16 B + hq + 4 i, columns 64 wx + 8 q .. +7
+  // ======================= output: rows 16 B + hq + 4 i, columns 64 wx + 8 q .. +7 of the tile
   const int col0 = X0 + 64 * wx + 8 * q;
+  if (wi.aux != ITEM_WHOLE) {
+    // one part of a split tile: store the partial, and the last part to finish reduces all parts in order
+    const uint2 sp = split_tab[wi.aux >> 12];
+    float* pbuf = part_buf + (size_t)(sp.x + (wi.aux & 0xFFFu)) * (TILE_W * TILE_H);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      float4* o = reinterpret_cast<float4*>(pbuf + (16 * B + hq + 4 * i) * TILE_W + 64 * wx + 8 * q);
+      o[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
+      o[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
+    }
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) s_last = atomicAdd(&done[wi.aux >> 12], 1u) == sp.y - 1;
+    __syncthreads();
+    if (!s_last) continue;
+    __threadfence();
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
+    for (uint32_t k = 0; k < sp.y; ++k) {
+      const float* pk = part_buf + (size_t)(sp.x + k) * (TILE_W * TILE_H);
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const float4* o = reinterpret_cast<const float4*>(pk + (16 * B + hq + 4 * i) * TILE_W + 64 * wx + 8 * q);
+        const float4 u = __ldcg(o), v = __ldcg(o + 1);
+        acc[i][0] = __fadd2_rn(acc[i][0], make_float2(u.x, u.y));
+        acc[i][1] = __fadd2_rn(acc[i][1], make_float2(u.z, u.w));
+        acc[i][2] = __fadd2_rn(acc[i][2], make_float2(v.x, v.y));
+        acc[i][3] = __fadd2_rn(acc[i][3], make_float2(v.z, v.w));
+      }
+    }
+  }
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
     const int row = Y0 + 16 * B + hq + 4 * i;  // band-relative
@@ -290,17 +335,21 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
         if (col0 + k < fp.W) o[k] = v[k];
     }
   }
+  }  // work loop
 }
 
 void init_tile_kernel() {
   cudaFuncSetAttribute(k_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
 }
 
-void launch_tile(const uint32_t* ids, const uint32_t* tile_off, const StarRec* rec, const FrameParams& fp,
-                 float* out, cudaStream_t st) {
+void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, float* out, const WorkItem* items,
+                 const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, cudaStream_t st) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
-  k_tile<<<(unsigned)ntiles, TILE_THREADS, sizeof(TileSmem), st>>>(ids, tile_off, rec, fp, out);
+  const int64_t maxitems = ntiles + part_cap;
+  const int64_t grid = maxitems;  // one CTA per possible item (parts first); CTAs past the item count exit at once
+  k_tile<<<(unsigned)grid, TILE_THREADS, sizeof(TileSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf, done,
+                                                                 hdr);
 }
 
 }  // namespace starsim
