@@ -83,6 +83,16 @@ int starsim_render_band(starsim_ctx* ctx, const float* x, const float* y, const 
                         int32_t width, int32_t height, int32_t row0, int32_t rows,
                         float sigma, int32_t roi, float gain, float* out_band, starsim_stream_t stream);
 
+/* The tiled render with the output stage fused into its epilogue: every pixel
+ * is written once as the gray value q = min(2^bits - 1, floor(v + 1/2)) (v <= 0 -> 0) of the same fp32 sum v that
+ * starsim_render computes, so the result equals starsim_quantize(starsim_render(...)) bit for bit, with a quarter
+ * (u8) or half (u16) of the image traffic and no separate pass.
+ *   out  (device) uint8_t[height*width] if bits == 8, uint16_t[height*width] if bits == 16.
+ * Same arguments and EINVAL cases as starsim_render, plus bits not 8 or 16. */
+int starsim_render_gray(starsim_ctx* ctx, const float* x, const float* y, const float* mag, int64_t n,
+                        int32_t width, int32_t height, float sigma, int32_t roi, float gain, int32_t bits,
+                        void* out, starsim_stream_t stream);
+
 /* The paper's own design, kept as the measured comparison (Fig. 6): zero the image, then one
  * warp per star adds g*mu into every ROI pixel with global fp32 reductions (red.global.add.f32).  Same arguments
  * and EINVAL cases as starsim_render.  The summation order is nondeterministic. */

@@ -4,9 +4,9 @@ The product is ``libstarsim.so`` (C ABI in ``include/starsim.h``; kernels in ``c
 ctypes binding.  :mod:`.dist` renders horizontal bands per GPU and assembles them with an NCCL all-gather.
 """
 from .starsim import (Context, StarsimError, starsim_create, starsim_destroy, starsim_render, starsim_render_band,
-                      starsim_render_atomic, starsim_upload_aos, starsim_quantize, starsim_get_bins, starsim_profile,
-                      starsim_kernel_times, LIB_PATH, KCLASSES)
+                      starsim_render_gray, starsim_render_atomic, starsim_upload_aos, starsim_quantize,
+                      starsim_get_bins, starsim_profile, starsim_kernel_times, LIB_PATH, KCLASSES)
 
 __all__ = ["Context", "StarsimError", "starsim_create", "starsim_destroy", "starsim_render", "starsim_render_band",
-           "starsim_render_atomic", "starsim_upload_aos", "starsim_quantize", "starsim_get_bins", "starsim_profile",
-           "starsim_kernel_times", "LIB_PATH", "KCLASSES"]
+           "starsim_render_gray", "starsim_render_atomic", "starsim_upload_aos", "starsim_quantize", "starsim_get_bins",
+           "starsim_profile", "starsim_kernel_times", "LIB_PATH", "KCLASSES"]

@@ -33,13 +33,13 @@ struct Launch {
 struct GraphKey {
   const void *x, *y, *mag, *out;
   int64_t n;
-  int32_t W, H, row0, rows, R;
+  int32_t W, H, row0, rows, R, obits;
   float sigma, gain;
   cudaStream_t st;
   uint64_t scratch_gen;
   bool operator==(const GraphKey& o) const {
     return x == o.x && y == o.y && mag == o.mag && out == o.out && n == o.n && W == o.W && H == o.H &&
-           row0 == o.row0 && rows == o.rows && R == o.R && sigma == o.sigma && gain == o.gain && st == o.st &&
+           row0 == o.row0 && rows == o.rows && R == o.R && obits == o.obits && sigma == o.sigma && gain == o.gain && st == o.st &&
            scratch_gen == o.scratch_gen;
   }
 };
@@ -189,7 +189,7 @@ int tiles_per_axis(int R, int tile, int ntiles_axis) {
 // Enqueue the tiled render on stream st: memset of the header + tile counters, k_prep, k_scan, k_scatter,
 // k_sortlists, k_tile.
 int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, const FrameParams& fp,
-                  int64_t ntiles, int tps, int part_cap, float* out, cudaStream_t st) {
+                  int64_t ntiles, int tps, int part_cap, void* out, cudaStream_t st) {
   Header* hdr = (Header*)c->zeroed.p;
   uint32_t* cnt = (uint32_t*)(hdr + 1);
   const size_t zbytes = sizeof(Header) + sizeof(uint32_t) * (CNT_STRIDE + 1) * (size_t)ntiles;
@@ -220,17 +220,22 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
 }
 
 int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
-                 int32_t row0, int32_t rows, float sigma, int32_t R, float gain, float* out, cudaStream_t st) {
+                 int32_t row0, int32_t rows, float sigma, int32_t R, float gain, int32_t obits, void* out,
+                 cudaStream_t st) {
   DevGuard g(c->dev);
   FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain);
-  fp.vec = (W % 4 == 0 && ((uintptr_t)out & 15) == 0) ? 1 : 0;
+  fp.obits = obits;
+  // one vector store per 8-pixel run: 32 B (fp32) / 8 B (u8) / 16 B (u16); rows must keep that alignment
+  const int vb = obits == 8 ? 8 : 16;
+  fp.vec = ((W * (obits ? obits / 8 : 4)) % vb == 0 && ((uintptr_t)out % vb) == 0) ? 1 : 0;
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   const int tps = tiles_per_axis(R, TILE_W, fp.ntx) * tiles_per_axis(R, TILE_H, fp.nty);
   const int64_t pmax = n * (int64_t)tps;
   if (pmax >= 0xFFFFFFFFll) return fail(c, STARSIM_EINVAL, "n * tiles-per-star >= 2^32 (pair counts are 32-bit)");
   const size_t zbytes = sizeof(Header) + sizeof(uint32_t) * (CNT_STRIDE + 1) * (size_t)ntiles;
-  // partial-tile buffers for split heavy tiles: at most P / SPLIT_LEN parts exist
-  const int part_cap = (int)std::min<int64_t>(PART_CAP, pmax / SPLIT_LEN + 1);
+  // partial-tile buffers for split heavy tiles (a fixed count, so that the split -- and the summation order -- of a
+  // tile is the same in a band render and in the full frame)
+  const int part_cap = PART_CAP;
   int rc;
   if ((rc = grow(c, c->rec, sizeof(StarRec) * (size_t)(n > 0 ? n : 1), "records"))) return rc;
   if ((rc = grow(c, c->slots, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "tile slots"))) return rc;
@@ -242,7 +247,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   if ((rc = grow(c, c->split_tab, sizeof(uint2) * (size_t)ntiles, "split table"))) return rc;
   if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
 
-  const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, sigma, gain, st, c->scratch_gen};
+  const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, sigma, gain, st, c->scratch_gen};
   if (st == nullptr || c->prof || !c->use_graphs) {
     if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st))) return rc;
   } else {
@@ -345,7 +350,7 @@ int starsim_render(starsim_ctx* c, const float* x, const float* y, const float* 
   if (!c) return STARSIM_EINVAL;
   int rc = validate_frame(c, x, y, mag, n, W, H, sigma, R, gain, out);
   if (rc) return rc;
-  return render_tiled(c, x, y, mag, n, W, H, 0, H, sigma, R, gain, out, (cudaStream_t)stream);
+  return render_tiled(c, x, y, mag, n, W, H, 0, H, sigma, R, gain, 0, out, (cudaStream_t)stream);
 }
 
 int starsim_render_band(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W,
@@ -355,7 +360,17 @@ int starsim_render_band(starsim_ctx* c, const float* x, const float* y, const fl
   int rc = validate_frame(c, x, y, mag, n, W, H, sigma, R, gain, out_band);
   if (rc) return rc;
   if (row0 < 0 || rows < 1 || (int64_t)row0 + rows > H) return fail(c, STARSIM_EINVAL, "band not inside the image");
-  return render_tiled(c, x, y, mag, n, W, H, row0, rows, sigma, R, gain, out_band, (cudaStream_t)stream);
+  return render_tiled(c, x, y, mag, n, W, H, row0, rows, sigma, R, gain, 0, out_band, (cudaStream_t)stream);
+}
+
+int starsim_render_gray(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W,
+                        int32_t H, float sigma, int32_t R, float gain, int32_t bits, void* out,
+                        starsim_stream_t stream) {
+  if (!c) return STARSIM_EINVAL;
+  int rc = validate_frame(c, x, y, mag, n, W, H, sigma, R, gain, out);
+  if (rc) return rc;
+  if (bits != 8 && bits != 16) return fail(c, STARSIM_EINVAL, "bits must be 8 or 16");
+  return render_tiled(c, x, y, mag, n, W, H, 0, H, sigma, R, gain, bits, out, (cudaStream_t)stream);
 }
 
 int starsim_render_atomic(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W,

@@ -69,11 +69,25 @@ struct FrameParams {
   int32_t row0, rows;    // band (row0 = 0, rows = H for a full frame)
   int32_t R;
   int32_t ntx, nty;      // tiles over the band
-  int32_t vec;           // 1 if out rows are 16-B aligned (W % 4 == 0 and out 16-B aligned): float4 stores
+  int32_t vec;           // 1 if every 8-pixel run of an out row is aligned for one vector store
+  int32_t obits;         // 0: fp32 image; 8 / 16: gray values quantised in the epilogue (u8 / u16 image)
   float kexp;            // -log2(e) / (2 sigma^2): exp(-d^2/(2 sigma^2)) = ex2(kexp * d^2)
   float sk;              // sqrt(log2(e) / (2 sigma^2)):  exp(-d^2/(2 sigma^2)) = ex2(-(d * sk)^2)
   double s_scale;        // A / (2 pi sigma^2), applied in fp64 before rounding s' to fp32
 };
+
+// Output stage: q = min(2^bits-1, floor(v + 1/2)), v <= 0 or NaN -> 0.  floor(v + 1/2) is taken
+// exactly as f + (v - f >= 1/2), f = floorf(v) (v - f is exact in fp32 for v >= 0); the rounded v + 0.5f would carry
+// across an integer for v = 0.49999997 (reading R13).
+__device__ __forceinline__ uint32_t quant1(float v, float qmax) {
+  float q = 0.f;
+  if (v > 0.f) {
+    const float f = floorf(v);
+    q = f + ((v - f >= 0.5f) ? 1.f : 0.f);
+    q = fminf(q, qmax);
+  }
+  return (uint32_t)q;
+}
 
 // MUFU.EX2 (2^x, flush-to-zero): the one SFU op per profile value.
 __device__ __forceinline__ float ex2_approx(float x) {

@@ -63,20 +63,8 @@ void launch_atomic(const float* x, const float* y, const float* m, int64_t n, co
 }
 
 // ---------------------------------------------------------------------------------------------------------------
-// k_quantize -- the Output stage: q = min(2^bits-1, floor(v + 1/2)), v <= 0 or NaN -> 0.
-// floor(v + 1/2) is taken exactly as f + (v - f >= 1/2), f = floorf(v) (v - f is exact in fp32 for v >= 0); the
-// rounded v + 0.5f would carry across an integer for v = 0.49999997 (reading R13).  4 pixels per thread.
+// k_quantize -- the Output stage on an fp32 image: quant1 (common.cuh) per pixel, 4 per thread.
 // ---------------------------------------------------------------------------------------------------------------
-__device__ __forceinline__ uint32_t quant1(float v, float qmax) {
-  float q = 0.f;
-  if (v > 0.f) {
-    const float f = floorf(v);
-    q = f + ((v - f >= 0.5f) ? 1.f : 0.f);
-    q = fminf(q, qmax);
-  }
-  return (uint32_t)q;
-}
-
 template <int BITS>
 __global__ void k_quantize(const float* __restrict__ img, int64_t npix, void* __restrict__ out) {
   const float qmax = BITS == 8 ? 255.f : 65535.f;

@@ -57,7 +57,7 @@ constexpr uint32_t ZERO_ENT = ZERO_GX * 32u << 16;  // gy byte offset 0, all-zer
 // ---------------------------------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __restrict__ ids,
                                                           const StarRec* __restrict__ rec, FrameParams fp,
-                                                          float* __restrict__ out, const WorkItem* __restrict__ items,
+                                                          void* __restrict__ out_, const WorkItem* __restrict__ items,
                                                           const uint2* __restrict__ split_tab,
                                                           float* __restrict__ part_buf, uint32_t* __restrict__ done,
                                                           Header* hdr) {
@@ -319,20 +319,60 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
       }
     }
   }
+  if (fp.obits == 0) {
+    float* out = reinterpret_cast<float*>(out_);
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const int row = Y0 + 16 * B + hq + 4 * i;  // band-relative
-    if (row >= fp.rows || col0 >= fp.W) continue;
-    float* o = out + (int64_t)row * fp.W + col0;
-    if (fp.vec && col0 + 8 <= fp.W) {
-      reinterpret_cast<float4*>(o)[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
-      reinterpret_cast<float4*>(o)[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
-    } else {
-      const float v[8] = {acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y,
-                          acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y};
+    for (int i = 0; i < 4; ++i) {
+      const int row = Y0 + 16 * B + hq + 4 * i;  // band-relative
+      if (row >= fp.rows || col0 >= fp.W) continue;
+      float* o = out + (int64_t)row * fp.W + col0;
+      if (fp.vec && col0 + 8 <= fp.W) {
+        reinterpret_cast<float4*>(o)[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
+        reinterpret_cast<float4*>(o)[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
+      } else {
+        const float v[8] = {acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y,
+                            acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y};
 #pragma unroll
-      for (int k = 0; k < 8; ++k)
-        if (col0 + k < fp.W) o[k] = v[k];
+        for (int k = 0; k < 8; ++k)
+          if (col0 + k < fp.W) o[k] = v[k];
+      }
+    }
+  } else {
+    // fused output stage (NEXT-1): the gray value of each pixel, exactly as k_quantize would compute it from the
+    // same fp32 sum, written as u8 / u16
+    const float qmax = fp.obits == 8 ? 255.f : 65535.f;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int row = Y0 + 16 * B + hq + 4 * i;
+      if (row >= fp.rows || col0 >= fp.W) continue;
+      uint32_t g[8];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        g[2 * k] = quant1(acc[i][k].x, qmax);
+        g[2 * k + 1] = quant1(acc[i][k].y, qmax);
+      }
+      const int64_t pix = (int64_t)row * fp.W + col0;
+      if (fp.obits == 8) {
+        uint8_t* o = reinterpret_cast<uint8_t*>(out_) + pix;
+        if (fp.vec && col0 + 8 <= fp.W) {
+          *reinterpret_cast<uint2*>(o) = make_uint2(g[0] | g[1] << 8 | g[2] << 16 | g[3] << 24,
+                                                    g[4] | g[5] << 8 | g[6] << 16 | g[7] << 24);
+        } else {
+#pragma unroll
+          for (int k = 0; k < 8; ++k)
+            if (col0 + k < fp.W) o[k] = (uint8_t)g[k];
+        }
+      } else {
+        uint16_t* o = reinterpret_cast<uint16_t*>(out_) + pix;
+        if (fp.vec && col0 + 8 <= fp.W) {
+          *reinterpret_cast<uint4*>(o) = make_uint4(g[0] | g[1] << 16, g[2] | g[3] << 16, g[4] | g[5] << 16,
+                                                    g[6] | g[7] << 16);
+        } else {
+#pragma unroll
+          for (int k = 0; k < 8; ++k)
+            if (col0 + k < fp.W) o[k] = (uint16_t)g[k];
+        }
+      }
     }
   }
   }  // work loop
@@ -342,7 +382,7 @@ void init_tile_kernel() {
   cudaFuncSetAttribute(k_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
 }
 
-void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, float* out, const WorkItem* items,
+void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, cudaStream_t st) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;

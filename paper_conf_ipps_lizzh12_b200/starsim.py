@@ -53,6 +53,8 @@ def lib():
         L.starsim_render.restype = ctypes.c_int
         L.starsim_render_band.argtypes = [vp, vp, vp, vp, i64, i32, i32, i32, i32, f32, i32, f32, vp, vp]
         L.starsim_render_band.restype = ctypes.c_int
+        L.starsim_render_gray.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, i32, vp, vp]
+        L.starsim_render_gray.restype = ctypes.c_int
         L.starsim_render_atomic.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
         L.starsim_render_atomic.restype = ctypes.c_int
         L.starsim_upload_aos.argtypes = [vp, vp, i64, vp, vp, vp, vp]
@@ -115,6 +117,15 @@ def starsim_render(h, x, y, mag, width, height, sigma, roi, gain, out, stream=No
     _check(h, lib().starsim_render(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
                                    _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
                                    int(roi), float(gain), _ptr(out, torch.float32, "out"), _stream(stream)))
+
+
+def starsim_render_gray(h, x, y, mag, width, height, sigma, roi, gain, bits, out, stream=None) -> None:
+    import torch
+    n = int(x.numel()) if x is not None else 0
+    dt = torch.uint8 if int(bits) == 8 else torch.uint16
+    _check(h, lib().starsim_render_gray(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
+                                        _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
+                                        int(roi), float(gain), int(bits), _ptr(out, dt, "out"), _stream(stream)))
 
 
 def starsim_render_band(h, x, y, mag, width, height, row0, rows, sigma, roi, gain, out_band, stream=None) -> None:
@@ -220,6 +231,13 @@ class Context:
     def render(self, x, y, mag, width, height, sigma, roi, gain, out=None, stream=None):
         out = self._out(height, width, out)
         starsim_render(self.h, x, y, mag, width, height, sigma, roi, gain, out, stream)
+        return out
+
+    def render_gray(self, x, y, mag, width, height, sigma, roi, gain, bits=8, out=None, stream=None):
+        import torch
+        if out is None:
+            out = torch.empty((height, width), dtype=torch.uint8 if bits == 8 else torch.uint16, device=x.device)
+        starsim_render_gray(self.h, x, y, mag, width, height, sigma, roi, gain, bits, out, stream)
         return out
 
     def render_band(self, x, y, mag, width, height, row0, rows, sigma, roi, gain, out=None, stream=None):

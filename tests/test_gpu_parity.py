@@ -205,6 +205,53 @@ def test_quantize_edge_values(torch_dev, ctx):
             assert np.array_equal(got, oracle.quantize(v.astype(np.float64), bits))
 
 
+# ---------------------------------------------------------------- fused gray output (NEXT-1)
+
+@pytest.mark.parametrize("bits", [8, 16])
+@pytest.mark.parametrize("W,H", [(1024, 1024), (1003, 517)])
+def test_render_gray_is_quantize_of_render(torch_dev, ctx, bits, W, H):
+    """starsim_render_gray == starsim_quantize(starsim_render) bit for bit (same fp32 sums, same exact rounding), on
+    vector-aligned and odd widths; and within +-1 LSB of quantising the fp64 oracle."""
+    torch, dev = torch_dev
+    f = synth.uniform_field(6000, W, H, seed=21, mag_lo=0.0, mag_hi=6.0)
+    A = synth.bench_gain(1.5, bits)
+    args = to_dev(torch_dev, f)
+    img = ctx.render(*args, W, H, 1.5, 9, A)
+    q_two_pass = ctx.quantize(img, bits).cpu().numpy()
+    q_fused = ctx.render_gray(*args, W, H, 1.5, 9, A, bits=bits).cpu().numpy()
+    assert q_fused.dtype == (np.uint8 if bits == 8 else np.uint16)
+    assert np.array_equal(q_fused, q_two_pass)
+    ref = oracle.quantize(oracle.render(f.x, f.y, f.mag, W, H, 1.5, 9, A, threads=_threads()), bits)
+    assert np.abs(q_fused.astype(np.int64) - ref.astype(np.int64)).max() <= 1
+
+
+# ---------------------------------------------------------------- heavy tiles (split into parts)
+
+def _dense_field(n, W, H, cx, cy, spread, seed):
+    u = synth.uniform01(seed, 0, 0, 3 * n)
+    x = (cx + (u[:n] - 0.5) * spread).astype(np.float32)
+    y = (cy + (u[n:2 * n] - 0.5) * spread).astype(np.float32)
+    m = (u[2 * n:] * 3.0).astype(np.float32)
+    return synth.Field(x, y, m)
+
+
+def test_heavy_tile_split_parity_and_bands(torch_dev, ctx):
+    """A tile with far more than SPLIT_LEN (1024) stars is rendered as several parts reduced in fixed order: parity
+    against the oracle, run-to-run determinism, and bitwise equality of tile-aligned bands with the frame."""
+    torch, dev = torch_dev
+    W, H, R, sigma = 512, 384, 15, 2.5
+    f = _dense_field(9000, W, H, 200.0, 150.0, 40.0, seed=31)
+    args = to_dev(torch_dev, f)
+    a = ctx.render(*args, W, H, sigma, R, 1.0)
+    tw, th, off, ids = ctx.get_bins()
+    assert int(np.diff(off).max()) > 4 * 1024  # some tile is split into >= 5 parts
+    ref = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads())
+    assert_parity(a.cpu().numpy(), ref, "heavy tile")
+    assert torch.equal(a, ctx.render(*args, W, H, sigma, R, 1.0))
+    bands = [ctx.render_band(*args, W, H, g * 64, 64, sigma, R, 1.0) for g in range(H // 64)]
+    assert torch.equal(torch.cat(bands, 0), a)
+
+
 # ---------------------------------------------------------------- boundary contract (T1)
 
 def test_einval_leaves_out_untouched(torch_dev, ctx):
