@@ -3,7 +3,7 @@
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config T] [--method tiled|atomic]
 
-A step is one frame: the whole hot path (per-star prep + binning + radix sort + CSR + tile accumulation) over one
+A step is one frame: the whole hot path (per-star prep + binning + per-tile sort + CSR + tile accumulation) over one
 synthetic catalogue resident in HBM, written to a device-resident fp32 image.  N=1 renders the north-star frame T
 (4096x4096, 1M uniform stars, R=15, sigma=2.5).  Under torchrun (N>1) the job is weak-scaled: the frame is
 4096 wide and 4096*N tall with N*1M stars, every rank renders its own 4096-row band and the
@@ -324,6 +324,32 @@ def run_ours(args, world, rank, local_rank):
     kernels = {k: {"ms_per_step": v[0] / args.steps, "launches_per_step": v[1] / args.steps} for k, v in kt.items()
                if v[1]}
 
+    # NEXT-1 variant (1 GPU, tiled): the same frame with the output stage fused -- u8 gray image written by k_tile
+    variants = {}
+    if world == 1 and args.method == "tiled":
+        gray = torch.empty((H, W), dtype=torch.uint8, device=dev)
+        Ag = synth.bench_gain(sigma, 8)
+
+        def gstep():
+            with torch.cuda.stream(stream):
+                ctx.render_gray(x, y, m, W, H, sigma, R, Ag, bits=8, out=gray, stream=stream)
+
+        for _ in range(max(3, args.warmup)):
+            gstep()
+        barrier()
+        g_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                for _ in range(args.steps)]
+        for i in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.fill_(float(i))
+                g_ev[i][0].record(stream)
+            gstep()
+            g_ev[i][1].record(stream)
+        barrier()
+        g_ms = sum(a.elapsed_time(b) for a, b in g_ev) / args.steps
+        variants["gray_u8"] = {"ms_per_step": g_ms, "frames_per_s": 1e3 / g_ms, "updates_per_s": U_frame / (g_ms * 1e-3),
+                               "note": "starsim_render_gray (output stage fused into k_tile, u8 image)"}
+
     # e2e: the same C-ABI call with host (pinned) catalogue in and image out, copies inside the timed region
     e2e = None
     if not args.no_e2e:
@@ -379,7 +405,7 @@ def run_ours(args, world, rank, local_rank):
             "clocks": clocks, "gpu_launches": int(round(launches * args.steps)),
             "gpu_launches_per_step": launches, "kernels": kernels,
             "ms_per_step_direct_launch": sum(ms_prof_steps) / len(ms_prof_steps),
-            "roofline": roofline, "e2e": e2e,
+            "roofline": roofline, "e2e": e2e, "variants": variants,
             "cpu_baseline": cpu}
     print(json.dumps(line), flush=True)
     ctx.close()

@@ -216,16 +216,23 @@ __device__ void sort_pass(const uint32_t* in, int len, int shift, uint32_t* out,
     __syncwarp();
   }
   __syncthreads();
-  // per digit: warp offsets inside the digit run, digit totals; then the exclusive scan over digits
-  uint32_t tot = 0;
-  if (tid < SORT_RADIX) {
+  // per digit: warp offsets inside the digit run, digit totals; then the exclusive scan over digits (DPT contiguous
+  // digits per thread)
+  constexpr int DPT = SORT_RADIX / SORT_THREADS;
+  uint32_t dtot[DPT], tot = 0;
+#pragma unroll
+  for (int k = 0; k < DPT; ++k) {
+    const int d = tid * DPT + k;
+    uint32_t run = 0;
 #pragma unroll
     for (int w = 0; w < NW; ++w) {
-      const uint32_t t = sm.wcnt[w][tid];
-      sm.wcnt[w][tid] = tot;
-      tot += t;
+      const uint32_t t = sm.wcnt[w][d];
+      sm.wcnt[w][d] = run;
+      run += t;
     }
-    if (dcount) dcount[tid] = tot;
+    if (dcount) dcount[d] = run;
+    dtot[k] = run;
+    tot += run;
   }
   uint32_t incl = tot;
 #pragma unroll
@@ -235,10 +242,15 @@ __device__ void sort_pass(const uint32_t* in, int len, int shift, uint32_t* out,
   }
   if (lane == 31) sm.wsum[warp] = incl;
   __syncthreads();
-  if (tid < SORT_RADIX) {
-    uint32_t pre = 0;
+  {
+    uint32_t pre = incl - tot;
     for (int w = 0; w < warp; ++w) pre += sm.wsum[w];
-    sm.dstart[tid] = pre + incl - tot + (gbase ? gbase[tid] : 0u);
+#pragma unroll
+    for (int k = 0; k < DPT; ++k) {
+      const int d = tid * DPT + k;
+      sm.dstart[d] = pre + (gbase ? gbase[d] : 0u);
+      pre += dtot[k];
+    }
   }
   __syncthreads();
 #pragma unroll

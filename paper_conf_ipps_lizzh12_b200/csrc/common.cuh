@@ -28,9 +28,9 @@ constexpr int GX_PAIRS = 768;                    // (star, strip) pairs per chun
 constexpr int CNT_STRIDE = 32;
 constexpr int PREP_THREADS = 256;
 // k_sortlists: one tile list per CTA; lists of up to SORT_CAP ids stay in shared memory
-constexpr int SORT_THREADS = 256;
-constexpr int SORT_CAP = 4096;
-constexpr int SORT_CHUNKS = SORT_CAP / SORT_THREADS;  // 32-item chunks per warp: SORT_CAP / 8 warps / 32 lanes
+constexpr int SORT_THREADS = 128;
+constexpr int SORT_CAP = 2048;
+constexpr int SORT_CHUNKS = SORT_CAP / SORT_THREADS;  // 32-item chunks per warp: SORT_CAP / (SORT_THREADS/32) / 32
 constexpr int SORT_BITS = 8;
 constexpr int SORT_RADIX = 1 << SORT_BITS;
 constexpr int SORT_NB = 1024;                    // buckets of the range bucket sort
@@ -38,10 +38,9 @@ constexpr int SORT_NB = 1024;                    // buckets of the range bucket 
 // Per-render header in device scratch, zeroed (with the tile counters) by one cudaMemsetAsync per render.
 struct Header {
   uint32_t P;                          // number of (tile, star) pairs
-  uint32_t next;                       // k_tile work queue: next item
-  uint32_t nitems;                     // k_tile work items (written by k_plan)
+  uint32_t nitems;                     // k_tile work items (written by k_scan)
   uint32_t nsplit;                     // tiles split into several items
-  uint32_t pad[28];
+  uint32_t pad[29];
 };
 
 // k_tile work item: stars [jb, je) of tile `tile`'s list; aux = ITEM_WHOLE, or (split index << 12 | part index) for
@@ -52,7 +51,6 @@ struct WorkItem {
 constexpr uint32_t ITEM_WHOLE = 0xFFFFFFFFu;
 constexpr int SPLIT_LEN = 1024;        // a tile list longer than this is split into parts of <= SPLIT_LEN stars
 constexpr int PART_CAP = 512;          // partial-tile buffers (128 x 64 fp32 each, 16 MB) available per render
-constexpr int TILE_CTAS_PER_SM = 3;    // persistent k_tile CTAs per SM
 
 // Star record written by k_prep, read by k_scatter and k_tile: {x, y, s', lo_x | lo_y << 16}.
 // s' = A * 2.512^-m / (2 pi sigma^2), evaluated in fp64 and rounded once to fp32.
