@@ -83,13 +83,18 @@ __global__ void __launch_bounds__(1024) k_scan(const uint32_t* __restrict__ cnt,
                                                uint32_t* __restrict__ tile_off, Header* hdr,
                                                WorkItem* __restrict__ items, uint2* __restrict__ split_tab,
                                                int part_cap) {
-  __shared__ uint3 s_w[32];
+  __shared__ uint3 s_w[33];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t per = (ntiles + 1023) / 1024;
   const int64_t a = min((int64_t)tid * per, ntiles), b = min(a + per, ntiles);
+  // the counts of this thread's tiles: loaded together (each sits on its own L2 line), kept for the second loop
+  constexpr int KEEP = 8;
+  uint32_t keep[KEEP];
+#pragma unroll
+  for (int k = 0; k < KEEP; ++k) keep[k] = a + k < b ? __ldcg(&cnt[(a + k) * CNT_STRIDE]) : 0u;
   uint3 sum = make_uint3(0, 0, 0);  // pairs, parts, split tiles
   for (int64_t t = a; t < b; ++t) {
-    const uint32_t c = cnt[t * CNT_STRIDE], np = parts_of(c);
+    const uint32_t c = t - a < KEEP ? keep[t - a] : __ldcg(&cnt[t * CNT_STRIDE]), np = parts_of(c);
     sum.x += c;
     sum.y += np;
     sum.z += np ? 1u : 0u;
@@ -107,18 +112,24 @@ __global__ void __launch_bounds__(1024) k_scan(const uint32_t* __restrict__ cnt,
   }
   if (lane == 31) s_w[warp] = incl;
   __syncthreads();
-  uint3 pre = make_uint3(incl.x - sum.x, incl.y - sum.y, incl.z - sum.z), tot = make_uint3(0, 0, 0);
-  for (int w = 0; w < 32; ++w) {
-    const uint3 v = s_w[w];
-    if (w < warp) {
-      pre.x += v.x;
-      pre.y += v.y;
-      pre.z += v.z;
+  if (warp == 0) {  // exclusive scan of the 32 warp sums; the total goes to s_w[32]
+    uint3 v = s_w[lane], w = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t vx = __shfl_up_sync(0xffffffffu, w.x, o), vy = __shfl_up_sync(0xffffffffu, w.y, o),
+                     vz = __shfl_up_sync(0xffffffffu, w.z, o);
+      if (lane >= o) {
+        w.x += vx;
+        w.y += vy;
+        w.z += vz;
+      }
     }
-    tot.x += v.x;
-    tot.y += v.y;
-    tot.z += v.z;
+    s_w[lane] = make_uint3(w.x - v.x, w.y - v.y, w.z - v.z);
+    if (lane == 31) s_w[32] = w;
   }
+  __syncthreads();
+  const uint3 wp = s_w[warp], tot = s_w[32];
+  const uint3 pre = make_uint3(wp.x + incl.x - sum.x, wp.y + incl.y - sum.y, wp.z + incl.z - sum.z);
   const bool split_on = tot.y <= (uint32_t)part_cap;
   const uint32_t nparts = split_on ? tot.y : 0u, nsplit = split_on ? tot.z : 0u;
   if (tid == 0) {
@@ -129,7 +140,7 @@ __global__ void __launch_bounds__(1024) k_scan(const uint32_t* __restrict__ cnt,
   }
   uint32_t run = pre.x, pb = pre.y, si = pre.z;
   for (int64_t t = a; t < b; ++t) {
-    const uint32_t c = cnt[t * CNT_STRIDE];
+    const uint32_t c = t - a < KEEP ? keep[t - a] : __ldcg(&cnt[t * CNT_STRIDE]);
     tile_off[t] = run;
     const uint32_t np = split_on ? parts_of(c) : 0u;
     if (np) {
