@@ -48,7 +48,7 @@ struct starsim_ctx {
   int dev = 0;
   int num_sms = 148;
   std::string err;
-  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, zeroed, stage;
+  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
@@ -205,7 +205,8 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
     if ((rc = check_launch(c, "k_prep"))) return rc;
   }
   timed(c, 2, st, [&] {
-    launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap, st);
+    launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap, c->partial.p,
+                st);
     launch_scatter(rec, n, fp, slots, tps, tile_off, ids, st);
   });
   if ((rc = check_launch(c, "k_scan/k_scatter"))) return rc;
@@ -245,6 +246,8 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   if ((rc = grow(c, c->zeroed, zbytes, "header+counters"))) return rc;
   if ((rc = grow(c, c->items, sizeof(WorkItem) * (size_t)(ntiles + part_cap), "work items"))) return rc;
   if ((rc = grow(c, c->split_tab, sizeof(uint2) * (size_t)ntiles, "split table"))) return rc;
+  if ((rc = grow(c, c->partial, sizeof(uint3) * (size_t)((ntiles + SCAN_TILES - 1) / SCAN_TILES), "scan partials")))
+    return rc;
   if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
 
   const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, sigma, gain, st, c->scratch_gen};
@@ -331,7 +334,7 @@ void starsim_destroy(starsim_ctx* c) {
     cudaDeviceSynchronize();
     if (c->have_graph) cudaGraphExecDestroy(c->gexec);
     Buf* bufs[] = {&c->rec, &c->slots, &c->ids, &c->tmp, &c->tile_off, &c->items, &c->split_tab, &c->parts,
-                   &c->zeroed, &c->stage};
+                   &c->partial, &c->zeroed, &c->stage};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {

@@ -2,8 +2,8 @@
 //   k_prep       a1: per star -- validity, s' in fp64, exact ROI origin, clip to the frame columns and band rows; the
 //                tiles its clipped ROI overlaps (row-major), and for each one a slot in that tile's list from an
 //                atomic counter (one ATOMG per (tile, star) pair).  Writes the 16-B star record.
-//   k_scan       a2: exclusive scan of the per-tile counts -> tile_off[ntiles+1] (one CTA), P; then k_tile's work
-//                list (heavy tiles split into parts).
+//   k_scan_a/b   a2: exclusive scan of the per-tile counts -> tile_off[ntiles+1], P; and k_tile's work list
+//                (heavy tiles split into parts).
 //   k_scatter    a3: ids[tile_off[tile] + slot] = star for every pair.
 //   k_sortlists  a4: sort every tile's list ascending (LSD radix on the star index in shared memory, 8-bit digits,
 //                stable warp-ballot ranking); lists longer than SORT_CAP are sorted in SORT_CAP chunks through a
@@ -79,83 +79,111 @@ __device__ __forceinline__ uint32_t parts_of(uint32_t len) {
   return min((len + SPLIT_LEN - 1) / SPLIT_LEN, 4095u);
 }
 
-__global__ void __launch_bounds__(1024) k_scan(const uint32_t* __restrict__ cnt, int64_t ntiles,
-                                               uint32_t* __restrict__ tile_off, Header* hdr,
-                                               WorkItem* __restrict__ items, uint2* __restrict__ split_tab,
-                                               int part_cap) {
-  __shared__ uint3 s_w[33];
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int64_t per = (ntiles + 1023) / 1024;
-  const int64_t a = min((int64_t)tid * per, ntiles), b = min(a + per, ntiles);
-  // the counts of this thread's tiles: loaded together (each sits on its own L2 line), kept for the second loop
-  constexpr int KEEP = 8;
-  uint32_t keep[KEEP];
-#pragma unroll
-  for (int k = 0; k < KEEP; ++k) keep[k] = a + k < b ? __ldcg(&cnt[(a + k) * CNT_STRIDE]) : 0u;
-  uint3 sum = make_uint3(0, 0, 0);  // pairs, parts, split tiles
-  for (int64_t t = a; t < b; ++t) {
-    const uint32_t c = t - a < KEEP ? keep[t - a] : __ldcg(&cnt[t * CNT_STRIDE]), np = parts_of(c);
-    sum.x += c;
-    sum.y += np;
-    sum.z += np ? 1u : 0u;
-  }
-  uint3 incl = sum;
+// Two kernels, SCAN_TILES tiles per CTA (SCAN_PER per thread): k_scan_a writes each CTA's sums (pairs, parts, split
+// tiles); k_scan_b re-reduces the sums of the CTAs before it and of all CTAs (a few hundred at most), scans its own
+// tiles and writes tile_off and the work items.
+__device__ __forceinline__ uint3 add3(uint3 a, uint3 b) { return make_uint3(a.x + b.x, a.y + b.y, a.z + b.z); }
+
+__device__ __forceinline__ uint3 warp_incl_scan3(uint3 v, int lane) {
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t vx = __shfl_up_sync(0xffffffffu, incl.x, o), vy = __shfl_up_sync(0xffffffffu, incl.y, o),
-                   vz = __shfl_up_sync(0xffffffffu, incl.z, o);
-    if (lane >= o) {
-      incl.x += vx;
-      incl.y += vy;
-      incl.z += vz;
-    }
+    const uint32_t x = __shfl_up_sync(0xffffffffu, v.x, o), y = __shfl_up_sync(0xffffffffu, v.y, o),
+                   z = __shfl_up_sync(0xffffffffu, v.z, o);
+    if (lane >= o) v = add3(v, make_uint3(x, y, z));
   }
+  return v;
+}
+
+// block-wide exclusive scan of uint3 (SCAN_THREADS threads); *total receives the block sum
+__device__ __forceinline__ uint3 block_excl_scan3(uint3 v, uint3* s_w, uint3* total) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint3 incl = warp_incl_scan3(v, lane);
   if (lane == 31) s_w[warp] = incl;
   __syncthreads();
-  if (warp == 0) {  // exclusive scan of the 32 warp sums; the total goes to s_w[32]
-    uint3 v = s_w[lane], w = v;
+  uint3 pre = make_uint3(0, 0, 0), tot = make_uint3(0, 0, 0);
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t vx = __shfl_up_sync(0xffffffffu, w.x, o), vy = __shfl_up_sync(0xffffffffu, w.y, o),
-                     vz = __shfl_up_sync(0xffffffffu, w.z, o);
-      if (lane >= o) {
-        w.x += vx;
-        w.y += vy;
-        w.z += vz;
-      }
-    }
-    s_w[lane] = make_uint3(w.x - v.x, w.y - v.y, w.z - v.z);
-    if (lane == 31) s_w[32] = w;
+  for (int w = 0; w < SCAN_THREADS / 32; ++w) {
+    const uint3 u = s_w[w];
+    if (w < warp) pre = add3(pre, u);
+    tot = add3(tot, u);
   }
   __syncthreads();
-  const uint3 wp = s_w[warp], tot = s_w[32];
-  const uint3 pre = make_uint3(wp.x + incl.x - sum.x, wp.y + incl.y - sum.y, wp.z + incl.z - sum.z);
-  const bool split_on = tot.y <= (uint32_t)part_cap;
-  const uint32_t nparts = split_on ? tot.y : 0u, nsplit = split_on ? tot.z : 0u;
-  if (tid == 0) {
-    hdr->P = tot.x;
-    tile_off[ntiles] = tot.x;
+  *total = tot;
+  return make_uint3(pre.x + incl.x - v.x, pre.y + incl.y - v.y, pre.z + incl.z - v.z);
+}
+
+__device__ __forceinline__ void load_counts(const uint32_t* cnt, int64_t ntiles, int64_t t0, uint32_t* c, uint3& sum) {
+  sum = make_uint3(0, 0, 0);
+#pragma unroll
+  for (int k = 0; k < SCAN_PER; ++k) c[k] = t0 + k < ntiles ? __ldcg(&cnt[(t0 + k) * CNT_STRIDE]) : 0u;
+#pragma unroll
+  for (int k = 0; k < SCAN_PER; ++k) {
+    const uint32_t np = parts_of(c[k]);
+    sum = add3(sum, make_uint3(c[k], np, np ? 1u : 0u));
+  }
+}
+
+__global__ void __launch_bounds__(SCAN_THREADS) k_scan_a(const uint32_t* __restrict__ cnt, int64_t ntiles,
+                                                         uint3* __restrict__ partial) {
+  __shared__ uint3 s_w[SCAN_THREADS / 32];
+  const int64_t t0 = (int64_t)blockIdx.x * SCAN_TILES + (int64_t)threadIdx.x * SCAN_PER;
+  uint32_t c[SCAN_PER];
+  uint3 sum, tot;
+  load_counts(cnt, ntiles, t0, c, sum);
+  block_excl_scan3(sum, s_w, &tot);
+  if (threadIdx.x == 0) partial[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(SCAN_THREADS) k_scan_b(const uint32_t* __restrict__ cnt, int64_t ntiles,
+                                                         const uint3* __restrict__ partial, int nblk,
+                                                         uint32_t* __restrict__ tile_off, Header* hdr,
+                                                         WorkItem* __restrict__ items,
+                                                         uint2* __restrict__ split_tab, int part_cap) {
+  __shared__ uint3 s_w[SCAN_THREADS / 32];
+  const int tid = threadIdx.x;
+  // sums of the CTAs before this one, and of all CTAs
+  uint3 before = make_uint3(0, 0, 0), all = make_uint3(0, 0, 0);
+  for (int k = tid; k < nblk; k += SCAN_THREADS) {
+    const uint3 u = partial[k];
+    if (k < (int)blockIdx.x) before = add3(before, u);
+    all = add3(all, u);
+  }
+  uint3 tb, ta;
+  block_excl_scan3(before, s_w, &tb);
+  block_excl_scan3(all, s_w, &ta);
+  const bool split_on = ta.y <= (uint32_t)part_cap;
+  const uint32_t nparts = split_on ? ta.y : 0u, nsplit = split_on ? ta.z : 0u;
+  if (blockIdx.x == 0 && tid == 0) {
+    hdr->P = ta.x;
+    tile_off[ntiles] = ta.x;
     hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
     hdr->nsplit = nsplit;
   }
-  uint32_t run = pre.x, pb = pre.y, si = pre.z;
-  for (int64_t t = a; t < b; ++t) {
-    const uint32_t c = t - a < KEEP ? keep[t - a] : __ldcg(&cnt[t * CNT_STRIDE]);
+  const int64_t t0 = (int64_t)blockIdx.x * SCAN_TILES + (int64_t)tid * SCAN_PER;
+  uint32_t c[SCAN_PER];
+  uint3 sum, tot;
+  load_counts(cnt, ntiles, t0, c, sum);
+  const uint3 ex = add3(tb, block_excl_scan3(sum, s_w, &tot));
+  uint32_t run = ex.x, pb = ex.y, si = ex.z;
+#pragma unroll
+  for (int k = 0; k < SCAN_PER; ++k) {
+    const int64_t t = t0 + k;
+    if (t >= ntiles) break;
     tile_off[t] = run;
-    const uint32_t np = split_on ? parts_of(c) : 0u;
+    const uint32_t np = split_on ? parts_of(c[k]) : 0u;
     if (np) {
       split_tab[si] = make_uint2(pb, np);
-      const uint32_t per_part = (c + np - 1) / np;
-      for (uint32_t k = 0; k < np; ++k)
-        items[pb + k] = WorkItem{(uint32_t)t, run + k * per_part, min(run + c, run + (k + 1) * per_part),
-                                 (si << 12) | k};
+      const uint32_t per_part = (c[k] + np - 1) / np;
+      for (uint32_t j = 0; j < np; ++j)
+        items[pb + j] = WorkItem{(uint32_t)t, run + j * per_part, min(run + c[k], run + (j + 1) * per_part),
+                                 (si << 12) | j};
       pb += np;
       ++si;
     } else {
       // whole tiles follow the parts, in tile order: index = nparts + (tiles before t that are not split)
-      items[nparts + (uint32_t)t - (split_on ? si : 0u)] = WorkItem{(uint32_t)t, run, run + c, ITEM_WHOLE};
+      items[nparts + (uint32_t)t - (split_on ? si : 0u)] = WorkItem{(uint32_t)t, run, run + c[k], ITEM_WHOLE};
     }
-    run += c;
+    run += c[k];
   }
 }
 
@@ -441,8 +469,11 @@ void launch_prep(const float* x, const float* y, const float* m, int64_t n, cons
 }
 
 void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items,
-                 uint2* split_tab, int part_cap, cudaStream_t st) {
-  k_scan<<<1, 1024, 0, st>>>(cnt, ntiles, tile_off, hdr, items, split_tab, part_cap);
+                 uint2* split_tab, int part_cap, void* partial, cudaStream_t st) {
+  const int nblk = (int)((ntiles + SCAN_TILES - 1) / SCAN_TILES);
+  k_scan_a<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (uint3*)partial);
+  k_scan_b<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (const uint3*)partial, nblk, tile_off, hdr, items, split_tab,
+                                         part_cap);
 }
 
 void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* slots, int tps,

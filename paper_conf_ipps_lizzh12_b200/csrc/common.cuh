@@ -27,6 +27,10 @@ constexpr int GX_PAIRS = 768;                    // (star, strip) pairs per chun
 // atomics of different tiles never serialise on one L2 line)
 constexpr int CNT_STRIDE = 32;
 constexpr int PREP_THREADS = 256;
+// k_scan_a / k_scan_b: SCAN_PER tiles per thread
+constexpr int SCAN_THREADS = 256;
+constexpr int SCAN_PER = 4;
+constexpr int SCAN_TILES = SCAN_THREADS * SCAN_PER;
 // k_sortlists: one tile list per CTA; lists of up to SORT_CAP ids stay in shared memory
 constexpr int SORT_THREADS = 128;
 constexpr int SORT_CAP = 2048;

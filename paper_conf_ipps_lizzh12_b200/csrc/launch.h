@@ -12,7 +12,7 @@ void init_tile_kernel();
 void launch_prep(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
                  uint32_t* cnt, uint32_t* slots, int tps, cudaStream_t st);
 void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items,
-                 uint2* split_tab, int part_cap, cudaStream_t st);
+                 uint2* split_tab, int part_cap, void* partial, cudaStream_t st);
 void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* slots, int tps,
                     const uint32_t* tile_off, uint32_t* ids, cudaStream_t st);
 void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, int64_t ntiles, int64_t n,
