@@ -201,51 +201,62 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
       S.len[tid] = n;
     }
     __syncthreads();
-    // profiles: thread = 4 values of one slot.  Band slot (row profile s' gy): rows 16 b + h4 + 4 i, i = 0..3;
-    // strip slot (column profile gx): columns 8 k + 4 half + i.  d = (pixel - centre) is exact before the scaling;
-    // values outside the ROI are 0.  FADD2/FMUL2 pairs, one MUFU.EX2 per value.
+    // profiles: thread = 8 values.  Band slot (row profile s' gy, [hq][i] = row 16 b + hq + 4 i): one thread per half
+    // slot (hq = 2h, 2h+1); strip slot (column profile gx, columns 8 k .. 8 k + 7, halves swizzled): one thread per
+    // slot.  d = (pixel - centre) is exact before the scaling; values outside the ROI are 0 (unsigned range test).
+    // FADD2/FMUL2 pairs, one MUFU.EX2 per value.
     {
-      const int ngq = S.ngy * 4;
-      for (int gq = tid; gq < ngq; gq += TILE_THREADS) {
-        const int k = gq >> 2, h4 = gq & 3;
+      const float2 sk2 = make_float2(sk, sk);
+      const int ngh = S.ngy * 2;
+      for (int g = tid; g < ngh; g += TILE_THREADS) {
+        const int k = g >> 1, hh = g & 1;
         const uint32_t own = S.gyown[k];
         const float4 pp = S.py[own & 0xFFu];
-        const int rel = 16 * (int)(own >> 8) + h4;                 // first row of this quad (tile-relative)
-        const int lo = (__float_as_int(pp.z) & 0xFF) - rel, hi = (__float_as_int(pp.z) >> 8) - rel;
-        const float b0f = (float)rel - pp.x;                       // exact
-        const float2 sk2 = make_float2(sk, sk);
-        float2 d01 = __fmul2_rn(__fadd2_rn(make_float2(b0f, b0f), make_float2(0.f, 4.f)), sk2);
-        float2 d23 = __fmul2_rn(__fadd2_rn(make_float2(b0f, b0f), make_float2(8.f, 12.f)), sk2);
-        d01 = __fmul2_rn(d01, make_float2(-d01.x, -d01.y));
-        d23 = __fmul2_rn(d23, make_float2(-d23.x, -d23.y));
-        float2 e01 = make_float2(ex2_approx(d01.x), ex2_approx(d01.y));
-        float2 e23 = make_float2(ex2_approx(d23.x), ex2_approx(d23.y));
-        e01 = __fmul2_rn(e01, make_float2(pp.y, pp.y));
-        e23 = __fmul2_rn(e23, make_float2(pp.y, pp.y));
-        const float4 v = make_float4(lo <= 0 && 0 <= hi ? e01.x : 0.f, lo <= 4 && 4 <= hi ? e01.y : 0.f,
-                                     lo <= 8 && 8 <= hi ? e23.x : 0.f, lo <= 12 && 12 <= hi ? e23.y : 0.f);
-        *reinterpret_cast<float4*>(&S.gy[k * 16 + h4 * 4]) = v;
+        const int rel = 16 * (int)(own >> 8) + 2 * hh;            // first row of this half slot (tile-relative)
+        const int prr = __float_as_int(pp.z);
+        const uint32_t u0 = (uint32_t)(rel - (prr & 0xFF)), span = (uint32_t)((prr >> 8) - (prr & 0xFF));
+        const float bf = (float)rel - pp.x;                         // exact
+        const float2 b2 = make_float2(bf, bf), s2 = make_float2(pp.y, pp.y);
+        float2 d[4] = {__fadd2_rn(b2, make_float2(0.f, 4.f)), __fadd2_rn(b2, make_float2(8.f, 12.f)),
+                       __fadd2_rn(b2, make_float2(1.f, 5.f)), __fadd2_rn(b2, make_float2(9.f, 13.f))};
+        float v[8];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          d[j] = __fmul2_rn(d[j], sk2);
+          d[j] = __fmul2_rn(d[j], make_float2(-d[j].x, -d[j].y));
+          const float2 e = __fmul2_rn(make_float2(ex2_approx(d[j].x), ex2_approx(d[j].y)), s2);
+          const int o0 = (j & 1) * 8 + (j >> 1), o1 = o0 + 4;       // row offsets of the pair
+          v[2 * j] = u0 + (uint32_t)o0 <= span ? e.x : 0.f;
+          v[2 * j + 1] = u0 + (uint32_t)o1 <= span ? e.y : 0.f;
+        }
+        // v = rows +0,+4,+8,+12 (quad hq=2hh) and +1,+5,+9,+13 (quad 2hh+1), [hq][i] order
+        float4* dst = reinterpret_cast<float4*>(&S.gy[k * 16 + hh * 8]);
+        dst[0] = make_float4(v[0], v[1], v[2], v[3]);
+        dst[1] = make_float4(v[4], v[5], v[6], v[7]);
       }
-      const int nxq = S.ngx * 2;
-      for (int gq = tid; gq < nxq; gq += TILE_THREADS) {
-        const uint32_t own = S.gxown[gq >> 1];
-        const int half = gq & 1;
+      const int nx = S.ngx;
+      for (int g = tid; g < nx; g += TILE_THREADS) {
+        const uint32_t own = S.gxown[g];
         const uint32_t slot = own & 0xFFFFu;
         const int k = (int)(slot & 15u);
         const float2 pp = S.px[own >> 16];
-        const int rel = 8 * k + 4 * half;
-        const int lo = (__float_as_int(pp.y) & 0xFF) - rel, hi = (__float_as_int(pp.y) >> 8) - rel;
-        const float b0f = (float)rel - pp.x;
-        const float2 sk2 = make_float2(sk, sk);
-        float2 d01 = __fmul2_rn(__fadd2_rn(make_float2(b0f, b0f), make_float2(0.f, 1.f)), sk2);
-        float2 d23 = __fmul2_rn(__fadd2_rn(make_float2(b0f, b0f), make_float2(2.f, 3.f)), sk2);
-        d01 = __fmul2_rn(d01, make_float2(-d01.x, -d01.y));
-        d23 = __fmul2_rn(d23, make_float2(-d23.x, -d23.y));
-        const float4 v = make_float4(lo <= 0 && 0 <= hi ? ex2_approx(d01.x) : 0.f,
-                                     lo <= 1 && 1 <= hi ? ex2_approx(d01.y) : 0.f,
-                                     lo <= 2 && 2 <= hi ? ex2_approx(d23.x) : 0.f,
-                                     lo <= 3 && 3 <= hi ? ex2_approx(d23.y) : 0.f);
-        *reinterpret_cast<float4*>(&S.gx[slot * 8 + ((half ^ ((k >> 2) & 1)) * 4)]) = v;
+        const int rel = 8 * k;
+        const int pcc = __float_as_int(pp.y);
+        const uint32_t u0 = (uint32_t)(rel - (pcc & 0xFF)), span = (uint32_t)((pcc >> 8) - (pcc & 0xFF));
+        const float bf = (float)rel - pp.x;
+        const float2 b2 = make_float2(bf, bf);
+        float v[8];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          float2 dd = __fmul2_rn(__fadd2_rn(b2, make_float2((float)(2 * j), (float)(2 * j + 1))), sk2);
+          dd = __fmul2_rn(dd, make_float2(-dd.x, -dd.y));
+          v[2 * j] = u0 + (uint32_t)(2 * j) <= span ? ex2_approx(dd.x) : 0.f;
+          v[2 * j + 1] = u0 + (uint32_t)(2 * j + 1) <= span ? ex2_approx(dd.y) : 0.f;
+        }
+        float* gs = &S.gx[slot * 8];
+        const int sw = ((k >> 2) & 1) * 4;
+        *reinterpret_cast<float4*>(gs + sw) = make_float4(v[0], v[1], v[2], v[3]);
+        *reinterpret_cast<float4*>(gs + (sw ^ 4)) = make_float4(v[4], v[5], v[6], v[7]);
       }
       // pad every list with all-zero entries up to the longest list of its warp
       if (tid < NBANDS * NSTRIPS) {
