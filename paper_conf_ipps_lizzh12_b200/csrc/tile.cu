@@ -38,7 +38,6 @@ struct TileSmem {
   uint32_t sb[TILE_WARPS][NSTRIPS];      // per-warp ballots: stars overlapping strip Q
   uint32_t lpre[NBANDS * NSTRIPS][TILE_WARPS];  // per (B,Q): entries of the warps before
   uint32_t rpre[NSTRIPS][TILE_WARPS];           // per Q: strip slots of the warps before
-  uint32_t len[NBANDS * NSTRIPS];
   uint32_t wsum[TILE_WARPS];
   float4 py[CHUNK];                      // per star: (y - IY0, s', r0 | r1 << 8, -)
   float2 px[CHUNK];                      // per star: (x - X0, c0 | c1 << 8)
@@ -154,8 +153,13 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
         run += __popc(S.sb[w][pq]);
       }
     }
-    uint32_t excl = incl - pk;
-    for (int w = 0; w < warp; ++w) excl += S.wsum[w];
+    uint32_t excl = incl - pk, ptot = 0;
+#pragma unroll
+    for (int w = 0; w < TILE_WARPS; ++w) {
+      const uint32_t u = S.wsum[w];
+      if (w < warp) excl += u;
+      ptot += u;
+    }
     const uint32_t gyb = excl & 0xFFFFu, gxb = excl >> 16;
     __syncthreads();
     // slots, list entries and the capacity check in one pass: a star whose slot or list position would overflow
@@ -185,29 +189,24 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
     }
     __syncthreads();
     const int ns = min(S.ns, nvalid);
-    if (tid == ns - 1) {
-      S.ngy = (int)(gyb + ngy);
-      S.ngx = (int)(gxb + ngx);
-    }
-    if (tid < NBANDS * NSTRIPS) {
-      const int pb = tid >> 4, pq = tid & 15;
-      uint32_t n = 0;
-#pragma unroll
-      for (int w = 0; w < TILE_WARPS; ++w) {
-        const int lo = ns - 32 * w;
-        const uint32_t below = lo >= 32 ? 0xffffffffu : (lo <= 0 ? 0u : ((1u << lo) - 1u));
-        n += __popc(S.bb[w][pb] & S.sb[w][pq] & below);
+    // slot totals of the chunk: the block totals, unless the chunk was cut short (rare: one more barrier)
+    int ngy_tot = (int)(ptot & 0xFFFFu), ngx_tot = (int)(ptot >> 16);
+    if (ns < nvalid) {
+      if (tid == ns - 1) {
+        S.ngy = (int)(gyb + ngy);
+        S.ngx = (int)(gxb + ngx);
       }
-      S.len[tid] = n;
+      __syncthreads();
+      ngy_tot = S.ngy;
+      ngx_tot = S.ngx;
     }
-    __syncthreads();
     // profiles: thread = 8 values.  Band slot (row profile s' gy, [hq][i] = row 16 b + hq + 4 i): one thread per half
     // slot (hq = 2h, 2h+1); strip slot (column profile gx, columns 8 k .. 8 k + 7, halves swizzled): one thread per
     // slot.  d = (pixel - centre) is exact before the scaling; values outside the ROI are 0 (unsigned range test).
     // FADD2/FMUL2 pairs, one MUFU.EX2 per value.
     {
       const float2 sk2 = make_float2(sk, sk);
-      const int ngh = S.ngy * 2;
+      const int ngh = ngy_tot * 2;
       for (int g = tid; g < ngh; g += TILE_THREADS) {
         const int k = g >> 1, hh = g & 1;
         const uint32_t own = S.gyown[k];
@@ -234,7 +233,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
         dst[0] = make_float4(v[0], v[1], v[2], v[3]);
         dst[1] = make_float4(v[4], v[5], v[6], v[7]);
       }
-      const int nx = S.ngx;
+      const int nx = ngx_tot;
       for (int g = tid; g < nx; g += TILE_THREADS) {
         const uint32_t own = S.gxown[g];
         const uint32_t slot = own & 0xFFFFu;
@@ -258,21 +257,24 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
         *reinterpret_cast<float4*>(gs + sw) = make_float4(v[0], v[1], v[2], v[3]);
         *reinterpret_cast<float4*>(gs + (sw ^ 4)) = make_float4(v[4], v[5], v[6], v[7]);
       }
-      // pad every list with all-zero entries up to the longest list of its warp
-      if (tid < NBANDS * NSTRIPS) {
-        const int pb = tid >> 4, pq = tid & 15, w0 = pq & 8;
-        uint32_t mxl = 0;
-#pragma unroll
-        for (int k = 0; k < 8; ++k) mxl = max(mxl, S.len[pb * NSTRIPS + w0 + k]);
-        for (uint32_t st = S.len[tid]; st < mxl; ++st) S.ent[(st * NBANDS + pb) * NSTRIPS + pq] = ZERO_ENT;
-      }
     }
+    // the length of this lane group's list (stars < ns), and the warp's longest; pad the own list with all-zero
+    // entries up to it (each list belongs to one lane group, so no other warp touches these entries)
+    uint32_t len = 0;
+#pragma unroll
+    for (int w = 0; w < TILE_WARPS; ++w) {
+      const int lo = ns - 32 * w;
+      const uint32_t below = lo >= 32 ? 0xffffffffu : (lo <= 0 ? 0u : ((1u << lo) - 1u));
+      len += __popc(S.bb[w][B] & S.sb[w][Q] & below);
+    }
+    const uint32_t steps = __reduce_max_sync(0xffffffffu, len);
+    uint32_t* ent = &S.ent[B * NSTRIPS + Q];
+    if (hq == 0)
+      for (uint32_t st = len; st < steps; ++st) ent[st * (NBANDS * NSTRIPS)] = ZERO_ENT;
     __syncthreads();
 
     // ======================= accumulate: lane group q walks the (padded) list of block (B, Q)
     {
-      const uint32_t steps = __reduce_max_sync(0xffffffffu, S.len[p]);
-      const uint32_t* ent = &S.ent[B * NSTRIPS + Q];
 #pragma unroll 4
       for (uint32_t st = 0; st < steps; ++st) {
         const uint32_t e = ent[st * (NBANDS * NSTRIPS)];
