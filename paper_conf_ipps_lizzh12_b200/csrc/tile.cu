@@ -109,7 +109,9 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
     }
     const int b0 = r0 >> 4, b1 = r1 >> 4, q0 = c0 >> 3, q1 = c1 >> 3;  // empty ranges when !valid
     const int ngy = valid ? b1 - b0 + 1 : 0, ngx = valid ? q1 - q0 + 1 : 0;
-    __syncthreads();  // the previous chunk's accumulate phase is done with the shared buffers
+    // No barrier here: this phase writes only S.bb, S.sb, S.wsum and S.ns, which the previous chunk stopped reading
+    // before its last barrier; the slot and list buffers are rewritten only after the next barrier, which every
+    // warp reaches after finishing its accumulation of the previous chunk.
     if (tid == 0) S.ns = CHUNK;
     {
       uint32_t bbv = 0, sbv = 0;
