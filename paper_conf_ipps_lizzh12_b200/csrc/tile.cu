@@ -93,14 +93,17 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
     for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
 
   const uint32_t j1 = wi.je;
+  // this thread's star record of the current chunk, loaded one chunk ahead (its latency hides behind the
+  // accumulation of the previous chunk)
+  StarRec rnext = {};
+  if (wi.jb + tid < j1) rnext = rec[ids[wi.jb + tid]];
   for (uint32_t base = wi.jb; base < j1;) {
     // ======================= prep: thread = star (base + tid)
     const int nvalid = (int)min((uint32_t)CHUNK, j1 - base);
     const bool valid = tid < nvalid;
-    StarRec r = {};
+    const StarRec r = rnext;
     int c0 = 0, c1 = -1, r0 = 0, r1 = -1;
     if (valid) {
-      r = rec[ids[base + tid]];
       const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
       c0 = max(lx, 0);
       c1 = min(lx + fp.R - 1, TWe - 1);
@@ -191,6 +194,9 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
     }
     __syncthreads();
     const int ns = min(S.ns, nvalid);
+    // next chunk's star id now (its record is requested just before the accumulation)
+    const uint32_t nb = base + (uint32_t)ns;
+    const uint32_t nid = nb + tid < j1 ? __ldg(&ids[nb + tid]) : 0u;
     // slot totals of the chunk: the block totals, unless the chunk was cut short (rare: one more barrier)
     int ngy_tot = (int)(ptot & 0xFFFFu), ngx_tot = (int)(ptot >> 16);
     if (ns < nvalid) {
@@ -275,6 +281,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
       for (uint32_t st = len; st < steps; ++st) ent[st * (NBANDS * NSTRIPS)] = ZERO_ENT;
     __syncthreads();
 
+    if (nb + tid < j1) rnext = rec[nid];
     // ======================= accumulate: lane group q walks the (padded) list of block (B, Q)
     {
 #pragma unroll 4
