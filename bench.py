@@ -349,6 +349,25 @@ def run_ours(args, world, rank, local_rank):
         g_ms = sum(a.elapsed_time(b) for a, b in g_ev) / args.steps
         variants["gray_u8"] = {"ms_per_step": g_ms, "frames_per_s": 1e3 / g_ms, "updates_per_s": U_frame / (g_ms * 1e-3),
                                "note": "starsim_render_gray (output stage fused into k_tile, u8 image)"}
+        # NEXT-2 variant: the same fp32 frame with the pixel-integrated PSF (erf profiles instead of exp)
+        ctx.set_psf("integrated")
+        for _ in range(max(3, args.warmup)):
+            step(x, y, m)
+        barrier()
+        i_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                for _ in range(args.steps)]
+        for i in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.fill_(float(i))
+                i_ev[i][0].record(stream)
+            step(x, y, m)
+            i_ev[i][1].record(stream)
+        barrier()
+        ctx.set_psf("point")
+        i_ms = sum(a.elapsed_time(b) for a, b in i_ev) / args.steps
+        variants["integrated_psf"] = {"ms_per_step": i_ms, "frames_per_s": 1e3 / i_ms,
+                                      "updates_per_s": U_frame / (i_ms * 1e-3),
+                                      "note": "starsim_set_psf(INTEGRATED): Eq. 2 integrated over each pixel (NEXT-2)"}
 
     # e2e: the same C-ABI call with host (pinned) catalogue in and image out, copies inside the timed region
     e2e = None

@@ -93,6 +93,16 @@ int starsim_render_gray(starsim_ctx* ctx, const float* x, const float* y, const 
                         int32_t width, int32_t height, float sigma, int32_t roi, float gain, int32_t bits,
                         void* out, starsim_stream_t stream);
 
+/* PSF model of the renders that follow on this ctx (all of render, render_band, render_gray, render_atomic):
+ *   STARSIM_PSF_POINT (default): Eq. 2 as the paper writes it, sampled at the pixel coordinate;
+ *   STARSIM_PSF_INTEGRATED: Eq. 2 integrated over the pixel square [px-1/2, px+1/2] x
+ *     [py-1/2, py+1/2], i.e. g(m) * P(px) * P(py) with P(p) = (erf((p+1/2-X)/(sqrt(2) s)) - erf((p-1/2-X)/(sqrt(2) s)))/2;
+ *     same ROI, clipping and summation order.  Still separable, so the tiled path is unchanged but for the profiles.
+ * EINVAL: ctx NULL or an unknown mode. */
+#define STARSIM_PSF_POINT 0
+#define STARSIM_PSF_INTEGRATED 1
+int starsim_set_psf(starsim_ctx* ctx, int32_t mode);
+
 /* The paper's own design, kept as the measured comparison (Fig. 6): zero the image, then one
  * warp per star adds g*mu into every ROI pixel with global fp32 reductions (red.global.add.f32).  Same arguments
  * and EINVAL cases as starsim_render.  The summation order is nondeterministic. */

@@ -52,17 +52,19 @@ def _load():
         lib.oracle_brightness.restype = f64
         lib.oracle_psf.argtypes = [f64, f64, f64, f64, f64]
         lib.oracle_psf.restype = f64
+        lib.oracle_psf_integrated.argtypes = [f64, f64, f64, f64, f64]
+        lib.oracle_psf_integrated.restype = f64
         lib.oracle_roi_lo.argtypes = [ctypes.c_float, i32]
         lib.oracle_roi_lo.restype = i64
         lib.oracle_star_roi.argtypes = [ctypes.c_float, ctypes.c_float, ctypes.c_float, i32, i32, i32, i64p]
         lib.oracle_star_roi.restype = ctypes.c_int
-        lib.oracle_render.argtypes = [f32p, f32p, f32p, i64, i32, i32, f64, i32, f64, f64p]
+        lib.oracle_render.argtypes = [f32p, f32p, f32p, i64, i32, i32, f64, i32, f64, i32, f64p]
         lib.oracle_render.restype = i64
-        lib.oracle_render_band.argtypes = [f32p, f32p, f32p, i64, i32, i32, i32, i32, f64, i32, f64, f64p]
+        lib.oracle_render_band.argtypes = [f32p, f32p, f32p, i64, i32, i32, i32, i32, f64, i32, f64, i32, f64p]
         lib.oracle_render_band.restype = None
-        lib.oracle_render_mt.argtypes = [f32p, f32p, f32p, i64, i32, i32, f64, i32, f64, f64p, i32]
+        lib.oracle_render_mt.argtypes = [f32p, f32p, f32p, i64, i32, i32, f64, i32, f64, i32, f64p, i32]
         lib.oracle_render_mt.restype = ctypes.c_int
-        lib.oracle_render_full.argtypes = [f32p, f32p, f32p, i64, i32, i32, f64, f64, f64p]
+        lib.oracle_render_full.argtypes = [f32p, f32p, f32p, i64, i32, i32, f64, f64, i32, f64p]
         lib.oracle_render_full.restype = None
         lib.oracle_bins.argtypes = [f32p, f32p, f32p, i64, i32, i32, i32, i32, i32, u32p, u32p, i64]
         lib.oracle_bins.restype = i64
@@ -89,9 +91,20 @@ def brightness(m: float, A: float) -> float:
     return _load().oracle_brightness(float(m), float(A))
 
 
-def psf(px: float, py: float, X: float, Y: float, sigma: float) -> float:
-    """Eq. 2 at pixel (px, py) for a star at (X, Y)."""
-    return _load().oracle_psf(float(px), float(py), float(X), float(Y), float(sigma))
+PSF_MODES = {"point": 0, "integrated": 1}
+
+
+def _mode(psf_mode):
+    if psf_mode not in PSF_MODES:
+        raise ValueError(f"psf must be one of {sorted(PSF_MODES)}")
+    return PSF_MODES[psf_mode]
+
+
+def psf(px: float, py: float, X: float, Y: float, sigma: float, mode: str = "point") -> float:
+    """Eq. 2 at pixel (px, py) for a star at (X, Y); mode "integrated": Eq. 2 integrated over the pixel
+    square (NEXT-2)."""
+    f = _load().oracle_psf_integrated if _mode(mode) else _load().oracle_psf
+    return f(float(px), float(py), float(X), float(Y), float(sigma))
 
 
 def roi_lo(c: float, R: int) -> int:
@@ -106,37 +119,42 @@ def star_roi(x: float, y: float, m: float, W: int, H: int, R: int):
     return tuple(out) if ok else None
 
 
-def render(x, y, mag, W: int, H: int, sigma: float, R: int, A: float, threads: int = 1, return_units: bool = False):
+def render(x, y, mag, W: int, H: int, sigma: float, R: int, A: float, threads: int = 1, return_units: bool = False,
+           psf: str = "point"):
     """The oracle image, fp64 (H, W), row-major with y = row: Eqs. 1-3 over square ROIs in star order (Fig. 5).
 
-    ``threads > 1`` splits rows over pthreads; the result is bitwise identical (same per-pixel order)."""
+    ``threads > 1`` splits rows over pthreads; the result is bitwise identical (same per-pixel order).
+    ``psf="integrated"``: the pixel-integrated variant of Eq. 2 (NEXT-2)."""
+    mode = _mode(psf)
     _, (px, py, pm), n = _stars(x, y, mag)
     img = np.empty((int(H), int(W)), dtype=np.float64)
     pimg = img.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
     lib = _load()
     if threads <= 1:
-        U = lib.oracle_render(px, py, pm, n, int(W), int(H), float(sigma), int(R), float(A), pimg)
+        U = lib.oracle_render(px, py, pm, n, int(W), int(H), float(sigma), int(R), float(A), mode, pimg)
     else:
-        if lib.oracle_render_mt(px, py, pm, n, int(W), int(H), float(sigma), int(R), float(A), pimg, int(threads)):
+        if lib.oracle_render_mt(px, py, pm, n, int(W), int(H), float(sigma), int(R), float(A), mode, pimg,
+                                int(threads)):
             raise MemoryError("oracle_render_mt")
         U = None
     return (img, U) if return_units else img
 
 
-def render_band(x, y, mag, W: int, H: int, row0: int, rows: int, sigma: float, R: int, A: float):
+def render_band(x, y, mag, W: int, H: int, row0: int, rows: int, sigma: float, R: int, A: float,
+                psf: str = "point"):
     """Rows [row0, row0+rows) of the oracle image, fp64 (rows, W)."""
     _, (px, py, pm), n = _stars(x, y, mag)
     img = np.empty((int(rows), int(W)), dtype=np.float64)
     _load().oracle_render_band(px, py, pm, n, int(W), int(H), int(row0), int(rows), float(sigma), int(R), float(A),
-                               img.ctypes.data_as(ctypes.POINTER(ctypes.c_double)))
+                               _mode(psf), img.ctypes.data_as(ctypes.POINTER(ctypes.c_double)))
     return img
 
 
-def render_full(x, y, mag, W: int, H: int, sigma: float, A: float):
+def render_full(x, y, mag, W: int, H: int, sigma: float, A: float, psf: str = "point"):
     """No ROI cut-off (Fig. 1 left): every star at every pixel.  Tiny inputs only."""
     _, (px, py, pm), n = _stars(x, y, mag)
     img = np.empty((int(H), int(W)), dtype=np.float64)
-    _load().oracle_render_full(px, py, pm, n, int(W), int(H), float(sigma), float(A),
+    _load().oracle_render_full(px, py, pm, n, int(W), int(H), float(sigma), float(A), _mode(psf),
                                img.ctypes.data_as(ctypes.POINTER(ctypes.c_double)))
     return img
 

@@ -21,6 +21,10 @@
  *   - stars with a non-finite x, y or m, or whose clipped ROI is empty, contribute nothing;
  *   - accumulation is fp64 in star-index order (the paper's loop order).
  *
+ * NEXT-2: a pixel-integrated variant of Eq. 2 -- the pixel value is the Gaussian of Eq. 2 integrated
+ * over the pixel square [px-1/2, px+1/2] x [py-1/2, py+1/2] instead of sampled at its centre (psf mode 1), with the
+ * same ROI, clipping and order.  Mode 0 is the paper's point-sampled Eq. 2.
+ *
  * Pins (tests/test_oracle_pins.py, all "-m 'not gpu'"): Poisson-summation closed form of the point-sampled ROI mass,
  * first moment (centroid), reflection/transpose symmetry, scipy.ndimage.correlate with a kernel built from
  * scipy.stats.norm.pdf, brute-force no-ROI evaluation on tiny inputs, superposition, integer translation, magnitude
@@ -43,6 +47,23 @@ double oracle_brightness(double m, double A) { return A * pow(2.512, -m); }
 double oracle_psf(double px, double py, double X, double Y, double delta) {
     double dx = px - X, dy = py - Y;
     return 1.0 / (2.0 * M_PI * delta * delta) * exp(-(dx * dx + dy * dy) / (2.0 * delta * delta));
+}
+
+/* NEXT-2: Eq. 2 integrated over the pixel square -- a product of two 1-D integrals of the normalised Gaussian,
+ * (1/2) [erf((p + 1/2 - X) / (sqrt(2) d)) - erf((p - 1/2 - X) / (sqrt(2) d))], each taken in the form without
+ * cancellation (erfc of the same-signed side). */
+static double pixel_mass_1d(double p, double X, double delta) {
+    double s = 1.0 / (sqrt(2.0) * delta);
+    double a = (p - 0.5 - X) * s, b = (p + 0.5 - X) * s;
+    if (a >= 0.0) return 0.5 * (erfc(a) - erfc(b));
+    if (b <= 0.0) return 0.5 * (erfc(-b) - erfc(-a));
+    return 0.5 * (erf(b) - erf(a));
+}
+double oracle_psf_integrated(double px, double py, double X, double Y, double delta) {
+    return pixel_mass_1d(px, X, delta) * pixel_mass_1d(py, Y, delta);
+}
+static double psf_of(int mode, double px, double py, double X, double Y, double delta) {
+    return mode ? oracle_psf_integrated(px, py, X, Y, delta) : oracle_psf(px, py, X, Y, delta);
 }
 
 /* First ROI column (or row) of a star at coordinate c: the R integers nearest to c, ties at k+1/2 upward, i.e.
@@ -81,7 +102,7 @@ int oracle_star_roi(float x, float y, float m, int32_t W, int32_t H, int32_t R, 
 /* Fig. 5 over rows [row0, row0+rows) of the image only; img is rows*W doubles, zeroed here.
  * Brightness is hoisted out of the pixel loop (reading R15: the value is identical). */
 static void render_rows(const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
-                        int32_t row0, int32_t rows, double delta, int32_t R, double A, double* img) {
+                        int32_t row0, int32_t rows, double delta, int32_t R, double A, int32_t mode, double* img) {
     memset(img, 0, sizeof(double) * (size_t)rows * (size_t)W);
     for (int64_t i = 0; i < n; ++i) {
         int64_t x0, x1, y0, y1;
@@ -93,14 +114,14 @@ static void render_rows(const float* x, const float* y, const float* mag, int64_
         for (int64_t py = y0; py <= y1; ++py)                            /* Fig. 5: pixelY over the ROI */
             for (int64_t px = x0; px <= x1; ++px)                        /* Fig. 5: pixelX over the ROI */
                 img[(size_t)(py - row0) * (size_t)W + (size_t)px] +=
-                    g * oracle_psf((double)px, (double)py, X, Y, delta); /* Eq. 3 */
+                    g * psf_of(mode, (double)px, (double)py, X, Y, delta); /* Eq. 3 */
     }
 }
 
 /* The oracle image (Eqs. 1-3, Fig. 5): img[py*W+px], fp64, H*W entries.  Returns U = sum of clipped ROI areas. */
 int64_t oracle_render(const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
-                      double delta, int32_t R, double A, double* img) {
-    render_rows(x, y, mag, n, W, H, 0, H, delta, R, A, img);
+                      double delta, int32_t R, double A, int32_t mode, double* img) {
+    render_rows(x, y, mag, n, W, H, 0, H, delta, R, A, mode, img);
     int64_t U = 0;
     for (int64_t i = 0; i < n; ++i) {
         int64_t x0, x1, y0, y1;
@@ -111,23 +132,23 @@ int64_t oracle_render(const float* x, const float* y, const float* mag, int64_t 
 
 /* Rows [row0, row0+rows) of the oracle image (used for band tests): img is rows*W. */
 void oracle_render_band(const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
-                        int32_t row0, int32_t rows, double delta, int32_t R, double A, double* img) {
-    render_rows(x, y, mag, n, W, H, row0, rows, delta, R, A, img);
+                        int32_t row0, int32_t rows, double delta, int32_t R, double A, int32_t mode, double* img) {
+    render_rows(x, y, mag, n, W, H, row0, rows, delta, R, A, mode, img);
 }
 
 /* Same image, the rows split over nthreads pthreads (each thread owns whole rows and walks the stars in index order,
  * so every pixel sees the same additions in the same order: the result is bitwise equal to oracle_render).
  * Used only to time the CPU baseline on all host cores. */
 struct band_job { const float *x, *y, *mag; int64_t n; int32_t W, H, row0, rows; double delta; int32_t R; double A;
-                  double* img; };
+                  int32_t mode; double* img; };
 static void* band_main(void* p) {
     struct band_job* j = (struct band_job*)p;
-    render_rows(j->x, j->y, j->mag, j->n, j->W, j->H, j->row0, j->rows, j->delta, j->R, j->A,
+    render_rows(j->x, j->y, j->mag, j->n, j->W, j->H, j->row0, j->rows, j->delta, j->R, j->A, j->mode,
                 j->img + (size_t)j->row0 * (size_t)j->W);
     return NULL;
 }
 int oracle_render_mt(const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
-                     double delta, int32_t R, double A, double* img, int32_t nthreads) {
+                     double delta, int32_t R, double A, int32_t mode, double* img, int32_t nthreads) {
     if (nthreads < 1) nthreads = 1;
     if (nthreads > H) nthreads = H;
     pthread_t* th = (pthread_t*)malloc(sizeof(pthread_t) * (size_t)nthreads);
@@ -135,7 +156,7 @@ int oracle_render_mt(const float* x, const float* y, const float* mag, int64_t n
     if (!th || !jobs) { free(th); free(jobs); return -1; }
     for (int t = 0; t < nthreads; ++t) {
         int32_t r0 = (int32_t)((int64_t)H * t / nthreads), r1 = (int32_t)((int64_t)H * (t + 1) / nthreads);
-        struct band_job j = {x, y, mag, n, W, H, r0, r1 - r0, delta, R, A, img};
+        struct band_job j = {x, y, mag, n, W, H, r0, r1 - r0, delta, R, A, mode, img};
         jobs[t] = j;
         pthread_create(&th[t], NULL, band_main, &jobs[t]);
     }
@@ -147,13 +168,13 @@ int oracle_render_mt(const float* x, const float* y, const float* mag, int64_t n
 /* No ROI cut-off (Fig. 1 left): every star against every pixel, pixel-centric (Fig. 3a).
  * For tiny inputs only.  Skips non-finite stars like the ROI version. */
 void oracle_render_full(const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
-                        double delta, double A, double* img) {
+                        double delta, double A, int32_t mode, double* img) {
     for (int32_t py = 0; py < H; ++py)
         for (int32_t px = 0; px < W; ++px) {
             double v = 0.0;
             for (int64_t i = 0; i < n; ++i) {
                 if (!isfinite(x[i]) || !isfinite(y[i]) || !isfinite(mag[i])) continue;
-                v += oracle_brightness((double)mag[i], A) * oracle_psf(px, py, (double)x[i], (double)y[i], delta);
+                v += oracle_brightness((double)mag[i], A) * psf_of(mode, px, py, (double)x[i], (double)y[i], delta);
             }
             img[(size_t)py * (size_t)W + (size_t)px] = v;
         }

@@ -5,8 +5,8 @@ ctypes binding.  :mod:`.dist` renders horizontal bands per GPU and assembles the
 """
 from .starsim import (Context, StarsimError, starsim_create, starsim_destroy, starsim_render, starsim_render_band,
                       starsim_render_gray, starsim_render_atomic, starsim_upload_aos, starsim_quantize,
-                      starsim_get_bins, starsim_profile, starsim_kernel_times, LIB_PATH, KCLASSES)
+                      starsim_get_bins, starsim_profile, starsim_kernel_times, starsim_set_psf, LIB_PATH, KCLASSES)
 
 __all__ = ["Context", "StarsimError", "starsim_create", "starsim_destroy", "starsim_render", "starsim_render_band",
            "starsim_render_gray", "starsim_render_atomic", "starsim_upload_aos", "starsim_quantize", "starsim_get_bins",
-           "starsim_profile", "starsim_kernel_times", "LIB_PATH", "KCLASSES"]
+           "starsim_profile", "starsim_kernel_times", "starsim_set_psf", "LIB_PATH", "KCLASSES"]

@@ -33,13 +33,13 @@ struct Launch {
 struct GraphKey {
   const void *x, *y, *mag, *out;
   int64_t n;
-  int32_t W, H, row0, rows, R, obits;
+  int32_t W, H, row0, rows, R, obits, psf;
   float sigma, gain;
   cudaStream_t st;
   uint64_t scratch_gen;
   bool operator==(const GraphKey& o) const {
     return x == o.x && y == o.y && mag == o.mag && out == o.out && n == o.n && W == o.W && H == o.H &&
-           row0 == o.row0 && rows == o.rows && R == o.R && obits == o.obits && sigma == o.sigma && gain == o.gain && st == o.st &&
+           row0 == o.row0 && rows == o.rows && R == o.R && obits == o.obits && psf == o.psf && sigma == o.sigma && gain == o.gain && st == o.st &&
            scratch_gen == o.scratch_gen;
   }
 };
@@ -47,6 +47,7 @@ struct GraphKey {
 struct starsim_ctx {
   int dev = 0;
   int num_sms = 148;
+  int32_t psf = 0;  // starsim_set_psf: 0 point-sampled Eq. 2, 1 pixel-integrated (NEXT-2)
   std::string err;
   Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
@@ -165,7 +166,8 @@ int validate_frame(starsim_ctx* c, const float* x, const float* y, const float* 
   return STARSIM_OK;
 }
 
-FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float sigma, int32_t R, float gain) {
+FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float sigma, int32_t R, float gain,
+                        int32_t psf) {
   FrameParams fp;
   fp.W = W;
   fp.H = H;
@@ -175,9 +177,11 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   fp.ntx = (W + TILE_W - 1) / TILE_W;
   fp.nty = (rows + TILE_H - 1) / TILE_H;
   const double s = (double)sigma;
-  fp.kexp = (float)(-1.0 / (2.0 * s * s * std::log(2.0)));   // exp(-d^2/(2 s^2)) = 2^(kexp d^2)
   fp.sk = (float)std::sqrt(1.0 / (2.0 * s * s * std::log(2.0)));  // exp(-d^2/(2 s^2)) = 2^(-(d sk)^2)
   fp.s_scale = (double)gain / (2.0 * M_PI * s * s);          // Eq. 1 gain with Eq. 2's 1/(2 pi s^2)
+  fp.psf = psf;
+  fp.kint = (float)(1.0 / (std::sqrt(2.0) * s));
+  if (psf) fp.s_scale = (double)gain;  // the pixel masses of the integrated PSF are already normalised
   return fp;
 }
 
@@ -224,7 +228,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
                  int32_t row0, int32_t rows, float sigma, int32_t R, float gain, int32_t obits, void* out,
                  cudaStream_t st) {
   DevGuard g(c->dev);
-  FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain);
+  FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain, c->psf);
   fp.obits = obits;
   // one vector store per 8-pixel run: 32 B (fp32) / 8 B (u8) / 16 B (u16); rows must keep that alignment
   const int vb = obits == 8 ? 8 : 16;
@@ -250,7 +254,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
     return rc;
   if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
 
-  const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, sigma, gain, st, c->scratch_gen};
+  const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, c->psf, sigma, gain, st, c->scratch_gen};
   if (st == nullptr || c->prof || !c->use_graphs) {
     if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st))) return rc;
   } else {
@@ -376,6 +380,15 @@ int starsim_render_gray(starsim_ctx* c, const float* x, const float* y, const fl
   return render_tiled(c, x, y, mag, n, W, H, 0, H, sigma, R, gain, bits, out, (cudaStream_t)stream);
 }
 
+int starsim_set_psf(starsim_ctx* c, int32_t mode) {
+  if (!c) return STARSIM_EINVAL;
+  if (mode != STARSIM_PSF_POINT && mode != STARSIM_PSF_INTEGRATED)
+    return fail(c, STARSIM_EINVAL, "psf mode must be STARSIM_PSF_POINT or STARSIM_PSF_INTEGRATED");
+  c->psf = mode;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
 int starsim_render_atomic(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W,
                           int32_t H, float sigma, int32_t R, float gain, float* out, starsim_stream_t stream) {
   if (!c) return STARSIM_EINVAL;
@@ -383,7 +396,7 @@ int starsim_render_atomic(starsim_ctx* c, const float* x, const float* y, const 
   if (rc) return rc;
   DevGuard g(c->dev);
   cudaStream_t st = (cudaStream_t)stream;
-  const FrameParams fp = make_params(W, H, 0, H, sigma, R, gain);
+  const FrameParams fp = make_params(W, H, 0, H, sigma, R, gain, c->psf);
   timed(c, 5, st, [&] { cudaMemsetAsync(out, 0, sizeof(float) * (size_t)W * H, st); });
   timed(c, 4, st, [&] { launch_atomic(x, y, mag, n, fp, out, st); });
   if ((rc = check_launch(c, "k_atomic"))) return rc;

@@ -73,8 +73,9 @@ struct FrameParams {
   int32_t ntx, nty;      // tiles over the band
   int32_t vec;           // 1 if every 8-pixel run of an out row is aligned for one vector store
   int32_t obits;         // 0: fp32 image; 8 / 16: gray values quantised in the epilogue (u8 / u16 image)
-  float kexp;            // -log2(e) / (2 sigma^2): exp(-d^2/(2 sigma^2)) = ex2(kexp * d^2)
+  int32_t psf;           // 0: Eq. 2 point-sampled (the paper); 1: Eq. 2 integrated over the pixel square (NEXT-2)
   float sk;              // sqrt(log2(e) / (2 sigma^2)):  exp(-d^2/(2 sigma^2)) = ex2(-(d * sk)^2)
+  float kint;            // 1 / (sqrt(2) sigma): the erf argument scale of the integrated PSF
   double s_scale;        // A / (2 pi sigma^2), applied in fp64 before rounding s' to fp32
 };
 
@@ -89,6 +90,15 @@ __device__ __forceinline__ uint32_t quant1(float v, float qmax) {
     q = fminf(q, qmax);
   }
   return (uint32_t)q;
+}
+
+// NEXT-2: the 1-D pixel mass of the normalised Gaussian between the pixel edges ta < tb (in units of sqrt(2) sigma):
+// Phi(tb) - Phi(ta), Phi(t) = erf(t)/2, from e = erfc(|t|) of each edge without cancellation.
+__device__ __forceinline__ float edge_erfc(float t) { return erfcf(fabsf(t)); }
+__device__ __forceinline__ float pix_mass(float ta, float ea, float tb, float eb) {
+  if (ta >= 0.f) return 0.5f * (ea - eb);
+  if (tb < 0.f) return 0.5f * (eb - ea);
+  return 1.f - 0.5f * (ea + eb);
 }
 
 // MUFU.EX2 (2^x, flush-to-zero): the one SFU op per profile value.

@@ -36,13 +36,26 @@ __global__ void __launch_bounds__(ATOM_WARPS * 32) k_atomic(const float* __restr
   s = __shfl_sync(0xffffffffu, s, 0);
   float* gx = s_prof + warp * 2 * fp.R;
   float* gy = gx + fp.R;
-  for (int c = lane; c < w; c += 32) {
-    const float d = (float)(cx0 + c) - x;
-    gx[c] = ex2_approx(fp.kexp * (d * d));
-  }
-  for (int r = lane; r < h; r += 32) {
-    const float d = (float)(cy0 + r) - y;
-    gy[r] = s * ex2_approx(fp.kexp * (d * d));
+  if (!fp.psf) {
+    for (int c = lane; c < w; c += 32) {
+      const float d = (float)(cx0 + c) - x;
+      const float e = d * fp.sk;
+      gx[c] = ex2_approx(-(e * e));
+    }
+    for (int r = lane; r < h; r += 32) {
+      const float d = (float)(cy0 + r) - y;
+      const float e = d * fp.sk;
+      gy[r] = s * ex2_approx(-(e * e));
+    }
+  } else {  // NEXT-2: pixel-integrated PSF, the pixel's 1-D masses between its edges
+    for (int c = lane; c < w; c += 32) {
+      const float d = (float)(cx0 + c) - x, ta = (d - 0.5f) * fp.kint, tb = (d + 0.5f) * fp.kint;
+      gx[c] = pix_mass(ta, edge_erfc(ta), tb, edge_erfc(tb));
+    }
+    for (int r = lane; r < h; r += 32) {
+      const float d = (float)(cy0 + r) - y, ta = (d - 0.5f) * fp.kint, tb = (d + 0.5f) * fp.kint;
+      gy[r] = s * pix_mass(ta, edge_erfc(ta), tb, edge_erfc(tb));
+    }
   }
   __syncwarp();
   const float inv_w = 1.0f / (float)w;

@@ -54,6 +54,7 @@ constexpr uint32_t ZERO_ENT = ZERO_GX * 32u << 16;  // gy byte offset 0, all-zer
 // directly; a part writes its 128 x 64 partial to part_buf, and the last part to finish (per-tile counter) sums the
 // parts in part order -- a fixed order, so the image stays deterministic.
 // ---------------------------------------------------------------------------------------------------------------
+template <bool INTEG>  // INTEG: the pixel-integrated PSF (NEXT-2) instead of the paper's point-sampled Eq. 2
 __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __restrict__ ids,
                                                           const StarRec* __restrict__ rec, FrameParams fp,
                                                           void* __restrict__ out_, const WorkItem* __restrict__ items,
@@ -227,14 +228,26 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
         float2 d[4] = {__fadd2_rn(b2, make_float2(0.f, 4.f)), __fadd2_rn(b2, make_float2(8.f, 12.f)),
                        __fadd2_rn(b2, make_float2(1.f, 5.f)), __fadd2_rn(b2, make_float2(9.f, 13.f))};
         float v[8];
+        if (!INTEG) {
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          d[j] = __fmul2_rn(d[j], sk2);
-          d[j] = __fmul2_rn(d[j], make_float2(-d[j].x, -d[j].y));
-          const float2 e = __fmul2_rn(make_float2(ex2_approx(d[j].x), ex2_approx(d[j].y)), s2);
-          const int o0 = (j & 1) * 8 + (j >> 1), o1 = o0 + 4;       // row offsets of the pair
-          v[2 * j] = u0 + (uint32_t)o0 <= span ? e.x : 0.f;
-          v[2 * j + 1] = u0 + (uint32_t)o1 <= span ? e.y : 0.f;
+          for (int j = 0; j < 4; ++j) {
+            d[j] = __fmul2_rn(d[j], sk2);
+            d[j] = __fmul2_rn(d[j], make_float2(-d[j].x, -d[j].y));
+            const float2 e = __fmul2_rn(make_float2(ex2_approx(d[j].x), ex2_approx(d[j].y)), s2);
+            const int o0 = (j & 1) * 8 + (j >> 1), o1 = o0 + 4;     // row offsets of the pair
+            v[2 * j] = u0 + (uint32_t)o0 <= span ? e.x : 0.f;
+            v[2 * j + 1] = u0 + (uint32_t)o1 <= span ? e.y : 0.f;
+          }
+        } else {
+          // pixel-integrated rows: the pairs (r, r+1) of the two quads share their middle edge
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const float dr = bf + (float)(4 * i);                     // exact
+            const float t0 = (dr - 0.5f) * fp.kint, t1 = (dr + 0.5f) * fp.kint, t2 = (dr + 1.5f) * fp.kint;
+            const float e0 = edge_erfc(t0), e1 = edge_erfc(t1), e2 = edge_erfc(t2);
+            v[i] = u0 + (uint32_t)(4 * i) <= span ? pp.y * pix_mass(t0, e0, t1, e1) : 0.f;
+            v[4 + i] = u0 + (uint32_t)(4 * i + 1) <= span ? pp.y * pix_mass(t1, e1, t2, e2) : 0.f;
+          }
         }
         // v = rows +0,+4,+8,+12 (quad hq=2hh) and +1,+5,+9,+13 (quad 2hh+1), [hq][i] order
         float4* dst = reinterpret_cast<float4*>(&S.gy[k * 16 + hh * 8]);
@@ -253,12 +266,24 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
         const float bf = (float)rel - pp.x;
         const float2 b2 = make_float2(bf, bf);
         float v[8];
+        if (!INTEG) {
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          float2 dd = __fmul2_rn(__fadd2_rn(b2, make_float2((float)(2 * j), (float)(2 * j + 1))), sk2);
-          dd = __fmul2_rn(dd, make_float2(-dd.x, -dd.y));
-          v[2 * j] = u0 + (uint32_t)(2 * j) <= span ? ex2_approx(dd.x) : 0.f;
-          v[2 * j + 1] = u0 + (uint32_t)(2 * j + 1) <= span ? ex2_approx(dd.y) : 0.f;
+          for (int j = 0; j < 4; ++j) {
+            float2 dd = __fmul2_rn(__fadd2_rn(b2, make_float2((float)(2 * j), (float)(2 * j + 1))), sk2);
+            dd = __fmul2_rn(dd, make_float2(-dd.x, -dd.y));
+            v[2 * j] = u0 + (uint32_t)(2 * j) <= span ? ex2_approx(dd.x) : 0.f;
+            v[2 * j + 1] = u0 + (uint32_t)(2 * j + 1) <= span ? ex2_approx(dd.y) : 0.f;
+          }
+        } else {
+          // pixel-integrated columns: 9 edges shared by the 8 consecutive columns
+          float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const float tn = (bf + (float)j + 0.5f) * fp.kint, en = edge_erfc(tn);
+            v[j] = u0 + (uint32_t)j <= span ? pix_mass(t, e, tn, en) : 0.f;
+            t = tn;
+            e = en;
+          }
         }
         float* gs = &S.gx[slot * 8];
         const int sw = ((k >> 2) & 1) * 4;
@@ -401,7 +426,8 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
 }
 
 void init_tile_kernel() {
-  cudaFuncSetAttribute(k_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
+  cudaFuncSetAttribute(k_tile<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
+  cudaFuncSetAttribute(k_tile<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
 }
 
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
@@ -410,8 +436,12 @@ void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp,
   if (ntiles <= 0) return;
   const int64_t maxitems = ntiles + part_cap;
   const int64_t grid = maxitems;  // one CTA per possible item (parts first); CTAs past the item count exit at once
-  k_tile<<<(unsigned)grid, TILE_THREADS, sizeof(TileSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf, done,
-                                                                 hdr);
+  if (fp.psf)
+    k_tile<true><<<(unsigned)grid, TILE_THREADS, sizeof(TileSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf,
+                                                                         done, hdr);
+  else
+    k_tile<false><<<(unsigned)grid, TILE_THREADS, sizeof(TileSmem), st>>>(ids, rec, fp, out, items, split_tab,
+                                                                          part_buf, done, hdr);
 }
 
 }  // namespace starsim

@@ -55,6 +55,8 @@ def lib():
         L.starsim_render_band.restype = ctypes.c_int
         L.starsim_render_gray.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, i32, vp, vp]
         L.starsim_render_gray.restype = ctypes.c_int
+        L.starsim_set_psf.argtypes = [vp, i32]
+        L.starsim_set_psf.restype = ctypes.c_int
         L.starsim_render_atomic.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
         L.starsim_render_atomic.restype = ctypes.c_int
         L.starsim_upload_aos.argtypes = [vp, vp, i64, vp, vp, vp, vp]
@@ -126,6 +128,13 @@ def starsim_render_gray(h, x, y, mag, width, height, sigma, roi, gain, bits, out
     _check(h, lib().starsim_render_gray(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
                                         _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
                                         int(roi), float(gain), int(bits), _ptr(out, dt, "out"), _stream(stream)))
+
+
+PSF_MODES = {"point": 0, "integrated": 1}
+
+
+def starsim_set_psf(h, mode) -> None:
+    _check(h, lib().starsim_set_psf(h, PSF_MODES.get(mode, mode) if isinstance(mode, str) else int(mode)))
 
 
 def starsim_render_band(h, x, y, mag, width, height, row0, rows, sigma, roi, gain, out_band, stream=None) -> None:
@@ -239,6 +248,10 @@ class Context:
             out = torch.empty((height, width), dtype=torch.uint8 if bits == 8 else torch.uint16, device=x.device)
         starsim_render_gray(self.h, x, y, mag, width, height, sigma, roi, gain, bits, out, stream)
         return out
+
+    def set_psf(self, mode="point"):
+        """"point" (Eq. 2 sampled at the pixel, the paper) or "integrated" (Eq. 2 integrated over the pixel)."""
+        starsim_set_psf(self.h, mode)
 
     def render_band(self, x, y, mag, width, height, row0, rows, sigma, roi, gain, out=None, stream=None):
         out = self._out(rows, width, out)

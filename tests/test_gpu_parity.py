@@ -341,3 +341,38 @@ def test_c5_sampled_rows(torch_dev, ctx):
     for row in [0, 1, 4095, 8191, 8192, 16383]:
         ref = oracle.render_band(f.x, f.y, f.mag, cfg.W, cfg.H, row, 1, cfg.sigma, cfg.R, A)
         assert_parity(img[row:row + 1].cpu().numpy(), ref, f"C5 row {row}")
+
+
+# ---------------------------------------------------------------- NEXT-2: pixel-integrated PSF
+
+@pytest.fixture()
+def ctx_integrated(ctx):
+    ctx.set_psf("integrated")
+    yield ctx
+    ctx.set_psf("point")
+
+
+@pytest.mark.parametrize("W,H,n,R,sigma", [(1024, 1024, 1000, 5, 1.0), (301, 177, 3000, 15, 2.5),
+                                           (256, 256, 400, 63, 10.5), (120, 90, 500, 7, 0.4)])
+def test_integrated_psf_parity(torch_dev, ctx_integrated, W, H, n, R, sigma):
+    f = synth.uniform_field(n, W, H, seed=R + n, mag_lo=0.0, mag_hi=3.0)
+    args = to_dev(torch_dev, f)
+    ref = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads(), psf="integrated")
+    assert_parity(ctx_integrated.render(*args, W, H, sigma, R, 1.0).cpu().numpy(), ref, f"integrated tiled {W}x{H}")
+    assert_parity(ctx_integrated.render_atomic(*args, W, H, sigma, R, 1.0).cpu().numpy(), ref,
+                  f"integrated atomic {W}x{H}")
+
+
+def test_integrated_psf_mode_switch_and_einval(torch_dev, ctx):
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import StarsimError
+    f = synth.uniform_field(500, 200, 200, seed=3, mag_lo=0.0, mag_hi=2.0)
+    args = to_dev(torch_dev, f)
+    a = ctx.render(*args, 200, 200, 1.5, 9, 1.0)
+    ctx.set_psf("integrated")
+    b = ctx.render(*args, 200, 200, 1.5, 9, 1.0)
+    ctx.set_psf("point")
+    c = ctx.render(*args, 200, 200, 1.5, 9, 1.0)
+    assert torch.equal(a, c) and not torch.equal(a, b)
+    with pytest.raises(StarsimError):
+        ctx.set_psf(7)

@@ -318,3 +318,56 @@ def test_even_roi_side_uses_nearest_pixels():
     cols = np.nonzero(img.any(axis=0))[0].tolist()
     rows = np.nonzero(img.any(axis=1))[0].tolist()
     assert cols == [9, 10, 11, 12] and rows == [9, 10, 11, 12]
+
+
+# ---------------------------------------------------------------- NEXT-2: pixel-integrated PSF (psf="integrated")
+
+def _erf_mass_1d(lo, hi, u, sigma):
+    """Telescoped closed form of the 1-D pixel masses over pixels lo..hi: (1/2)[erf((hi+1/2-u)/(sqrt2 s)) -
+    erf((lo-1/2-u)/(sqrt2 s))] (the per-pixel differences cancel pairwise)."""
+    s = math.sqrt(2.0) * sigma
+    return 0.5 * (math.erf((hi + 0.5 - u) / s) - math.erf((lo - 0.5 - u) / s))
+
+
+@pytest.mark.parametrize("sigma", [0.5, 1.0, 2.5])
+@pytest.mark.parametrize("u,v", [(0.0, 0.0), (0.3, -0.45), (-0.49, 0.2)])
+@pytest.mark.parametrize("R", [5, 15])
+def test_integrated_roi_mass_telescopes(sigma, u, v, R):
+    x, y, m = star(40 + u, 40 + v)
+    img = oracle.render(x, y, m, 81, 81, sigma, R, 1.0, psf="integrated")
+    lx, ly = oracle.roi_lo(float(x[0]), R), oracle.roi_lo(float(y[0]), R)
+    expect = (_erf_mass_1d(lx, lx + R - 1, float(x[0]), sigma) * _erf_mass_1d(ly, ly + R - 1, float(y[0]), sigma))
+    assert abs(img.sum() - expect) < 1e-13
+    # exactly the ROI pixels are lit
+    assert np.count_nonzero(img) == R * R
+
+
+@pytest.mark.parametrize("sigma,X,Y,px,py", [(0.7, 10.3, 9.8, 10, 10), (0.7, 10.3, 9.8, 11, 9),
+                                             (1.5, 4.0, 4.0, 6, 3), (0.4, 2.5, 2.5, 2, 3)])
+def test_integrated_pixel_equals_numerical_quadrature(sigma, X, Y, px, py):
+    from scipy import integrate
+    f = lambda yy, xx: math.exp(-((xx - X) ** 2 + (yy - Y) ** 2) / (2 * sigma * sigma)) / (2 * math.pi * sigma ** 2)
+    q, err = integrate.dblquad(f, px - 0.5, px + 0.5, py - 0.5, py + 0.5, epsabs=1e-14, epsrel=1e-12)
+    assert abs(oracle.psf(px, py, X, Y, sigma, "integrated") - q) < 1e-12
+
+
+def test_integrated_tends_to_point_sampled_for_wide_psf():
+    # for sigma >> 1 px the pixel integral of the Gaussian is its centre value times (1 + f''/(24 f) per axis):
+    # (a - b) / b = [(dx^2/s^2 - 1) + (dy^2/s^2 - 1)] / (24 s^2) + O(s^-4)   (midpoint rule error, exact 2nd order)
+    s = 20.0
+    for px, py in [(0, 0), (3, -2), (10, 7)]:
+        dx, dy = px - 0.2, py + 0.1
+        a = oracle.psf(px, py, 0.2, -0.1, s, "integrated")
+        b = oracle.psf(px, py, 0.2, -0.1, s, "point")
+        pred = ((dx * dx / (s * s) - 1.0) + (dy * dy / (s * s) - 1.0)) / (24.0 * s * s)
+        assert abs((a - b) / b - pred) < 2e-7
+
+
+def test_integrated_symmetric_and_full_evaluation_bitwise():
+    x, y, m = star(12, 12)
+    img = oracle.render(x, y, m, 25, 25, 1.3, 9, 1.0, psf="integrated")
+    assert np.array_equal(img, img[::-1, ::-1]) and np.array_equal(img, img.T)
+    f = synth.uniform_field(30, 24, 20, seed=5, mag_lo=0.0, mag_hi=3.0)
+    a = oracle.render(f.x, f.y, f.mag, 24, 20, 1.1, 2 * 24 + 1, 1.0, psf="integrated")
+    b = oracle.render_full(f.x, f.y, f.mag, 24, 20, 1.1, 1.0, psf="integrated")
+    assert np.array_equal(a, b)
