@@ -103,6 +103,16 @@ int starsim_render_gray(starsim_ctx* ctx, const float* x, const float* y, const 
 #define STARSIM_PSF_INTEGRATED 1
 int starsim_set_psf(starsim_ctx* ctx, int32_t mode);
 
+/* Tile-accumulation kernel of the tiled renders that follow on this ctx (render, render_band, render_gray).  Both
+ * compute Eqs. 2-3 per tile in fp32 registers with the separable PSF and write every pixel once;
+ * they differ in how a tile's star list is walked, hence in the (deterministic) per-pixel summation order:
+ *   STARSIM_TILE_AUTO (default): for R <= 17 the sorted-corner-bin kernel, else the list kernel;
+ *   STARSIM_TILE_LISTS: always the per-block entry-list kernel (the comparison / any R).
+ * EINVAL: ctx NULL or an unknown mode. */
+#define STARSIM_TILE_AUTO 0
+#define STARSIM_TILE_LISTS 1
+int starsim_set_tile_kernel(starsim_ctx* ctx, int32_t mode);
+
 /* The paper's own design, kept as the measured comparison (Fig. 6): zero the image, then one
  * warp per star adds g*mu into every ROI pixel with global fp32 reductions (red.global.add.f32).  Same arguments
  * and EINVAL cases as starsim_render.  The summation order is nondeterministic. */

@@ -33,13 +33,13 @@ struct Launch {
 struct GraphKey {
   const void *x, *y, *mag, *out;
   int64_t n;
-  int32_t W, H, row0, rows, R, obits, psf;
+  int32_t W, H, row0, rows, R, obits, psf, tile_impl;
   float sigma, gain;
   cudaStream_t st;
   uint64_t scratch_gen;
   bool operator==(const GraphKey& o) const {
     return x == o.x && y == o.y && mag == o.mag && out == o.out && n == o.n && W == o.W && H == o.H &&
-           row0 == o.row0 && rows == o.rows && R == o.R && obits == o.obits && psf == o.psf && sigma == o.sigma && gain == o.gain && st == o.st &&
+           row0 == o.row0 && rows == o.rows && R == o.R && obits == o.obits && psf == o.psf && tile_impl == o.tile_impl && sigma == o.sigma && gain == o.gain && st == o.st &&
            scratch_gen == o.scratch_gen;
   }
 };
@@ -48,6 +48,7 @@ struct starsim_ctx {
   int dev = 0;
   int num_sms = 148;
   int32_t psf = 0;  // starsim_set_psf: 0 point-sampled Eq. 2, 1 pixel-integrated (NEXT-2)
+  int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto (sorted bins when R <= 17), 1 per-block lists
   std::string err;
   Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
@@ -180,6 +181,9 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   fp.sk = (float)std::sqrt(1.0 / (2.0 * s * s * std::log(2.0)));  // exp(-d^2/(2 s^2)) = 2^(-(d sk)^2)
   fp.s_scale = (double)gain / (2.0 * M_PI * s * s);          // Eq. 1 gain with Eq. 2's 1/(2 pi s^2)
   fp.psf = psf;
+  fp.tile_impl = 0;
+  fp.obits = 0;
+  fp.vec = 0;
   fp.kint = (float)(1.0 / (std::sqrt(2.0) * s));
   if (psf) fp.s_scale = (double)gain;  // the pixel masses of the integrated PSF are already normalised
   return fp;
@@ -230,6 +234,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   DevGuard g(c->dev);
   FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain, c->psf);
   fp.obits = obits;
+  fp.tile_impl = c->tile_impl;
   // one vector store per 8-pixel run: 32 B (fp32) / 8 B (u8) / 16 B (u16); rows must keep that alignment
   const int vb = obits == 8 ? 8 : 16;
   fp.vec = ((W * (obits ? obits / 8 : 4)) % vb == 0 && ((uintptr_t)out % vb) == 0) ? 1 : 0;
@@ -254,7 +259,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
     return rc;
   if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
 
-  const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, c->psf, sigma, gain, st, c->scratch_gen};
+  const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, c->psf, c->tile_impl, sigma, gain, st, c->scratch_gen};
   if (st == nullptr || c->prof || !c->use_graphs) {
     if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st))) return rc;
   } else {
@@ -385,6 +390,15 @@ int starsim_set_psf(starsim_ctx* c, int32_t mode) {
   if (mode != STARSIM_PSF_POINT && mode != STARSIM_PSF_INTEGRATED)
     return fail(c, STARSIM_EINVAL, "psf mode must be STARSIM_PSF_POINT or STARSIM_PSF_INTEGRATED");
   c->psf = mode;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
+int starsim_set_tile_kernel(starsim_ctx* c, int32_t mode) {
+  if (!c) return STARSIM_EINVAL;
+  if (mode != STARSIM_TILE_AUTO && mode != STARSIM_TILE_LISTS)
+    return fail(c, STARSIM_EINVAL, "tile kernel mode must be STARSIM_TILE_AUTO or STARSIM_TILE_LISTS");
+  c->tile_impl = mode;
   c->err.clear();
   return STARSIM_OK;
 }

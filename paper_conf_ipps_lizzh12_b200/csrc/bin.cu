@@ -492,6 +492,9 @@ void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, in
   k_sortlists<<<(unsigned)ntiles, SORT_THREADS, 0, st>>>(ids, tmp, tile_off, passes);
 }
 
-void init_kernels() { init_tile_kernel(); }
+void init_kernels() {
+  init_tile_kernel();
+  init_tile_sb_kernel();
+}
 
 }  // namespace starsim

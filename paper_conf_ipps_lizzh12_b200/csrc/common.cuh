@@ -22,6 +22,7 @@ constexpr int GY_CAP = 384;                      // band slots (16 floats: the r
 constexpr int RCAP = 56;                         // strip slots (8 floats: the column profile on one strip) per strip
 constexpr int LCAP = 32;                         // entries per (band, strip) list per chunk
 constexpr int GX_PAIRS = 768;                    // (star, strip) pairs per chunk
+constexpr int SB_MAXR = 17;                      // tile_sb.cu: an ROI of side <= 17 spans <= 2 bands and <= 3 strips
 
 // k_prep: one star per thread; per-tile counters CNT_STRIDE words apart (one 128-B line each, so that the
 // atomics of different tiles never serialise on one L2 line)
@@ -74,6 +75,7 @@ struct FrameParams {
   int32_t vec;           // 1 if every 8-pixel run of an out row is aligned for one vector store
   int32_t obits;         // 0: fp32 image; 8 / 16: gray values quantised in the epilogue (u8 / u16 image)
   int32_t psf;           // 0: Eq. 2 point-sampled (the paper); 1: Eq. 2 integrated over the pixel square (NEXT-2)
+  int32_t tile_impl;     // 0: sorted-bin tile kernel when R <= SB_MAXR (tile_sb.cu), else the list kernel; 1: always the list kernel (tile.cu)
   float sk;              // sqrt(log2(e) / (2 sigma^2)):  exp(-d^2/(2 sigma^2)) = ex2(-(d * sk)^2)
   float kint;            // 1 / (sqrt(2) sigma): the erf argument scale of the integrated PSF
   double s_scale;        // A / (2 pi sigma^2), applied in fp64 before rounding s' to fp32

@@ -9,6 +9,7 @@ namespace starsim {
 
 void init_kernels();
 void init_tile_kernel();
+void init_tile_sb_kernel();
 void launch_prep(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
                  uint32_t* cnt, uint32_t* slots, int tps, cudaStream_t st);
 void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items,
@@ -19,6 +20,9 @@ void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, in
                       cudaStream_t st);
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, cudaStream_t st);
+void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
+                    const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr,
+                    cudaStream_t st);
 void launch_atomic(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, float* out,
                    cudaStream_t st);
 void launch_quantize(const float* img, int64_t npix, int bits, void* out, int num_sms, cudaStream_t st);

@@ -27,6 +27,7 @@
 
 #include "common.cuh"
 #include "launch.h"
+#include "tile_common.cuh"
 
 namespace starsim {
 
@@ -332,96 +333,8 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
   }
 
   // ======================= output: rows 16 B + hq + 4 i, columns 64 wx + 8 q .. +7 of the tile
-  const int col0 = X0 + 64 * wx + 8 * q;
-  if (wi.aux != ITEM_WHOLE) {
-    // one part of a split tile: store the partial, and the last part to finish reduces all parts in order
-    const uint2 sp = split_tab[wi.aux >> 12];
-    float* pbuf = part_buf + (size_t)(sp.x + (wi.aux & 0xFFFu)) * (TILE_W * TILE_H);
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      float4* o = reinterpret_cast<float4*>(pbuf + (16 * B + hq + 4 * i) * TILE_W + 64 * wx + 8 * q);
-      o[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
-      o[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
-    }
-    __threadfence();
-    __syncthreads();
-    if (tid == 0) s_last = atomicAdd(&done[wi.aux >> 12], 1u) == sp.y - 1;
-    __syncthreads();
-    if (!s_last) continue;
-    __threadfence();
-#pragma unroll
-    for (int i = 0; i < 4; ++i)
-#pragma unroll
-      for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
-    for (uint32_t k = 0; k < sp.y; ++k) {
-      const float* pk = part_buf + (size_t)(sp.x + k) * (TILE_W * TILE_H);
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const float4* o = reinterpret_cast<const float4*>(pk + (16 * B + hq + 4 * i) * TILE_W + 64 * wx + 8 * q);
-        const float4 u = __ldcg(o), v = __ldcg(o + 1);
-        acc[i][0] = __fadd2_rn(acc[i][0], make_float2(u.x, u.y));
-        acc[i][1] = __fadd2_rn(acc[i][1], make_float2(u.z, u.w));
-        acc[i][2] = __fadd2_rn(acc[i][2], make_float2(v.x, v.y));
-        acc[i][3] = __fadd2_rn(acc[i][3], make_float2(v.z, v.w));
-      }
-    }
-  }
-  if (fp.obits == 0) {
-    float* out = reinterpret_cast<float*>(out_);
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int row = Y0 + 16 * B + hq + 4 * i;  // band-relative
-      if (row >= fp.rows || col0 >= fp.W) continue;
-      float* o = out + (int64_t)row * fp.W + col0;
-      if (fp.vec && col0 + 8 <= fp.W) {
-        reinterpret_cast<float4*>(o)[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
-        reinterpret_cast<float4*>(o)[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
-      } else {
-        const float v[8] = {acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y,
-                            acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y};
-#pragma unroll
-        for (int k = 0; k < 8; ++k)
-          if (col0 + k < fp.W) o[k] = v[k];
-      }
-    }
-  } else {
-    // fused output stage (NEXT-1): the gray value of each pixel, exactly as k_quantize would compute it from the
-    // same fp32 sum, written as u8 / u16
-    const float qmax = fp.obits == 8 ? 255.f : 65535.f;
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int row = Y0 + 16 * B + hq + 4 * i;
-      if (row >= fp.rows || col0 >= fp.W) continue;
-      uint32_t g[8];
-#pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        g[2 * k] = quant1(acc[i][k].x, qmax);
-        g[2 * k + 1] = quant1(acc[i][k].y, qmax);
-      }
-      const int64_t pix = (int64_t)row * fp.W + col0;
-      if (fp.obits == 8) {
-        uint8_t* o = reinterpret_cast<uint8_t*>(out_) + pix;
-        if (fp.vec && col0 + 8 <= fp.W) {
-          *reinterpret_cast<uint2*>(o) = make_uint2(g[0] | g[1] << 8 | g[2] << 16 | g[3] << 24,
-                                                    g[4] | g[5] << 8 | g[6] << 16 | g[7] << 24);
-        } else {
-#pragma unroll
-          for (int k = 0; k < 8; ++k)
-            if (col0 + k < fp.W) o[k] = (uint8_t)g[k];
-        }
-      } else {
-        uint16_t* o = reinterpret_cast<uint16_t*>(out_) + pix;
-        if (fp.vec && col0 + 8 <= fp.W) {
-          *reinterpret_cast<uint4*>(o) = make_uint4(g[0] | g[1] << 16, g[2] | g[3] << 16, g[4] | g[5] << 16,
-                                                    g[6] | g[7] << 16);
-        } else {
-#pragma unroll
-          for (int k = 0; k < 8; ++k)
-            if (col0 + k < fp.W) o[k] = (uint16_t)g[k];
-        }
-      }
-    }
-  }
+  if (!tile_reduce_parts(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last)) continue;
+  tile_store(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
   }  // work loop
 }
 
@@ -432,6 +345,10 @@ void init_tile_kernel() {
 
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, cudaStream_t st) {
+  if (fp.R <= SB_MAXR && fp.tile_impl == 0) {
+    launch_tile_sb(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, st);
+    return;
+  }
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
   const int64_t maxitems = ntiles + part_cap;

@@ -1,0 +1,114 @@
+// Pieces shared by the two tile-accumulation kernels (tile.cu: per-block entry lists, any R; tile_sb.cu: sorted
+// corner bins, R <= SB_MAXR).  Both use the same lane layout: warp (wx, B) owns the 64 x 16 block at tile columns
+// 64 wx, rows 16 B; lane group q = lane/4 owns the 8-column strip Q = 8 wx + q, lane hq = lane%4 the rows
+// 16 B + hq + 4 i (i = 0..3), as 4 x 4 float2 accumulators (columns 8 Q + 2 k, 8 Q + 2 k + 1 in acc[i][k]).
+#pragma once
+#include "common.cuh"
+
+namespace starsim {
+
+// A whole tile is written to `out` directly; a part of a split heavy tile (wi.aux != ITEM_WHOLE) writes its
+// 128 x 64 partial to part_buf, and the last part to finish (per-tile counter) sums the parts in part order -- a
+// fixed order, so the image stays deterministic.  Returns false for a part that is not the last one (nothing left
+// to write); on true, acc holds the tile's final sums.  Contains block barriers: every thread of the CTA calls it.
+__device__ __forceinline__ bool tile_reduce_parts(float2 (&acc)[4][4], const WorkItem& wi,
+                                                  const uint2* __restrict__ split_tab, float* __restrict__ part_buf,
+                                                  uint32_t* __restrict__ done, int B, int wx, int q, int hq,
+                                                  int* s_last) {
+  if (wi.aux == ITEM_WHOLE) return true;
+  const int tid = threadIdx.x;
+  const uint2 sp = split_tab[wi.aux >> 12];
+  float* pbuf = part_buf + (size_t)(sp.x + (wi.aux & 0xFFFu)) * (TILE_W * TILE_H);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    float4* o = reinterpret_cast<float4*>(pbuf + (16 * B + hq + 4 * i) * TILE_W + 64 * wx + 8 * q);
+    o[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
+    o[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
+  }
+  __threadfence();
+  __syncthreads();
+  if (tid == 0) *s_last = atomicAdd(&done[wi.aux >> 12], 1u) == sp.y - 1;
+  __syncthreads();
+  if (!*s_last) return false;
+  __threadfence();
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
+  for (uint32_t k = 0; k < sp.y; ++k) {
+    const float* pk = part_buf + (size_t)(sp.x + k) * (TILE_W * TILE_H);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float4* o = reinterpret_cast<const float4*>(pk + (16 * B + hq + 4 * i) * TILE_W + 64 * wx + 8 * q);
+      const float4 u = __ldcg(o), v = __ldcg(o + 1);
+      acc[i][0] = __fadd2_rn(acc[i][0], make_float2(u.x, u.y));
+      acc[i][1] = __fadd2_rn(acc[i][1], make_float2(u.z, u.w));
+      acc[i][2] = __fadd2_rn(acc[i][2], make_float2(v.x, v.y));
+      acc[i][3] = __fadd2_rn(acc[i][3], make_float2(v.z, v.w));
+    }
+  }
+  return true;
+}
+
+// Write the lane's 4 rows x 8 columns of the tile (rows Y0 + 16 B + hq + 4 i of the band, columns col0 .. col0+7):
+// fp32, or (fused output stage, NEXT-1) the gray value of each pixel exactly as k_quantize computes it from the same
+// fp32 sum, as u8 / u16.  Coalesced: the 8 lane groups of a warp store 8 adjacent 8-pixel runs of a row.
+__device__ __forceinline__ void tile_store(const float2 (&acc)[4][4], const FrameParams& fp, void* __restrict__ out_,
+                                           int Y0, int col0, int B, int hq) {
+  if (fp.obits == 0) {
+    float* out = reinterpret_cast<float*>(out_);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int row = Y0 + 16 * B + hq + 4 * i;  // band-relative
+      if (row >= fp.rows || col0 >= fp.W) continue;
+      float* o = out + (int64_t)row * fp.W + col0;
+      if (fp.vec && col0 + 8 <= fp.W) {
+        reinterpret_cast<float4*>(o)[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
+        reinterpret_cast<float4*>(o)[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
+      } else {
+        const float v[8] = {acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y,
+                            acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y};
+#pragma unroll
+        for (int k = 0; k < 8; ++k)
+          if (col0 + k < fp.W) o[k] = v[k];
+      }
+    }
+  } else {
+    const float qmax = fp.obits == 8 ? 255.f : 65535.f;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int row = Y0 + 16 * B + hq + 4 * i;
+      if (row >= fp.rows || col0 >= fp.W) continue;
+      uint32_t g[8];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        g[2 * k] = quant1(acc[i][k].x, qmax);
+        g[2 * k + 1] = quant1(acc[i][k].y, qmax);
+      }
+      const int64_t pix = (int64_t)row * fp.W + col0;
+      if (fp.obits == 8) {
+        uint8_t* o = reinterpret_cast<uint8_t*>(out_) + pix;
+        if (fp.vec && col0 + 8 <= fp.W) {
+          *reinterpret_cast<uint2*>(o) = make_uint2(g[0] | g[1] << 8 | g[2] << 16 | g[3] << 24,
+                                                    g[4] | g[5] << 8 | g[6] << 16 | g[7] << 24);
+        } else {
+#pragma unroll
+          for (int k = 0; k < 8; ++k)
+            if (col0 + k < fp.W) o[k] = (uint8_t)g[k];
+        }
+      } else {
+        uint16_t* o = reinterpret_cast<uint16_t*>(out_) + pix;
+        if (fp.vec && col0 + 8 <= fp.W) {
+          *reinterpret_cast<uint4*>(o) = make_uint4(g[0] | g[1] << 16, g[2] | g[3] << 16, g[4] | g[5] << 16,
+                                                    g[6] | g[7] << 16);
+        } else {
+#pragma unroll
+          for (int k = 0; k < 8; ++k)
+            if (col0 + k < fp.W) o[k] = (uint16_t)g[k];
+        }
+      }
+    }
+  }
+}
+
+}  // namespace starsim

@@ -1,0 +1,297 @@
+// Tile accumulation with sorted corner bins (DESIGN.md §The tile kernel) -- the kernel for
+// R <= SB_MAXR (every BASELINE config except the wide-ROI end of the C4 sweep, which uses tile.cu).
+//
+// Same contract, tile geometry, lane layout and epilogue as tile.cu (tile_common.cuh): one CTA renders one 128 x 64
+// tile (or one part of a split heavy tile) from its CSR star list, accumulating Eq. 3's sum of separable Eq. 2 terms
+// [s' gy(r)] * gx(c) in fp32 registers, and writes every pixel once.  What differs is how a chunk of up to 256 stars
+// is prepared and walked:
+//
+//   sort   (thread = star): the star's ROI clipped to the tile starts in band b0 = r0/16 and strip q0 = c0/8 (its
+//          "corner bin", 4 x 16 bins).  A stable counting sort by corner bin (warp match + per-warp histogram + one
+//          scan) gives the star its sorted index j.  For R <= 17 the ROI spans at most 2 bands and 3 strips, so the
+//          stars that can touch the block (B, Q) of lane group q are exactly those with corner bins
+//          (B-1, Q-2..Q) and (B, Q-2..Q): two contiguous ranges of the sorted order.  No per-block lists are built.
+//   prep   (thread = star): its row profile s' gy on its two bands b0, b0+1 (16-float band slots in the [hq][i]
+//          order the lanes read) and its column profile gx on strips q0..q0+2 (8-float strip slots in a ring of
+//          4 indexed by Q & 3), zero outside the ROI, at fixed places of sorted star j: one MUFU.EX2 per value.
+//   accumulate (warp): lane group q walks its two ranges (band slot 1 for the corner band B-1, band slot 0 for B),
+//          padded with an all-zero slot to the warp's longest walk; a step is three LDS.128 (4 row factors, 8 column
+//          factors) and 16 FFMA2.  Stars of a range that do not reach the block read all-zero slots (exact zeros).
+//
+// Bank conflicts: strip slot of strip Q sits at ring position Q & 3 with its two 16-B halves swapped when bit 2 of
+// Q is set, so the 8 lane groups of a warp always hit 8 distinct bank quads; band slot k of star j sits in the half
+// (j ^ k) & 1 of the star's 128 B, spreading the groups of a warp over both halves.
+//
+// Summation order of a pixel: range 1 then range 2, each in sorted order (corner bin, then the tile list's star
+// order) -- deterministic, and a function of the tile's own list only, so band renders stay bitwise equal to the
+// frame (reading R12).  No atomics on the image.
+#include <algorithm>
+
+#include "common.cuh"
+#include "launch.h"
+#include "tile_common.cuh"
+
+namespace starsim {
+
+constexpr int SB_NBIN = NBANDS * NSTRIPS;  // 64 corner bins (band-major)
+constexpr uint32_t SB_ZJ = CHUNK;           // the all-zero slot
+
+struct SbSmem {
+  float gy[(CHUNK + 1) * 32];    // sorted star j: two 16-float band slots, slot k at j*32 + ((j ^ k) & 1) * 16
+  float gx[(CHUNK + 1) * 32];    // sorted star j: ring of four 8-float strip slots, strip Q at j*32 + (Q & 3) * 8
+  uint32_t hist[TILE_WARPS][SB_NBIN];      // per warp: stars of each corner bin
+  uint32_t binoff[SB_NBIN][TILE_WARPS];    // per bin: stars of the bin in the warps before
+  uint32_t binstart[SB_NBIN + 1];          // exclusive scan of the bin totals (bin-major)
+};
+
+template <bool INTEG>
+__global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __restrict__ ids,
+                                                             const StarRec* __restrict__ rec, FrameParams fp,
+                                                             void* __restrict__ out_,
+                                                             const WorkItem* __restrict__ items,
+                                                             const uint2* __restrict__ split_tab,
+                                                             float* __restrict__ part_buf,
+                                                             uint32_t* __restrict__ done, Header* hdr) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  SbSmem& S = *reinterpret_cast<SbSmem*>(smem_raw);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  // exp(-d^2 / 2 sigma^2) = 2^(-(d * sk)^2); d = pixel - centre is formed exactly (tile-relative integer minus the
+  // tile-relative centre, both exact in fp32) before the one scaling rounding.
+  const float sk = fp.sk;
+
+  const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
+  const int Q = 8 * wx + q;
+  const int swz = (Q >> 2) & 1;
+  const uint32_t gy_base = (uint32_t)__cvta_generic_to_shared(S.gy) + 16u * hq;
+  const uint32_t gx_base = (uint32_t)__cvta_generic_to_shared(S.gx) + 32u * (Q & 3);
+  // the strip halves of lanes with swz = 1 are stored swapped: those lanes load columns 4-7 first and hold them in
+  // acc[i][0..1] until the epilogue swaps them back (so both loads use the same address + an immediate offset)
+  __shared__ int s_last;
+  if (tid < 32) {
+    S.gy[SB_ZJ * 32 + tid] = 0.f;
+    S.gx[SB_ZJ * 32 + tid] = 0.f;
+  }
+
+  if (blockIdx.x >= __ldcg(&hdr->nitems)) return;
+  const WorkItem wi = items[blockIdx.x];
+  const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
+  const int X0 = tx * TILE_W;    // first column of the tile
+  const int Y0 = ty * TILE_H;    // first row of the tile, relative to the band
+  const int IY0 = fp.row0 + Y0;  // first image row of the tile
+  const int TWe = min(TILE_W, fp.W - X0), THe = min(TILE_H, fp.rows - Y0);
+  float2 acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
+
+  const uint32_t j1 = wi.je;
+  StarRec rnext = {};
+  if (wi.jb + tid < j1) rnext = rec[ids[wi.jb + tid]];
+  for (uint32_t base = wi.jb; base < j1; base += CHUNK) {
+    // ======================= sort: thread = star (base + tid) of the tile's list
+    const int nvalid = (int)min((uint32_t)CHUNK, j1 - base);
+    const StarRec r = rnext;
+    int c0 = 0, c1 = -1, r0 = 0, r1 = -1;
+    uint32_t key = SB_NBIN;
+    if (tid < nvalid) {
+      const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
+      c0 = max(lx, 0);
+      c1 = min(lx + fp.R - 1, TWe - 1);
+      r0 = max(ly, 0);
+      r1 = min(ly + fp.R - 1, THe - 1);
+      if (c0 <= c1 && r0 <= r1) key = (uint32_t)((r0 >> 4) * NSTRIPS + (c0 >> 3));
+    }
+    const uint32_t peers = __match_any_sync(0xffffffffu, key);
+    const uint32_t rank = __popc(peers & lt);
+    // No barrier before this: the previous chunk's readers of hist (warp 0's scan) finished before its second
+    // barrier; binstart / the slots are rewritten only after the next barrier.
+    S.hist[warp][lane] = 0u;
+    S.hist[warp][lane + 32] = 0u;
+    __syncwarp();
+    if (rank == 0 && key < SB_NBIN) S.hist[warp][key] = __popc(peers);
+    // next chunk's star id now (its record is requested just before the accumulation)
+    const uint32_t nb = base + CHUNK;
+    const uint32_t nid = nb + tid < j1 ? __ldg(&ids[nb + tid]) : 0u;
+    __syncthreads();
+    if (warp == 0) {
+      uint32_t tot[2];
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int bin = 2 * lane + h;
+        uint32_t run = 0;
+#pragma unroll
+        for (int w = 0; w < TILE_WARPS; ++w) {
+          S.binoff[bin][w] = run;
+          run += S.hist[w][bin];
+        }
+        tot[h] = run;
+      }
+      const uint32_t s = tot[0] + tot[1];
+      uint32_t incl = s;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += v;
+      }
+      S.binstart[2 * lane] = incl - s;
+      S.binstart[2 * lane + 1] = incl - s + tot[0];
+      if (lane == 31) S.binstart[SB_NBIN] = incl;
+    }
+    __syncthreads();
+    // ======================= prep: the star's profiles at its sorted place j
+    if (key < SB_NBIN) {
+      const uint32_t j = S.binstart[key] + S.binoff[key][warp] + rank;
+      const float yr = r.y - (float)IY0, xr = r.x - (float)X0;  // exact
+      const float2 sk2 = make_float2(sk, sk), s2 = make_float2(r.s, r.s);
+      const int b0 = r0 >> 4, q0 = c0 >> 3;
+      // band slots: the 8 quads (band k, row group h: rows h + 4 i) are written in an order rotated by the lane, so
+      // that each STS.128 of the warp hits all 8 bank quads (slot half (j ^ k) & 1 = u & 1, h = u >> 1)
+      const int ra0 = r0 - 16 * b0, rb0 = r1 - 16 * b0;      // ROI rows relative to band b0 (band b0+1: -16)
+      const uint32_t m0 = (0xFFFFFFFFu >> (31 - min(rb0, 31))) & (0xFFFFFFFFu << ra0);  // ROI rows over both bands
+      const float bf0 = (float)(16 * b0) - yr;              // exact
+#pragma unroll
+      for (int c = 0; c < 8; ++c) {
+        const int u = (c + lane) & 7;
+        const int hh = u >> 1, k = (u ^ (int)j) & 1;
+        const uint32_t m = m0 >> (16 * k + hh);            // bit 4 i: row hh + 4 i of band b0 + k in the ROI
+        const float bf = bf0 + (float)(16 * k + hh);        // exact
+        float v[4];
+        if (!INTEG) {
+          const float2 bb = make_float2(bf, bf);
+#pragma unroll
+          for (int i = 0; i < 4; i += 2) {
+            float2 d = __fadd2_rn(bb, make_float2((float)(4 * i), (float)(4 * i + 4)));
+            d = __fmul2_rn(d, sk2);
+            d = __fmul2_rn(d, make_float2(-d.x, -d.y));
+            const float2 e = __fmul2_rn(make_float2(ex2_approx(d.x), ex2_approx(d.y)), s2);
+            v[i] = (m >> (4 * i)) & 1u ? e.x : 0.f;
+            v[i + 1] = (m >> (4 * i + 4)) & 1u ? e.y : 0.f;
+          }
+        } else {
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const float t0 = (bf + (float)(4 * i) - 0.5f) * fp.kint, t1 = (bf + (float)(4 * i) + 0.5f) * fp.kint;
+            v[i] = (m >> (4 * i)) & 1u ? r.s * pix_mass(t0, edge_erfc(t0), t1, edge_erfc(t1)) : 0.f;
+          }
+        }
+        *reinterpret_cast<float4*>(&S.gy[j * 32 + (u & 1) * 16 + hh * 4]) = make_float4(v[0], v[1], v[2], v[3]);
+      }
+#pragma unroll
+      for (int k = 0; k < 3; ++k) {
+        const int Qs = q0 + k;
+        const int rel = 8 * Qs;                              // first column of the strip (tile-relative)
+        const int lo = max(c0 - rel, 0), hi = min(c1 - rel, 7);
+        const uint32_t m = hi >= lo ? ((0xFFu >> (7 - hi)) & (0xFFu << lo)) : 0u;
+        const float bf = (float)rel - xr;                    // exact
+        float v[8];
+        if (!INTEG) {
+#pragma unroll
+          for (int p = 0; p < 8; p += 2) {
+            float2 d = __fmul2_rn(__fadd2_rn(make_float2(bf, bf), make_float2((float)p, (float)(p + 1))), sk2);
+            d = __fmul2_rn(d, make_float2(-d.x, -d.y));
+            v[p] = (m >> p) & 1u ? ex2_approx(d.x) : 0.f;
+            v[p + 1] = (m >> (p + 1)) & 1u ? ex2_approx(d.y) : 0.f;
+          }
+        } else {
+          float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
+#pragma unroll
+          for (int p = 0; p < 8; ++p) {
+            const float tn = (bf + (float)p + 0.5f) * fp.kint, en = edge_erfc(tn);
+            v[p] = (m >> p) & 1u ? pix_mass(t, e, tn, en) : 0.f;
+            t = tn;
+            e = en;
+          }
+        }
+        float* gs = &S.gx[j * 32 + (Qs & 3) * 8];
+        const int sw = ((Qs >> 2) & 1) * 4;
+        *reinterpret_cast<float4*>(gs + sw) = make_float4(v[0], v[1], v[2], v[3]);
+        *reinterpret_cast<float4*>(gs + (sw ^ 4)) = make_float4(v[4], v[5], v[6], v[7]);
+      }
+    }
+    // this lane group's two ranges of the sorted order: corner bins (B-1, qlo..Q) then (B, qlo..Q)
+    const int qlo = max(Q - 2, 0);
+    const uint32_t s2r = S.binstart[B * NSTRIPS + qlo], e2r = S.binstart[B * NSTRIPS + Q + 1];
+    uint32_t s1r = 0, e1r = 0;
+    if (B > 0) {
+      s1r = S.binstart[(B - 1) * NSTRIPS + qlo];
+      e1r = S.binstart[(B - 1) * NSTRIPS + Q + 1];
+    }
+    const uint32_t len1 = e1r - s1r, L = len1 + (e2r - s2r);
+    const uint32_t steps = __reduce_max_sync(0xffffffffu, L);
+    // step t of the walk reads sorted star j = t + c (c = s1r in range 1, s2r - len1 in range 2); its band slot
+    // k (1 in range 1, 0 in range 2) sits in half (j ^ k) & 1 = (t & 1) ^ ((c + k) & 1).  So per range and per
+    // parity of t the gy address is base + 128 t: the loop below runs step pairs (even, odd).
+    const uint32_t c1v = s1r, c2v = s2r - len1;
+    const uint32_t e1 = (c1v + 1u) & 1u, e2 = c2v & 1u;
+    const uint32_t g1e = gy_base + c1v * 128u + e1 * 64u, g1o = gy_base + c1v * 128u + (e1 ^ 1u) * 64u;
+    const uint32_t g2e = gy_base + c2v * 128u + e2 * 64u, g2o = gy_base + c2v * 128u + (e2 ^ 1u) * 64u;
+    const uint32_t x1 = gx_base + c1v * 128u, x2 = gx_base + c2v * 128u;
+    const uint32_t gz = gy_base + SB_ZJ * 128u, xz = gx_base + SB_ZJ * 128u;
+    __syncthreads();
+
+    if (nb + tid < j1) rnext = rec[nid];
+    // ======================= accumulate: lane group q walks its two ranges (padded with the zero slot)
+#pragma unroll 2
+    for (uint32_t st = 0; st < steps; st += 2) {
+#pragma unroll
+      for (uint32_t o = 0; o < 2; ++o) {
+        const uint32_t t = st + o;
+        const bool in1 = t < len1, in = t < L;
+        uint32_t ga = (in1 ? (o ? g1o : g1e) : (o ? g2o : g2e)) + t * 128u;
+        uint32_t xa = (in1 ? x1 : x2) + t * 128u;
+        ga = in ? ga : gz;
+        xa = in ? xa : xz;
+        float4 g, a, c;
+        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(g.x), "=f"(g.y), "=f"(g.z), "=f"(g.w) : "r"(ga));
+        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "r"(xa));
+        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(c.x), "=f"(c.y), "=f"(c.z), "=f"(c.w) : "r"(xa + 16u));
+        const float gi[4] = {g.x, g.y, g.z, g.w};
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const float2 gg = make_float2(gi[i], gi[i]);
+          acc[i][0] = __ffma2_rn(gg, make_float2(a.x, a.y), acc[i][0]);
+          acc[i][1] = __ffma2_rn(gg, make_float2(a.z, a.w), acc[i][1]);
+          acc[i][2] = __ffma2_rn(gg, make_float2(c.x, c.y), acc[i][2]);
+          acc[i][3] = __ffma2_rn(gg, make_float2(c.z, c.w), acc[i][3]);
+        }
+      }
+    }
+  }
+
+  // ======================= output
+  if (swz) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float2 t0 = acc[i][0], t1 = acc[i][1];
+      acc[i][0] = acc[i][2];
+      acc[i][1] = acc[i][3];
+      acc[i][2] = t0;
+      acc[i][3] = t1;
+    }
+  }
+  if (!tile_reduce_parts(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last)) return;
+  tile_store(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+}
+
+void init_tile_sb_kernel() {
+  cudaFuncSetAttribute(k_tile_sb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SbSmem));
+  cudaFuncSetAttribute(k_tile_sb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SbSmem));
+}
+
+void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
+                    const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr,
+                    cudaStream_t st) {
+  const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
+  if (ntiles <= 0) return;
+  const int64_t grid = ntiles + part_cap;  // one CTA per possible item (parts first); the rest exit at once
+  if (fp.psf)
+    k_tile_sb<true><<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab,
+                                                                          part_buf, done, hdr);
+  else
+    k_tile_sb<false><<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab,
+                                                                           part_buf, done, hdr);
+}
+
+}  // namespace starsim

@@ -57,6 +57,8 @@ def lib():
         L.starsim_render_gray.restype = ctypes.c_int
         L.starsim_set_psf.argtypes = [vp, i32]
         L.starsim_set_psf.restype = ctypes.c_int
+        L.starsim_set_tile_kernel.argtypes = [vp, i32]
+        L.starsim_set_tile_kernel.restype = ctypes.c_int
         L.starsim_render_atomic.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
         L.starsim_render_atomic.restype = ctypes.c_int
         L.starsim_upload_aos.argtypes = [vp, vp, i64, vp, vp, vp, vp]
@@ -135,6 +137,13 @@ PSF_MODES = {"point": 0, "integrated": 1}
 
 def starsim_set_psf(h, mode) -> None:
     _check(h, lib().starsim_set_psf(h, PSF_MODES.get(mode, mode) if isinstance(mode, str) else int(mode)))
+
+
+TILE_KERNELS = {"auto": 0, "lists": 1}
+
+
+def starsim_set_tile_kernel(h, mode) -> None:
+    _check(h, lib().starsim_set_tile_kernel(h, TILE_KERNELS.get(mode, mode) if isinstance(mode, str) else int(mode)))
 
 
 def starsim_render_band(h, x, y, mag, width, height, row0, rows, sigma, roi, gain, out_band, stream=None) -> None:
@@ -252,6 +261,10 @@ class Context:
     def set_psf(self, mode="point"):
         """"point" (Eq. 2 sampled at the pixel, the paper) or "integrated" (Eq. 2 integrated over the pixel)."""
         starsim_set_psf(self.h, mode)
+
+    def set_tile_kernel(self, mode="auto"):
+        """"auto" (sorted-corner-bin kernel for R <= 17, else the list kernel) or "lists" (always the list kernel)."""
+        starsim_set_tile_kernel(self.h, mode)
 
     def render_band(self, x, y, mag, width, height, row0, rows, sigma, roi, gain, out=None, stream=None):
         out = self._out(rows, width, out)

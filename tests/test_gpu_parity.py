@@ -29,10 +29,13 @@ def torch_dev():
     return torch, torch.device("cuda:0")
 
 
-@pytest.fixture(scope="module")
-def ctx(torch_dev):
+@pytest.fixture(scope="module", params=["auto", "lists"])
+def ctx(torch_dev, request):
+    """Every test runs against both tile kernels: "auto" (the sorted-corner-bin kernel for R <= 17, the list kernel
+    above) and "lists" (the per-block entry-list kernel for every R)."""
     from paper_conf_ipps_lizzh12_b200 import Context
     c = Context(0)
+    c.set_tile_kernel(request.param)
     yield c
     c.close()
 

@@ -27,6 +27,7 @@ def main():
     ap.add_argument("--n", type=int, default=0)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--atomic", action="store_true")
+    ap.add_argument("--tile", default="auto", help="tile kernel: auto | lists")
     a = ap.parse_args()
     cfg = synth.CONFIGS[a.config]
     if a.R:
@@ -37,6 +38,7 @@ def main():
     gain = synth.bench_gain(cfg.sigma)
     out = torch.empty((cfg.H, cfg.W), dtype=torch.float32, device=dev)
     with Context(0) as ctx:
+        ctx.set_tile_kernel(a.tile)
         fn = ctx.render_atomic if a.atomic else ctx.render
         for _ in range(a.reps + 2):
             fn(x, y, m, cfg.W, cfg.H, cfg.sigma, cfg.R, gain, out=out)
