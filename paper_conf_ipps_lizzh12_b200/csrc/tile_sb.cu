@@ -33,7 +33,10 @@
 
 namespace starsim {
 
-constexpr int SB_NBIN = NBANDS * NSTRIPS;  // 64 corner bins (band-major)
+// corner bins: band key 0..4 (0 = the ROI comes in over the tile's top edge, else 1 + band) x strip key 0..16 (0 =
+// it comes in over the left edge, else 1 + strip), band-major
+constexpr int SB_NSK = NSTRIPS + 1;
+constexpr int SB_NBIN = (NBANDS + 1) * SB_NSK;  // 85
 constexpr uint32_t SB_ZJ = CHUNK;           // the all-zero slot
 
 struct SbSmem {
@@ -101,7 +104,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
       c1 = min(lx + fp.R - 1, TWe - 1);
       r0 = max(ly, 0);
       r1 = min(ly + fp.R - 1, THe - 1);
-      if (c0 <= c1 && r0 <= r1) key = (uint32_t)((r0 >> 4) * NSTRIPS + (c0 >> 3));
+      if (c0 <= c1 && r0 <= r1) key = (uint32_t)((ly < 0 ? 0 : 1 + (r0 >> 4)) * SB_NSK + (lx < 0 ? 0 : 1 + (c0 >> 3)));
     }
     const uint32_t peers = __match_any_sync(0xffffffffu, key);
     const uint32_t rank = __popc(peers & lt);
@@ -109,6 +112,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
     // barrier; binstart / the slots are rewritten only after the next barrier.
     S.hist[warp][lane] = 0u;
     S.hist[warp][lane + 32] = 0u;
+    if (lane < SB_NBIN - 64) S.hist[warp][lane + 64] = 0u;
     __syncwarp();
     if (rank == 0 && key < SB_NBIN) S.hist[warp][key] = __popc(peers);
     // next chunk's star id now (its record is requested just before the accumulation)
@@ -116,28 +120,34 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
     const uint32_t nid = nb + tid < j1 ? __ldg(&ids[nb + tid]) : 0u;
     __syncthreads();
     if (warp == 0) {
-      uint32_t tot[2];
+      uint32_t tot[3], sum = 0;
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const int bin = 2 * lane + h;
+      for (int h = 0; h < 3; ++h) {
+        const int bin = 3 * lane + h;
         uint32_t run = 0;
+        if (bin < SB_NBIN) {
 #pragma unroll
-        for (int w = 0; w < TILE_WARPS; ++w) {
-          S.binoff[bin][w] = run;
-          run += S.hist[w][bin];
+          for (int w = 0; w < TILE_WARPS; ++w) {
+            S.binoff[bin][w] = run;
+            run += S.hist[w][bin];
+          }
         }
         tot[h] = run;
+        sum += run;
       }
-      const uint32_t s = tot[0] + tot[1];
-      uint32_t incl = s;
+      uint32_t incl = sum;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
         if (lane >= o) incl += v;
       }
-      S.binstart[2 * lane] = incl - s;
-      S.binstart[2 * lane + 1] = incl - s + tot[0];
-      if (lane == 31) S.binstart[SB_NBIN] = incl;
+      uint32_t ex = incl - sum;
+#pragma unroll
+      for (int h = 0; h < 3; ++h) {
+        const int bin = 3 * lane + h;
+        if (bin <= SB_NBIN) S.binstart[bin] = ex;  // bin SB_NBIN (lane 28, h 1) receives the total
+        ex += tot[h];
+      }
     }
     __syncthreads();
     // ======================= prep: the star's profiles at its sorted place j
@@ -145,7 +155,8 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
       const uint32_t j = S.binstart[key] + S.binoff[key][warp] + rank;
       const float yr = r.y - (float)IY0, xr = r.x - (float)X0;  // exact
       const float2 sk2 = make_float2(sk, sk), s2 = make_float2(r.s, r.s);
-      const int b0 = r0 >> 4, q0 = c0 >> 3;
+      // first band / strip of the slots: the corner bin's (-1 for an ROI that comes in over the top / left edge)
+      const int b0 = (int)(key / SB_NSK) - 1, q0 = (int)(key % SB_NSK) - 1;
       // band slots: the 8 quads (band k, row group h: rows h + 4 i) are written in an order rotated by the lane, so
       // that each STS.128 of the warp hits all 8 bank quads (slot half (j ^ k) & 1 = u & 1, h = u >> 1)
       const int ra0 = r0 - 16 * b0, rb0 = r1 - 16 * b0;      // ROI rows relative to band b0 (band b0+1: -16)
@@ -211,13 +222,10 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
       }
     }
     // this lane group's two ranges of the sorted order: corner bins (B-1, qlo..Q) then (B, qlo..Q)
-    const int qlo = max(Q - 2, 0);
-    const uint32_t s2r = S.binstart[B * NSTRIPS + qlo], e2r = S.binstart[B * NSTRIPS + Q + 1];
-    uint32_t s1r = 0, e1r = 0;
-    if (B > 0) {
-      s1r = S.binstart[(B - 1) * NSTRIPS + qlo];
-      e1r = S.binstart[(B - 1) * NSTRIPS + Q + 1];
-    }
+    // strip keys max(Q-2, -1) + 1 .. Q + 1; band key B (corner band B-1, incl. the top-edge key 0), then B + 1
+    const int sklo = max(Q - 1, 0);
+    const uint32_t s1r = S.binstart[B * SB_NSK + sklo], e1r = S.binstart[B * SB_NSK + Q + 2];
+    const uint32_t s2r = S.binstart[(B + 1) * SB_NSK + sklo], e2r = S.binstart[(B + 1) * SB_NSK + Q + 2];
     const uint32_t len1 = e1r - s1r, L = len1 + (e2r - s2r);
     const uint32_t steps = __reduce_max_sync(0xffffffffu, L);
     // step t of the walk reads sorted star j = t + c (c = s1r in range 1, s2r - len1 in range 2); its band slot
