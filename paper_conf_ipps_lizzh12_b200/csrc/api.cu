@@ -24,6 +24,7 @@ struct Buf {
 
 struct Launch {
   int kclass;
+  int n;  // kernels enqueued between the two events
   cudaEvent_t a, b;
 };
 
@@ -50,7 +51,7 @@ struct starsim_ctx {
   int32_t psf = 0;  // starsim_set_psf: 0 point-sampled Eq. 2, 1 pixel-integrated (NEXT-2)
   int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto (sorted bins when R <= 17), 1 per-block lists
   std::string err;
-  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage;
+  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
@@ -134,12 +135,12 @@ cudaEvent_t get_event(starsim_ctx* c) {
 
 // Run `launch` on stream st, bracketed by CUDA events on the same stream when profiling is on.
 template <typename F>
-void timed(starsim_ctx* c, int kclass, cudaStream_t st, F&& launch) {
+void timed(starsim_ctx* c, int kclass, cudaStream_t st, F&& launch, int nlaunch = 1) {
   if (!c->prof) {
     launch();
     return;
   }
-  Launch l{kclass, get_event(c), get_event(c)};
+  Launch l{kclass, nlaunch, get_event(c), get_event(c)};
   cudaEventRecord(l.a, st);
   launch();
   cudaEventRecord(l.b, st);
@@ -189,6 +190,9 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   return fp;
 }
 
+// the deterministic binning of dbin.cu applies (DB_MAXT tiles, an ROI over at most 2 x 2 tiles)
+bool dbin_ok(const FrameParams& fp, int64_t ntiles) { return ntiles <= DB_MAXT && fp.R <= DB_MAXR; }
+
 int tiles_per_axis(int R, int tile, int ntiles_axis) {
   int t = (R - 1 + tile - 1) / tile + 1;
   return t < ntiles_axis ? t : ntiles_axis;
@@ -207,19 +211,44 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
   uint32_t* slots = (uint32_t*)c->slots.p;
   StarRec* rec = (StarRec*)c->rec.p;
   int rc;
-  timed(c, 5, st, [&] { cudaMemsetAsync(hdr, 0, zbytes, st); });
-  if (n > 0) {
-    timed(c, 0, st, [&] { launch_prep(x, y, mag, n, fp, rec, cnt, slots, tps, st); });
-    if ((rc = check_launch(c, "k_prep"))) return rc;
+  if (dbin_ok(fp, ntiles)) {
+    // deterministic counting sort (dbin.cu): no memset, no atomics on global counters, no per-tile sort
+    uint32_t* C = (uint32_t*)c->cmat.p;
+    if (n > 0) {
+      timed(c, 0, st, [&] { launch_dcount(x, y, mag, n, fp, rec, C, (int)ntiles, st); });
+      if ((rc = check_launch(c, "k_dcount"))) return rc;
+    }
+    timed(
+        c, 2, st,
+        [&] {
+          launch_dcolscan(C, n, (int)ntiles, cnt, st);
+          launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap,
+                      c->partial.p, done, st);
+        },
+        3);
+    if ((rc = check_launch(c, "k_dcolscan/k_scan"))) return rc;
+    if (n > 0) {
+      timed(c, 1, st, [&] { launch_dplace(rec, n, fp, C, (int)ntiles, tile_off, ids, st); });
+      if ((rc = check_launch(c, "k_dplace"))) return rc;
+    }
+  } else {
+    timed(c, 5, st, [&] { cudaMemsetAsync(hdr, 0, zbytes, st); });
+    if (n > 0) {
+      timed(c, 0, st, [&] { launch_prep(x, y, mag, n, fp, rec, cnt, slots, tps, st); });
+      if ((rc = check_launch(c, "k_prep"))) return rc;
+    }
+    timed(
+        c, 2, st,
+        [&] {
+          launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap,
+                      c->partial.p, done, st);
+          launch_scatter(rec, n, fp, slots, tps, tile_off, ids, st);
+        },
+        n > 0 ? 3 : 2);
+    if ((rc = check_launch(c, "k_scan/k_scatter"))) return rc;
+    timed(c, 1, st, [&] { launch_sortlists(ids, (uint32_t*)c->tmp.p, tile_off, ntiles, n, st); });
+    if ((rc = check_launch(c, "k_sortlists"))) return rc;
   }
-  timed(c, 2, st, [&] {
-    launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap, c->partial.p,
-                st);
-    launch_scatter(rec, n, fp, slots, tps, tile_off, ids, st);
-  });
-  if ((rc = check_launch(c, "k_scan/k_scatter"))) return rc;
-  timed(c, 1, st, [&] { launch_sortlists(ids, (uint32_t*)c->tmp.p, tile_off, ntiles, n, st); });
-  if ((rc = check_launch(c, "k_sortlists"))) return rc;
   timed(c, 3, st, [&] {
     launch_tile(ids, rec, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p, part_cap, done,
                 hdr, st);
@@ -248,9 +277,10 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   const int part_cap = PART_CAP;
   int rc;
   if ((rc = grow(c, c->rec, sizeof(StarRec) * (size_t)(n > 0 ? n : 1), "records"))) return rc;
-  if ((rc = grow(c, c->slots, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "tile slots"))) return rc;
+  const bool old_bins = !dbin_ok(fp, ntiles);  // bin.cu's pipeline needs the slot and sort scratch
+  if (old_bins && (rc = grow(c, c->slots, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "tile slots"))) return rc;
   if ((rc = grow(c, c->ids, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "tile lists"))) return rc;
-  if ((rc = grow(c, c->tmp, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "sort scratch"))) return rc;
+  if (old_bins && (rc = grow(c, c->tmp, sizeof(uint32_t) * (size_t)(pmax > 0 ? pmax : 1), "sort scratch"))) return rc;
   if ((rc = grow(c, c->tile_off, sizeof(uint32_t) * (size_t)(ntiles + 1), "tile offsets"))) return rc;
   if ((rc = grow(c, c->zeroed, zbytes, "header+counters"))) return rc;
   if ((rc = grow(c, c->items, sizeof(WorkItem) * (size_t)(ntiles + part_cap), "work items"))) return rc;
@@ -258,6 +288,10 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   if ((rc = grow(c, c->partial, sizeof(uint3) * (size_t)((ntiles + SCAN_TILES - 1) / SCAN_TILES), "scan partials")))
     return rc;
   if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
+  if (dbin_ok(fp, ntiles) &&
+      (rc = grow(c, c->cmat, sizeof(uint32_t) * (size_t)ntiles * (size_t)(dbin_ctas(n) > 0 ? dbin_ctas(n) : 1),
+                 "count matrix")))
+    return rc;
 
   const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, c->psf, c->tile_impl, sigma, gain, st, c->scratch_gen};
   if (st == nullptr || c->prof || !c->use_graphs) {
@@ -343,7 +377,7 @@ void starsim_destroy(starsim_ctx* c) {
     cudaDeviceSynchronize();
     if (c->have_graph) cudaGraphExecDestroy(c->gexec);
     Buf* bufs[] = {&c->rec, &c->slots, &c->ids, &c->tmp, &c->tile_off, &c->items, &c->split_tab, &c->parts,
-                   &c->partial, &c->zeroed, &c->stage};
+                   &c->partial, &c->zeroed, &c->stage, &c->cmat};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {
@@ -503,7 +537,7 @@ int starsim_kernel_times(starsim_ctx* c, double* ms, int64_t* launches) {
     float t = 0;
     cudaEventElapsedTime(&t, l.a, l.b);
     c->ms[l.kclass] += t;
-    c->launches[l.kclass] += 1;
+    c->launches[l.kclass] += l.n;
     c->ev_pool.push_back(l.a);
     c->ev_pool.push_back(l.b);
   }

@@ -14,18 +14,9 @@
 
 #include "common.cuh"
 #include "launch.h"
+#include "prep.cuh"
 
 namespace starsim {
-
-// Clipped ROI of a star against the frame columns and the band rows; false if empty.
-__device__ __forceinline__ bool clip_roi(const FrameParams& fp, int lx, int ly, int& cx0, int& cx1, int& cy0,
-                                         int& cy1) {
-  cx0 = max(lx, 0);
-  cx1 = min(lx + fp.R - 1, fp.W - 1);
-  cy0 = max(ly, fp.row0);
-  cy1 = min(ly + fp.R - 1, fp.row0 + fp.rows - 1);
-  return cx0 <= cx1 && cy0 <= cy1;
-}
 
 // ---------------------------------------------------------------------------------------------------------------
 // k_prep -- step a1.  Per star: reject non-finite x, y, mag (reading R11); s' = A 2.512^-m / (2 pi sigma^2) in fp64
@@ -38,30 +29,15 @@ __global__ void __launch_bounds__(PREP_THREADS) k_prep(const float* __restrict__
                                                        uint32_t* __restrict__ slots, int tps) {
   const int64_t i = (int64_t)blockIdx.x * PREP_THREADS + threadIdx.x;
   if (i >= n) return;
-  const float x = X[i], y = Y[i], m = M[i];
-  const float R = (float)fp.R;
-  bool ok = isfinite(x) && isfinite(y) && isfinite(m);
-  // pre-filter far-off stars (keeps the int conversions exact); the exact test is the clip below
-  ok = ok && x > -R - 2.f && x < (float)fp.W + R + 2.f && y > (float)fp.row0 - R - 2.f &&
-       y < (float)(fp.row0 + fp.rows) + R + 2.f;
-  StarRec r;
-  r.x = x;
-  r.y = y;
-  r.s = 0.f;
-  r.lo = LO_CULLED;
-  if (ok) {
-    const int lx = roi_lo_exact(x, fp.R), ly = roi_lo_exact(y, fp.R);
-    int cx0, cx1, cy0, cy1;
-    if (clip_roi(fp, lx, ly, cx0, cx1, cy0, cy1)) {
-      r.lo = ((uint32_t)(uint16_t)(int16_t)lx) | ((uint32_t)(uint16_t)(int16_t)ly << 16);
-      r.s = (float)(fp.s_scale * exp2(-(double)m * 1.3288364642295399628));  // 2.512^-m, Eq. 1
-      const int tx0 = cx0 / TILE_W, tx1 = cx1 / TILE_W;
-      const int ty0 = (cy0 - fp.row0) / TILE_H, ty1 = (cy1 - fp.row0) / TILE_H;
-      uint32_t* sl = slots + i * tps;
-      int k = 0;
-      for (int ty = ty0; ty <= ty1; ++ty)
-        for (int tx = tx0; tx <= tx1; ++tx) sl[k++] = atomicAdd(&cnt[(int64_t)(ty * fp.ntx + tx) * CNT_STRIDE], 1u);
-    }
+  int cx0, cx1, cy0, cy1;
+  const StarRec r = prep_star(X[i], Y[i], M[i], fp, cx0, cx1, cy0, cy1);
+  if (r.lo != LO_CULLED) {
+    const int tx0 = cx0 / TILE_W, tx1 = cx1 / TILE_W;
+    const int ty0 = (cy0 - fp.row0) / TILE_H, ty1 = (cy1 - fp.row0) / TILE_H;
+    uint32_t* sl = slots + i * tps;
+    int k = 0;
+    for (int ty = ty0; ty <= ty1; ++ty)
+      for (int tx = tx0; tx <= tx1; ++tx) sl[k++] = atomicAdd(&cnt[(int64_t)(ty * fp.ntx + tx) * CNT_STRIDE], 1u);
   }
   rec[i] = r;
 }
@@ -138,7 +114,8 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_b(const uint32_t* __restr
                                                          const uint3* __restrict__ partial, int nblk,
                                                          uint32_t* __restrict__ tile_off, Header* hdr,
                                                          WorkItem* __restrict__ items,
-                                                         uint2* __restrict__ split_tab, int part_cap) {
+                                                         uint2* __restrict__ split_tab, int part_cap,
+                                                         uint32_t* __restrict__ done) {
   __shared__ uint3 s_w[SCAN_THREADS / 32];
   const int tid = threadIdx.x;
   // sums of the CTAs before this one, and of all CTAs
@@ -173,6 +150,7 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_b(const uint32_t* __restr
     const uint32_t np = split_on ? parts_of(c[k]) : 0u;
     if (np) {
       split_tab[si] = make_uint2(pb, np);
+      done[si] = 0u;  // the parts' completion counter (k_tile)
       const uint32_t per_part = (c[k] + np - 1) / np;
       for (uint32_t j = 0; j < np; ++j)
         items[pb + j] = WorkItem{(uint32_t)t, run + j * per_part, min(run + c[k], run + (j + 1) * per_part),
@@ -469,11 +447,11 @@ void launch_prep(const float* x, const float* y, const float* m, int64_t n, cons
 }
 
 void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items,
-                 uint2* split_tab, int part_cap, void* partial, cudaStream_t st) {
+                 uint2* split_tab, int part_cap, void* partial, uint32_t* done, cudaStream_t st) {
   const int nblk = (int)((ntiles + SCAN_TILES - 1) / SCAN_TILES);
   k_scan_a<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (uint3*)partial);
   k_scan_b<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (const uint3*)partial, nblk, tile_off, hdr, items, split_tab,
-                                         part_cap);
+                                         part_cap, done);
 }
 
 void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* slots, int tps,
@@ -495,6 +473,7 @@ void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, in
 void init_kernels() {
   init_tile_kernel();
   init_tile_sb_kernel();
+  init_dbin_kernels();
 }
 
 }  // namespace starsim

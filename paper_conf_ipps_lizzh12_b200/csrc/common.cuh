@@ -28,6 +28,9 @@ constexpr int SB_MAXR = 17;                      // tile_sb.cu: an ROI of side <
 // atomics of different tiles never serialise on one L2 line)
 constexpr int CNT_STRIDE = 32;
 constexpr int PREP_THREADS = 256;
+// dbin.cu (deterministic binning): frames / bands with at most DB_MAXT tiles and R <= DB_MAXR
+constexpr int DB_MAXT = 2048;
+constexpr int DB_MAXR = 65;                      // an ROI then overlaps at most 2 x 2 tiles
 // k_scan_a / k_scan_b: SCAN_PER tiles per thread
 constexpr int SCAN_THREADS = 256;
 constexpr int SCAN_PER = 4;

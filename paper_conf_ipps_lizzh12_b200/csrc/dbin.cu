@@ -1,0 +1,237 @@
+// Deterministic binning: a stable counting sort of the (tile, star)
+// pairs by tile, with no global atomics and no per-tile sort.  Used when the frame (or band) has at most DB_MAXT
+// tiles and an ROI overlaps at most 2 x 2 tiles (R <= 65); bin.cu's atomic-slot pipeline covers the rest.
+//
+//   k_dcount     a1 + counts: CTA c takes stars [c*DB_CTA, (c+1)*DB_CTA); per star the record of step a1
+//                (prep_star); per tile the number of pairs of the CTA (shared-memory atomics -- counts do not depend
+//                on order) -> C[tile][c].
+//   k_dcolscan   per tile (one warp): exclusive scan of C[tile][0..nCTA) in CTA order (in place) and the tile's
+//                total -> cnt[tile] (then bin.cu's k_scan_a/b: tile_off, the work list).
+//   k_dplace     CTA c again: its pairs are grouped by tile in shared memory (slots from shared-memory atomics, in
+//                arbitrary order); a pair's rank in its group is the number of the group's stars with a smaller
+//                index, and it goes to tile_off[t] + C[t][c] + rank: every tile list holds its stars in ascending
+//                star index -- the unique CSR (reading R18), bit-exact, with no sort pass over the lists and no
+//                atomics on global memory.  (Groups are (tile, 2048-star block) pairs: a few stars each.)
+#include "common.cuh"
+#include "launch.h"
+#include "prep.cuh"
+
+namespace starsim {
+
+constexpr int DB_CTA = 8192;                     // stars per CTA (one column of the count matrix)
+constexpr int DC_THREADS = 1024;                 // k_dcount: DB_CTA / DC_THREADS stars per thread
+constexpr int DC_PER = DB_CTA / DC_THREADS;
+constexpr int DP_THREADS = 1024;                 // k_dplace
+constexpr int DP_WARPS = DP_THREADS / 32;
+constexpr int DP_KEYS = DB_CTA * 4;              // at most 2 x 2 tiles per star
+constexpr int DP_SPT = DB_CTA / DP_THREADS;      // stars per thread (strided by DP_THREADS)
+constexpr int DCS_THREADS = 256;
+static_assert(DB_MAXT <= 65536 && DB_CTA <= 65536, "tile ids, slots and star indices are 16-bit in k_dplace");
+
+__global__ void __launch_bounds__(DC_THREADS) k_dcount(const float* __restrict__ X, const float* __restrict__ Y,
+                                                       const float* __restrict__ M, int64_t n, FrameParams fp,
+                                                       StarRec* __restrict__ rec, uint32_t* __restrict__ C,
+                                                       int nCTA, int ntiles) {
+  __shared__ uint32_t cnt[DB_MAXT];
+  const int tid = threadIdx.x, cta = blockIdx.x;
+  for (int t = tid; t < ntiles; t += DC_THREADS) cnt[t] = 0u;
+  // all loads of the thread's stars first (one memory latency, not DC_PER)
+  const int64_t i0 = (int64_t)cta * DB_CTA + tid;
+  float xs[DC_PER], ys[DC_PER], ms[DC_PER];
+#pragma unroll
+  for (int k = 0; k < DC_PER; ++k) {
+    const int64_t i = i0 + (int64_t)k * DC_THREADS;
+    const bool in = i < n;
+    xs[k] = in ? __ldg(&X[i]) : 0.f;
+    ys[k] = in ? __ldg(&Y[i]) : 0.f;
+    ms[k] = in ? __ldg(&M[i]) : 0.f;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int k = 0; k < DC_PER; ++k) {
+    const int64_t i = i0 + (int64_t)k * DC_THREADS;
+    if (i >= n) break;
+    int cx0, cx1, cy0, cy1;
+    const StarRec r = prep_star(xs[k], ys[k], ms[k], fp, cx0, cx1, cy0, cy1);
+    rec[i] = r;
+    if (r.lo != LO_CULLED) {
+      const int tx0 = cx0 / TILE_W, tx1 = cx1 / TILE_W;
+      const int ty0 = (cy0 - fp.row0) / TILE_H, ty1 = (cy1 - fp.row0) / TILE_H;
+      for (int ty = ty0; ty <= ty1; ++ty)
+        for (int tx = tx0; tx <= tx1; ++tx) atomicAdd(&cnt[ty * fp.ntx + tx], 1u);
+    }
+  }
+  __syncthreads();
+  for (int t = tid; t < ntiles; t += DC_THREADS) C[(int64_t)t * nCTA + cta] = cnt[t];
+}
+
+__global__ void __launch_bounds__(DCS_THREADS) k_dcolscan(uint32_t* __restrict__ C, int nCTA, int ntiles,
+                                                         uint32_t* __restrict__ cnt) {
+  const int lane = threadIdx.x & 31;
+  const int t = blockIdx.x * (DCS_THREADS / 32) + (threadIdx.x >> 5);
+  if (t >= ntiles) return;
+  uint32_t* row = C + (int64_t)t * nCTA;
+  uint32_t run = 0;
+  for (int c0 = 0; c0 < nCTA; c0 += 32) {
+    const bool in = c0 + lane < nCTA;
+    const uint32_t v = in ? row[c0 + lane] : 0u;
+    uint32_t incl = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += u;
+    }
+    if (in) row[c0 + lane] = run + incl - v;
+    run += __shfl_sync(0xffffffffu, incl, 31);
+  }
+  if (lane == 0) cnt[(int64_t)t * CNT_STRIDE] = run;
+}
+
+// block-wide exclusive scan of one value per thread (DP_THREADS); returns the prefix, *total the sum
+__device__ __forceinline__ uint32_t dp_block_scan(uint32_t v, uint32_t* s_w, uint32_t* total) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint32_t incl = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += u;
+  }
+  if (lane == 31) s_w[warp] = incl;
+  __syncthreads();
+  uint32_t pre = 0, tot = 0;
+#pragma unroll
+  for (int w = 0; w < DP_WARPS; ++w) {
+    const uint32_t u = s_w[w];
+    pre += w < warp ? u : 0u;
+    tot += u;
+  }
+  __syncthreads();
+  *total = tot;
+  return pre + incl - v;
+}
+
+struct DpSmem {
+  uint32_t gstart[DB_MAXT + 1];  // per tile: pairs of the CTA, then the first position of the tile's group
+  uint32_t cur[DB_MAXT];         // per tile: next free slot of its group; then the tile list position of the group
+  uint16_t arr[DP_KEYS];          // the CTA's star indices grouped by tile (in arbitrary order inside a group)
+  uint32_t s_w[DP_WARPS];
+};
+
+// the tiles of the star with ROI origin lo (not culled): [tx0, tx1] x [ty0, ty1]
+__device__ __forceinline__ void star_tiles(const FrameParams& fp, uint32_t lo, int& tx0, int& tx1, int& ty0, int& ty1) {
+  int cx0, cx1, cy0, cy1;
+  clip_roi(fp, lo_x_of(lo), lo_y_of(lo), cx0, cx1, cy0, cy1);
+  tx0 = cx0 / TILE_W;
+  tx1 = cx1 / TILE_W;
+  ty0 = (cy0 - fp.row0) / TILE_H;
+  ty1 = (cy1 - fp.row0) / TILE_H;
+}
+
+__global__ void __launch_bounds__(DP_THREADS) k_dplace(const StarRec* __restrict__ rec, int64_t n, FrameParams fp,
+                                                       const uint32_t* __restrict__ C, int nCTA, int ntiles,
+                                                       const uint32_t* __restrict__ tile_off,
+                                                       uint32_t* __restrict__ ids) {
+  extern __shared__ __align__(16) unsigned char dsm_raw[];
+  DpSmem& S = *reinterpret_cast<DpSmem*>(dsm_raw);
+  const int tid = threadIdx.x, cta = blockIdx.x;
+  const int64_t c0 = (int64_t)cta * DB_CTA;
+  for (int t = tid; t <= ntiles; t += DP_THREADS) S.gstart[t] = 0u;
+  uint32_t lo[DP_SPT];
+#pragma unroll
+  for (int k = 0; k < DP_SPT; ++k) {
+    const int64_t i = c0 + tid + k * DP_THREADS;
+    lo[k] = i < n ? __ldg(&rec[i].lo) : LO_CULLED;
+  }
+  __syncthreads();
+  // group sizes
+#pragma unroll
+  for (int k = 0; k < DP_SPT; ++k) {
+    if (lo[k] == LO_CULLED) continue;
+    int tx0, tx1, ty0, ty1;
+    star_tiles(fp, lo[k], tx0, tx1, ty0, ty1);
+    for (int ty = ty0; ty <= ty1; ++ty)
+      for (int tx = tx0; tx <= tx1; ++tx) atomicAdd(&S.gstart[ty * fp.ntx + tx], 1u);
+  }
+  __syncthreads();
+  // exclusive scan of the group sizes (TPT consecutive tiles per thread)
+  {
+    constexpr int TPT = (DB_MAXT + DP_THREADS - 1) / DP_THREADS;
+    uint32_t c[TPT], sum = 0;
+#pragma unroll
+    for (int k = 0; k < TPT; ++k) {
+      const int t = tid * TPT + k;
+      c[k] = t < ntiles ? S.gstart[t] : 0u;
+      sum += c[k];
+    }
+    uint32_t tot;
+    uint32_t run = dp_block_scan(sum, S.s_w, &tot);
+#pragma unroll
+    for (int k = 0; k < TPT; ++k) {
+      const int t = tid * TPT + k;
+      if (t < ntiles) {
+        S.gstart[t] = run;
+        S.cur[t] = run;
+      }
+      run += c[k];
+    }
+    if (tid == 0) S.gstart[ntiles] = tot;
+  }
+  __syncthreads();
+  // group the star indices by tile
+#pragma unroll
+  for (int k = 0; k < DP_SPT; ++k) {
+    if (lo[k] == LO_CULLED) continue;
+    int tx0, tx1, ty0, ty1;
+    star_tiles(fp, lo[k], tx0, tx1, ty0, ty1);
+    for (int ty = ty0; ty <= ty1; ++ty)
+      for (int tx = tx0; tx <= tx1; ++tx)
+        S.arr[atomicAdd(&S.cur[ty * fp.ntx + tx], 1u)] = (uint16_t)(tid + k * DP_THREADS);
+  }
+  __syncthreads();
+  // first list position of every group: tile_off[t] + (pairs of tile t in the CTAs before)
+  for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = tile_off[t] + C[(int64_t)t * nCTA + cta];
+  __syncthreads();
+  // a pair's rank in its group = the group's stars with a smaller index
+#pragma unroll
+  for (int k = 0; k < DP_SPT; ++k) {
+    if (lo[k] == LO_CULLED) continue;
+    const uint32_t idx = (uint32_t)(tid + k * DP_THREADS);
+    int tx0, tx1, ty0, ty1;
+    star_tiles(fp, lo[k], tx0, tx1, ty0, ty1);
+    for (int ty = ty0; ty <= ty1; ++ty)
+      for (int tx = tx0; tx <= tx1; ++tx) {
+        const int t = ty * fp.ntx + tx;
+        const uint32_t g0 = S.gstart[t], g1 = S.gstart[t + 1];
+        uint32_t rank = 0;
+        for (uint32_t u = g0; u < g1; ++u) rank += S.arr[u] < idx ? 1u : 0u;
+        ids[S.cur[t] + rank] = (uint32_t)c0 + idx;
+      }
+  }
+}
+
+size_t dbin_smem(int) { return sizeof(DpSmem); }
+
+int dbin_ctas(int64_t n) { return (int)((n + DB_CTA - 1) / DB_CTA); }
+
+void init_dbin_kernels() {
+  cudaFuncSetAttribute(k_dplace, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DpSmem));
+}
+
+void launch_dcount(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
+                   uint32_t* C, int ntiles, cudaStream_t st) {
+  const int nc = dbin_ctas(n);
+  if (nc > 0) k_dcount<<<nc, DC_THREADS, 0, st>>>(x, y, m, n, fp, rec, C, nc, ntiles);
+}
+
+void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, cudaStream_t st) {
+  constexpr int wpb = DCS_THREADS / 32;
+  k_dcolscan<<<(ntiles + wpb - 1) / wpb, DCS_THREADS, 0, st>>>(C, dbin_ctas(n), ntiles, cnt);
+}
+
+void launch_dplace(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,
+                   const uint32_t* tile_off, uint32_t* ids, cudaStream_t st) {
+  const int nc = dbin_ctas(n);
+  if (nc > 0) k_dplace<<<nc, DP_THREADS, sizeof(DpSmem), st>>>(rec, n, fp, C, nc, ntiles, tile_off, ids);
+}
+
+}  // namespace starsim

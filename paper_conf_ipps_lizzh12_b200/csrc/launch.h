@@ -10,10 +10,18 @@ namespace starsim {
 void init_kernels();
 void init_tile_kernel();
 void init_tile_sb_kernel();
+void init_dbin_kernels();
+size_t dbin_smem(int ntiles);
+int dbin_ctas(int64_t n);
+void launch_dcount(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
+                   uint32_t* C, int ntiles, cudaStream_t st);
+void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, cudaStream_t st);
+void launch_dplace(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,
+                   const uint32_t* tile_off, uint32_t* ids, cudaStream_t st);
 void launch_prep(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
                  uint32_t* cnt, uint32_t* slots, int tps, cudaStream_t st);
 void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items,
-                 uint2* split_tab, int part_cap, void* partial, cudaStream_t st);
+                 uint2* split_tab, int part_cap, void* partial, uint32_t* done, cudaStream_t st);
 void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* slots, int tps,
                     const uint32_t* tile_off, uint32_t* ids, cudaStream_t st);
 void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, int64_t ntiles, int64_t n,
