@@ -251,7 +251,7 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
   }
   timed(c, 3, st, [&] {
     launch_tile(ids, rec, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p, part_cap, done,
-                hdr, st);
+                hdr, c->num_sms, st);
   });
   if ((rc = check_launch(c, "k_tile"))) return rc;
   return STARSIM_OK;

@@ -135,6 +135,7 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_b(const uint32_t* __restr
     tile_off[ntiles] = ta.x;
     hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
     hdr->nsplit = nsplit;
+    hdr->next_item = 0u;
   }
   const int64_t t0 = (int64_t)blockIdx.x * SCAN_TILES + (int64_t)tid * SCAN_PER;
   uint32_t c[SCAN_PER];

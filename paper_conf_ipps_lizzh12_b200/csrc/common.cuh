@@ -48,7 +48,8 @@ struct Header {
   uint32_t P;                          // number of (tile, star) pairs
   uint32_t nitems;                     // k_tile work items (written by k_scan)
   uint32_t nsplit;                     // tiles split into several items
-  uint32_t pad[29];
+  uint32_t next_item;                  // k_tile_sb: the next work item a persistent CTA takes (k_scan zeroes it)
+  uint32_t pad[28];
 };
 
 // k_tile work item: stars [jb, je) of tile `tile`'s list; aux = ITEM_WHOLE, or (split index << 12 | part index) for

@@ -18,7 +18,7 @@
 
 namespace starsim {
 
-constexpr int DB_CTA = 8192;                     // stars per CTA (one column of the count matrix)
+constexpr int DB_CTA = 4096;                     // stars per CTA (one column of the count matrix)
 constexpr int DC_THREADS = 1024;                 // k_dcount: DB_CTA / DC_THREADS stars per thread
 constexpr int DC_PER = DB_CTA / DC_THREADS;
 constexpr int DP_THREADS = 1024;                 // k_dplace
@@ -117,41 +117,55 @@ struct DpSmem {
   uint32_t s_w[DP_WARPS];
 };
 
-// the tiles of the star with ROI origin lo (not culled): [tx0, tx1] x [ty0, ty1]
-__device__ __forceinline__ void star_tiles(const FrameParams& fp, uint32_t lo, int& tx0, int& tx1, int& ty0, int& ty1) {
+// the tiles of the star with ROI origin lo, packed: first tile t0 | dx << 16 | dy << 17 (it also covers t0 + 1 if dx,
+// t0 + ntx if dy, t0 + ntx + 1 if both); DP_NONE if the star is culled
+constexpr uint32_t DP_NONE = 0xFFFFFFFFu;
+__device__ __forceinline__ uint32_t star_tiles(const FrameParams& fp, uint32_t lo) {
+  if (lo == LO_CULLED) return DP_NONE;
   int cx0, cx1, cy0, cy1;
-  clip_roi(fp, lo_x_of(lo), lo_y_of(lo), cx0, cx1, cy0, cy1);
-  tx0 = cx0 / TILE_W;
-  tx1 = cx1 / TILE_W;
-  ty0 = (cy0 - fp.row0) / TILE_H;
-  ty1 = (cy1 - fp.row0) / TILE_H;
+  clip_roi(fp, lo_x_of(lo), lo_y_of(lo), cx0, cx1, cy0, cy1);  // cx0, cy0 - row0 >= 0: plain shifts
+  const int tx0 = cx0 >> 7, ty0 = (cy0 - fp.row0) >> 6;
+  const uint32_t dx = (uint32_t)((cx1 >> 7) - tx0), dy = (uint32_t)(((cy1 - fp.row0) >> 6) - ty0);
+  return (uint32_t)(ty0 * fp.ntx + tx0) | dx << 16 | dy << 17;
+}
+
+// the e-th tile (e = 0..3, in row-major order) of a packed box, or -1
+__device__ __forceinline__ int box_tile(uint32_t code, int e, int ntx) {
+  if (code == DP_NONE) return -1;
+  const int dx = (int)((code >> 16) & 1u), dy = (int)((code >> 17) & 1u);
+  const int ex = e & 1, ey = e >> 1;
+  if (ex > dx || ey > dy) return -1;
+  // row-major order inside the box: (0,0), (0,1), (1,0), (1,1) -> skip e = 1 when dx = 0 is handled by the test
+  return (int)(code & 0xFFFFu) + ey * ntx + ex;
 }
 
 __global__ void __launch_bounds__(DP_THREADS) k_dplace(const StarRec* __restrict__ rec, int64_t n, FrameParams fp,
                                                        const uint32_t* __restrict__ C, int nCTA, int ntiles,
                                                        const uint32_t* __restrict__ tile_off,
                                                        uint32_t* __restrict__ ids) {
+  static_assert(TILE_W == 128 && TILE_H == 64, "star_tiles shifts");
   extern __shared__ __align__(16) unsigned char dsm_raw[];
   DpSmem& S = *reinterpret_cast<DpSmem*>(dsm_raw);
   const int tid = threadIdx.x, cta = blockIdx.x;
   const int64_t c0 = (int64_t)cta * DB_CTA;
   for (int t = tid; t <= ntiles; t += DP_THREADS) S.gstart[t] = 0u;
-  uint32_t lo[DP_SPT];
+  uint32_t code[DP_SPT];
 #pragma unroll
   for (int k = 0; k < DP_SPT; ++k) {
     const int64_t i = c0 + tid + k * DP_THREADS;
-    lo[k] = i < n ? __ldg(&rec[i].lo) : LO_CULLED;
+    code[k] = i < n ? __ldg(&rec[i].lo) : LO_CULLED;
   }
+#pragma unroll
+  for (int k = 0; k < DP_SPT; ++k) code[k] = star_tiles(fp, code[k]);
   __syncthreads();
   // group sizes
 #pragma unroll
-  for (int k = 0; k < DP_SPT; ++k) {
-    if (lo[k] == LO_CULLED) continue;
-    int tx0, tx1, ty0, ty1;
-    star_tiles(fp, lo[k], tx0, tx1, ty0, ty1);
-    for (int ty = ty0; ty <= ty1; ++ty)
-      for (int tx = tx0; tx <= tx1; ++tx) atomicAdd(&S.gstart[ty * fp.ntx + tx], 1u);
-  }
+  for (int k = 0; k < DP_SPT; ++k)
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int t = box_tile(code[k], e, fp.ntx);
+      if (t >= 0) atomicAdd(&S.gstart[t], 1u);
+    }
   __syncthreads();
   // exclusive scan of the group sizes (TPT consecutive tiles per thread)
   {
@@ -177,16 +191,14 @@ __global__ void __launch_bounds__(DP_THREADS) k_dplace(const StarRec* __restrict
     if (tid == 0) S.gstart[ntiles] = tot;
   }
   __syncthreads();
-  // group the star indices by tile
+  // group the star indices by tile (arbitrary order inside a group)
 #pragma unroll
-  for (int k = 0; k < DP_SPT; ++k) {
-    if (lo[k] == LO_CULLED) continue;
-    int tx0, tx1, ty0, ty1;
-    star_tiles(fp, lo[k], tx0, tx1, ty0, ty1);
-    for (int ty = ty0; ty <= ty1; ++ty)
-      for (int tx = tx0; tx <= tx1; ++tx)
-        S.arr[atomicAdd(&S.cur[ty * fp.ntx + tx], 1u)] = (uint16_t)(tid + k * DP_THREADS);
-  }
+  for (int k = 0; k < DP_SPT; ++k)
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int t = box_tile(code[k], e, fp.ntx);
+      if (t >= 0) S.arr[atomicAdd(&S.cur[t], 1u)] = (uint16_t)(tid + k * DP_THREADS);
+    }
   __syncthreads();
   // first list position of every group: tile_off[t] + (pairs of tile t in the CTAs before)
   for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = tile_off[t] + C[(int64_t)t * nCTA + cta];
@@ -194,18 +206,16 @@ __global__ void __launch_bounds__(DP_THREADS) k_dplace(const StarRec* __restrict
   // a pair's rank in its group = the group's stars with a smaller index
 #pragma unroll
   for (int k = 0; k < DP_SPT; ++k) {
-    if (lo[k] == LO_CULLED) continue;
     const uint32_t idx = (uint32_t)(tid + k * DP_THREADS);
-    int tx0, tx1, ty0, ty1;
-    star_tiles(fp, lo[k], tx0, tx1, ty0, ty1);
-    for (int ty = ty0; ty <= ty1; ++ty)
-      for (int tx = tx0; tx <= tx1; ++tx) {
-        const int t = ty * fp.ntx + tx;
-        const uint32_t g0 = S.gstart[t], g1 = S.gstart[t + 1];
-        uint32_t rank = 0;
-        for (uint32_t u = g0; u < g1; ++u) rank += S.arr[u] < idx ? 1u : 0u;
-        ids[S.cur[t] + rank] = (uint32_t)c0 + idx;
-      }
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int t = box_tile(code[k], e, fp.ntx);
+      if (t < 0) continue;
+      const uint32_t g0 = S.gstart[t], g1 = S.gstart[t + 1];
+      uint32_t rank = 0;
+      for (uint32_t u = g0; u < g1; ++u) rank += S.arr[u] < idx ? 1u : 0u;
+      ids[S.cur[t] + rank] = (uint32_t)c0 + idx;
+    }
   }
 }
 

@@ -27,9 +27,10 @@ void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, const 
 void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, int64_t ntiles, int64_t n,
                       cudaStream_t st);
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
-                 const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, cudaStream_t st);
+                 const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
+                 cudaStream_t st);
 void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
-                    const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr,
+                    const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
                     cudaStream_t st);
 void launch_atomic(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, float* out,
                    cudaStream_t st);

@@ -77,6 +77,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
   }
 
   if (blockIdx.x >= __ldcg(&hdr->nitems)) return;
+  {
   const WorkItem wi = items[blockIdx.x];
   const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
   const int X0 = tx * TILE_W;    // first column of the tile
@@ -241,31 +242,33 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
 
     if (nb + tid < j1) rnext = rec[nid];
     // ======================= accumulate: lane group q walks its two ranges (padded with the zero slot)
-#pragma unroll 2
-    for (uint32_t st = 0; st < steps; st += 2) {
+    auto step = [&](uint32_t t, bool odd) {
+      const bool in1 = t < len1, in = t < L;
+      uint32_t ga = (in1 ? (odd ? g1o : g1e) : (odd ? g2o : g2e)) + t * 128u;
+      uint32_t xa = (in1 ? x1 : x2) + t * 128u;
+      ga = in ? ga : gz;
+      xa = in ? xa : xz;
+      float4 g, a, c;
+      asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(g.x), "=f"(g.y), "=f"(g.z), "=f"(g.w) : "r"(ga));
+      asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "r"(xa));
+      asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(c.x), "=f"(c.y), "=f"(c.z), "=f"(c.w) : "r"(xa + 16u));
+      const float gi[4] = {g.x, g.y, g.z, g.w};
 #pragma unroll
-      for (uint32_t o = 0; o < 2; ++o) {
-        const uint32_t t = st + o;
-        const bool in1 = t < len1, in = t < L;
-        uint32_t ga = (in1 ? (o ? g1o : g1e) : (o ? g2o : g2e)) + t * 128u;
-        uint32_t xa = (in1 ? x1 : x2) + t * 128u;
-        ga = in ? ga : gz;
-        xa = in ? xa : xz;
-        float4 g, a, c;
-        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(g.x), "=f"(g.y), "=f"(g.z), "=f"(g.w) : "r"(ga));
-        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "r"(xa));
-        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(c.x), "=f"(c.y), "=f"(c.z), "=f"(c.w) : "r"(xa + 16u));
-        const float gi[4] = {g.x, g.y, g.z, g.w};
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const float2 gg = make_float2(gi[i], gi[i]);
-          acc[i][0] = __ffma2_rn(gg, make_float2(a.x, a.y), acc[i][0]);
-          acc[i][1] = __ffma2_rn(gg, make_float2(a.z, a.w), acc[i][1]);
-          acc[i][2] = __ffma2_rn(gg, make_float2(c.x, c.y), acc[i][2]);
-          acc[i][3] = __ffma2_rn(gg, make_float2(c.z, c.w), acc[i][3]);
-        }
+      for (int i = 0; i < 4; ++i) {
+        const float2 gg = make_float2(gi[i], gi[i]);
+        acc[i][0] = __ffma2_rn(gg, make_float2(a.x, a.y), acc[i][0]);
+        acc[i][1] = __ffma2_rn(gg, make_float2(a.z, a.w), acc[i][1]);
+        acc[i][2] = __ffma2_rn(gg, make_float2(c.x, c.y), acc[i][2]);
+        acc[i][3] = __ffma2_rn(gg, make_float2(c.z, c.w), acc[i][3]);
       }
+    };
+    uint32_t st = 0;
+#pragma unroll 2
+    for (; st + 1 < steps; st += 2) {
+      step(st, false);
+      step(st + 1, true);
     }
+    if (st < steps) step(st, false);
   }
 
   // ======================= output
@@ -279,8 +282,9 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
       acc[i][3] = t1;
     }
   }
-  if (!tile_reduce_parts(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last)) return;
-  tile_store(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+  if (tile_reduce_parts(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last))
+    tile_store(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+  }
 }
 
 void init_tile_sb_kernel() {
@@ -289,10 +293,11 @@ void init_tile_sb_kernel() {
 }
 
 void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
-                    const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr,
+                    const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
                     cudaStream_t st) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
+  (void)num_sms;
   const int64_t grid = ntiles + part_cap;  // one CTA per possible item (parts first); the rest exit at once
   if (fp.psf)
     k_tile_sb<true><<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab,

@@ -305,7 +305,7 @@ def test_kernel_times_recorded(torch_dev, ctx):
     ctx.render(*args, cfg.W, cfg.H, cfg.sigma, cfg.R, 1.0)
     t = ctx.kernel_times()
     ctx.profile(False)
-    assert t["tile"][1] == 1 and t["tile"][0] > 0 and t["prep"][1] == 1 and t["sort"][1] == 1 and t["csr"][1] == 1
+    assert t["tile"][1] == 1 and t["tile"][0] > 0 and t["prep"][1] == 1 and t["sort"][1] == 1 and t["csr"][1] in (2, 3)
 
 
 # ---------------------------------------------------------------- B200-scale frames (full images, threaded oracle)
