@@ -333,8 +333,8 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
   }
 
   // ======================= output: rows 16 B + hq + 4 i, columns 64 wx + 8 q .. +7 of the tile
-  if (!tile_reduce_parts(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last)) continue;
-  tile_store(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+  if (!tile_reduce_parts<false>(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last)) continue;
+  tile_store<false>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
   }  // work loop
 }
 

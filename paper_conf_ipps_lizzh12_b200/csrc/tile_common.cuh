@@ -1,16 +1,21 @@
 // Pieces shared by the two tile-accumulation kernels (tile.cu: per-block entry lists, any R; tile_sb.cu: sorted
 // corner bins, R <= SB_MAXR).  Both use the same lane layout: warp (wx, B) owns the 64 x 16 block at tile columns
 // 64 wx, rows 16 B; lane group q = lane/4 owns the 8-column strip Q = 8 wx + q, lane hq = lane%4 the rows
-// 16 B + hq + 4 i (i = 0..3), as 4 x 4 float2 accumulators (columns 8 Q + 2 k, 8 Q + 2 k + 1 in acc[i][k]).
+// 16 B + hq + 4 i (tile.cu, CONTIG = false) or 16 B + 4 hq + i (tile_sb.cu, CONTIG = true), i = 0..3, as 4 x 4 float2
+// accumulators (columns 8 Q + 2 k, 8 Q + 2 k + 1 in acc[i][k]).
 #pragma once
 #include "common.cuh"
 
 namespace starsim {
 
+template <bool CONTIG>
+__device__ __forceinline__ int lane_row(int B, int hq, int i) { return CONTIG ? 16 * B + 4 * hq + i : 16 * B + hq + 4 * i; }
+
 // A whole tile is written to `out` directly; a part of a split heavy tile (wi.aux != ITEM_WHOLE) writes its
 // 128 x 64 partial to part_buf, and the last part to finish (per-tile counter) sums the parts in part order -- a
 // fixed order, so the image stays deterministic.  Returns false for a part that is not the last one (nothing left
 // to write); on true, acc holds the tile's final sums.  Contains block barriers: every thread of the CTA calls it.
+template <bool CONTIG>
 __device__ __forceinline__ bool tile_reduce_parts(float2 (&acc)[4][4], const WorkItem& wi,
                                                   const uint2* __restrict__ split_tab, float* __restrict__ part_buf,
                                                   uint32_t* __restrict__ done, int B, int wx, int q, int hq,
@@ -21,7 +26,7 @@ __device__ __forceinline__ bool tile_reduce_parts(float2 (&acc)[4][4], const Wor
   float* pbuf = part_buf + (size_t)(sp.x + (wi.aux & 0xFFFu)) * (TILE_W * TILE_H);
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
-    float4* o = reinterpret_cast<float4*>(pbuf + (16 * B + hq + 4 * i) * TILE_W + 64 * wx + 8 * q);
+    float4* o = reinterpret_cast<float4*>(pbuf + lane_row<CONTIG>(B, hq, i) * TILE_W + 64 * wx + 8 * q);
     o[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
     o[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
   }
@@ -39,7 +44,7 @@ __device__ __forceinline__ bool tile_reduce_parts(float2 (&acc)[4][4], const Wor
     const float* pk = part_buf + (size_t)(sp.x + k) * (TILE_W * TILE_H);
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
-      const float4* o = reinterpret_cast<const float4*>(pk + (16 * B + hq + 4 * i) * TILE_W + 64 * wx + 8 * q);
+      const float4* o = reinterpret_cast<const float4*>(pk + lane_row<CONTIG>(B, hq, i) * TILE_W + 64 * wx + 8 * q);
       const float4 u = __ldcg(o), v = __ldcg(o + 1);
       acc[i][0] = __fadd2_rn(acc[i][0], make_float2(u.x, u.y));
       acc[i][1] = __fadd2_rn(acc[i][1], make_float2(u.z, u.w));
@@ -50,16 +55,17 @@ __device__ __forceinline__ bool tile_reduce_parts(float2 (&acc)[4][4], const Wor
   return true;
 }
 
-// Write the lane's 4 rows x 8 columns of the tile (rows Y0 + 16 B + hq + 4 i of the band, columns col0 .. col0+7):
+// Write the lane's 4 rows x 8 columns of the tile (rows Y0 + lane_row(B, hq, i) of the band, columns col0 .. col0+7):
 // fp32, or (fused output stage, NEXT-1) the gray value of each pixel exactly as k_quantize computes it from the same
 // fp32 sum, as u8 / u16.  Coalesced: the 8 lane groups of a warp store 8 adjacent 8-pixel runs of a row.
+template <bool CONTIG>
 __device__ __forceinline__ void tile_store(const float2 (&acc)[4][4], const FrameParams& fp, void* __restrict__ out_,
                                            int Y0, int col0, int B, int hq) {
   if (fp.obits == 0) {
     float* out = reinterpret_cast<float*>(out_);
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
-      const int row = Y0 + 16 * B + hq + 4 * i;  // band-relative
+      const int row = Y0 + lane_row<CONTIG>(B, hq, i);  // band-relative
       if (row >= fp.rows || col0 >= fp.W) continue;
       float* o = out + (int64_t)row * fp.W + col0;
       if (fp.vec && col0 + 8 <= fp.W) {
@@ -77,7 +83,7 @@ __device__ __forceinline__ void tile_store(const float2 (&acc)[4][4], const Fram
     const float qmax = fp.obits == 8 ? 255.f : 65535.f;
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
-      const int row = Y0 + 16 * B + hq + 4 * i;
+      const int row = Y0 + lane_row<CONTIG>(B, hq, i);
       if (row >= fp.rows || col0 >= fp.W) continue;
       uint32_t g[8];
 #pragma unroll

@@ -37,18 +37,20 @@ namespace starsim {
 // it comes in over the left edge, else 1 + strip), band-major
 constexpr int SB_NSK = NSTRIPS + 1;
 constexpr int SB_NBIN = (NBANDS + 1) * SB_NSK;  // 85
-constexpr uint32_t SB_ZJ = CHUNK;           // the all-zero slot
+constexpr int SB_CHUNK = CHUNK;             // stars per chunk (<= TILE_THREADS; 192 with 4 CTAs/SM measured slower: spills)
+constexpr int SB_MINB = 3;                  // CTAs per SM (80 registers, 70 KB shared memory)
+constexpr uint32_t SB_ZJ = SB_CHUNK;        // the all-zero slot
 
 struct SbSmem {
-  float gy[(CHUNK + 1) * 32];    // sorted star j: two 16-float band slots, slot k at j*32 + ((j ^ k) & 1) * 16
-  float gx[(CHUNK + 1) * 32];    // sorted star j: ring of four 8-float strip slots, strip Q at j*32 + (Q & 3) * 8
+  float gy[(SB_CHUNK + 1) * 32];    // sorted star j: two 16-float band slots, slot k at j*32 + ((j ^ k) & 1) * 16
+  float gx[(SB_CHUNK + 1) * 32];    // sorted star j: ring of four 8-float strip slots, strip Q at j*32 + (Q & 3) * 8
   uint32_t hist[TILE_WARPS][SB_NBIN];      // per warp: stars of each corner bin
   uint32_t binoff[SB_NBIN][TILE_WARPS];    // per bin: stars of the bin in the warps before
   uint32_t binstart[SB_NBIN + 1];          // exclusive scan of the bin totals (bin-major)
 };
 
 template <bool INTEG>
-__global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __restrict__ ids,
+__global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_t* __restrict__ ids,
                                                              const StarRec* __restrict__ rec, FrameParams fp,
                                                              void* __restrict__ out_,
                                                              const WorkItem* __restrict__ items,
@@ -92,10 +94,10 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
 
   const uint32_t j1 = wi.je;
   StarRec rnext = {};
-  if (wi.jb + tid < j1) rnext = rec[ids[wi.jb + tid]];
-  for (uint32_t base = wi.jb; base < j1; base += CHUNK) {
+  if (tid < SB_CHUNK && wi.jb + tid < j1) rnext = rec[ids[wi.jb + tid]];
+  for (uint32_t base = wi.jb; base < j1; base += SB_CHUNK) {
     // ======================= sort: thread = star (base + tid) of the tile's list
-    const int nvalid = (int)min((uint32_t)CHUNK, j1 - base);
+    const int nvalid = (int)min((uint32_t)SB_CHUNK, j1 - base);
     const StarRec r = rnext;
     int c0 = 0, c1 = -1, r0 = 0, r1 = -1;
     uint32_t key = SB_NBIN;
@@ -117,8 +119,8 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
     __syncwarp();
     if (rank == 0 && key < SB_NBIN) S.hist[warp][key] = __popc(peers);
     // next chunk's star id now (its record is requested just before the accumulation)
-    const uint32_t nb = base + CHUNK;
-    const uint32_t nid = nb + tid < j1 ? __ldg(&ids[nb + tid]) : 0u;
+    const uint32_t nb = base + SB_CHUNK;
+    const uint32_t nid = tid < SB_CHUNK && nb + tid < j1 ? __ldg(&ids[nb + tid]) : 0u;
     __syncthreads();
     if (warp == 0) {
       uint32_t tot[3], sum = 0;
@@ -158,37 +160,48 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
       const float2 sk2 = make_float2(sk, sk), s2 = make_float2(r.s, r.s);
       // first band / strip of the slots: the corner bin's (-1 for an ROI that comes in over the top / left edge)
       const int b0 = (int)(key / SB_NSK) - 1, q0 = (int)(key % SB_NSK) - 1;
-      // band slots: the 8 quads (band k, row group h: rows h + 4 i) are written in an order rotated by the lane, so
-      // that each STS.128 of the warp hits all 8 bank quads (slot half (j ^ k) & 1 = u & 1, h = u >> 1)
+      // band slots (lane hq reads rows 4 hq .. 4 hq + 3 of a band): the two bands b0, b0+1 are 8 row quads w = 0..7
+      // (band w >> 2, rows 4 (w & 3) ..) of which the ROI's <= 17 rows touch at most 5 consecutive ones, from
+      // qfirst: iterations c = 0..4 compute quads qfirst + c, c = 5..7 store the other three as zeros (mod 8)
       const int ra0 = r0 - 16 * b0, rb0 = r1 - 16 * b0;      // ROI rows relative to band b0 (band b0+1: -16)
       const uint32_t m0 = (0xFFFFFFFFu >> (31 - min(rb0, 31))) & (0xFFFFFFFFu << ra0);  // ROI rows over both bands
       const float bf0 = (float)(16 * b0) - yr;              // exact
+      const int qfirst = ra0 >> 2;
 #pragma unroll
       for (int c = 0; c < 8; ++c) {
-        const int u = (c + lane) & 7;
-        const int hh = u >> 1, k = (u ^ (int)j) & 1;
-        const uint32_t m = m0 >> (16 * k + hh);            // bit 4 i: row hh + 4 i of band b0 + k in the ROI
-        const float bf = bf0 + (float)(16 * k + hh);        // exact
+        const int w = (qfirst + c) & 7;
+        const int k = w >> 2, hh = w & 3;
+        float4* dst = reinterpret_cast<float4*>(&S.gy[j * 32 + ((j ^ (uint32_t)k) & 1u) * 16 + hh * 4]);
+        if (c >= 5) {
+          *dst = make_float4(0.f, 0.f, 0.f, 0.f);
+          continue;
+        }
+        const uint32_t m = m0 >> (4 * w);                  // bit i: row 4 w + i of the window in the ROI
+        const float bf = bf0 + (float)(4 * w);              // exact
         float v[4];
         if (!INTEG) {
           const float2 bb = make_float2(bf, bf);
 #pragma unroll
           for (int i = 0; i < 4; i += 2) {
-            float2 d = __fadd2_rn(bb, make_float2((float)(4 * i), (float)(4 * i + 4)));
+            float2 d = __fadd2_rn(bb, make_float2((float)i, (float)(i + 1)));
             d = __fmul2_rn(d, sk2);
             d = __fmul2_rn(d, make_float2(-d.x, -d.y));
             const float2 e = __fmul2_rn(make_float2(ex2_approx(d.x), ex2_approx(d.y)), s2);
-            v[i] = (m >> (4 * i)) & 1u ? e.x : 0.f;
-            v[i + 1] = (m >> (4 * i + 4)) & 1u ? e.y : 0.f;
+            v[i] = (m >> i) & 1u ? e.x : 0.f;
+            v[i + 1] = (m >> (i + 1)) & 1u ? e.y : 0.f;
           }
         } else {
+          // pixel-integrated rows: the 4 consecutive rows share their 5 edges
+          float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
 #pragma unroll
           for (int i = 0; i < 4; ++i) {
-            const float t0 = (bf + (float)(4 * i) - 0.5f) * fp.kint, t1 = (bf + (float)(4 * i) + 0.5f) * fp.kint;
-            v[i] = (m >> (4 * i)) & 1u ? r.s * pix_mass(t0, edge_erfc(t0), t1, edge_erfc(t1)) : 0.f;
+            const float tn = (bf + (float)i + 0.5f) * fp.kint, en = edge_erfc(tn);
+            v[i] = (m >> i) & 1u ? r.s * pix_mass(t, e, tn, en) : 0.f;
+            t = tn;
+            e = en;
           }
         }
-        *reinterpret_cast<float4*>(&S.gy[j * 32 + (u & 1) * 16 + hh * 4]) = make_float4(v[0], v[1], v[2], v[3]);
+        *dst = make_float4(v[0], v[1], v[2], v[3]);
       }
 #pragma unroll
       for (int k = 0; k < 3; ++k) {
@@ -240,7 +253,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
     const uint32_t gz = gy_base + SB_ZJ * 128u, xz = gx_base + SB_ZJ * 128u;
     __syncthreads();
 
-    if (nb + tid < j1) rnext = rec[nid];
+    if (tid < SB_CHUNK && nb + tid < j1) rnext = rec[nid];
     // ======================= accumulate: lane group q walks its two ranges (padded with the zero slot)
     auto step = [&](uint32_t t, bool odd) {
       const bool in1 = t < len1, in = t < L;
@@ -282,8 +295,8 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile_sb(const uint32_t* __r
       acc[i][3] = t1;
     }
   }
-  if (tile_reduce_parts(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last))
-    tile_store(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+  if (tile_reduce_parts<true>(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last))
+    tile_store<true>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
   }
 }
 
