@@ -109,6 +109,16 @@ int starsim_set_psf(starsim_ctx* ctx, int32_t mode);
  *   STARSIM_TILE_AUTO (default): for R <= 17 the sorted-corner-bin kernel, else the list kernel;
  *   STARSIM_TILE_LISTS: always the per-block entry-list kernel (the comparison / any R).
  * EINVAL: ctx NULL or an unknown mode. */
+/* Binning pipeline of the tiled renders that follow on this ctx.  Both produce the same CSR (each tile's list in
+ * ascending star index, reading R18 of DESIGN.md), hence the same image bit for bit:
+ *   STARSIM_BIN_AUTO (default): the deterministic counting sort (dbin.cu, no global atomics) when the frame or band
+ *     has <= 2048 tiles and R <= 65, else the atomic-slot pipeline;
+ *   STARSIM_BIN_ATOMIC: always the atomic-slot pipeline (per-tile counters, scatter, per-tile sort).
+ * EINVAL: ctx NULL or an unknown mode. */
+#define STARSIM_BIN_AUTO 0
+#define STARSIM_BIN_ATOMIC 1
+int starsim_set_binning(starsim_ctx* ctx, int32_t mode);
+
 #define STARSIM_TILE_AUTO 0
 #define STARSIM_TILE_LISTS 1
 int starsim_set_tile_kernel(starsim_ctx* ctx, int32_t mode);

@@ -34,13 +34,13 @@ struct Launch {
 struct GraphKey {
   const void *x, *y, *mag, *out;
   int64_t n;
-  int32_t W, H, row0, rows, R, obits, psf, tile_impl;
+  int32_t W, H, row0, rows, R, obits, psf, tile_impl, bin_impl;
   float sigma, gain;
   cudaStream_t st;
   uint64_t scratch_gen;
   bool operator==(const GraphKey& o) const {
     return x == o.x && y == o.y && mag == o.mag && out == o.out && n == o.n && W == o.W && H == o.H &&
-           row0 == o.row0 && rows == o.rows && R == o.R && obits == o.obits && psf == o.psf && tile_impl == o.tile_impl && sigma == o.sigma && gain == o.gain && st == o.st &&
+           row0 == o.row0 && rows == o.rows && R == o.R && obits == o.obits && psf == o.psf && tile_impl == o.tile_impl && bin_impl == o.bin_impl && sigma == o.sigma && gain == o.gain && st == o.st &&
            scratch_gen == o.scratch_gen;
   }
 };
@@ -50,6 +50,7 @@ struct starsim_ctx {
   int num_sms = 148;
   int32_t psf = 0;  // starsim_set_psf: 0 point-sampled Eq. 2, 1 pixel-integrated (NEXT-2)
   int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto (sorted bins when R <= 17), 1 per-block lists
+  int32_t bin_impl = 0;   // starsim_set_binning: 0 auto (dbin.cu when it applies), 1 always bin.cu's pipeline
   std::string err;
   Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
@@ -183,6 +184,7 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   fp.s_scale = (double)gain / (2.0 * M_PI * s * s);          // Eq. 1 gain with Eq. 2's 1/(2 pi s^2)
   fp.psf = psf;
   fp.tile_impl = 0;
+  fp.bin_impl = 0;
   fp.obits = 0;
   fp.vec = 0;
   fp.kint = (float)(1.0 / (std::sqrt(2.0) * s));
@@ -191,7 +193,7 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
 }
 
 // the deterministic binning of dbin.cu applies (DB_MAXT tiles, an ROI over at most 2 x 2 tiles)
-bool dbin_ok(const FrameParams& fp, int64_t ntiles) { return ntiles <= DB_MAXT && fp.R <= DB_MAXR; }
+bool dbin_ok(const FrameParams& fp, int64_t ntiles) { return fp.bin_impl == 0 && ntiles <= DB_MAXT && fp.R <= DB_MAXR; }
 
 int tiles_per_axis(int R, int tile, int ntiles_axis) {
   int t = (R - 1 + tile - 1) / tile + 1;
@@ -225,7 +227,7 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
           launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap,
                       c->partial.p, done, st);
         },
-        3);
+        1 + scan_launches(ntiles));
     if ((rc = check_launch(c, "k_dcolscan/k_scan"))) return rc;
     if (n > 0) {
       timed(c, 1, st, [&] { launch_dplace(rec, n, fp, C, (int)ntiles, tile_off, ids, st); });
@@ -244,7 +246,7 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
                       c->partial.p, done, st);
           launch_scatter(rec, n, fp, slots, tps, tile_off, ids, st);
         },
-        n > 0 ? 3 : 2);
+        (n > 0 ? 1 : 0) + scan_launches(ntiles));
     if ((rc = check_launch(c, "k_scan/k_scatter"))) return rc;
     timed(c, 1, st, [&] { launch_sortlists(ids, (uint32_t*)c->tmp.p, tile_off, ntiles, n, st); });
     if ((rc = check_launch(c, "k_sortlists"))) return rc;
@@ -264,6 +266,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain, c->psf);
   fp.obits = obits;
   fp.tile_impl = c->tile_impl;
+  fp.bin_impl = c->bin_impl;
   // one vector store per 8-pixel run: 32 B (fp32) / 8 B (u8) / 16 B (u16); rows must keep that alignment
   const int vb = obits == 8 ? 8 : 16;
   fp.vec = ((W * (obits ? obits / 8 : 4)) % vb == 0 && ((uintptr_t)out % vb) == 0) ? 1 : 0;
@@ -293,7 +296,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
                  "count matrix")))
     return rc;
 
-  const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, c->psf, c->tile_impl, sigma, gain, st, c->scratch_gen};
+  const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, c->psf, c->tile_impl, c->bin_impl, sigma, gain, st, c->scratch_gen};
   if (st == nullptr || c->prof || !c->use_graphs) {
     if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st))) return rc;
   } else {
@@ -424,6 +427,15 @@ int starsim_set_psf(starsim_ctx* c, int32_t mode) {
   if (mode != STARSIM_PSF_POINT && mode != STARSIM_PSF_INTEGRATED)
     return fail(c, STARSIM_EINVAL, "psf mode must be STARSIM_PSF_POINT or STARSIM_PSF_INTEGRATED");
   c->psf = mode;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
+int starsim_set_binning(starsim_ctx* c, int32_t mode) {
+  if (!c) return STARSIM_EINVAL;
+  if (mode != STARSIM_BIN_AUTO && mode != STARSIM_BIN_ATOMIC)
+    return fail(c, STARSIM_EINVAL, "binning mode must be STARSIM_BIN_AUTO or STARSIM_BIN_ATOMIC");
+  c->bin_impl = mode;
   c->err.clear();
   return STARSIM_OK;
 }

@@ -166,6 +166,63 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_b(const uint32_t* __restr
   }
 }
 
+// k_scan_one: the same as k_scan_a + k_scan_b in a single CTA of SCAN1_THREADS threads (SCAN_PER tiles each), for
+// frames / bands of at most SCAN1_TILES tiles: one launch instead of two.
+constexpr int SCAN1_THREADS = 1024;
+constexpr int SCAN1_TILES = SCAN1_THREADS * SCAN_PER;
+
+__global__ void __launch_bounds__(SCAN1_THREADS) k_scan_one(const uint32_t* __restrict__ cnt, int64_t ntiles,
+                                                             uint32_t* __restrict__ tile_off, Header* hdr,
+                                                             WorkItem* __restrict__ items,
+                                                             uint2* __restrict__ split_tab, int part_cap,
+                                                             uint32_t* __restrict__ done) {
+  __shared__ uint3 s_w[SCAN1_THREADS / 32];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t t0 = (int64_t)tid * SCAN_PER;
+  uint32_t c[SCAN_PER];
+  uint3 sum;
+  load_counts(cnt, ntiles, t0, c, sum);
+  const uint3 incl = warp_incl_scan3(sum, lane);
+  if (lane == 31) s_w[warp] = incl;
+  __syncthreads();
+  uint3 pre = make_uint3(0, 0, 0), ta = make_uint3(0, 0, 0);
+  for (int w = 0; w < SCAN1_THREADS / 32; ++w) {
+    const uint3 u = s_w[w];
+    if (w < warp) pre = add3(pre, u);
+    ta = add3(ta, u);
+  }
+  const bool split_on = ta.y <= (uint32_t)part_cap;
+  const uint32_t nparts = split_on ? ta.y : 0u, nsplit = split_on ? ta.z : 0u;
+  if (tid == 0) {
+    hdr->P = ta.x;
+    tile_off[ntiles] = ta.x;
+    hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
+    hdr->nsplit = nsplit;
+    hdr->next_item = 0u;
+  }
+  uint32_t run = pre.x + incl.x - sum.x, pb = pre.y + incl.y - sum.y, si = pre.z + incl.z - sum.z;
+#pragma unroll
+  for (int k = 0; k < SCAN_PER; ++k) {
+    const int64_t t = t0 + k;
+    if (t >= ntiles) break;
+    tile_off[t] = run;
+    const uint32_t np = split_on ? parts_of(c[k]) : 0u;
+    if (np) {
+      split_tab[si] = make_uint2(pb, np);
+      done[si] = 0u;
+      const uint32_t per_part = (c[k] + np - 1) / np;
+      for (uint32_t j = 0; j < np; ++j)
+        items[pb + j] = WorkItem{(uint32_t)t, run + j * per_part, min(run + c[k], run + (j + 1) * per_part),
+                                 (si << 12) | j};
+      pb += np;
+      ++si;
+    } else {
+      items[nparts + (uint32_t)t - (split_on ? si : 0u)] = WorkItem{(uint32_t)t, run, run + c[k], ITEM_WHOLE};
+    }
+    run += c[k];
+  }
+}
+
 // ---------------------------------------------------------------------------------------------------------------
 // k_scatter -- step a3: every (tile, star) pair to its slot.
 // ---------------------------------------------------------------------------------------------------------------
@@ -447,8 +504,14 @@ void launch_prep(const float* x, const float* y, const float* m, int64_t n, cons
                                                                                      tps);
 }
 
+int scan_launches(int64_t ntiles) { return ntiles <= SCAN1_TILES ? 1 : 2; }
+
 void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items,
                  uint2* split_tab, int part_cap, void* partial, uint32_t* done, cudaStream_t st) {
+  if (ntiles <= SCAN1_TILES) {
+    k_scan_one<<<1, SCAN1_THREADS, 0, st>>>(cnt, ntiles, tile_off, hdr, items, split_tab, part_cap, done);
+    return;
+  }
   const int nblk = (int)((ntiles + SCAN_TILES - 1) / SCAN_TILES);
   k_scan_a<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (uint3*)partial);
   k_scan_b<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (const uint3*)partial, nblk, tile_off, hdr, items, split_tab,

@@ -20,6 +20,7 @@ void launch_dplace(const StarRec* rec, int64_t n, const FrameParams& fp, const u
                    const uint32_t* tile_off, uint32_t* ids, cudaStream_t st);
 void launch_prep(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
                  uint32_t* cnt, uint32_t* slots, int tps, cudaStream_t st);
+int scan_launches(int64_t ntiles);  // kernels launch_scan enqueues (1 or 2)
 void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items,
                  uint2* split_tab, int part_cap, void* partial, uint32_t* done, cudaStream_t st);
 void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* slots, int tps,

@@ -57,6 +57,8 @@ def lib():
         L.starsim_render_gray.restype = ctypes.c_int
         L.starsim_set_psf.argtypes = [vp, i32]
         L.starsim_set_psf.restype = ctypes.c_int
+        L.starsim_set_binning.argtypes = [vp, i32]
+        L.starsim_set_binning.restype = ctypes.c_int
         L.starsim_set_tile_kernel.argtypes = [vp, i32]
         L.starsim_set_tile_kernel.restype = ctypes.c_int
         L.starsim_render_atomic.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
@@ -137,6 +139,13 @@ PSF_MODES = {"point": 0, "integrated": 1}
 
 def starsim_set_psf(h, mode) -> None:
     _check(h, lib().starsim_set_psf(h, PSF_MODES.get(mode, mode) if isinstance(mode, str) else int(mode)))
+
+
+BINNINGS = {"auto": 0, "atomic": 1}
+
+
+def starsim_set_binning(h, mode) -> None:
+    _check(h, lib().starsim_set_binning(h, BINNINGS.get(mode, mode) if isinstance(mode, str) else int(mode)))
 
 
 TILE_KERNELS = {"auto": 0, "lists": 1}
@@ -261,6 +270,10 @@ class Context:
     def set_psf(self, mode="point"):
         """"point" (Eq. 2 sampled at the pixel, the paper) or "integrated" (Eq. 2 integrated over the pixel)."""
         starsim_set_psf(self.h, mode)
+
+    def set_binning(self, mode="auto"):
+        """"auto" (deterministic counting sort when the frame has <= 2048 tiles and R <= 65) or "atomic"."""
+        starsim_set_binning(self.h, mode)
 
     def set_tile_kernel(self, mode="auto"):
         """"auto" (sorted-corner-bin kernel for R <= 17, else the list kernel) or "lists" (always the list kernel)."""

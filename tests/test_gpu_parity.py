@@ -379,3 +379,62 @@ def test_integrated_psf_mode_switch_and_einval(torch_dev, ctx):
     assert torch.equal(a, c) and not torch.equal(a, b)
     with pytest.raises(StarsimError):
         ctx.set_psf(7)
+
+
+# ---------------------------------------------------------------- the two binning pipelines and tile kernels agree
+
+@pytest.mark.parametrize("name,W,H,n,R,kind", [("uniform", 700, 530, 20000, 15, "uniform"),
+                                                ("clustered", 1024, 768, 30000, 9, "clustered"),
+                                                ("adversarial", 300, 200, 3000, 5, "adversarial"),
+                                                ("wide", 640, 512, 2000, 65, "uniform")])
+def test_binning_pipelines_identical(torch_dev, name, W, H, n, R, kind):
+    """dbin.cu (deterministic counting sort) and bin.cu (atomic slots + per-tile sort) build the same CSR, so the
+    image is bitwise the same; both equal the oracle's bins (reading R18)."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context
+    if kind == "clustered":
+        f = synth.clustered_field(n, W, H, seed=21)
+    elif kind == "adversarial":
+        f = synth.adversarial_field(n, W, H, R, seed=22)
+    else:
+        f = synth.uniform_field(n, W, H, seed=23, mag_hi=2.0)
+    args = to_dev(torch_dev, f)
+    res = {}
+    for mode in ("auto", "atomic"):
+        with Context(0) as c:
+            c.set_binning(mode)
+            img = c.render(*args, W, H, R / 6, R, 1.0)
+            res[mode] = (img, c.get_bins())
+    (ia, (tw, th, oa, da)), (ib, (_, _, ob, db)) = res["auto"], res["atomic"]
+    ntiles = (-(-W // tw)) * (-(-H // th))
+    assert np.array_equal(oa[:ntiles + 1], ob[:ntiles + 1]) and np.array_equal(da, db)
+    assert torch.equal(ia, ib)
+    ref_off, ref_ids = oracle.bins(f.x, f.y, f.mag, W, H, R, tw, th)
+    assert np.array_equal(oa[:ntiles + 1], ref_off) and np.array_equal(da, ref_ids)
+
+
+def test_tile_kernels_agree_within_rounding(torch_dev):
+    """k_tile_sb and k_tile sum each pixel in different (fixed) orders: equal up to fp32 rounding, both at parity."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context
+    W, H, R = 1000, 700, 15
+    f = synth.uniform_field(60000, W, H, seed=24, mag_hi=2.0)
+    args = to_dev(torch_dev, f)
+    out = {}
+    for mode in ("auto", "lists"):
+        with Context(0) as c:
+            c.set_tile_kernel(mode)
+            out[mode] = c.render(*args, W, H, 2.5, R, 1.0).double().cpu().numpy()
+    ref = oracle.render(f.x, f.y, f.mag, W, H, 2.5, R, 1.0, threads=_threads())
+    for mode in out:
+        assert_parity(out[mode], ref, f"tile kernel {mode}")
+    peak = float(np.abs(ref).max())
+    assert float(np.abs(out["auto"] - out["lists"]).max()) <= 1e-5 * peak
+
+
+def test_mode_setters_einval(torch_dev):
+    from paper_conf_ipps_lizzh12_b200 import Context, StarsimError
+    with Context(0) as c:
+        for fn in (c.set_binning, c.set_tile_kernel):
+            with pytest.raises(StarsimError):
+                fn(7)
