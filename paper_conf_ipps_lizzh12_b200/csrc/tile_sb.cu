@@ -78,9 +78,23 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
     S.gx[SB_ZJ * 32 + tid] = 0.f;
   }
 
-  if (blockIdx.x >= __ldcg(&hdr->nitems)) return;
-  {
-  const WorkItem wi = items[blockIdx.x];
+  // Persistent CTAs (SB_MINB per SM): item blockIdx.x first, then items from a counter k_scan zeroed (parts of heavy
+  // tiles come first).  The next item's index is fetched when an item starts, its WorkItem when the first chunk's
+  // profiles are done, its first star ids before the last chunk's accumulation and its records after it: the
+  // latency of starting a tile hides behind the previous tile's work.
+  __shared__ uint32_t s_next;
+  const uint32_t nitems = __ldcg(&hdr->nitems);
+  uint32_t item = blockIdx.x;
+  if (item >= nitems) return;
+  WorkItem wi = items[item];
+  StarRec rnext = {};
+  if (tid < SB_CHUNK && wi.jb + tid < wi.je) rnext = rec[ids[wi.jb + tid]];
+  for (;;) {
+  uint32_t nxt = 0;
+  if (tid == 0) nxt = atomicAdd(&hdr->next_item, 1u) + gridDim.x;
+  uint32_t item_n = 0xFFFFFFFFu, nid0 = 0;
+  WorkItem wn = {0u, 0u, 0u, 0u};
+  bool fetched = false;
   const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
   const int X0 = tx * TILE_W;    // first column of the tile
   const int Y0 = ty * TILE_H;    // first row of the tile, relative to the band
@@ -93,8 +107,6 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
     for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
 
   const uint32_t j1 = wi.je;
-  StarRec rnext = {};
-  if (tid < SB_CHUNK && wi.jb + tid < j1) rnext = rec[ids[wi.jb + tid]];
   for (uint32_t base = wi.jb; base < j1; base += SB_CHUNK) {
     // ======================= sort: thread = star (base + tid) of the tile's list
     const int nvalid = (int)min((uint32_t)SB_CHUNK, j1 - base);
@@ -251,9 +263,20 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
     const uint32_t g2e = gy_base + c2v * 128u + e2 * 64u, g2o = gy_base + c2v * 128u + (e2 ^ 1u) * 64u;
     const uint32_t x1 = gx_base + c1v * 128u, x2 = gx_base + c2v * 128u;
     const uint32_t gz = gy_base + SB_ZJ * 128u, xz = gx_base + SB_ZJ * 128u;
+    const bool first = base == wi.jb, last = nb >= j1;
+    if (first && tid == 0) s_next = nxt;
     __syncthreads();
 
-    if (tid < SB_CHUNK && nb + tid < j1) rnext = rec[nid];
+    if (first) {
+      fetched = true;
+      item_n = s_next;
+      if (item_n < nitems) wn = items[item_n];
+    }
+    if (!last) {
+      if (tid < SB_CHUNK && nb + tid < j1) rnext = rec[nid];
+    } else if (item_n < nitems && tid < SB_CHUNK && wn.jb + tid < wn.je) {
+      nid0 = __ldg(&ids[wn.jb + tid]);
+    }
     // ======================= accumulate: lane group q walks its two ranges (padded with the zero slot)
     auto step = [&](uint32_t t, bool odd) {
       const bool in1 = t < len1, in = t < L;
@@ -297,7 +320,21 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
   }
   if (tile_reduce_parts<true>(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last))
     tile_store<true>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+  if (!fetched) {  // an item with an empty list ran no chunk
+    if (tid == 0) s_next = nxt;
+    __syncthreads();
+    item_n = s_next;
+    if (item_n < nitems) {
+      wn = items[item_n];
+      if (tid < SB_CHUNK && wn.jb + tid < wn.je) nid0 = __ldg(&ids[wn.jb + tid]);
+    }
   }
+  if (item_n >= nitems) break;
+  rnext = StarRec{};
+  if (tid < SB_CHUNK && wn.jb + tid < wn.je) rnext = rec[nid0];
+  wi = wn;
+  item = item_n;
+  }  // work loop
 }
 
 void init_tile_sb_kernel() {
@@ -310,8 +347,7 @@ void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& 
                     cudaStream_t st) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
-  (void)num_sms;
-  const int64_t grid = ntiles + part_cap;  // one CTA per possible item (parts first); the rest exit at once
+  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)SB_MINB * num_sms);  // persistent CTAs
   if (fp.psf)
     k_tile_sb<true><<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab,
                                                                           part_buf, done, hdr);
