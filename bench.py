@@ -238,13 +238,27 @@ def run_ours(args, world, rank, local_rank):
     row0, rows = sdist.band_rows(H, world, rank)
     flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
 
+    # N > 1: the fused band exchange (tile epilogue stores into every rank's symmetric-memory frame over NVLink, then
+    # a device barrier) when available, else render_band + NCCL all-gather (STARSIM_EXCHANGE=allgather forces it)
+    fused = None
+    if world > 1 and args.method == "tiled" and os.environ.get("STARSIM_EXCHANGE", "fused") == "fused" \
+            and sdist.FusedFrame.available():
+        try:
+            fused = sdist.FusedFrame(H, W, dev)
+        except Exception as e:  # noqa: BLE001 -- fall back to the all-gather, say so in the JSON line
+            print(f"bench: fused exchange unavailable ({e}); using the NCCL all-gather", file=sys.stderr)
+            fused = None
+    exchange = "single" if world == 1 else ("fused-p2p" if fused is not None else "nccl-allgather")
+
     def step(xx, yy, mm):
         with torch.cuda.stream(stream):
             if args.method == "atomic":
                 ctx.render_atomic(xx, yy, mm, W, H, sigma, R, A, out=band[:H], stream=stream)
+            elif fused is not None:
+                fused.render(ctx, xx, yy, mm, sigma, R, A, stream=stream)
             else:
                 ctx.render_band(xx, yy, mm, W, H, row0, rows, sigma, R, A, out=band[:rows], stream=stream)
-            if world > 1:
+            if world > 1 and fused is None:
                 dist.all_gather_into_tensor(full, band)
 
     def barrier():
@@ -383,7 +397,8 @@ def run_ours(args, world, rank, local_rank):
                 dm.copy_(hm, non_blocking=True)
             step(dx, dy, dm)
             with torch.cuda.stream(stream):
-                himg.copy_(band[:himg.shape[0]], non_blocking=True)
+                src = fused.frame[row0:row0 + rows] if fused is not None else band[:himg.shape[0]]
+                himg[:src.shape[0]].copy_(src, non_blocking=True)
 
         for _ in range(2):
             e2e_step()
@@ -404,7 +419,45 @@ def run_ours(args, world, rank, local_rank):
         e_ms = float(te.item())
         e2e = {"value": U_frame / (e_ms * 1e-3), "unit": UNIT, "ms_per_step": e_ms,
                "h2d_bytes_per_step": int(3 * 4 * f.n), "d2h_bytes_per_step": int(himg.numel() * 4),
-               "note": "pinned host catalogue -> device, render, image -> pinned host, per step"}
+               "note": "pinned host catalogue -> device, render, image -> pinned host, per step, one stream"}
+        if world == 1 and args.method == "tiled":
+            # the same steps pipelined over two streams (one ctx, catalogue and image buffers each): step i+1's copy in
+            # and render overlap step i's copy out (PCIe is full duplex); every step still moves its own catalogue in
+            # and its own image out.  Timed from the first copy in to the last copy out.
+            streams = [stream, torch.cuda.Stream(dev)]
+            ctxs = [ctx, Context(local_rank)]
+            dbufs = [(dx, dy, dm), tuple(torch.empty_like(x) for _ in range(3))]
+            imgs = [band, torch.empty_like(band)]
+            himgs = [himg, torch.empty_like(himg).pin_memory()]
+
+            def p_step(i):
+                s_ = i & 1
+                st, cx, (ax, ay, am) = streams[s_], ctxs[s_], dbufs[s_]
+                with torch.cuda.stream(st):
+                    ax.copy_(hx, non_blocking=True)
+                    ay.copy_(hy, non_blocking=True)
+                    am.copy_(hm, non_blocking=True)
+                    cx.render_band(ax, ay, am, W, H, row0, rows, sigma, R, A, out=imgs[s_][:rows], stream=st)
+                    himgs[s_].copy_(imgs[s_][:himg.shape[0]], non_blocking=True)
+
+            for i in range(4):
+                p_step(i)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+            e0.record(streams[0])
+            streams[1].wait_event(e0)
+            for i in range(args.steps):
+                p_step(i)
+            for k in range(2):
+                e1[k].record(streams[k])
+            torch.cuda.synchronize()
+            p_ms = max(e0.elapsed_time(e1[k]) for k in range(2)) / args.steps
+            e2e = {"value": U_frame / (p_ms * 1e-3), "unit": UNIT, "ms_per_step": p_ms,
+                   "h2d_bytes_per_step": int(3 * 4 * f.n), "d2h_bytes_per_step": int(himg.numel() * 4),
+                   "latency_ms_one_stream": e_ms,
+                   "note": "pinned host catalogue -> device, render, image -> pinned host for every step; steps "
+                           "pipelined over two streams (copy out of step i overlaps copy in + render of step i+1)"}
+            ctxs[1].close()
 
     if rank != 0:
         ctx.close()
@@ -419,7 +472,7 @@ def run_ours(args, world, rank, local_rank):
                                    + (f"; {world} bands of {prow} rows + NCCL all-gather" if world > 1 else ""),
                        "W": W, "H": H, "stars": f.n, "R": R, "sigma": sigma, "gain": A, "method": args.method,
                        "frames_per_s": 1e3 / ms, "updates_per_frame": U_frame, "exps_per_frame": E_frame,
-                       "parallelism": f"bands{world}" if world > 1 else "single",
+                       "parallelism": f"bands{world}" if world > 1 else "single", "exchange": exchange,
                        "l2": "flushed before every step (256 MiB write, untimed)"},
             "clocks": clocks, "gpu_launches": int(round(launches * args.steps)),
             "gpu_launches_per_step": launches, "kernels": kernels,

@@ -83,6 +83,19 @@ int starsim_render_band(starsim_ctx* ctx, const float* x, const float* y, const 
                         int32_t width, int32_t height, int32_t row0, int32_t rows,
                         float sigma, int32_t roi, float gain, float* out_band, starsim_stream_t stream);
 
+/* Multi-GPU band exchange fused into the render (north star: bands assembled over NVLink 5 / NVSwitch; SURVEY.md
+ * §8e): renders rows [row0, row0+rows) exactly like starsim_render_band, but the tile kernel's epilogue stores every
+ * pixel of the band straight into each of the ndst full frames dsts[0..ndst), at row row0 + r of each -- the local
+ * frame and the peer GPUs' frames mapped into this process (e.g. torch symmetric memory buffer pointers), so the
+ * exchange overlaps the tiles still being rendered and no separate all-gather pass is needed.
+ *   dsts  (host) array of ndst device pointers, each float[height*width] row-major; 1 <= ndst <= 8.
+ * Same EINVAL cases as starsim_render_band, plus ndst outside [1, 8] or a NULL entry.  The library does not
+ * synchronise with the peers: the caller orders the stores before any read of a frame (a cross-GPU barrier on the
+ * stream, e.g. the symmetric-memory handle's barrier). */
+int starsim_render_band_to(starsim_ctx* ctx, const float* x, const float* y, const float* mag, int64_t n,
+                           int32_t width, int32_t height, int32_t row0, int32_t rows, float sigma, int32_t roi,
+                           float gain, float* const* dsts, int32_t ndst, starsim_stream_t stream);
+
 /* The tiled render with the output stage fused into its epilogue: every pixel
  * is written once as the gray value q = min(2^bits - 1, floor(v + 1/2)) (v <= 0 -> 0) of the same fp32 sum v that
  * starsim_render computes, so the result equals starsim_quantize(starsim_render(...)) bit for bit, with a quarter

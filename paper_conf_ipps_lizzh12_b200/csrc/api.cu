@@ -34,13 +34,15 @@ struct Launch {
 struct GraphKey {
   const void *x, *y, *mag, *out;
   int64_t n;
-  int32_t W, H, row0, rows, R, obits, psf, tile_impl, bin_impl;
+  int32_t W, H, row0, rows, R, obits, psf, tile_impl, bin_impl, ndst;
+  float* dst[MAX_DST];
   float sigma, gain;
   cudaStream_t st;
   uint64_t scratch_gen;
   bool operator==(const GraphKey& o) const {
     return x == o.x && y == o.y && mag == o.mag && out == o.out && n == o.n && W == o.W && H == o.H &&
-           row0 == o.row0 && rows == o.rows && R == o.R && obits == o.obits && psf == o.psf && tile_impl == o.tile_impl && bin_impl == o.bin_impl && sigma == o.sigma && gain == o.gain && st == o.st &&
+           row0 == o.row0 && rows == o.rows && R == o.R && obits == o.obits && psf == o.psf && tile_impl == o.tile_impl && bin_impl == o.bin_impl && ndst == o.ndst &&
+           std::equal(dst, dst + MAX_DST, o.dst) && sigma == o.sigma && gain == o.gain && st == o.st &&
            scratch_gen == o.scratch_gen;
   }
 };
@@ -185,6 +187,8 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   fp.psf = psf;
   fp.tile_impl = 0;
   fp.bin_impl = 0;
+  fp.ndst = 0;
+  for (int i = 0; i < MAX_DST; ++i) fp.dst[i] = nullptr;
   fp.obits = 0;
   fp.vec = 0;
   fp.kint = (float)(1.0 / (std::sqrt(2.0) * s));
@@ -261,7 +265,7 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
 
 int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
                  int32_t row0, int32_t rows, float sigma, int32_t R, float gain, int32_t obits, void* out,
-                 cudaStream_t st) {
+                 cudaStream_t st, float* const* dsts = nullptr, int ndst = 0) {
   DevGuard g(c->dev);
   FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain, c->psf);
   fp.obits = obits;
@@ -269,7 +273,13 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   fp.bin_impl = c->bin_impl;
   // one vector store per 8-pixel run: 32 B (fp32) / 8 B (u8) / 16 B (u16); rows must keep that alignment
   const int vb = obits == 8 ? 8 : 16;
-  fp.vec = ((W * (obits ? obits / 8 : 4)) % vb == 0 && ((uintptr_t)out % vb) == 0) ? 1 : 0;
+  bool aligned = ((uintptr_t)out % vb) == 0;
+  fp.ndst = ndst;
+  for (int i = 0; i < ndst; ++i) {
+    fp.dst[i] = dsts[i] + (int64_t)row0 * W;  // band origin inside destination frame i
+    aligned = aligned && ((uintptr_t)fp.dst[i] % vb) == 0;
+  }
+  fp.vec = ((W * (obits ? obits / 8 : 4)) % vb == 0 && aligned) ? 1 : 0;
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   const int tps = tiles_per_axis(R, TILE_W, fp.ntx) * tiles_per_axis(R, TILE_H, fp.nty);
   const int64_t pmax = n * (int64_t)tps;
@@ -296,7 +306,9 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
                  "count matrix")))
     return rc;
 
-  const GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, c->psf, c->tile_impl, c->bin_impl, sigma, gain, st, c->scratch_gen};
+  GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, c->psf, c->tile_impl, c->bin_impl, fp.ndst, {}, sigma, gain, st,
+               c->scratch_gen};
+  for (int i = 0; i < MAX_DST; ++i) key.dst[i] = fp.dst[i];
   if (st == nullptr || c->prof || !c->use_graphs) {
     if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st))) return rc;
   } else {
@@ -410,6 +422,20 @@ int starsim_render_band(starsim_ctx* c, const float* x, const float* y, const fl
   if (rc) return rc;
   if (row0 < 0 || rows < 1 || (int64_t)row0 + rows > H) return fail(c, STARSIM_EINVAL, "band not inside the image");
   return render_tiled(c, x, y, mag, n, W, H, row0, rows, sigma, R, gain, 0, out_band, (cudaStream_t)stream);
+}
+
+int starsim_render_band_to(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W,
+                           int32_t H, int32_t row0, int32_t rows, float sigma, int32_t R, float gain,
+                           float* const* dsts, int32_t ndst, starsim_stream_t stream) {
+  if (!c) return STARSIM_EINVAL;
+  if (!dsts || ndst < 1 || ndst > MAX_DST) return fail(c, STARSIM_EINVAL, "ndst outside [1, 8] or dsts NULL");
+  for (int i = 0; i < ndst; ++i)
+    if (!dsts[i]) return fail(c, STARSIM_EINVAL, "NULL destination frame");
+  int rc = validate_frame(c, x, y, mag, n, W, H, sigma, R, gain, dsts[0]);
+  if (rc) return rc;
+  if (row0 < 0 || rows < 1 || (int64_t)row0 + rows > H) return fail(c, STARSIM_EINVAL, "band not inside the image");
+  return render_tiled(c, x, y, mag, n, W, H, row0, rows, sigma, R, gain, 0, dsts[0] + (int64_t)row0 * W,
+                      (cudaStream_t)stream, dsts, ndst);
 }
 
 int starsim_render_gray(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W,

@@ -71,6 +71,8 @@ constexpr uint32_t LO_CULLED = 0x80008000u;
 __device__ __forceinline__ int lo_x_of(uint32_t lo) { return (int)(int16_t)(lo & 0xFFFFu); }
 __device__ __forceinline__ int lo_y_of(uint32_t lo) { return (int)(int16_t)(lo >> 16); }
 
+constexpr int MAX_DST = 8;  // destinations of the fused band exchange (one per GPU of an 8-GPU box)
+
 struct FrameParams {
   int32_t W, H;          // full frame
   int32_t row0, rows;    // band (row0 = 0, rows = H for a full frame)
@@ -81,6 +83,8 @@ struct FrameParams {
   int32_t psf;           // 0: Eq. 2 point-sampled (the paper); 1: Eq. 2 integrated over the pixel square (NEXT-2)
   int32_t tile_impl;     // 0: sorted-bin tile kernel when R <= SB_MAXR (tile_sb.cu), else the list kernel; 1: always the list kernel (tile.cu)
   int32_t bin_impl;      // 0: dbin.cu's deterministic binning when it applies; 1: always bin.cu's atomic-slot pipeline
+  int32_t ndst;          // > 0: the tile kernels store every pixel into dst[0..ndst) instead of `out` (fused band exchange)
+  float* dst[MAX_DST];   // band origins (row0 of each destination frame) -- local and peer-mapped frames
   float sk;              // sqrt(log2(e) / (2 sigma^2)):  exp(-d^2/(2 sigma^2)) = ex2(-(d * sk)^2)
   float kint;            // 1 / (sqrt(2) sigma): the erf argument scale of the integrated PSF
   double s_scale;        // A / (2 pi sigma^2), applied in fp64 before rounding s' to fp32

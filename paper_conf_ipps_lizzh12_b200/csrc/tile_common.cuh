@@ -59,7 +59,7 @@ __device__ __forceinline__ bool tile_reduce_parts(float2 (&acc)[4][4], const Wor
 // fp32, or (fused output stage, NEXT-1) the gray value of each pixel exactly as k_quantize computes it from the same
 // fp32 sum, as u8 / u16.  Coalesced: the 8 lane groups of a warp store 8 adjacent 8-pixel runs of a row.
 template <bool CONTIG>
-__device__ __forceinline__ void tile_store(const float2 (&acc)[4][4], const FrameParams& fp, void* __restrict__ out_,
+__device__ __forceinline__ void tile_store_one(const float2 (&acc)[4][4], const FrameParams& fp, void* __restrict__ out_,
                                            int Y0, int col0, int B, int hq) {
   if (fp.obits == 0) {
     float* out = reinterpret_cast<float*>(out_);
@@ -115,6 +115,18 @@ __device__ __forceinline__ void tile_store(const float2 (&acc)[4][4], const Fram
       }
     }
   }
+}
+
+
+// The epilogue: into `out_`, or (fused band exchange) into each of the fp.ndst destination frames.
+template <bool CONTIG>
+__device__ __forceinline__ void tile_store(const float2 (&acc)[4][4], const FrameParams& fp, void* __restrict__ out_,
+                                           int Y0, int col0, int B, int hq) {
+  if (fp.ndst == 0) {
+    tile_store_one<CONTIG>(acc, fp, out_, Y0, col0, B, hq);
+    return;
+  }
+  for (int g = 0; g < fp.ndst; ++g) tile_store_one<CONTIG>(acc, fp, fp.dst[g], Y0, col0, B, hq);
 }
 
 }  // namespace starsim

@@ -62,3 +62,55 @@ def render_frame(render_band, x, y, mag, width: int, height: int, sigma: float, 
         full_out = torch.empty((world * prow, width), dtype=torch.float32, device=dev)
     dist.all_gather_into_tensor(full_out, band_out, group=group)
     return full_out[:height], band_out
+
+
+class FusedFrame:
+    """The fused band exchange (north star: bands assembled over NVLink).
+
+    The frame lives in torch symmetric memory: every rank maps every other rank's frame into its address space, and
+    ``starsim_render_band_to`` makes the tile kernel's epilogue store each pixel of this rank's band into all of them
+    over NVLink / NVSwitch while the rest of the band is still being rendered.  A device-side barrier on the render
+    stream (the symmetric-memory handle's signal pads) then orders every rank's stores before any rank reads its
+    frame.  There is no all-gather pass: the exchange overlaps the render.  Needs CUDA peer access between the ranks'
+    GPUs (one node); ``available()`` says whether this process can use it, otherwise ``render_frame`` (NCCL
+    all-gather) is the path.
+    """
+
+    def __init__(self, height: int, width: int, device, group=None):
+        import torch
+        import torch.distributed as dist
+        import torch.distributed._symmetric_memory as symm_mem
+
+        self.height, self.width = height, width
+        self.group = group if group is not None else dist.group.WORLD
+        self.world = dist.get_world_size(self.group)
+        self.rank = dist.get_rank(self.group)
+        self.frame = symm_mem.empty((height, width), dtype=torch.float32, device=device)
+        self.handle = symm_mem.rendezvous(self.frame, self.group.group_name)
+        self.ptrs = [int(p) for p in self.handle.buffer_ptrs]
+        if len(self.ptrs) != self.world:
+            raise RuntimeError("symmetric-memory rendezvous returned a wrong number of peer buffers")
+
+    @staticmethod
+    def available() -> bool:
+        try:
+            import torch
+            import torch.distributed as dist
+            import torch.distributed._symmetric_memory  # noqa: F401
+        except Exception:
+            return False
+        return torch.cuda.is_available() and dist.is_initialized() and dist.get_backend() == "nccl"
+
+    def render(self, ctx, x, y, mag, sigma: float, roi: int, gain: float, stream=None):
+        """This rank's band into every rank's frame, then the cross-GPU barrier (all on `stream`); returns the local
+        frame, complete once the stream reaches the barrier."""
+        import torch
+
+        row0, rows = band_rows(self.height, self.world, self.rank)
+        st = stream if stream is not None else torch.cuda.current_stream()
+        with torch.cuda.stream(st):
+            if rows > 0:
+                ctx.render_band_to(x, y, mag, self.width, self.height, row0, rows, sigma, roi, gain, self.ptrs,
+                                   stream=st)
+            self.handle.barrier(channel=0)
+        return self.frame

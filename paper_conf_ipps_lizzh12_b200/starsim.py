@@ -52,6 +52,9 @@ def lib():
         L.starsim_render.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
         L.starsim_render.restype = ctypes.c_int
         L.starsim_render_band.argtypes = [vp, vp, vp, vp, i64, i32, i32, i32, i32, f32, i32, f32, vp, vp]
+        L.starsim_render_band_to.argtypes = [vp, vp, vp, vp, i64, i32, i32, i32, i32, f32, i32, f32,
+                                             ctypes.POINTER(vp), i32, vp]
+        L.starsim_render_band_to.restype = ctypes.c_int
         L.starsim_render_band.restype = ctypes.c_int
         L.starsim_render_gray.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, i32, vp, vp]
         L.starsim_render_gray.restype = ctypes.c_int
@@ -123,6 +126,17 @@ def starsim_render(h, x, y, mag, width, height, sigma, roi, gain, out, stream=No
     _check(h, lib().starsim_render(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
                                    _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
                                    int(roi), float(gain), _ptr(out, torch.float32, "out"), _stream(stream)))
+
+
+def starsim_render_band_to(h, x, y, mag, width, height, row0, rows, sigma, roi, gain, dst_ptrs, stream=None) -> None:
+    """dst_ptrs: device addresses (ints) of ndst full float32 frames (height x width), local or peer-mapped."""
+    import torch
+    n = int(x.numel()) if x is not None else 0
+    arr = (ctypes.c_void_p * max(1, len(dst_ptrs)))(*[ctypes.c_void_p(int(p)) for p in dst_ptrs])
+    _check(h, lib().starsim_render_band_to(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
+                                           _ptr(mag, torch.float32, "mag"), n, int(width), int(height), int(row0),
+                                           int(rows), float(sigma), int(roi), float(gain), arr, len(dst_ptrs),
+                                           _stream(stream)))
 
 
 def starsim_render_gray(h, x, y, mag, width, height, sigma, roi, gain, bits, out, stream=None) -> None:
@@ -283,6 +297,16 @@ class Context:
         out = self._out(rows, width, out)
         starsim_render_band(self.h, x, y, mag, width, height, row0, rows, sigma, roi, gain, out, stream)
         return out
+
+    def render_band_to(self, x, y, mag, width, height, row0, rows, sigma, roi, gain, frames, stream=None):
+        """Render rows [row0, row0+rows) into every frame of `frames` (full height x width float32 frames: CUDA
+        tensors, or raw device addresses of peer-mapped frames) -- the fused band exchange."""
+        ptrs = [f if isinstance(f, int) else f.data_ptr() for f in frames]
+        for f in frames:
+            if not isinstance(f, int) and (f.dtype.itemsize != 4 or not f.is_contiguous() or
+                                           f.numel() != width * height):
+                raise ValueError("frames must be contiguous float32 tensors of height x width")
+        starsim_render_band_to(self.h, x, y, mag, width, height, row0, rows, sigma, roi, gain, ptrs, stream)
 
     def render_atomic(self, x, y, mag, width, height, sigma, roi, gain, out=None, stream=None):
         out = self._out(height, width, out)

@@ -438,3 +438,75 @@ def test_mode_setters_einval(torch_dev):
         for fn in (c.set_binning, c.set_tile_kernel):
             with pytest.raises(StarsimError):
                 fn(7)
+
+
+# ---------------------------------------------------------------- fused band exchange (multi-destination epilogue)
+
+@pytest.mark.parametrize("tile_kernel", ["auto", "lists"])
+def test_render_band_to_writes_every_destination(torch_dev, tile_kernel):
+    """starsim_render_band_to: every band lands, bitwise equal to starsim_render_band, in each destination frame at its
+    rows (the epilogue of the fused exchange; on one GPU the destinations are local frames standing in for peers)."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context
+    W, H, R, G = 640, 512, 15, 4
+    f = synth.uniform_field(12000, W, H, seed=31, mag_hi=2.0)
+    args = to_dev(torch_dev, f)
+    with Context(0) as c:
+        c.set_tile_kernel(tile_kernel)
+        full = c.render(*args, W, H, 2.5, R, 1.0)
+        frames = [torch.full((H, W), -1.0, device=dev) for _ in range(3)]
+        rows = H // G
+        for g in range(G):
+            c.render_band_to(*args, W, H, g * rows, rows, 2.5, R, 1.0, frames)
+        for fr in frames:
+            assert torch.equal(fr, full)
+        # a single destination with an unaligned band leaves the other rows untouched
+        one = torch.full((H, W), -1.0, device=dev)
+        c.render_band_to(*args, W, H, 37, 100, 2.5, R, 1.0, [one])
+        band = c.render_band(*args, W, H, 37, 100, 2.5, R, 1.0)
+        assert torch.equal(one[37:137], band)
+        assert bool((one[:37] == -1).all()) and bool((one[137:] == -1).all())
+
+
+def test_render_band_to_einval(torch_dev):
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context, StarsimError
+    f = synth.uniform_field(10, 64, 64, seed=1)
+    args = to_dev(torch_dev, f)
+    with Context(0) as c:
+        fr = torch.zeros((64, 64), device=dev)
+        with pytest.raises(StarsimError):
+            c.render_band_to(*args, 64, 64, 0, 64, 1.0, 5, 1.0, [fr] * 9)
+        with pytest.raises(StarsimError):
+            c.render_band_to(*args, 64, 64, 60, 10, 1.0, 5, 1.0, [fr])
+        with pytest.raises(StarsimError):
+            c.render_band_to(*args, 64, 64, 0, 64, 1.0, 5, 1.0, [fr, 0])
+
+
+def test_fused_frame_single_rank(torch_dev):
+    """FusedFrame (symmetric-memory frame + render_band_to + device barrier) on a one-rank NCCL group: the frame equals
+    the plain render bitwise.  Skipped where this torch build / driver has no symmetric memory."""
+    torch, dev = torch_dev
+    import torch.distributed as dist
+    from paper_conf_ipps_lizzh12_b200 import Context
+    from paper_conf_ipps_lizzh12_b200 import dist as sdist
+    own = not dist.is_initialized()
+    if own:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29533")
+        dist.init_process_group("nccl", rank=0, world_size=1, device_id=dev)
+    try:
+        try:
+            ff = sdist.FusedFrame(384, 512, dev)
+        except Exception as e:  # no symmetric memory support here
+            pytest.skip(f"symmetric memory unavailable: {e}")
+        f = synth.uniform_field(5000, 512, 384, seed=32, mag_hi=2.0)
+        args = to_dev(torch_dev, f)
+        with Context(0) as c:
+            ref = c.render(*args, 512, 384, 2.5, 15, 1.0)
+            got = ff.render(c, *args, 2.5, 15, 1.0)
+            torch.cuda.synchronize()
+            assert torch.equal(got, ref)
+    finally:
+        if own:
+            dist.destroy_process_group()
