@@ -383,6 +383,31 @@ def run_ours(args, world, rank, local_rank):
                                       "updates_per_s": U_frame / (i_ms * 1e-3),
                                       "note": "starsim_set_psf(INTEGRATED): Eq. 2 integrated over each pixel (NEXT-2)"}
 
+        # the paper's two star-centric designs on the same frame: the atomic simulator and its lookup-table variant
+        for name, fn_, note in (("atomic", ctx.render_atomic, "starsim_render_atomic: the paper's parallel simulator "
+                                 "(Fig. 6), red.global.add per ROI pixel, nondeterministic order"),
+                                ("lut", ctx.render_lut, "starsim_render_lut: the paper's adaptive simulator "
+                                 "(PAPER.md:158-168), table at the ROI centre (reading R20, approximate off-centre)")):
+            if world > 1:
+                break
+            a_out = torch.empty((H, W), dtype=torch.float32, device=dev)
+            for _ in range(2):
+                fn_(x, y, m, W, H, sigma, R, A, out=a_out, stream=stream)
+            torch.cuda.synchronize()
+            a_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                    for _ in range(args.steps)]
+            for i in range(args.steps):
+                with torch.cuda.stream(stream):
+                    flush.fill_(float(i))
+                    a_ev[i][0].record(stream)
+                    fn_(x, y, m, W, H, sigma, R, A, out=a_out, stream=stream)
+                    a_ev[i][1].record(stream)
+            torch.cuda.synchronize()
+            a_ms = sum(a.elapsed_time(b) for a, b in a_ev) / args.steps
+            variants[name] = {"ms_per_step": a_ms, "frames_per_s": 1e3 / a_ms, "updates_per_s": U_frame / (a_ms * 1e-3),
+                              "note": note}
+            del a_out
+
     # e2e: the same C-ABI call with host (pinned) catalogue in and image out, copies inside the timed region
     e2e = None
     if not args.no_e2e:

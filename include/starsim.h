@@ -143,6 +143,18 @@ int starsim_render_atomic(starsim_ctx* ctx, const float* x, const float* y, cons
                           int32_t width, int32_t height, float sigma, int32_t roi, float gain,
                           float* out, starsim_stream_t stream);
 
+/* NEXT-4: the paper's adaptive simulator (Fig. 8), kept as a second measured comparison: the
+ * intensity matrix of Eq. 2 over the R x R ROI for a star at the ROI's centre is tabulated once (the magnitude only
+ * scales it: Eq. 1's s' times the one matrix is the paper's magnitude x ROI table), and every star adds s' times the
+ * table into its ROI with global fp32 reductions.  Reading R20: each star is taken at the centre of its
+ * ROI -- the R nearest pixels of R7, i.e. snapped to the nearest pixel centre for odd R -- so the result is exact
+ * for stars on pixel centres and an approximation otherwise (that is the paper's design).  Same arguments and EINVAL
+ * cases as starsim_render_atomic, plus roi > 63.  Honours starsim_set_psf.  Summation order nondeterministic. */
+#define STARSIM_MAX_LUT_ROI 63
+int starsim_render_lut(starsim_ctx* ctx, const float* x, const float* y, const float* mag, int64_t n,
+                       int32_t width, int32_t height, float sigma, int32_t roi, float gain,
+                       float* out, starsim_stream_t stream);
+
 /* Upload the paper's AoS star records {float mag, posX, posY}[n] (Fig. 6 step 4) from host memory
  * `host_aos` (host, any alignment) and split them into the device SoA arrays x, y, mag (device, float[n] each).
  * The host->device copy goes through a ctx-owned staging buffer on `stream`; the call returns once the host

@@ -140,6 +140,25 @@ def render(x, y, mag, W: int, H: int, sigma: float, R: int, A: float, threads: i
     return (img, U) if return_units else img
 
 
+def lut_positions(x, y, R: int):
+    """Reading R20 (the adaptive simulator): every star taken at the centre of its ROI, i.e. at
+    roi_lo(c, R) + (R - 1) / 2 on each axis (exact in fp32); non-finite coordinates are kept (the star is skipped)."""
+    def snap(c):
+        c64 = np.asarray(c, dtype=np.float32).astype(np.float64)
+        fin = np.isfinite(c64)
+        c0 = np.where(fin, c64, 0.0)
+        fl = np.floor(c0)
+        lo = (fl + (c0 >= fl + 0.5) - (R - 1) // 2) if R % 2 else (fl + 1 - R // 2)  # reading R7, exact in fp64
+        return np.where(fin, lo + 0.5 * (R - 1), c64).astype(np.float32)
+    return snap(x), snap(y)
+
+
+def render_lut(x, y, mag, W: int, H: int, sigma: float, R: int, A: float, threads: int = 1, psf: str = "point"):
+    """The adaptive simulator's image (NEXT-4): ``render`` with every star at its ROI centre."""
+    sx, sy = lut_positions(x, y, R)
+    return render(sx, sy, mag, W, H, sigma, R, A, threads=threads, psf=psf)
+
+
 def render_band(x, y, mag, W: int, H: int, row0: int, rows: int, sigma: float, R: int, A: float,
                 psf: str = "point"):
     """Rows [row0, row0+rows) of the oracle image, fp64 (rows, W)."""

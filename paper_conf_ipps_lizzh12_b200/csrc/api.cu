@@ -490,6 +490,22 @@ int starsim_render_atomic(starsim_ctx* c, const float* x, const float* y, const 
   return STARSIM_OK;
 }
 
+int starsim_render_lut(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W,
+                       int32_t H, float sigma, int32_t R, float gain, float* out, starsim_stream_t stream) {
+  if (!c) return STARSIM_EINVAL;
+  int rc = validate_frame(c, x, y, mag, n, W, H, sigma, R, gain, out);
+  if (rc) return rc;
+  if (R > STARSIM_MAX_LUT_ROI) return fail(c, STARSIM_EINVAL, "roi > 63 for the lookup-table kernel");
+  DevGuard g(c->dev);
+  cudaStream_t st = (cudaStream_t)stream;
+  const FrameParams fp = make_params(W, H, 0, H, sigma, R, gain, c->psf);
+  timed(c, 5, st, [&] { cudaMemsetAsync(out, 0, sizeof(float) * (size_t)W * H, st); });
+  timed(c, 4, st, [&] { launch_lut(x, y, mag, n, fp, out, st); });
+  if ((rc = check_launch(c, "k_lut"))) return rc;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
 int starsim_upload_aos(starsim_ctx* c, const void* host_aos, int64_t n, float* x, float* y, float* mag,
                        starsim_stream_t stream) {
   if (!c) return STARSIM_EINVAL;

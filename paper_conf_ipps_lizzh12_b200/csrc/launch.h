@@ -35,6 +35,8 @@ void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& 
                     cudaStream_t st);
 void launch_atomic(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, float* out,
                    cudaStream_t st);
+void launch_lut(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, float* out,
+                cudaStream_t st);
 void launch_quantize(const float* img, int64_t npix, int bits, void* out, int num_sms, cudaStream_t st);
 void launch_split_aos(const float* aos, int64_t n, float* x, float* y, float* m, int num_sms, cudaStream_t st);
 

@@ -1,4 +1,5 @@
-// The comparison kernel (the paper's atomic star-centric design), the output quantiser and the AoS upload split.
+// The comparison kernels (the paper's atomic star-centric design and its lookup-table variant), the output quantiser
+// and the AoS upload split.
 #include "common.cuh"
 #include "launch.h"
 
@@ -73,6 +74,69 @@ void launch_atomic(const float* x, const float* y, const float* m, int64_t n, co
   const unsigned blocks = (unsigned)((n + ATOM_WARPS - 1) / ATOM_WARPS);
   const size_t smem = sizeof(float) * 2 * fp.R * ATOM_WARPS;
   k_atomic<<<blocks, ATOM_WARPS * 32, smem, st>>>(x, y, m, n, fp, out);
+}
+
+// ---------------------------------------------------------------------------------------------------------------
+// k_lut -- NEXT-4: the paper's adaptive simulator (Fig. 8) re-shaped for sm_100a.  The paper
+// pre-builds a lookup table of a star's intensity matrix over its ROI (per magnitude) and replaces the per-pixel
+// evaluation of Eqs. 1-2 by table reads.  Here the R x R matrix of Eq. 2 for a star at the centre of its ROI is
+// built once per CTA in shared memory (the magnitude only scales it, so one matrix times the star's s' is the
+// paper's 3-D table exactly), and each warp adds s' * LUT[r][c] into its star's ROI pixels with global fp32
+// reductions (reading R20: the star sits at its ROI's centre -- exact for stars on pixel centres, odd R).
+// ---------------------------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(ATOM_WARPS * 32) k_lut(const float* __restrict__ X, const float* __restrict__ Y,
+                                                         const float* __restrict__ M, int64_t n, FrameParams fp,
+                                                         float* __restrict__ out) {
+  extern __shared__ float s_lut[];  // [R][R], then the 1-D centred profile [R]
+  const int R = fp.R;
+  float* g1 = s_lut + R * R;
+  const float cen = 0.5f * (float)(R - 1);  // exact
+  for (int k = threadIdx.x; k < R; k += blockDim.x) {
+    const float d = (float)k - cen;  // exact
+    if (!fp.psf) {
+      const float e = d * fp.sk;
+      g1[k] = ex2_approx(-(e * e));
+    } else {
+      const float ta = (d - 0.5f) * fp.kint, tb = (d + 0.5f) * fp.kint;
+      g1[k] = pix_mass(ta, edge_erfc(ta), tb, edge_erfc(tb));
+    }
+  }
+  __syncthreads();
+  for (int k = threadIdx.x; k < R * R; k += blockDim.x) s_lut[k] = g1[k / R] * g1[k % R];
+  __syncthreads();
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t i = (int64_t)blockIdx.x * ATOM_WARPS + warp;
+  if (i >= n) return;
+  const float x = X[i], y = Y[i], m = M[i];
+  const float Rf = (float)R;
+  if (!(isfinite(x) && isfinite(y) && isfinite(m))) return;
+  if (!(x > -Rf - 2.f && x < (float)fp.W + Rf + 2.f && y > (float)fp.row0 - Rf - 2.f &&
+        y < (float)(fp.row0 + fp.rows) + Rf + 2.f))
+    return;
+  const int lx = roi_lo_exact(x, R), ly = roi_lo_exact(y, R);
+  const int cx0 = max(lx, 0), cx1 = min(lx + R - 1, fp.W - 1);
+  const int cy0 = max(ly, fp.row0), cy1 = min(ly + R - 1, fp.row0 + fp.rows - 1);
+  if (cx0 > cx1 || cy0 > cy1) return;
+  const int w = cx1 - cx0 + 1, h = cy1 - cy0 + 1;
+  float s = 0.f;
+  if (lane == 0) s = (float)(fp.s_scale * pow(2.512, -(double)m));  // Eq. 1, the table's magnitude axis
+  s = __shfl_sync(0xffffffffu, s, 0);
+  const float* lut = s_lut + (cy0 - ly) * R + (cx0 - lx);
+  const float inv_w = 1.0f / (float)w;
+  float* o = out + (int64_t)(cy0 - fp.row0) * fp.W + cx0;
+  for (int p = lane; p < w * h; p += 32) {
+    const int r = __float2int_rz(((float)p + 0.5f) * inv_w);
+    const int c = p - r * w;
+    atomicAdd(o + (int64_t)r * fp.W + c, s * lut[r * R + c]);
+  }
+}
+
+void launch_lut(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, float* out,
+                cudaStream_t st) {
+  if (n <= 0) return;
+  const unsigned blocks = (unsigned)((n + ATOM_WARPS - 1) / ATOM_WARPS);
+  const size_t smem = sizeof(float) * (size_t)(fp.R * fp.R + fp.R);
+  k_lut<<<blocks, ATOM_WARPS * 32, smem, st>>>(x, y, m, n, fp, out);
 }
 
 // ---------------------------------------------------------------------------------------------------------------

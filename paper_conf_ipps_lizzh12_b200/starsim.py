@@ -66,6 +66,8 @@ def lib():
         L.starsim_set_tile_kernel.restype = ctypes.c_int
         L.starsim_render_atomic.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
         L.starsim_render_atomic.restype = ctypes.c_int
+        L.starsim_render_lut.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
+        L.starsim_render_lut.restype = ctypes.c_int
         L.starsim_upload_aos.argtypes = [vp, vp, i64, vp, vp, vp, vp]
         L.starsim_upload_aos.restype = ctypes.c_int
         L.starsim_quantize.argtypes = [vp, vp, i64, i32, vp, vp]
@@ -182,6 +184,14 @@ def starsim_render_atomic(h, x, y, mag, width, height, sigma, roi, gain, out, st
     import torch
     n = int(x.numel()) if x is not None else 0
     _check(h, lib().starsim_render_atomic(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
+                                          _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
+                                          int(roi), float(gain), _ptr(out, torch.float32, "out"), _stream(stream)))
+
+
+def starsim_render_lut(h, x, y, mag, width, height, sigma, roi, gain, out, stream=None) -> None:
+    import torch
+    n = int(x.numel()) if x is not None else 0
+    _check(h, lib().starsim_render_lut(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
                                           _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
                                           int(roi), float(gain), _ptr(out, torch.float32, "out"), _stream(stream)))
 
@@ -311,6 +321,11 @@ class Context:
     def render_atomic(self, x, y, mag, width, height, sigma, roi, gain, out=None, stream=None):
         out = self._out(height, width, out)
         starsim_render_atomic(self.h, x, y, mag, width, height, sigma, roi, gain, out, stream)
+        return out
+
+    def render_lut(self, x, y, mag, width, height, sigma, roi, gain, out=None, stream=None):
+        out = self._out(height, width, out)
+        starsim_render_lut(self.h, x, y, mag, width, height, sigma, roi, gain, out, stream)
         return out
 
     def upload_aos(self, host_aos, stream=None):

@@ -510,3 +510,28 @@ def test_fused_frame_single_rank(torch_dev):
     finally:
         if own:
             dist.destroy_process_group()
+
+
+# ---------------------------------------------------------------- NEXT-4: lookup-table (adaptive simulator) comparison
+
+@pytest.mark.parametrize("W,H,n,R,sigma,kind", [(1024, 1024, 1000, 5, 1.0, "uniform"), (700, 530, 5000, 15, 2.5, "adv"),
+                                                 (300, 200, 2000, 10, 1.7, "uniform"), (512, 384, 3000, 63, 10.5, "uniform")])
+def test_lut_parity(torch_dev, ctx, W, H, n, R, sigma, kind):
+    """starsim_render_lut against the oracle's render_lut (reading R20), and exact vs render for pixel-centred stars."""
+    f = synth.adversarial_field(n, W, H, R, seed=41) if kind == "adv" else synth.uniform_field(n, W, H, seed=42,
+                                                                                                  mag_hi=2.0)
+    ref = oracle.render_lut(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads())
+    got = ctx.render_lut(*to_dev(torch_dev, f), W, H, sigma, R, 1.0).cpu().numpy()
+    assert_parity(got, ref, f"lut {W}x{H} R={R}")
+    if R % 2:
+        fc = synth.Field(np.round(f.x).astype(np.float32), np.round(f.y).astype(np.float32), f.mag)
+        ref_c = oracle.render(fc.x, fc.y, fc.mag, W, H, sigma, R, 1.0, threads=_threads())
+        got_c = ctx.render_lut(*to_dev(torch_dev, fc), W, H, sigma, R, 1.0).cpu().numpy()
+        assert_parity(got_c, ref_c, f"lut pixel-centred R={R}")
+
+
+def test_lut_einval(torch_dev, ctx):
+    from paper_conf_ipps_lizzh12_b200 import StarsimError
+    f = synth.uniform_field(10, 64, 64, seed=1)
+    with pytest.raises(StarsimError):
+        ctx.render_lut(*to_dev(torch_dev, f), 64, 64, 1.0, 65, 1.0)

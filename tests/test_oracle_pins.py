@@ -371,3 +371,43 @@ def test_integrated_symmetric_and_full_evaluation_bitwise():
     a = oracle.render(f.x, f.y, f.mag, 24, 20, 1.1, 2 * 24 + 1, 1.0, psf="integrated")
     b = oracle.render_full(f.x, f.y, f.mag, 24, 20, 1.1, 1.0, psf="integrated")
     assert np.array_equal(a, b)
+
+
+# ---------------------------------------------------------------- NEXT-4: the adaptive simulator's table (reading R20)
+
+@pytest.mark.parametrize("R", [1, 2, 5, 10, 15, 16])
+def test_lut_positions_are_the_roi_centres(R):
+    """lut_positions snaps every coordinate to the centre of its ROI: lo + (R-1)/2 with lo the oracle's exact roi_lo
+    (pinned above against Fraction), checked on the adversarial coordinates."""
+    cs = np.array(_adversarial_coords()[:4000], dtype=np.float32)
+    sx, _ = oracle.lut_positions(cs, cs, R)
+    for c, s in zip(cs, sx):
+        assert float(s) == oracle.roi_lo(float(c), R) + 0.5 * (R - 1)
+        # the snapped star has the same ROI (the table is laid over the star's own R nearest pixels)
+        assert oracle.roi_lo(float(s), R) == oracle.roi_lo(float(c), R)
+
+
+def test_lut_equals_render_for_pixel_centred_stars():
+    """For stars on pixel centres and odd R the table is exact: render_lut == render bitwise; sub-pixel stars move."""
+    rng_ = np.random.default_rng(40)
+    W, H, R = 120, 90, 9
+    x = rng_.integers(-5, W + 5, 300).astype(np.float32)
+    y = rng_.integers(-5, H + 5, 300).astype(np.float32)
+    m = rng_.uniform(0, 5, 300).astype(np.float32)
+    a = oracle.render_lut(x, y, m, W, H, 1.5, R, 1.0)
+    b = oracle.render(x, y, m, W, H, 1.5, R, 1.0)
+    assert np.array_equal(a, b)
+    c = oracle.render_lut(x + np.float32(0.3), y - np.float32(0.2), m, W, H, 1.5, R, 1.0)
+    assert np.array_equal(c, b)                      # |offset| < 1/2: same centres
+    d = oracle.render(x + np.float32(0.3), y - np.float32(0.2), m, W, H, 1.5, R, 1.0)
+    assert not np.array_equal(d, b)
+
+
+def test_lut_star_mass_is_the_centred_closed_form():
+    """A sub-pixel star rendered by the table carries the centred ROI mass g * M1(0)^2 (C1: 0.98181476105437437),
+    not its own sub-pixel mass, and its image is symmetric about the ROI centre."""
+    x, y, m = star(10.3, 9.8)
+    img = oracle.render_lut(x, y, m, 21, 21, 1.0, 5, 1.0)
+    assert abs(img.sum() - 0.98181476105437437) < 1e-13
+    assert np.array_equal(img, img[::-1, ::-1]) and np.array_equal(img, img.T)
+    assert img[10, 10] == img.max()

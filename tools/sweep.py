@@ -1,5 +1,5 @@
 #!/usr/bin/env python
-"""Star-count and ROI sweeps of the tiled path against the atomic comparison kernel (the C3 / C4
+"""Star-count and ROI sweeps of the tiled path against the atomic and lookup-table comparison kernels (the C3 / C4
 "selection" study, the B200 analogue of the paper's Table III).
 
     python tools/sweep.py [--sweep c3|c4|all] [--steps 10] [--warmup 3] > profiles/<round>_sweep.jsonl
@@ -61,8 +61,8 @@ def run_point(ctx, label, cfg, f, steps, warmup, stream, flush, out):
     gain = synth.bench_gain(cfg.sigma)
     U = units(f, cfg)
     res = {}
-    for method in ("tiled", "atomic"):
-        fn_ = ctx.render if method == "tiled" else ctx.render_atomic
+    for method in ("tiled", "atomic", "lut"):
+        fn_ = {"tiled": ctx.render, "atomic": ctx.render_atomic, "lut": ctx.render_lut}[method]
         med, lo, hi = time_frames(lambda: fn_(x, y, m, cfg.W, cfg.H, cfg.sigma, cfg.R, gain, out=out, stream=stream),
                                   steps, warmup, stream, flush)
         line = {"sweep": label, "W": cfg.W, "H": cfg.H, "stars": f.n, "R": cfg.R, "sigma": cfg.sigma,
@@ -78,7 +78,8 @@ def run_point(ctx, label, cfg, f, steps, warmup, stream, flush, out):
         res[method] = med
         print(json.dumps(line), flush=True)
     print(json.dumps({"sweep": label, "stars": f.n, "R": cfg.R, "winner": min(res, key=res.get),
-                      "atomic_over_tiled": res["atomic"] / res["tiled"]}), flush=True)
+                      "atomic_over_tiled": res["atomic"] / res["tiled"], "lut_over_atomic": res["lut"] / res["atomic"]}),
+          flush=True)
 
 
 def main():
