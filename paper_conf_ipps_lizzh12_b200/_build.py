@@ -35,7 +35,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and up_to_date():
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, *ARCH, *FLAGS, "-o", tmp, *sources(), "-lcudart"]
+    extra = os.environ.get("STARSIM_NVCC_EXTRA", "").split()  # e.g. -DSTARSIM_SB_TIMING (debug builds only)
+    cmd = [NVCC, *ARCH, *FLAGS, *extra, "-o", tmp, *sources(), "-lcudart"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     log = os.path.join(PKG, "build.log")
     with open(log, "w") as fh:

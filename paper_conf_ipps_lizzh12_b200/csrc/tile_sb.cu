@@ -33,6 +33,16 @@
 
 namespace starsim {
 
+#ifdef STARSIM_SB_TIMING
+// per-phase SM cycles summed over warps (debug builds only): sort, scan, profiles, wait, accumulate, chunks
+__device__ unsigned long long g_sb_prof[6];
+#define SB_T(v) const long long v = clock64()
+#define SB_ACC(k, d) if (lane == 0) atomicAdd(&g_sb_prof[k], (unsigned long long)(d))
+#else
+#define SB_T(v)
+#define SB_ACC(k, d)
+#endif
+
 // corner bins: band key 0..4 (0 = the ROI comes in over the tile's top edge, else 1 + band) x strip key 0..16 (0 =
 // it comes in over the left edge, else 1 + strip), band-major
 constexpr int SB_NSK = NSTRIPS + 1;
@@ -45,7 +55,7 @@ struct SbSmem {
   float gy[(SB_CHUNK + 1) * 32];    // sorted star j: two 16-float band slots, slot k at j*32 + ((j ^ k) & 1) * 16
   float gx[(SB_CHUNK + 1) * 32];    // sorted star j: ring of four 8-float strip slots, strip Q at j*32 + (Q & 3) * 8
   uint32_t hist[TILE_WARPS][SB_NBIN];      // per warp: stars of each corner bin
-  uint32_t binoff[SB_NBIN][TILE_WARPS];    // per bin: stars of the bin in the warps before
+  uint32_t binoff[TILE_WARPS][SB_NBIN];    // per warp, per bin: stars of the bin in the warps before
   uint32_t binstart[SB_NBIN + 1];          // exclusive scan of the bin totals (bin-major)
 };
 
@@ -121,6 +131,7 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
       r1 = min(ly + fp.R - 1, THe - 1);
       if (c0 <= c1 && r0 <= r1) key = (uint32_t)((ly < 0 ? 0 : 1 + (r0 >> 4)) * SB_NSK + (lx < 0 ? 0 : 1 + (c0 >> 3)));
     }
+    SB_T(t0);
     const uint32_t peers = __match_any_sync(0xffffffffu, key);
     const uint32_t rank = __popc(peers & lt);
     // No barrier before this: the previous chunk's readers of hist (warp 0's scan) finished before its second
@@ -134,18 +145,21 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
     const uint32_t nb = base + SB_CHUNK;
     const uint32_t nid = tid < SB_CHUNK && nb + tid < j1 ? __ldg(&ids[nb + tid]) : 0u;
     __syncthreads();
+    SB_T(t1);
     if (warp == 0) {
+      // per bin: its 8 histogram words first (independent loads), then the prefix over the warps
       uint32_t tot[3], sum = 0;
 #pragma unroll
       for (int h = 0; h < 3; ++h) {
         const int bin = 3 * lane + h;
-        uint32_t run = 0;
-        if (bin < SB_NBIN) {
+        uint32_t c[TILE_WARPS];
 #pragma unroll
-          for (int w = 0; w < TILE_WARPS; ++w) {
-            S.binoff[bin][w] = run;
-            run += S.hist[w][bin];
-          }
+        for (int w = 0; w < TILE_WARPS; ++w) c[w] = bin < SB_NBIN ? S.hist[w][bin] : 0u;
+        uint32_t run = 0;
+#pragma unroll
+        for (int w = 0; w < TILE_WARPS; ++w) {
+          if (bin < SB_NBIN) S.binoff[w][bin] = run;
+          run += c[w];
         }
         tot[h] = run;
         sum += run;
@@ -165,9 +179,10 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
       }
     }
     __syncthreads();
+    SB_T(t2);
     // ======================= prep: the star's profiles at its sorted place j
     if (key < SB_NBIN) {
-      const uint32_t j = S.binstart[key] + S.binoff[key][warp] + rank;
+      const uint32_t j = S.binstart[key] + S.binoff[warp][key] + rank;
       const float yr = r.y - (float)IY0, xr = r.x - (float)X0;  // exact
       const float2 sk2 = make_float2(sk, sk), s2 = make_float2(r.s, r.s);
       // first band / strip of the slots: the corner bin's (-1 for an ROI that comes in over the top / left edge)
@@ -265,7 +280,9 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
     const uint32_t gz = gy_base + SB_ZJ * 128u, xz = gx_base + SB_ZJ * 128u;
     const bool first = base == wi.jb, last = nb >= j1;
     if (first && tid == 0) s_next = nxt;
+    SB_T(t3);
     __syncthreads();
+    SB_T(t4);
 
     if (first) {
       fetched = true;
@@ -305,6 +322,17 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
       step(st + 1, true);
     }
     if (st < steps) step(st, false);
+#ifdef STARSIM_SB_TIMING
+    {
+      SB_T(t5);
+      SB_ACC(0, t1 - t0);
+      SB_ACC(1, t2 - t1);
+      SB_ACC(2, t3 - t2);
+      SB_ACC(3, t4 - t3);
+      SB_ACC(4, t5 - t4);
+      SB_ACC(5, 1);
+    }
+#endif
   }
 
   // ======================= output
@@ -336,6 +364,20 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
   item = item_n;
   }  // work loop
 }
+
+#ifdef STARSIM_SB_TIMING
+extern "C" int starsim_debug_sb_timing(double* out6, int reset) {
+  unsigned long long h[6];
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(h, g_sb_prof, sizeof(h));
+  for (int i = 0; i < 6; ++i) out6[i] = (double)h[i];
+  if (reset) {
+    unsigned long long z[6] = {0, 0, 0, 0, 0, 0};
+    cudaMemcpyToSymbol(g_sb_prof, z, sizeof(z));
+  }
+  return 0;
+}
+#endif
 
 void init_tile_sb_kernel() {
   cudaFuncSetAttribute(k_tile_sb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SbSmem));
