@@ -17,7 +17,7 @@ import threading
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libstarsim.so")
+LIB_PATH = os.environ.get("STARSIM_LIB") or os.path.join(_PKG, "libstarsim.so")  # override: A/B tooling only
 
 STARSIM_OK, STARSIM_EINVAL, STARSIM_ENOMEM, STARSIM_ECUDA, STARSIM_ENODEV = 0, -1, -2, -3, -4
 KCLASSES = ("prep", "sort", "csr", "tile", "atomic", "memset", "quantize", "aos")
