@@ -193,16 +193,14 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
       const int ra0 = r0 - 16 * b0, rb0 = r1 - 16 * b0;      // ROI rows relative to band b0 (band b0+1: -16)
       const uint32_t m0 = (0xFFFFFFFFu >> (31 - min(rb0, 31))) & (0xFFFFFFFFu << ra0);  // ROI rows over both bands
       const float bf0 = (float)(16 * b0) - yr;              // exact
-      const int qfirst = ra0 >> 2;
 #pragma unroll
       for (int c = 0; c < 8; ++c) {
-        const int w = (qfirst + c) & 7;
-        const int k = w >> 2, hh = w & 3;
-        float4* dst = reinterpret_cast<float4*>(&S.gy[j * 32 + ((j ^ (uint32_t)k) & 1u) * 16 + hh * 4]);
-        if (c >= 5) {
-          *dst = make_float4(0.f, 0.f, 0.f, 0.f);
-          continue;
-        }
+        // lane-rotated order: u = (c + lane) & 7 picks the slot half u & 1 and the row group u >> 1, so the 8 lanes
+        // of each quarter warp store to 8 distinct bank quads
+        const int u = (c + lane) & 7;
+        const int hh = u >> 1, k = (u ^ (int)j) & 1;
+        const int w = 4 * k + hh;
+        float4* dst = reinterpret_cast<float4*>(&S.gy[j * 32 + (u & 1) * 16 + hh * 4]);
         const uint32_t m = m0 >> (4 * w);                  // bit i: row 4 w + i of the window in the ROI
         const float bf = bf0 + (float)(4 * w);              // exact
         float v[4];
