@@ -43,6 +43,8 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="T")
     ap.add_argument("--method", default="tiled", choices=["tiled", "atomic"])
+    ap.add_argument("--tile-kernel", default="auto", choices=["auto", "lists", "sb"],
+                    help="starsim_set_tile_kernel mode (A/B comparisons; the default is the product path)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     return ap.parse_args()
@@ -230,6 +232,7 @@ def run_ours(args, world, rank, local_rank):
     A = synth.bench_gain(sigma)
     U_frame, E_frame = units_of(f, W, H, R)
     ctx = Context(local_rank)
+    ctx.set_tile_kernel(args.tile_kernel)
     stream = torch.cuda.Stream(dev)
     x, y, m = (torch.from_numpy(a).to(dev) for a in (f.x, f.y, f.mag))
     prow = sdist.padded_band_rows(H, world)

@@ -51,7 +51,7 @@ struct starsim_ctx {
   int dev = 0;
   int num_sms = 148;
   int32_t psf = 0;  // starsim_set_psf: 0 point-sampled Eq. 2, 1 pixel-integrated (NEXT-2)
-  int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto (sorted bins when R <= 17), 1 per-block lists
+  int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto (warp-specialised sorted bins when R <= 17), 1 lists, 2 sorted bins
   int32_t bin_impl = 0;   // starsim_set_binning: 0 auto (dbin.cu when it applies), 1 always bin.cu's pipeline
   std::string err;
   Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat;
@@ -468,8 +468,8 @@ int starsim_set_binning(starsim_ctx* c, int32_t mode) {
 
 int starsim_set_tile_kernel(starsim_ctx* c, int32_t mode) {
   if (!c) return STARSIM_EINVAL;
-  if (mode != STARSIM_TILE_AUTO && mode != STARSIM_TILE_LISTS)
-    return fail(c, STARSIM_EINVAL, "tile kernel mode must be STARSIM_TILE_AUTO or STARSIM_TILE_LISTS");
+  if (mode != STARSIM_TILE_AUTO && mode != STARSIM_TILE_LISTS && mode != STARSIM_TILE_SB)
+    return fail(c, STARSIM_EINVAL, "tile kernel mode must be STARSIM_TILE_AUTO, STARSIM_TILE_LISTS or STARSIM_TILE_SB");
   c->tile_impl = mode;
   c->err.clear();
   return STARSIM_OK;

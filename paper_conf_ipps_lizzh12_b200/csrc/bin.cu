@@ -537,6 +537,7 @@ void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, in
 void init_kernels() {
   init_tile_kernel();
   init_tile_sb_kernel();
+  init_tile_ws_kernel();
   init_dbin_kernels();
 }
 

@@ -81,7 +81,7 @@ struct FrameParams {
   int32_t vec;           // 1 if every 8-pixel run of an out row is aligned for one vector store
   int32_t obits;         // 0: fp32 image; 8 / 16: gray values quantised in the epilogue (u8 / u16 image)
   int32_t psf;           // 0: Eq. 2 point-sampled (the paper); 1: Eq. 2 integrated over the pixel square (NEXT-2)
-  int32_t tile_impl;     // 0: sorted-bin tile kernel when R <= SB_MAXR (tile_sb.cu), else the list kernel; 1: always the list kernel (tile.cu)
+  int32_t tile_impl;     // 0: warp-specialised sorted-bin kernel when R <= SB_MAXR (tile_ws.cu), else the list kernel; 1: always the list kernel (tile.cu); 2: tile_sb.cu when R <= SB_MAXR
   int32_t bin_impl;      // 0: dbin.cu's deterministic binning when it applies; 1: always bin.cu's atomic-slot pipeline
   int32_t ndst;          // > 0: the tile kernels store every pixel into dst[0..ndst) instead of `out` (fused band exchange)
   float* dst[MAX_DST];   // band origins (row0 of each destination frame) -- local and peer-mapped frames

@@ -28,7 +28,7 @@ constexpr int DP_SPT = DB_CTA / DP_THREADS;      // stars per thread (strided by
 constexpr int DCS_THREADS = 256;
 static_assert(DB_MAXT <= 65536 && DB_CTA <= 65536, "tile ids, slots and star indices are 16-bit in k_dplace");
 
-__global__ void __launch_bounds__(DC_THREADS) k_dcount(const float* __restrict__ X, const float* __restrict__ Y,
+__global__ void __launch_bounds__(DC_THREADS, 2) k_dcount(const float* __restrict__ X, const float* __restrict__ Y,
                                                        const float* __restrict__ M, int64_t n, FrameParams fp,
                                                        StarRec* __restrict__ rec, uint32_t* __restrict__ C,
                                                        int nCTA, int ntiles) {
@@ -139,7 +139,7 @@ __device__ __forceinline__ int box_tile(uint32_t code, int e, int ntx) {
   return (int)(code & 0xFFFFu) + ey * ntx + ex;
 }
 
-__global__ void __launch_bounds__(DP_THREADS) k_dplace(const StarRec* __restrict__ rec, int64_t n, FrameParams fp,
+__global__ void __launch_bounds__(DP_THREADS, 2) k_dplace(const StarRec* __restrict__ rec, int64_t n, FrameParams fp,
                                                        const uint32_t* __restrict__ C, int nCTA, int ntiles,
                                                        const uint32_t* __restrict__ tile_off,
                                                        uint32_t* __restrict__ ids) {

@@ -10,6 +10,7 @@ namespace starsim {
 void init_kernels();
 void init_tile_kernel();
 void init_tile_sb_kernel();
+void init_tile_ws_kernel();
 void init_dbin_kernels();
 size_t dbin_smem(int ntiles);
 int dbin_ctas(int64_t n);
@@ -31,6 +32,9 @@ void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
                  cudaStream_t st);
 void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
+                    const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
+                    cudaStream_t st);
+void launch_tile_ws(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
                     cudaStream_t st);
 void launch_atomic(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, float* out,

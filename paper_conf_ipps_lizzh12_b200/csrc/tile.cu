@@ -347,6 +347,10 @@ void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
                  cudaStream_t st) {
   if (fp.R <= SB_MAXR && fp.tile_impl == 0) {
+    launch_tile_ws(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st);
+    return;
+  }
+  if (fp.R <= SB_MAXR && fp.tile_impl == 2) {
     launch_tile_sb(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st);
     return;
   }

@@ -11,11 +11,22 @@ namespace starsim {
 template <bool CONTIG>
 __device__ __forceinline__ int lane_row(int B, int hq, int i) { return CONTIG ? 16 * B + 4 * hq + i : 16 * B + hq + 4 * i; }
 
+// Barrier over the threads that own the tile's accumulators: the whole CTA (NBAR = 0), or -- in the warp-specialised
+// kernel, whose producer warps never take part -- named barrier 2 over the first NBAR threads.
+template <int NBAR>
+__device__ __forceinline__ void acc_barrier() {
+  if (NBAR == 0)
+    __syncthreads();
+  else
+    asm volatile("bar.sync 2, %0;" ::"n"(NBAR) : "memory");
+}
+
 // A whole tile is written to `out` directly; a part of a split heavy tile (wi.aux != ITEM_WHOLE) writes its
 // 128 x 64 partial to part_buf, and the last part to finish (per-tile counter) sums the parts in part order -- a
 // fixed order, so the image stays deterministic.  Returns false for a part that is not the last one (nothing left
-// to write); on true, acc holds the tile's final sums.  Contains block barriers: every thread of the CTA calls it.
-template <bool CONTIG>
+// to write); on true, acc holds the tile's final sums.  Contains barriers (acc_barrier<NBAR>): every accumulating
+// thread calls it.
+template <bool CONTIG, int NBAR = 0>
 __device__ __forceinline__ bool tile_reduce_parts(float2 (&acc)[4][4], const WorkItem& wi,
                                                   const uint2* __restrict__ split_tab, float* __restrict__ part_buf,
                                                   uint32_t* __restrict__ done, int B, int wx, int q, int hq,
@@ -31,9 +42,9 @@ __device__ __forceinline__ bool tile_reduce_parts(float2 (&acc)[4][4], const Wor
     o[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
   }
   __threadfence();
-  __syncthreads();
+  acc_barrier<NBAR>();
   if (tid == 0) *s_last = atomicAdd(&done[wi.aux >> 12], 1u) == sp.y - 1;
-  __syncthreads();
+  acc_barrier<NBAR>();
   if (!*s_last) return false;
   __threadfence();
 #pragma unroll

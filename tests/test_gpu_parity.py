@@ -29,10 +29,11 @@ def torch_dev():
     return torch, torch.device("cuda:0")
 
 
-@pytest.fixture(scope="module", params=["auto", "lists"])
+@pytest.fixture(scope="module", params=["auto", "lists", "sb"])
 def ctx(torch_dev, request):
-    """Every test runs against both tile kernels: "auto" (the sorted-corner-bin kernel for R <= 17, the list kernel
-    above) and "lists" (the per-block entry-list kernel for every R)."""
+    """Every test runs against the three tile kernels: "auto" (the warp-specialised sorted-corner-bin kernel for
+    R <= 17, the list kernel above), "lists" (the per-block entry-list kernel for every R) and "sb" (the sorted-bin
+    kernel with both roles in every warp)."""
     from paper_conf_ipps_lizzh12_b200 import Context
     c = Context(0)
     c.set_tile_kernel(request.param)
@@ -432,6 +433,27 @@ def test_tile_kernels_agree_within_rounding(torch_dev):
     assert float(np.abs(out["auto"] - out["lists"]).max()) <= 1e-5 * peak
 
 
+@pytest.mark.parametrize("psf", ["point", "integrated"])
+@pytest.mark.parametrize("W,H,n,R,seed", [(1000, 700, 60000, 15, 24), (4096, 4096, 1000000, 15, 1),
+                                          (301, 177, 3000, 17, 5), (700, 500, 0, 9, 6)])
+def test_ws_equals_sb_bitwise(torch_dev, psf, W, H, n, R, seed):
+    """The warp-specialised kernel (auto) sums every pixel in k_tile_sb's order: the images are identical bit for bit,
+    also with heavy tiles split into parts (the clustered field) and with the integrated PSF."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context
+    f = synth.uniform_field(n, W, H, seed=seed, mag_hi=15.0)
+    if n == 60000:
+        f = _dense_field(n, W, H, 500.0, 350.0, 120.0, seed=seed)
+    args = to_dev(torch_dev, f)
+    out = {}
+    for mode in ("auto", "sb"):
+        with Context(0) as c:
+            c.set_tile_kernel(mode)
+            c.set_psf(psf)
+            out[mode] = c.render(*args, W, H, R / 6, R, 1.0)
+    assert torch.equal(out["auto"], out["sb"])
+
+
 def test_mode_setters_einval(torch_dev):
     from paper_conf_ipps_lizzh12_b200 import Context, StarsimError
     with Context(0) as c:
@@ -442,7 +464,7 @@ def test_mode_setters_einval(torch_dev):
 
 # ---------------------------------------------------------------- fused band exchange (multi-destination epilogue)
 
-@pytest.mark.parametrize("tile_kernel", ["auto", "lists"])
+@pytest.mark.parametrize("tile_kernel", ["auto", "lists", "sb"])
 def test_render_band_to_writes_every_destination(torch_dev, tile_kernel):
     """starsim_render_band_to: every band lands, bitwise equal to starsim_render_band, in each destination frame at its
     rows (the epilogue of the fused exchange; on one GPU the destinations are local frames standing in for peers)."""
