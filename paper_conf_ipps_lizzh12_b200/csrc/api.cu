@@ -219,23 +219,28 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
   int rc;
   if (dbin_ok(fp, ntiles)) {
     // deterministic counting sort (dbin.cu): no memset, no atomics on global counters, no per-tile sort
+    // (step a2 runs inside k_dplace; an empty catalogue has no k_dplace, so k_scan plans its all-empty tiles)
     uint32_t* C = (uint32_t*)c->cmat.p;
     if (n > 0) {
       timed(c, 0, st, [&] { launch_dcount(x, y, mag, n, fp, rec, C, (int)ntiles, st); });
       if ((rc = check_launch(c, "k_dcount"))) return rc;
-    }
-    timed(
-        c, 2, st,
-        [&] {
-          launch_dcolscan(C, n, (int)ntiles, cnt, st);
-          launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap,
-                      c->partial.p, done, st);
-        },
-        1 + scan_launches(ntiles));
-    if ((rc = check_launch(c, "k_dcolscan/k_scan"))) return rc;
-    if (n > 0) {
-      timed(c, 1, st, [&] { launch_dplace(rec, n, fp, C, (int)ntiles, tile_off, ids, st); });
+      timed(c, 2, st, [&] { launch_dcolscan(C, n, (int)ntiles, cnt, 1, st); });  // dense totals for k_dplace
+      if ((rc = check_launch(c, "k_dcolscan"))) return rc;
+      timed(c, 1, st, [&] {
+        launch_dplace(rec, n, fp, C, (int)ntiles, cnt, tile_off, hdr, (WorkItem*)c->items.p,
+                      (uint2*)c->split_tab.p, part_cap, done, ids, st);
+      });
       if ((rc = check_launch(c, "k_dplace"))) return rc;
+    } else {
+      timed(
+          c, 2, st,
+          [&] {
+            launch_dcolscan(C, n, (int)ntiles, cnt, CNT_STRIDE, st);
+            launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap,
+                        c->partial.p, done, st);
+          },
+          1 + scan_launches(ntiles));
+      if ((rc = check_launch(c, "k_dcolscan/k_scan"))) return rc;
     }
   } else {
     timed(c, 5, st, [&] { cudaMemsetAsync(hdr, 0, zbytes, st); });

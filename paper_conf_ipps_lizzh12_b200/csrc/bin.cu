@@ -14,6 +14,7 @@
 
 #include "common.cuh"
 #include "launch.h"
+#include "plan.cuh"
 #include "prep.cuh"
 
 namespace starsim {
@@ -50,26 +51,9 @@ __global__ void __launch_bounds__(PREP_THREADS) k_prep(const float* __restrict__
 //   on the tile's own list, so it is the same for any band decomposition.  If the parts would need more than
 //   `part_cap` partial buffers, nothing is split.
 // ---------------------------------------------------------------------------------------------------------------
-__device__ __forceinline__ uint32_t parts_of(uint32_t len) {
-  if (len <= (uint32_t)SPLIT_LEN) return 0u;
-  return min((len + SPLIT_LEN - 1) / SPLIT_LEN, 4095u);
-}
-
 // Two kernels, SCAN_TILES tiles per CTA (SCAN_PER per thread): k_scan_a writes each CTA's sums (pairs, parts, split
 // tiles); k_scan_b re-reduces the sums of the CTAs before it and of all CTAs (a few hundred at most), scans its own
 // tiles and writes tile_off and the work items.
-__device__ __forceinline__ uint3 add3(uint3 a, uint3 b) { return make_uint3(a.x + b.x, a.y + b.y, a.z + b.z); }
-
-__device__ __forceinline__ uint3 warp_incl_scan3(uint3 v, int lane) {
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t x = __shfl_up_sync(0xffffffffu, v.x, o), y = __shfl_up_sync(0xffffffffu, v.y, o),
-                   z = __shfl_up_sync(0xffffffffu, v.z, o);
-    if (lane >= o) v = add3(v, make_uint3(x, y, z));
-  }
-  return v;
-}
-
 // block-wide exclusive scan of uint3 (SCAN_THREADS threads); *total receives the block sum
 __device__ __forceinline__ uint3 block_excl_scan3(uint3 v, uint3* s_w, uint3* total) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -147,22 +131,7 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_b(const uint32_t* __restr
   for (int k = 0; k < SCAN_PER; ++k) {
     const int64_t t = t0 + k;
     if (t >= ntiles) break;
-    tile_off[t] = run;
-    const uint32_t np = split_on ? parts_of(c[k]) : 0u;
-    if (np) {
-      split_tab[si] = make_uint2(pb, np);
-      done[si] = 0u;  // the parts' completion counter (k_tile)
-      const uint32_t per_part = (c[k] + np - 1) / np;
-      for (uint32_t j = 0; j < np; ++j)
-        items[pb + j] = WorkItem{(uint32_t)t, run + j * per_part, min(run + c[k], run + (j + 1) * per_part),
-                                 (si << 12) | j};
-      pb += np;
-      ++si;
-    } else {
-      // whole tiles follow the parts, in tile order: index = nparts + (tiles before t that are not split)
-      items[nparts + (uint32_t)t - (split_on ? si : 0u)] = WorkItem{(uint32_t)t, run, run + c[k], ITEM_WHOLE};
-    }
-    run += c[k];
+    plan_tile((uint32_t)t, c[k], run, pb, si, nparts, split_on, tile_off, items, split_tab, done);
   }
 }
 
@@ -205,21 +174,7 @@ __global__ void __launch_bounds__(SCAN1_THREADS) k_scan_one(const uint32_t* __re
   for (int k = 0; k < SCAN_PER; ++k) {
     const int64_t t = t0 + k;
     if (t >= ntiles) break;
-    tile_off[t] = run;
-    const uint32_t np = split_on ? parts_of(c[k]) : 0u;
-    if (np) {
-      split_tab[si] = make_uint2(pb, np);
-      done[si] = 0u;
-      const uint32_t per_part = (c[k] + np - 1) / np;
-      for (uint32_t j = 0; j < np; ++j)
-        items[pb + j] = WorkItem{(uint32_t)t, run + j * per_part, min(run + c[k], run + (j + 1) * per_part),
-                                 (si << 12) | j};
-      pb += np;
-      ++si;
-    } else {
-      items[nparts + (uint32_t)t - (split_on ? si : 0u)] = WorkItem{(uint32_t)t, run, run + c[k], ITEM_WHOLE};
-    }
-    run += c[k];
+    plan_tile((uint32_t)t, c[k], run, pb, si, nparts, split_on, tile_off, items, split_tab, done);
   }
 }
 

@@ -6,14 +6,16 @@
 //                (prep_star); per tile the number of pairs of the CTA (shared-memory atomics -- counts do not depend
 //                on order) -> C[tile][c].
 //   k_dcolscan   per tile (one warp): exclusive scan of C[tile][0..nCTA) in CTA order (in place) and the tile's
-//                total -> cnt[tile] (then bin.cu's k_scan_a/b: tile_off, the work list).
-//   k_dplace     CTA c again: its pairs are grouped by tile in shared memory (slots from shared-memory atomics, in
+//                total -> cnt[tile].
+//   k_dplace     CTA c again: step a2 first (every CTA scans the tile totals; CTA c writes tile_off and the work
+//                items of the tiles t = c mod nCTA -- no scan launch between the two), then its pairs are grouped by tile in shared memory (slots from shared-memory atomics, in
 //                arbitrary order); a pair's rank in its group is the number of the group's stars with a smaller
 //                index, and it goes to tile_off[t] + C[t][c] + rank: every tile list holds its stars in ascending
 //                star index -- the unique CSR (reading R18), bit-exact, with no sort pass over the lists and no
 //                atomics on global memory.  (Groups are (tile, 2048-star block) pairs: a few stars each.)
 #include "common.cuh"
 #include "launch.h"
+#include "plan.cuh"
 #include "prep.cuh"
 
 namespace starsim {
@@ -26,6 +28,7 @@ constexpr int DP_WARPS = DP_THREADS / 32;
 constexpr int DP_KEYS = DB_CTA * 4;              // at most 2 x 2 tiles per star
 constexpr int DP_SPT = DB_CTA / DP_THREADS;      // stars per thread (strided by DP_THREADS)
 constexpr int DCS_THREADS = 256;
+constexpr int DCS_PER = 8;                       // k_dcolscan: consecutive CTA counts per lane
 static_assert(DB_MAXT <= 65536 && DB_CTA <= 65536, "tile ids, slots and star indices are 16-bit in k_dplace");
 
 __global__ void __launch_bounds__(DC_THREADS, 2) k_dcount(const float* __restrict__ X, const float* __restrict__ Y,
@@ -66,25 +69,36 @@ __global__ void __launch_bounds__(DC_THREADS, 2) k_dcount(const float* __restric
 }
 
 __global__ void __launch_bounds__(DCS_THREADS) k_dcolscan(uint32_t* __restrict__ C, int nCTA, int ntiles,
-                                                         uint32_t* __restrict__ cnt) {
+                                                         uint32_t* __restrict__ cnt, int cstride) {
   const int lane = threadIdx.x & 31;
   const int t = blockIdx.x * (DCS_THREADS / 32) + (threadIdx.x >> 5);
   if (t >= ntiles) return;
   uint32_t* row = C + (int64_t)t * nCTA;
+  // lane l takes the DCS_PER consecutive CTAs [DCS_PER l, DCS_PER (l + 1)): all loads first, one warp scan
   uint32_t run = 0;
-  for (int c0 = 0; c0 < nCTA; c0 += 32) {
-    const bool in = c0 + lane < nCTA;
-    const uint32_t v = in ? row[c0 + lane] : 0u;
-    uint32_t incl = v;
+  for (int b0 = 0; b0 < nCTA; b0 += 32 * DCS_PER) {
+    const int j0 = b0 + lane * DCS_PER;
+    uint32_t v[DCS_PER], sum = 0;
+#pragma unroll
+    for (int k = 0; k < DCS_PER; ++k) {
+      v[k] = j0 + k < nCTA ? row[j0 + k] : 0u;
+      sum += v[k];
+    }
+    uint32_t incl = sum;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
       const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
       if (lane >= o) incl += u;
     }
-    if (in) row[c0 + lane] = run + incl - v;
+    uint32_t ex = run + incl - sum;
+#pragma unroll
+    for (int k = 0; k < DCS_PER; ++k) {
+      if (j0 + k < nCTA) row[j0 + k] = ex;
+      ex += v[k];
+    }
     run += __shfl_sync(0xffffffffu, incl, 31);
   }
-  if (lane == 0) cnt[(int64_t)t * CNT_STRIDE] = run;
+  if (lane == 0) cnt[(int64_t)t * cstride] = run;
 }
 
 // block-wide exclusive scan of one value per thread (DP_THREADS); returns the prefix, *total the sum
@@ -111,6 +125,8 @@ __device__ __forceinline__ uint32_t dp_block_scan(uint32_t v, uint32_t* s_w, uin
 }
 
 struct DpSmem {
+  uint32_t toff[DB_MAXT];        // step a2, computed by every CTA: the first list position of every tile
+  uint3 s_w3[DP_WARPS];
   uint32_t gstart[DB_MAXT + 1];  // per tile: pairs of the CTA, then the first position of the tile's group
   uint32_t cur[DB_MAXT];         // per tile: next free slot of its group; then the tile list position of the group
   uint16_t arr[DP_KEYS];          // the CTA's star indices grouped by tile (in arbitrary order inside a group)
@@ -139,15 +155,83 @@ __device__ __forceinline__ int box_tile(uint32_t code, int e, int ntx) {
   return (int)(code & 0xFFFFu) + ey * ntx + ex;
 }
 
+// Step a2 inside k_dplace (no separate scan launch): every CTA scans the DB_MAXT tile totals k_dcolscan wrote (2 per
+// thread) into S.toff, and CTA c writes tile_off, the work items, the split table and the header for the tiles
+// t = c mod nCTA -- the same values k_scan_one computes (plan_tile).
+__device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restrict__ cnt, int ntiles, int nCTA,
+                                              uint32_t* __restrict__ tile_off, Header* hdr,
+                                              WorkItem* __restrict__ items, uint2* __restrict__ split_tab,
+                                              int part_cap, uint32_t* __restrict__ done) {
+  constexpr int TPT = DB_MAXT / DP_THREADS;
+  static_assert(TPT * DP_THREADS == DB_MAXT, "tiles per thread");
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, cta = blockIdx.x;
+  uint32_t c[TPT];
+  uint3 sum = make_uint3(0u, 0u, 0u);
+#pragma unroll
+  for (int k = 0; k < TPT; ++k) {
+    const int t = tid * TPT + k;
+    c[k] = t < ntiles ? __ldcg(&cnt[t]) : 0u;  // dense totals (k_dcolscan with cstride 1)
+    const uint32_t np = parts_of(c[k]);
+    sum = add3(sum, make_uint3(c[k], np, np ? 1u : 0u));
+  }
+  const uint3 incl = warp_incl_scan3(sum, lane);
+  if (lane == 31) S.s_w3[warp] = incl;
+  __syncthreads();
+  if (warp == 0) {  // exclusive scan of the warp sums; the total in the last slot's inclusive value
+    const uint3 v = S.s_w3[lane];
+    const uint3 wi = warp_incl_scan3(v, lane);
+    __syncwarp();
+    S.s_w3[lane] = make_uint3(wi.x - v.x, wi.y - v.y, wi.z - v.z);
+    const uint3 ta = make_uint3(__shfl_sync(0xffffffffu, wi.x, 31), __shfl_sync(0xffffffffu, wi.y, 31),
+                                __shfl_sync(0xffffffffu, wi.z, 31));
+    if (lane == 0) {
+      S.gstart[0] = ta.x;  // borrowed for the totals until gstart is cleared after the next barrier
+      S.gstart[1] = ta.y;
+      S.gstart[2] = ta.z;
+    }
+  }
+  __syncthreads();
+  const uint3 pre = S.s_w3[warp];
+  const uint3 ta = make_uint3(S.gstart[0], S.gstart[1], S.gstart[2]);
+  const bool split_on = ta.y <= (uint32_t)part_cap;
+  const uint32_t nparts = split_on ? ta.y : 0u, nsplit = split_on ? ta.z : 0u;
+  uint32_t run = pre.x + incl.x - sum.x, pb = pre.y + incl.y - sum.y, si = pre.z + incl.z - sum.z;
+  if (cta == 0 && tid == 0) {
+    hdr->P = ta.x;
+    tile_off[ntiles] = ta.x;
+    hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
+    hdr->nsplit = nsplit;
+    hdr->next_item = 0u;
+  }
+#pragma unroll
+  for (int k = 0; k < TPT; ++k) {
+    const int t = tid * TPT + k;
+    if (t >= ntiles) break;
+    S.toff[t] = run;
+    if (t % nCTA == cta) {
+      plan_tile((uint32_t)t, c[k], run, pb, si, nparts, split_on, tile_off, items, split_tab, done);
+    } else {
+      const uint32_t np = split_on ? parts_of(c[k]) : 0u;
+      run += c[k];
+      pb += np;
+      si += np ? 1u : 0u;
+    }
+  }
+  __syncthreads();
+}
+
 __global__ void __launch_bounds__(DP_THREADS, 2) k_dplace(const StarRec* __restrict__ rec, int64_t n, FrameParams fp,
                                                        const uint32_t* __restrict__ C, int nCTA, int ntiles,
-                                                       const uint32_t* __restrict__ tile_off,
-                                                       uint32_t* __restrict__ ids) {
+                                                       const uint32_t* __restrict__ cnt, uint32_t* __restrict__ tile_off,
+                                                       Header* hdr, WorkItem* __restrict__ items,
+                                                       uint2* __restrict__ split_tab, int part_cap,
+                                                       uint32_t* __restrict__ done, uint32_t* __restrict__ ids) {
   static_assert(TILE_W == 128 && TILE_H == 64, "star_tiles shifts");
   extern __shared__ __align__(16) unsigned char dsm_raw[];
   DpSmem& S = *reinterpret_cast<DpSmem*>(dsm_raw);
   const int tid = threadIdx.x, cta = blockIdx.x;
   const int64_t c0 = (int64_t)cta * DB_CTA;
+  dp_scan_tiles(S, cnt, ntiles, nCTA, tile_off, hdr, items, split_tab, part_cap, done);
   for (int t = tid; t <= ntiles; t += DP_THREADS) S.gstart[t] = 0u;
   uint32_t code[DP_SPT];
 #pragma unroll
@@ -201,7 +285,7 @@ __global__ void __launch_bounds__(DP_THREADS, 2) k_dplace(const StarRec* __restr
     }
   __syncthreads();
   // first list position of every group: tile_off[t] + (pairs of tile t in the CTAs before)
-  for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = tile_off[t] + C[(int64_t)t * nCTA + cta];
+  for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = S.toff[t] + C[(int64_t)t * nCTA + cta];
   __syncthreads();
   // a pair's rank in its group = the group's stars with a smaller index
 #pragma unroll
@@ -233,15 +317,18 @@ void launch_dcount(const float* x, const float* y, const float* m, int64_t n, co
   if (nc > 0) k_dcount<<<nc, DC_THREADS, 0, st>>>(x, y, m, n, fp, rec, C, nc, ntiles);
 }
 
-void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, cudaStream_t st) {
+void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstride, cudaStream_t st) {
   constexpr int wpb = DCS_THREADS / 32;
-  k_dcolscan<<<(ntiles + wpb - 1) / wpb, DCS_THREADS, 0, st>>>(C, dbin_ctas(n), ntiles, cnt);
+  k_dcolscan<<<(ntiles + wpb - 1) / wpb, DCS_THREADS, 0, st>>>(C, dbin_ctas(n), ntiles, cnt, cstride);
 }
 
 void launch_dplace(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,
-                   const uint32_t* tile_off, uint32_t* ids, cudaStream_t st) {
+                   const uint32_t* cnt, uint32_t* tile_off, Header* hdr, WorkItem* items, uint2* split_tab,
+                   int part_cap, uint32_t* done, uint32_t* ids, cudaStream_t st) {
   const int nc = dbin_ctas(n);
-  if (nc > 0) k_dplace<<<nc, DP_THREADS, sizeof(DpSmem), st>>>(rec, n, fp, C, nc, ntiles, tile_off, ids);
+  if (nc > 0)
+    k_dplace<<<nc, DP_THREADS, sizeof(DpSmem), st>>>(rec, n, fp, C, nc, ntiles, cnt, tile_off, hdr, items, split_tab,
+                                                      part_cap, done, ids);
 }
 
 }  // namespace starsim

@@ -1,0 +1,51 @@
+// Step a2's per-tile planning (DESIGN.md §Heavy tiles), shared by k_scan_one / k_scan_b (bin.cu) and the fused scan
+// of k_dplace (dbin.cu): tile_off, and k_tile's work items -- a tile whose list is longer than SPLIT_LEN becomes
+// ceil(len / SPLIT_LEN) items over consecutive star ranges (its parts), every other tile one item; parts come first.
+// The split depends only on the tile's own list, so it is the same for any band decomposition.  If the parts would
+// need more than `part_cap` partial buffers, nothing is split.
+#pragma once
+#include "common.cuh"
+
+namespace starsim {
+
+__device__ __forceinline__ uint32_t parts_of(uint32_t len) {
+  if (len <= (uint32_t)SPLIT_LEN) return 0u;
+  return min((len + SPLIT_LEN - 1) / SPLIT_LEN, 4095u);
+}
+
+__device__ __forceinline__ uint3 add3(uint3 a, uint3 b) { return make_uint3(a.x + b.x, a.y + b.y, a.z + b.z); }
+
+__device__ __forceinline__ uint3 warp_incl_scan3(uint3 v, int lane) {
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t x = __shfl_up_sync(0xffffffffu, v.x, o), y = __shfl_up_sync(0xffffffffu, v.y, o),
+                   z = __shfl_up_sync(0xffffffffu, v.z, o);
+    if (lane >= o) v = add3(v, make_uint3(x, y, z));
+  }
+  return v;
+}
+
+// Tile t with c stars: (run, pb, si) = (pairs, parts, split tiles) of the tiles before it on entry, after it on
+// return.  Writes tile_off[t], its items (and split table entry, zeroed completion counter, if it is split).
+__device__ __forceinline__ void plan_tile(uint32_t t, uint32_t c, uint32_t& run, uint32_t& pb, uint32_t& si,
+                                          uint32_t nparts, bool split_on, uint32_t* __restrict__ tile_off,
+                                          WorkItem* __restrict__ items, uint2* __restrict__ split_tab,
+                                          uint32_t* __restrict__ done) {
+  tile_off[t] = run;
+  const uint32_t np = split_on ? parts_of(c) : 0u;
+  if (np) {
+    split_tab[si] = make_uint2(pb, np);
+    done[si] = 0u;  // the parts' completion counter (k_tile)
+    const uint32_t per_part = (c + np - 1) / np;
+    for (uint32_t j = 0; j < np; ++j)
+      items[pb + j] = WorkItem{t, run + j * per_part, min(run + c, run + (j + 1) * per_part), (si << 12) | j};
+    pb += np;
+    ++si;
+  } else {
+    // whole tiles follow the parts, in tile order: index = nparts + (tiles before t that are not split)
+    items[nparts + t - (split_on ? si : 0u)] = WorkItem{t, run, run + c, ITEM_WHOLE};
+  }
+  run += c;
+}
+
+}  // namespace starsim
