@@ -145,13 +145,13 @@ __device__ __forceinline__ uint32_t star_tiles(const FrameParams& fp, uint32_t l
   return (uint32_t)(ty0 * fp.ntx + tx0) | dx << 16 | dy << 17;
 }
 
-// the e-th tile (e = 0..3, in row-major order) of a packed box, or -1
+// tiles of a packed box (0 if the star is culled) and its e-th tile, e < box_n (row-major order inside the box)
+__device__ __forceinline__ int box_n(uint32_t code) {
+  return code == DP_NONE ? 0 : (1 + (int)((code >> 16) & 1u)) << (int)((code >> 17) & 1u);
+}
 __device__ __forceinline__ int box_tile(uint32_t code, int e, int ntx) {
-  if (code == DP_NONE) return -1;
-  const int dx = (int)((code >> 16) & 1u), dy = (int)((code >> 17) & 1u);
-  const int ex = e & 1, ey = e >> 1;
-  if (ex > dx || ey > dy) return -1;
-  // row-major order inside the box: (0,0), (0,1), (1,0), (1,1) -> skip e = 1 when dx = 0 is handled by the test
+  const int dx = (int)((code >> 16) & 1u);
+  const int ex = e & dx, ey = e >> dx;
   return (int)(code & 0xFFFFu) + ey * ntx + ex;
 }
 
@@ -244,12 +244,10 @@ __global__ void __launch_bounds__(DP_THREADS, 2) k_dplace(const StarRec* __restr
   __syncthreads();
   // group sizes
 #pragma unroll
-  for (int k = 0; k < DP_SPT; ++k)
-#pragma unroll
-    for (int e = 0; e < 4; ++e) {
-      const int t = box_tile(code[k], e, fp.ntx);
-      if (t >= 0) atomicAdd(&S.gstart[t], 1u);
-    }
+  for (int k = 0; k < DP_SPT; ++k) {
+    const int nb = box_n(code[k]);
+    for (int e = 0; e < nb; ++e) atomicAdd(&S.gstart[box_tile(code[k], e, fp.ntx)], 1u);
+  }
   __syncthreads();
   // exclusive scan of the group sizes (TPT consecutive tiles per thread)
   {
@@ -277,12 +275,11 @@ __global__ void __launch_bounds__(DP_THREADS, 2) k_dplace(const StarRec* __restr
   __syncthreads();
   // group the star indices by tile (arbitrary order inside a group)
 #pragma unroll
-  for (int k = 0; k < DP_SPT; ++k)
-#pragma unroll
-    for (int e = 0; e < 4; ++e) {
-      const int t = box_tile(code[k], e, fp.ntx);
-      if (t >= 0) S.arr[atomicAdd(&S.cur[t], 1u)] = (uint16_t)(tid + k * DP_THREADS);
-    }
+  for (int k = 0; k < DP_SPT; ++k) {
+    const int nb = box_n(code[k]);
+    for (int e = 0; e < nb; ++e)
+      S.arr[atomicAdd(&S.cur[box_tile(code[k], e, fp.ntx)], 1u)] = (uint16_t)(tid + k * DP_THREADS);
+  }
   __syncthreads();
   // first list position of every group: tile_off[t] + (pairs of tile t in the CTAs before)
   for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = S.toff[t] + C[(int64_t)t * nCTA + cta];
@@ -291,10 +288,9 @@ __global__ void __launch_bounds__(DP_THREADS, 2) k_dplace(const StarRec* __restr
 #pragma unroll
   for (int k = 0; k < DP_SPT; ++k) {
     const uint32_t idx = (uint32_t)(tid + k * DP_THREADS);
-#pragma unroll
-    for (int e = 0; e < 4; ++e) {
+    const int nb = box_n(code[k]);
+    for (int e = 0; e < nb; ++e) {
       const int t = box_tile(code[k], e, fp.ntx);
-      if (t < 0) continue;
       const uint32_t g0 = S.gstart[t], g1 = S.gstart[t + 1];
       uint32_t rank = 0;
       for (uint32_t u = g0; u < g1; ++u) rank += S.arr[u] < idx ? 1u : 0u;
