@@ -43,7 +43,7 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="T")
     ap.add_argument("--method", default="tiled", choices=["tiled", "atomic"])
-    ap.add_argument("--tile-kernel", default="auto", choices=["auto", "lists", "sb"],
+    ap.add_argument("--tile-kernel", default="auto", choices=["auto", "lists", "sb", "ws"],
                     help="starsim_set_tile_kernel mode (A/B comparisons; the default is the product path)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")

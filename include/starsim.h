@@ -119,12 +119,13 @@ int starsim_set_psf(starsim_ctx* ctx, int32_t mode);
 /* Tile-accumulation kernel of the tiled renders that follow on this ctx (render, render_band, render_gray).  Both
  * compute Eqs. 2-3 per tile in fp32 registers with the separable PSF and write every pixel once;
  * they differ in how a tile's star list is walked, hence in the (deterministic) per-pixel summation order:
- *   STARSIM_TILE_AUTO (default): for R <= 17 the warp-specialised sorted-corner-bin kernel (producer warps sort
- *     and evaluate profiles into a ring of shared-memory stages while consumer warps accumulate),
- *     else the list kernel;
+ *   STARSIM_TILE_AUTO (default): for R <= 17, STARSIM_TILE_WS on dense frames (expected list length per 128 x 64
+ *     tile n (127 + R)(63 + R) / (width rows) >= 100, point PSF), else STARSIM_TILE_SB; for R > 17 the list kernel;
  *   STARSIM_TILE_LISTS: always the per-block entry-list kernel (the comparison / any R);
- *   STARSIM_TILE_SB: for R <= 17 the sorted-corner-bin kernel with both roles in every warp (the round-1b kernel,
- *     same summation order as AUTO, hence the same image bit for bit), else the list kernel.
+ *   STARSIM_TILE_SB: for R <= 17 the sorted-corner-bin kernel with both roles in every warp, else the list kernel;
+ *   STARSIM_TILE_WS: for R <= 17 the warp-specialised sorted-corner-bin kernel (producer warps sort and evaluate
+ *     profiles into a ring of shared-memory stages while consumer warps accumulate), else the list
+ *     kernel.  SB and WS sum every pixel in the same order: the same image bit for bit.
  * EINVAL: ctx NULL or an unknown mode. */
 /* Binning pipeline of the tiled renders that follow on this ctx.  Both produce the same CSR (each tile's list in
  * ascending star index, reading R18 of DESIGN.md), hence the same image bit for bit:
@@ -139,6 +140,7 @@ int starsim_set_binning(starsim_ctx* ctx, int32_t mode);
 #define STARSIM_TILE_AUTO 0
 #define STARSIM_TILE_LISTS 1
 #define STARSIM_TILE_SB 2
+#define STARSIM_TILE_WS 3
 int starsim_set_tile_kernel(starsim_ctx* ctx, int32_t mode);
 
 /* The paper's own design, kept as the measured comparison (Fig. 6): zero the image, then one

@@ -51,7 +51,7 @@ struct starsim_ctx {
   int dev = 0;
   int num_sms = 148;
   int32_t psf = 0;  // starsim_set_psf: 0 point-sampled Eq. 2, 1 pixel-integrated (NEXT-2)
-  int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto (warp-specialised sorted bins when R <= 17), 1 lists, 2 sorted bins
+  int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto, 1 lists, 2 sorted bins, 3 warp-specialised sorted bins
   int32_t bin_impl = 0;   // starsim_set_binning: 0 auto (dbin.cu when it applies), 1 always bin.cu's pipeline
   std::string err;
   Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat;
@@ -275,6 +275,13 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain, c->psf);
   fp.obits = obits;
   fp.tile_impl = c->tile_impl;
+  if (fp.tile_impl == STARSIM_TILE_AUTO) {
+    // the warp-specialised kernel wins on dense frames (its per-item pipeline latency and static item order cost
+    // more than they save on sparse, clustered and integrated-PSF frames: DESIGN.md §9): expected list length per
+    // tile for a uniform field, n (128 + R - 1)(64 + R - 1) / (W rows)
+    const double per_tile = (double)n * (TILE_W + R - 1) * (TILE_H + R - 1) / ((double)W * (rows > 0 ? rows : 1));
+    fp.tile_impl = (c->psf == 0 && per_tile >= WS_MIN_PER_TILE) ? STARSIM_TILE_WS : STARSIM_TILE_SB;
+  }
   fp.bin_impl = c->bin_impl;
   // one vector store per 8-pixel run: 32 B (fp32) / 8 B (u8) / 16 B (u16); rows must keep that alignment
   const int vb = obits == 8 ? 8 : 16;
@@ -473,8 +480,8 @@ int starsim_set_binning(starsim_ctx* c, int32_t mode) {
 
 int starsim_set_tile_kernel(starsim_ctx* c, int32_t mode) {
   if (!c) return STARSIM_EINVAL;
-  if (mode != STARSIM_TILE_AUTO && mode != STARSIM_TILE_LISTS && mode != STARSIM_TILE_SB)
-    return fail(c, STARSIM_EINVAL, "tile kernel mode must be STARSIM_TILE_AUTO, STARSIM_TILE_LISTS or STARSIM_TILE_SB");
+  if (mode != STARSIM_TILE_AUTO && mode != STARSIM_TILE_LISTS && mode != STARSIM_TILE_SB && mode != STARSIM_TILE_WS)
+    return fail(c, STARSIM_EINVAL, "tile kernel mode must be STARSIM_TILE_AUTO, _LISTS, _SB or _WS");
   c->tile_impl = mode;
   c->err.clear();
   return STARSIM_OK;

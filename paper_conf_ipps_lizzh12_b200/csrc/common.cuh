@@ -22,6 +22,7 @@ constexpr int GY_CAP = 384;                      // band slots (16 floats: the r
 constexpr int RCAP = 56;                         // strip slots (8 floats: the column profile on one strip) per strip
 constexpr int LCAP = 32;                         // entries per (band, strip) list per chunk
 constexpr int GX_PAIRS = 768;                    // (star, strip) pairs per chunk
+constexpr int WS_MIN_PER_TILE = 100;            // STARSIM_TILE_AUTO picks tile_ws.cu from this expected list length
 constexpr int SB_MAXR = 17;                      // tile_sb.cu: an ROI of side <= 17 spans <= 2 bands and <= 3 strips
 
 // k_prep: one star per thread; per-tile counters CNT_STRIDE words apart (one 128-B line each, so that the
@@ -81,7 +82,7 @@ struct FrameParams {
   int32_t vec;           // 1 if every 8-pixel run of an out row is aligned for one vector store
   int32_t obits;         // 0: fp32 image; 8 / 16: gray values quantised in the epilogue (u8 / u16 image)
   int32_t psf;           // 0: Eq. 2 point-sampled (the paper); 1: Eq. 2 integrated over the pixel square (NEXT-2)
-  int32_t tile_impl;     // 0: warp-specialised sorted-bin kernel when R <= SB_MAXR (tile_ws.cu), else the list kernel; 1: always the list kernel (tile.cu); 2: tile_sb.cu when R <= SB_MAXR
+  int32_t tile_impl;     // resolved by render_tiled: 1 the list kernel (tile.cu); 2 tile_sb.cu, 3 tile_ws.cu when R <= SB_MAXR (else tile.cu)
   int32_t bin_impl;      // 0: dbin.cu's deterministic binning when it applies; 1: always bin.cu's atomic-slot pipeline
   int32_t ndst;          // > 0: the tile kernels store every pixel into dst[0..ndst) instead of `out` (fused band exchange)
   float* dst[MAX_DST];   // band origins (row0 of each destination frame) -- local and peer-mapped frames

@@ -36,10 +36,20 @@ constexpr int WS_CONS = 8;                           // consumer warps
 #define WS_PGROUPS 1                                 // producer groups: group g produces the chunks c = g mod WS_PGROUPS
 #endif
 constexpr int WS_THREADS = 32 * (WS_PGROUPS * WS_PROD + WS_CONS);
-constexpr int WS_NSTAGE = 2;                         // depth of the chunk ring (chunk c in stage c mod WS_NSTAGE)
+#ifndef WS_NSTAGE_OPT
+#define WS_NSTAGE_OPT 2
+#endif
+#ifndef WS_RSTAGE_OPT
+#define WS_RSTAGE_OPT SPLIT_LEN
+#endif
+#ifndef WS_WALK_UNROLL
+#define WS_WALK_UNROLL 2
+#endif
+constexpr int WS_UNROLL = WS_WALK_UNROLL;              // walk steps per loop iteration (pairs of even/odd)
+constexpr int WS_NSTAGE = WS_NSTAGE_OPT;              // depth of the chunk ring (chunk c in stage c mod WS_NSTAGE)
 constexpr uint32_t WS_ZJ = WS_CHUNK;                 // the all-zero slot of every stage
 constexpr uint32_t WS_LAST = 1u, WS_STOP = 2u;       // chunk flags
-constexpr int WS_RSTAGE = SPLIT_LEN;                 // star records of a work item staged in shared memory
+constexpr int WS_RSTAGE = WS_RSTAGE_OPT;             // star records of a work item staged in shared memory
 constexpr int WS_RPT = WS_RSTAGE / WS_CHUNK;         // ... per producer thread
 
 struct WsStage {
@@ -406,7 +416,7 @@ __device__ __forceinline__ void ws_consumer(WsSmem& S, const FrameParams& fp, vo
 #ifdef WS_NOWALK
     st = steps;
 #endif
-#pragma unroll 2
+#pragma unroll WS_UNROLL
     for (; st + 1 < steps; st += 2) {
       step(st, false);
       step(st + 1, true);

@@ -8,7 +8,7 @@ STARSIM_PARITY_LOG=gpurun_out/${TAG}_parity.jsonl timeout 900 python -m pytest t
 timeout 400 python bench.py > gpurun_out/${TAG}_bench_T.json 2> gpurun_out/bench.err
 timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv \
   python tools/profile_frame.py --reps 3 > /dev/null 2>&1
-timeout 600 ncu --set full --import-source on --clock-control none -k regex:k_ -s 12 -c 6 -f -o gpurun_out/${TAG}_full \
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:k_ -s 8 -c 4 -f -o gpurun_out/${TAG}_full \
   python tools/profile_frame.py --reps 1 > gpurun_out/ncu_full.log 2>&1
 timeout 900 python tools/sweep.py --sweep all > gpurun_out/${TAG}_sweep.jsonl 2> gpurun_out/sweep.err
 tail -2 gpurun_out/gpu_tests.log

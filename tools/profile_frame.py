@@ -27,7 +27,7 @@ def main():
     ap.add_argument("--n", type=int, default=0)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--atomic", action="store_true")
-    ap.add_argument("--tile", default="auto", help="tile kernel: auto | lists")
+    ap.add_argument("--tile", default="auto", help="tile kernel: auto | lists | sb")
     a = ap.parse_args()
     cfg = synth.CONFIGS[a.config]
     if a.R:
