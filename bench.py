@@ -409,6 +409,24 @@ def run_ours(args, world, rank, local_rank):
             a_ms = sum(a.elapsed_time(b) for a, b in a_ev) / args.steps
             variants[name] = {"ms_per_step": a_ms, "frames_per_s": 1e3 / a_ms, "updates_per_s": U_frame / (a_ms * 1e-3),
                               "note": note}
+            if name == "atomic":  # NEXT-3: the same star-centric kernel with the pixel-circle ROI
+                ctx.set_roi("circle")
+                fn_(x, y, m, W, H, sigma, R, A, out=a_out, stream=stream)
+                torch.cuda.synchronize()
+                c_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                        for _ in range(args.steps)]
+                for i in range(args.steps):
+                    with torch.cuda.stream(stream):
+                        flush.fill_(float(i))
+                        c_ev[i][0].record(stream)
+                        fn_(x, y, m, W, H, sigma, R, A, out=a_out, stream=stream)
+                        c_ev[i][1].record(stream)
+                torch.cuda.synchronize()
+                ctx.set_roi("square")
+                c_ms = sum(a.elapsed_time(b) for a, b in c_ev) / args.steps
+                variants["atomic_circle"] = {"ms_per_step": c_ms, "frames_per_s": 1e3 / c_ms,
+                                             "note": "starsim_set_roi(CIRCLE) + starsim_render_atomic: the paper's "
+                                                     "'pixel circle' ROI (NEXT-3, reading R21)"}
             del a_out
 
     # e2e: the same C-ABI call with host (pinned) catalogue in and image out, copies inside the timed region

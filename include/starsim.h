@@ -116,6 +116,18 @@ int starsim_render_gray(starsim_ctx* ctx, const float* x, const float* y, const 
 #define STARSIM_PSF_INTEGRATED 1
 int starsim_set_psf(starsim_ctx* ctx, int32_t mode);
 
+/* ROI shape of the renders that follow on this ctx (reading R21):
+ *   STARSIM_ROI_SQUARE (default): the R x R square of reading R5/R7 (Fig. 1 caption PAPER.md:19, Fig. 5);
+ *   STARSIM_ROI_CIRCLE: the paper's literal "pixel circle" -- the pixels of that square whose centres lie
+ *     in the circle inscribed in it: ROI row / column offsets (i, j) with (2j - (R-1))^2 + (2i - (R-1))^2 <= R^2,
+ *     an exact integer test, then clipped to the image.  Supported by starsim_render_atomic and starsim_render_lut;
+ *     the tiled renders (render, render_band, render_band_to, render_gray), which accumulate separable rectangular
+ *     ROIs, return EINVAL while it is set.
+ * EINVAL: ctx NULL or an unknown shape. */
+#define STARSIM_ROI_SQUARE 0
+#define STARSIM_ROI_CIRCLE 1
+int starsim_set_roi(starsim_ctx* ctx, int32_t shape);
+
 /* Tile-accumulation kernel of the tiled renders that follow on this ctx (render, render_band, render_gray).  Both
  * compute Eqs. 2-3 per tile in fp32 registers with the separable PSF and write every pixel once;
  * they differ in how a tile's star list is walked, hence in the (deterministic) per-pixel summation order:

@@ -57,6 +57,8 @@ def _load():
         lib.oracle_roi_lo.argtypes = [ctypes.c_float, i32]
         lib.oracle_roi_lo.restype = i64
         lib.oracle_star_roi.argtypes = [ctypes.c_float, ctypes.c_float, ctypes.c_float, i32, i32, i32, i64p]
+        lib.oracle_in_circle.argtypes = [ctypes.c_int64, ctypes.c_int64, i32]
+        lib.oracle_in_circle.restype = ctypes.c_int
         lib.oracle_star_roi.restype = ctypes.c_int
         lib.oracle_render.argtypes = [f32p, f32p, f32p, i64, i32, i32, f64, i32, f64, i32, f64p]
         lib.oracle_render.restype = i64
@@ -92,12 +94,21 @@ def brightness(m: float, A: float) -> float:
 
 
 PSF_MODES = {"point": 0, "integrated": 1}
+ROI_SHAPES = {"square": 0, "circle": 2}  # NEXT-3 (reading R21): the paper's "pixel circle", mode bit 1
 
 
-def _mode(psf_mode):
+def _mode(psf_mode, roi="square"):
     if psf_mode not in PSF_MODES:
         raise ValueError(f"psf must be one of {sorted(PSF_MODES)}")
-    return PSF_MODES[psf_mode]
+    if roi not in ROI_SHAPES:
+        raise ValueError(f"roi must be one of {sorted(ROI_SHAPES)}")
+    return PSF_MODES[psf_mode] | ROI_SHAPES[roi]
+
+
+def in_circle(i: int, j: int, R: int) -> bool:
+    """NEXT-3 (reading R21): is ROI pixel (row offset i, column offset j) inside the circle inscribed in the R x R
+    square ROI?"""
+    return bool(_load().oracle_in_circle(int(i), int(j), int(R)))
 
 
 def psf(px: float, py: float, X: float, Y: float, sigma: float, mode: str = "point") -> float:
@@ -120,12 +131,13 @@ def star_roi(x: float, y: float, m: float, W: int, H: int, R: int):
 
 
 def render(x, y, mag, W: int, H: int, sigma: float, R: int, A: float, threads: int = 1, return_units: bool = False,
-           psf: str = "point"):
+           psf: str = "point", roi: str = "square"):
     """The oracle image, fp64 (H, W), row-major with y = row: Eqs. 1-3 over square ROIs in star order (Fig. 5).
 
     ``threads > 1`` splits rows over pthreads; the result is bitwise identical (same per-pixel order).
-    ``psf="integrated"``: the pixel-integrated variant of Eq. 2 (NEXT-2)."""
-    mode = _mode(psf)
+    ``psf="integrated"``: the pixel-integrated variant of Eq. 2 (NEXT-2); ``roi="circle"``: the pixel circle
+    inscribed in the square ROI (NEXT-3, reading R21); U then counts the circle's pixels."""
+    mode = _mode(psf, roi)
     _, (px, py, pm), n = _stars(x, y, mag)
     img = np.empty((int(H), int(W)), dtype=np.float64)
     pimg = img.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
@@ -153,10 +165,11 @@ def lut_positions(x, y, R: int):
     return snap(x), snap(y)
 
 
-def render_lut(x, y, mag, W: int, H: int, sigma: float, R: int, A: float, threads: int = 1, psf: str = "point"):
+def render_lut(x, y, mag, W: int, H: int, sigma: float, R: int, A: float, threads: int = 1, psf: str = "point",
+               roi: str = "square"):
     """The adaptive simulator's image (NEXT-4): ``render`` with every star at its ROI centre."""
     sx, sy = lut_positions(x, y, R)
-    return render(sx, sy, mag, W, H, sigma, R, A, threads=threads, psf=psf)
+    return render(sx, sy, mag, W, H, sigma, R, A, threads=threads, psf=psf, roi=roi)
 
 
 def render_band(x, y, mag, W: int, H: int, row0: int, rows: int, sigma: float, R: int, A: float,

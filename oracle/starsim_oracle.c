@@ -25,6 +25,12 @@
  * over the pixel square [px-1/2, px+1/2] x [py-1/2, py+1/2] instead of sampled at its centre (psf mode 1), with the
  * same ROI, clipping and order.  Mode 0 is the paper's point-sampled Eq. 2.
  *
+ * NEXT-3 (reading R21): the paper's literal "pixel circle" ROI -- mode bit 1.
+ * The ROI is then the pixels of the square ROI above whose centres lie in the circle inscribed in that square: with
+ * lo_x, lo_y its first column and row, pixel (px,py) belongs iff
+ *   (2 (px - lo_x) - (R - 1))^2 + (2 (py - lo_y) - (R - 1))^2 <= R^2      (integers: an exact decision),
+ * then clipped to the image as before.
+ *
  * Pins (tests/test_oracle_pins.py, all "-m 'not gpu'"): Poisson-summation closed form of the point-sampled ROI mass,
  * first moment (centroid), reflection/transpose symmetry, scipy.ndimage.correlate with a kernel built from
  * scipy.stats.norm.pdf, brute-force no-ROI evaluation on tiny inputs, superposition, integer translation, magnitude
@@ -63,8 +69,16 @@ double oracle_psf_integrated(double px, double py, double X, double Y, double de
     return pixel_mass_1d(px, X, delta) * pixel_mass_1d(py, Y, delta);
 }
 static double psf_of(int mode, double px, double py, double X, double Y, double delta) {
-    return mode ? oracle_psf_integrated(px, py, X, Y, delta) : oracle_psf(px, py, X, Y, delta);
+    return (mode & 1) ? oracle_psf_integrated(px, py, X, Y, delta) : oracle_psf(px, py, X, Y, delta);
 }
+
+/* NEXT-3 (reading R21): is ROI pixel (i, j) = (row, column) offsets from the square's first row/column inside the
+ * circle inscribed in the R x R square? */
+static int in_circle(int64_t i, int64_t j, int32_t R) {
+    int64_t u = 2 * j - (R - 1), v = 2 * i - (R - 1);
+    return u * u + v * v <= (int64_t)R * R;
+}
+int oracle_in_circle(int64_t i, int64_t j, int32_t R) { return in_circle(i, j, R); }
 
 /* First ROI column (or row) of a star at coordinate c: the R integers nearest to c, ties at k+1/2 upward, i.e.
  * lo = floor(c + 1 - R/2) in exact arithmetic (reading R7).  With f = floor(c) (exact):
@@ -109,12 +123,15 @@ static void render_rows(const float* x, const float* y, const float* mag, int64_
         if (!star_roi(x[i], y[i], mag[i], W, H, R, &x0, &x1, &y0, &y1)) continue;
         double g = oracle_brightness((double)mag[i], A);              /* Eq. 1 */
         double X = (double)x[i], Y = (double)y[i];
+        int64_t lx = oracle_roi_lo(x[i], R), ly = oracle_roi_lo(y[i], R); /* the square's first column / row */
         if (y0 < row0) y0 = row0;
         if (y1 > row0 + rows - 1) y1 = row0 + rows - 1;
         for (int64_t py = y0; py <= y1; ++py)                            /* Fig. 5: pixelY over the ROI */
-            for (int64_t px = x0; px <= x1; ++px)                        /* Fig. 5: pixelX over the ROI */
+            for (int64_t px = x0; px <= x1; ++px) {                      /* Fig. 5: pixelX over the ROI */
+                if ((mode & 2) && !in_circle(py - ly, px - lx, R)) continue; /* NEXT-3: the pixel circle */
                 img[(size_t)(py - row0) * (size_t)W + (size_t)px] +=
                     g * psf_of(mode, (double)px, (double)py, X, Y, delta); /* Eq. 3 */
+            }
     }
 }
 
@@ -125,7 +142,11 @@ int64_t oracle_render(const float* x, const float* y, const float* mag, int64_t 
     int64_t U = 0;
     for (int64_t i = 0; i < n; ++i) {
         int64_t x0, x1, y0, y1;
-        if (star_roi(x[i], y[i], mag[i], W, H, R, &x0, &x1, &y0, &y1)) U += (x1 - x0 + 1) * (y1 - y0 + 1);
+        if (!star_roi(x[i], y[i], mag[i], W, H, R, &x0, &x1, &y0, &y1)) continue;
+        if (!(mode & 2)) { U += (x1 - x0 + 1) * (y1 - y0 + 1); continue; }
+        int64_t lx = oracle_roi_lo(x[i], R), ly = oracle_roi_lo(y[i], R);
+        for (int64_t py = y0; py <= y1; ++py)
+            for (int64_t px = x0; px <= x1; ++px) U += in_circle(py - ly, px - lx, R);
     }
     return U;
 }

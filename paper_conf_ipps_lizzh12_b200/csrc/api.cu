@@ -51,6 +51,7 @@ struct starsim_ctx {
   int dev = 0;
   int num_sms = 148;
   int32_t psf = 0;  // starsim_set_psf: 0 point-sampled Eq. 2, 1 pixel-integrated (NEXT-2)
+  int32_t roi = 0;  // starsim_set_roi: 0 square, 1 pixel circle (NEXT-3; atomic and lookup-table renders only)
   int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto, 1 lists, 2 sorted bins, 3 warp-specialised sorted bins
   int32_t bin_impl = 0;   // starsim_set_binning: 0 auto (dbin.cu when it applies), 1 always bin.cu's pipeline
   std::string err;
@@ -185,6 +186,7 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   fp.sk = (float)std::sqrt(1.0 / (2.0 * s * s * std::log(2.0)));  // exp(-d^2/(2 s^2)) = 2^(-(d sk)^2)
   fp.s_scale = (double)gain / (2.0 * M_PI * s * s);          // Eq. 1 gain with Eq. 2's 1/(2 pi s^2)
   fp.psf = psf;
+  fp.roi = 0;
   fp.tile_impl = 0;
   fp.bin_impl = 0;
   fp.ndst = 0;
@@ -271,6 +273,10 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
 int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
                  int32_t row0, int32_t rows, float sigma, int32_t R, float gain, int32_t obits, void* out,
                  cudaStream_t st, float* const* dsts = nullptr, int ndst = 0) {
+  if (c->roi != STARSIM_ROI_SQUARE)
+    return fail(c, STARSIM_EINVAL,
+                "circular ROI (NEXT-3): the tiled renders accumulate separable square ROIs; use starsim_render_atomic "
+                "or starsim_render_lut");
   DevGuard g(c->dev);
   FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain, c->psf);
   fp.obits = obits;
@@ -469,6 +475,15 @@ int starsim_set_psf(starsim_ctx* c, int32_t mode) {
   return STARSIM_OK;
 }
 
+int starsim_set_roi(starsim_ctx* c, int32_t shape) {
+  if (!c) return STARSIM_EINVAL;
+  if (shape != STARSIM_ROI_SQUARE && shape != STARSIM_ROI_CIRCLE)
+    return fail(c, STARSIM_EINVAL, "roi shape must be STARSIM_ROI_SQUARE or STARSIM_ROI_CIRCLE");
+  c->roi = shape;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
 int starsim_set_binning(starsim_ctx* c, int32_t mode) {
   if (!c) return STARSIM_EINVAL;
   if (mode != STARSIM_BIN_AUTO && mode != STARSIM_BIN_ATOMIC)
@@ -494,7 +509,8 @@ int starsim_render_atomic(starsim_ctx* c, const float* x, const float* y, const 
   if (rc) return rc;
   DevGuard g(c->dev);
   cudaStream_t st = (cudaStream_t)stream;
-  const FrameParams fp = make_params(W, H, 0, H, sigma, R, gain, c->psf);
+  FrameParams fp = make_params(W, H, 0, H, sigma, R, gain, c->psf);
+  fp.roi = c->roi;
   timed(c, 5, st, [&] { cudaMemsetAsync(out, 0, sizeof(float) * (size_t)W * H, st); });
   timed(c, 4, st, [&] { launch_atomic(x, y, mag, n, fp, out, st); });
   if ((rc = check_launch(c, "k_atomic"))) return rc;
@@ -510,7 +526,8 @@ int starsim_render_lut(starsim_ctx* c, const float* x, const float* y, const flo
   if (R > STARSIM_MAX_LUT_ROI) return fail(c, STARSIM_EINVAL, "roi > 63 for the lookup-table kernel");
   DevGuard g(c->dev);
   cudaStream_t st = (cudaStream_t)stream;
-  const FrameParams fp = make_params(W, H, 0, H, sigma, R, gain, c->psf);
+  FrameParams fp = make_params(W, H, 0, H, sigma, R, gain, c->psf);
+  fp.roi = c->roi;
   timed(c, 5, st, [&] { cudaMemsetAsync(out, 0, sizeof(float) * (size_t)W * H, st); });
   timed(c, 4, st, [&] { launch_lut(x, y, mag, n, fp, out, st); });
   if ((rc = check_launch(c, "k_lut"))) return rc;

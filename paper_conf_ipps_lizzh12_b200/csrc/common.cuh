@@ -82,6 +82,7 @@ struct FrameParams {
   int32_t vec;           // 1 if every 8-pixel run of an out row is aligned for one vector store
   int32_t obits;         // 0: fp32 image; 8 / 16: gray values quantised in the epilogue (u8 / u16 image)
   int32_t psf;           // 0: Eq. 2 point-sampled (the paper); 1: Eq. 2 integrated over the pixel square (NEXT-2)
+  int32_t roi;           // 0: square ROI (reading R5); 1: the pixel circle inscribed in it (NEXT-3, reading R21)
   int32_t tile_impl;     // resolved by render_tiled: 1 the list kernel (tile.cu); 2 tile_sb.cu, 3 tile_ws.cu when R <= SB_MAXR (else tile.cu)
   int32_t bin_impl;      // 0: dbin.cu's deterministic binning when it applies; 1: always bin.cu's atomic-slot pipeline
   int32_t ndst;          // > 0: the tile kernels store every pixel into dst[0..ndst) instead of `out` (fused band exchange)
@@ -111,6 +112,13 @@ __device__ __forceinline__ float pix_mass(float ta, float ea, float tb, float eb
   if (ta >= 0.f) return 0.5f * (ea - eb);
   if (tb < 0.f) return 0.5f * (eb - ea);
   return 1.f - 0.5f * (ea + eb);
+}
+
+// NEXT-3 (reading R21): ROI pixel at row / column offsets (i, j) from the square ROI's first row / column lies in the
+// circle inscribed in the R x R square iff (2j - (R-1))^2 + (2i - (R-1))^2 <= R^2 (integers: exact).
+__device__ __forceinline__ bool in_roi_circle(int i, int j, int R) {
+  const int u = 2 * j - (R - 1), v = 2 * i - (R - 1);
+  return u * u + v * v <= R * R;
 }
 
 // MUFU.EX2 (2^x, flush-to-zero): the one SFU op per profile value.

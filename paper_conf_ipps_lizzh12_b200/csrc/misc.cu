@@ -64,6 +64,7 @@ __global__ void __launch_bounds__(ATOM_WARPS * 32) k_atomic(const float* __restr
   for (int p = lane; p < w * h; p += 32) {
     const int r = __float2int_rz(((float)p + 0.5f) * inv_w);
     const int c = p - r * w;
+    if (fp.roi && !in_roi_circle(cy0 + r - ly, cx0 + c - lx, fp.R)) continue;  // NEXT-3: the pixel circle
     atomicAdd(o + (int64_t)r * fp.W + c, gy[r] * gx[c]);
   }
 }
@@ -127,6 +128,7 @@ __global__ void __launch_bounds__(ATOM_WARPS * 32) k_lut(const float* __restrict
   for (int p = lane; p < w * h; p += 32) {
     const int r = __float2int_rz(((float)p + 0.5f) * inv_w);
     const int c = p - r * w;
+    if (fp.roi && !in_roi_circle(cy0 + r - ly, cx0 + c - lx, R)) continue;  // NEXT-3: the pixel circle
     atomicAdd(o + (int64_t)r * fp.W + c, s * lut[r * R + c]);
   }
 }

@@ -60,6 +60,8 @@ def lib():
         L.starsim_render_gray.restype = ctypes.c_int
         L.starsim_set_psf.argtypes = [vp, i32]
         L.starsim_set_psf.restype = ctypes.c_int
+        L.starsim_set_roi.argtypes = [vp, i32]
+        L.starsim_set_roi.restype = ctypes.c_int
         L.starsim_set_binning.argtypes = [vp, i32]
         L.starsim_set_binning.restype = ctypes.c_int
         L.starsim_set_tile_kernel.argtypes = [vp, i32]
@@ -155,6 +157,13 @@ PSF_MODES = {"point": 0, "integrated": 1}
 
 def starsim_set_psf(h, mode) -> None:
     _check(h, lib().starsim_set_psf(h, PSF_MODES.get(mode, mode) if isinstance(mode, str) else int(mode)))
+
+
+ROI_SHAPES = {"square": 0, "circle": 1}
+
+
+def starsim_set_roi(h, shape) -> None:
+    _check(h, lib().starsim_set_roi(h, ROI_SHAPES.get(shape, shape) if isinstance(shape, str) else int(shape)))
 
 
 BINNINGS = {"auto": 0, "atomic": 1}
@@ -294,6 +303,11 @@ class Context:
     def set_psf(self, mode="point"):
         """"point" (Eq. 2 sampled at the pixel, the paper) or "integrated" (Eq. 2 integrated over the pixel)."""
         starsim_set_psf(self.h, mode)
+
+    def set_roi(self, shape="square"):
+        """"square" (the R x R ROI, reading R5) or "circle" (the pixel circle inscribed in it, NEXT-3; the atomic and
+        lookup-table renders only -- the tiled renders then fail with EINVAL)."""
+        starsim_set_roi(self.h, shape)
 
     def set_binning(self, mode="auto"):
         """"auto" (deterministic counting sort when the frame has <= 2048 tiles and R <= 65) or "atomic"."""

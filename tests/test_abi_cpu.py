@@ -32,7 +32,7 @@ def test_header_declares_the_boundary():
     for want in ["starsim_create", "starsim_destroy", "starsim_last_error", "starsim_render", "starsim_render_band",
                  "starsim_render_gray", "starsim_render_atomic", "starsim_upload_aos", "starsim_quantize",
                  "starsim_get_bins", "starsim_profile", "starsim_kernel_times", "starsim_set_psf",
-                 "starsim_set_tile_kernel", "starsim_set_binning",
+                 "starsim_set_tile_kernel", "starsim_set_binning", "starsim_set_roi",
                  "starsim_render_band_to", "starsim_render_lut"]:
         assert want in names
 

@@ -457,7 +457,7 @@ def test_ws_equals_sb_bitwise(torch_dev, psf, W, H, n, R, seed):
 def test_mode_setters_einval(torch_dev):
     from paper_conf_ipps_lizzh12_b200 import Context, StarsimError
     with Context(0) as c:
-        for fn in (c.set_binning, c.set_tile_kernel):
+        for fn in (c.set_binning, c.set_tile_kernel, c.set_roi):
             with pytest.raises(StarsimError):
                 fn(7)
 
@@ -557,3 +557,29 @@ def test_lut_einval(torch_dev, ctx):
     f = synth.uniform_field(10, 64, 64, seed=1)
     with pytest.raises(StarsimError):
         ctx.render_lut(*to_dev(torch_dev, f), 64, 64, 1.0, 65, 1.0)
+
+
+# ---------------------------------------------------------------- NEXT-3: the "pixel circle" ROI (reading R21)
+
+@pytest.mark.parametrize("W,H,n,R,sigma,kind", [(1024, 1024, 1000, 5, 1.0, "uniform"), (700, 530, 5000, 15, 2.5, "adv"),
+                                                 (300, 200, 2000, 10, 1.7, "uniform"), (512, 384, 3000, 63, 10.5, "uniform")])
+def test_circle_roi_parity(torch_dev, ctx, W, H, n, R, sigma, kind):
+    """starsim_set_roi(CIRCLE): the atomic and lookup-table renders against the oracle's circle ROI; the tiled renders
+    refuse it (EINVAL) and work again once the square ROI is back."""
+    from paper_conf_ipps_lizzh12_b200 import StarsimError
+    f = synth.adversarial_field(n, W, H, R, seed=43) if kind == "adv" else synth.uniform_field(n, W, H, seed=44,
+                                                                                                  mag_hi=2.0)
+    args = to_dev(torch_dev, f)
+    ctx.set_roi("circle")
+    try:
+        ref = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads(), roi="circle")
+        assert_parity(ctx.render_atomic(*args, W, H, sigma, R, 1.0).cpu().numpy(), ref, f"circle atomic R={R}")
+        if R <= 63:
+            ref_l = oracle.render_lut(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads(), roi="circle")
+            assert_parity(ctx.render_lut(*args, W, H, sigma, R, 1.0).cpu().numpy(), ref_l, f"circle lut R={R}")
+        with pytest.raises(StarsimError):
+            ctx.render(*args, W, H, sigma, R, 1.0)
+    finally:
+        ctx.set_roi("square")
+    ref_sq = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads())
+    assert_parity(ctx.render(*args, W, H, sigma, R, 1.0).cpu().numpy(), ref_sq, f"square after circle R={R}")

@@ -411,3 +411,52 @@ def test_lut_star_mass_is_the_centred_closed_form():
     assert abs(img.sum() - 0.98181476105437437) < 1e-13
     assert np.array_equal(img, img[::-1, ::-1]) and np.array_equal(img, img.T)
     assert img[10, 10] == img.max()
+
+
+# ---------------------------------------------------------------- NEXT-3: the "pixel circle" ROI (reading R21)
+
+# Gauss's circle problem: N(n) = #{(u, v) in Z^2 : u^2 + v^2 <= n} (OEIS A057655: N(6) = 21, N(12) = 37, N(20) = 69,
+# N(56) = 177).  For odd R the circle inscribed in the R x R ROI is centred on a pixel with radius R/2, so it holds
+# N(floor(R^2/4)) pixels; for R = 4 the centre is a pixel corner and the pixels are the 12 half-integer points
+# (+-1/2, +-1/2), (+-1/2, +-3/2), (+-3/2, +-1/2) within radius 2.
+@pytest.mark.parametrize("R,count", [(5, 21), (7, 37), (9, 69), (15, 177), (4, 12)])
+def test_circle_roi_holds_the_gauss_circle_count(R, count):
+    x, y, m = star(40.0, 40.0)
+    img, U = oracle.render(x, y, m, 81, 81, 1e4, R, 1.0, return_units=True, roi="circle")  # flat PSF: all > 0
+    assert int(np.count_nonzero(img)) == count and U == count
+    sq = oracle.render(x, y, m, 81, 81, 1e4, R, 1.0, roi="square")
+    assert int(np.count_nonzero(sq)) == R * R
+
+
+@pytest.mark.parametrize("R", [5, 8, 15])
+def test_circle_roi_is_the_square_minus_its_corners(R):
+    """Inside the circle the value is the square ROI's bitwise; the square's four corner pixels are always outside,
+    the four edge midpoints (odd R) inside; and a pixel-centred star's circle image is dihedrally symmetric."""
+    x, y, m = star(30.0, 30.0, 0.5)
+    sq = oracle.render(x, y, m, 61, 61, 2.0, R, 1.0)
+    ci = oracle.render(x, y, m, 61, 61, 2.0, R, 1.0, roi="circle")
+    inside = ci != 0
+    assert np.array_equal(ci[inside], sq[inside]) and np.all(sq[~inside & (sq != 0)] > 0)
+    lo = oracle.roi_lo(30.0, R)
+    for (py, px) in [(lo, lo), (lo, lo + R - 1), (lo + R - 1, lo), (lo + R - 1, lo + R - 1)]:
+        assert ci[py, px] == 0 and sq[py, px] > 0
+    if R % 2:
+        c = lo + (R - 1) // 2
+        for (py, px) in [(lo, c), (c, lo), (lo + R - 1, c), (c, lo + R - 1)]:
+            assert ci[py, px] > 0
+        for t in (ci.T, ci[::-1, :], ci[:, ::-1], ci[::-1, ::-1].T):
+            assert np.array_equal(t, ci)
+
+
+def test_circle_roi_superposition_and_clipping():
+    """The circle only masks: linear in the catalogue, and a circle cut by the image border keeps exactly the in-image
+    pixels of the full circle rendered in a larger frame (shifted by a whole number of pixels)."""
+    f = synth.uniform_field(40, 64, 48, seed=3, mag_hi=3.0)
+    a = oracle.render(f.x[:20], f.y[:20], f.mag[:20], 64, 48, 1.3, 9, 1.0, roi="circle")
+    b = oracle.render(f.x[20:], f.y[20:], f.mag[20:], 64, 48, 1.3, 9, 1.0, roi="circle")
+    ab = oracle.render(f.x, f.y, f.mag, 64, 48, 1.3, 9, 1.0, roi="circle")
+    assert np.allclose(a + b, ab, rtol=1e-14, atol=0)
+    x, y, m = star(1.0, 2.0)
+    small = oracle.render(x, y, m, 20, 20, 1.5, 11, 1.0, roi="circle")
+    big = oracle.render(x + 10, y + 10, m, 40, 40, 1.5, 11, 1.0, roi="circle")
+    assert np.array_equal(small, big[10:30, 10:30])
