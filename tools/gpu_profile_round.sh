@@ -4,6 +4,7 @@
 set -u
 TAG=${1:-r1b}
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1
 STARSIM_PARITY_LOG=gpurun_out/${TAG}_parity.jsonl timeout 900 python -m pytest tests -m gpu -q > gpurun_out/gpu_tests.log 2>&1
 timeout 400 python bench.py > gpurun_out/${TAG}_bench_T.json 2> gpurun_out/bench.err
 timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv \
