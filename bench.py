@@ -234,11 +234,14 @@ def run_ours(args, world, rank, local_rank):
     ctx = Context(local_rank)
     ctx.set_tile_kernel(args.tile_kernel)
     stream = torch.cuda.Stream(dev)
-    x, y, m = (torch.from_numpy(a).to(dev) for a in (f.x, f.y, f.mag))
     prow = sdist.padded_band_rows(H, world)
+    row0, rows = sdist.band_rows(H, world, rank)
+    # N > 1: each rank holds the stars whose ROI rows meet its band (the per-band catalogue query, done once on the
+    # host before the timed region; same tile lists as the whole catalogue, so the same image bit for bit)
+    lf = f if world == 1 else synth.Field(*(a[sdist.band_star_mask(f.y, row0, rows, R)] for a in (f.x, f.y, f.mag)))
+    x, y, m = (torch.from_numpy(a).to(dev) for a in (lf.x, lf.y, lf.mag))
     band = torch.zeros((prow, W), dtype=torch.float32, device=dev)
     full = torch.empty((world * prow, W), dtype=torch.float32, device=dev) if world > 1 else None
-    row0, rows = sdist.band_rows(H, world, rank)
     flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
 
     # N > 1: the fused band exchange (tile epilogue stores into every rank's symmetric-memory frame over NVLink, then
@@ -335,8 +338,8 @@ def run_ours(args, world, rank, local_rank):
                               f"f={sm_mhz:.0f} MHz; U={U_band}, E={E_band}; frac at 1965 MHz = "
                               f"{(achieved / peak_max) if achieved else 0:.3f}",
                 "kernel_ms": tile_ms,
-                "hbm": {"bytes": 4 * W * (rows if world > 1 else H) + 16 * f.n,
-                        "achieved_GBps": (4 * W * (rows if world > 1 else H) + 16 * f.n) / (tile_ms * 1e-3) / 1e9,
+                "hbm": {"bytes": 4 * W * (rows if world > 1 else H) + 16 * lf.n,
+                        "achieved_GBps": (4 * W * (rows if world > 1 else H) + 16 * lf.n) / (tile_ms * 1e-3) / 1e9,
                         "peak_GBps": peaks.get("hbm_gbs"), "peak_source": peak_src}}
     kernels = {k: {"ms_per_step": v[0] / args.steps, "launches_per_step": v[1] / args.steps} for k, v in kt.items()
                if v[1]}
@@ -432,7 +435,7 @@ def run_ours(args, world, rank, local_rank):
     # e2e: the same C-ABI call with host (pinned) catalogue in and image out, copies inside the timed region
     e2e = None
     if not args.no_e2e:
-        hx, hy, hm = (torch.from_numpy(a).pin_memory() for a in (f.x, f.y, f.mag))
+        hx, hy, hm = (torch.from_numpy(a).pin_memory() for a in (lf.x, lf.y, lf.mag))
         himg = torch.empty((rows if world > 1 else H, W), dtype=torch.float32).pin_memory()
         dx, dy, dm = (torch.empty_like(x) for _ in range(3))
 
@@ -464,8 +467,9 @@ def run_ours(args, world, rank, local_rank):
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
         e_ms = float(te.item())
         e2e = {"value": U_frame / (e_ms * 1e-3), "unit": UNIT, "ms_per_step": e_ms,
-               "h2d_bytes_per_step": int(3 * 4 * f.n), "d2h_bytes_per_step": int(himg.numel() * 4),
-               "note": "pinned host catalogue -> device, render, image -> pinned host, per step, one stream"}
+               "h2d_bytes_per_step": int(3 * 4 * lf.n), "d2h_bytes_per_step": int(himg.numel() * 4),
+               "note": "pinned host catalogue -> device, render, image -> pinned host, per step, one stream"
+                       + ("; per rank: its band's catalogue in, its band out (max over ranks)" if world > 1 else "")}
         if world == 1 and args.method == "tiled":
             # the same steps pipelined over two streams (one ctx, catalogue and image buffers each): step i+1's copy in
             # and render overlap step i's copy out (PCIe is full duplex); every step still moves its own catalogue in
@@ -519,6 +523,9 @@ def run_ours(args, world, rank, local_rank):
                        "W": W, "H": H, "stars": f.n, "R": R, "sigma": sigma, "gain": A, "method": args.method,
                        "frames_per_s": 1e3 / ms, "updates_per_frame": U_frame, "exps_per_frame": E_frame,
                        "parallelism": f"bands{world}" if world > 1 else "single", "exchange": exchange,
+                       "catalogue": "whole frame" if world == 1 else
+                                    f"per rank: the stars whose ROI rows meet its band (rank 0: {lf.n} of {f.n}; "
+                                    "selected on the host before the timed region, dist.band_star_mask)",
                        "l2": "flushed before every step (256 MiB write, untimed)"},
             "clocks": clocks, "gpu_launches": int(round(launches * args.steps)),
             "gpu_launches_per_step": launches, "kernels": kernels,

@@ -1,9 +1,9 @@
 """Multi-GPU frames: horizontal bands, one per rank, assembled with one all-gather.
 
 The paper is single-GPU and names multi-GPU scaling as future work (Sec. V).  Here the image is split
-into G horizontal bands of whole 32-row tiles; every rank holds the full catalogue, renders its band with
-``starsim_render_band`` (stars are routed to a band iff their clipped ROI rows intersect it -- done inside the
-library's binning pass), and ``torch.distributed.all_gather_into_tensor`` concatenates the bands: row-major band
+into G horizontal bands of whole 64-row tiles; every rank renders its band with ``starsim_render_band`` (stars are
+routed to a band iff their ROI rows intersect it: ``band_star_mask`` selects a rank's catalogue, and the library's
+binning pass clips every star to the band), and ``torch.distributed.all_gather_into_tensor`` concatenates the bands: row-major band
 concatenation *is* the frame, so there is no re-layout.  With tile-aligned band edges the assembled frame is bitwise
 equal to the single-GPU render (same per-pixel star order).
 
@@ -26,6 +26,23 @@ def band_rows(height: int, world: int, rank: int, align: int = TILE_H) -> tuple[
     row0 = min(height, t0 * align)
     row1 = min(height, t1 * align)
     return row0, row1 - row0
+
+
+def band_star_mask(y, row0: int, rows: int, roi: int):
+    """The stars routed to band [row0, row0 + rows): those whose ROI rows meet it, as a boolean
+    mask over the catalogue (host, numpy).  The ROI's first row is the exact rule of reading R7 (the R rows nearest
+    y, ties at k + 1/2 upward), evaluated exactly in fp64 on the fp32 coordinate; stars with a non-finite y are left
+    out (they contribute nothing).  Keeping the catalogue order, a band rendered from ``catalogue[mask]`` has the same
+    tile lists, in the same relative order, as the band rendered from the whole catalogue: the same image bit for bit.
+    This is the per-band catalogue query of a distributed render (the catalogue retrieval itself is out of scope,
+    SURVEY.md §8f); bench.py applies it before the timed region, so no rank bins stars of other bands."""
+    import numpy as np
+    y64 = np.asarray(y, dtype=np.float32).astype(np.float64)
+    fin = np.isfinite(y64)
+    yc = np.where(fin, y64, 0.0)
+    fy = np.floor(yc)
+    ly = (fy + (yc >= fy + 0.5) - (roi - 1) // 2) if roi % 2 else (fy + 1 - roi // 2)
+    return fin & (ly <= row0 + rows - 1) & (ly + roi - 1 >= row0)
 
 
 def padded_band_rows(height: int, world: int, align: int = TILE_H) -> int:

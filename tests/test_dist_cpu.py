@@ -27,6 +27,26 @@ def test_band_rows_partition_every_row():
             assert rows == list(range(H))
 
 
+@pytest.mark.parametrize("R", [1, 4, 9, 15])
+def test_band_star_mask_routes_exactly_the_stars_whose_roi_meets_the_band(R):
+    """band_star_mask against the oracle's clipped ROI rows (reading R7, exact) on adversarial coordinates: a star is
+    routed to a band iff its clipped ROI rows meet it; every contributing star reaches at least one band."""
+    import oracle
+    import synth
+    W, H, G = 70, 256, 4
+    f = synth.adversarial_field(3000, W, H, R, seed=7)
+    masks = [sdist.band_star_mask(f.y, *sdist.band_rows(H, G, g), R) for g in range(G)]
+    for i in range(f.n):
+        roi = oracle.star_roi(float(f.x[i]), float(f.y[i]), float(f.mag[i]), W, H, R)
+        if roi is None:
+            continue
+        y0, y1 = roi[2], roi[3]
+        for g in range(G):
+            r0, n = sdist.band_rows(H, G, g)
+            assert bool(masks[g][i]) == (y0 <= r0 + n - 1 and y1 >= r0), (i, g)
+        assert any(m[i] for m in masks)
+
+
 def _free_port():
     s = socket.socket()
     s.bind(("127.0.0.1", 0))
@@ -44,7 +64,9 @@ def _worker(rank, world, port, W, H, q):
     f = synth.uniform_field(600, W, H, seed=3)
 
     def render_band(x, y, mag, width, height, row0, rows, sigma, roi, gain, out):
-        img = oracle.render_band(f.x, f.y, f.mag, width, height, row0, rows, sigma, roi, gain)
+        # the rank's own catalogue: the stars routed to its band (bench.py does the same before its timed region)
+        sel = sdist.band_star_mask(f.y, row0, rows, roi)
+        img = oracle.render_band(f.x[sel], f.y[sel], f.mag[sel], width, height, row0, rows, sigma, roi, gain)
         out.copy_(torch.from_numpy(img.astype(np.float32)))
 
     x = torch.zeros(1)
