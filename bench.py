@@ -324,13 +324,14 @@ def run_ours(args, world, rank, local_rank):
     peak_max, _ = fp32_sfu_peak_updates(1965.0, U_band, E_band)
     achieved = U_band / (tile_ms * 1e-3) if args.method == "tiled" else None
     peaks, peak_src = load_peaks()
-    traffic = None
+    traffic, ncu_tile = None, {}
     prof = os.path.join(ROOT, "profiles", "ncu_tile_traffic.json")
     if os.path.exists(prof):
         try:
-            traffic = json.load(open(prof)).get(cfg.name, {}).get("dram_bytes_per_launch")
+            ncu_tile = json.load(open(prof)).get(cfg.name, {})
+            traffic = ncu_tile.get("dram_bytes_per_launch")
         except Exception:
-            traffic = None
+            traffic, ncu_tile = None, {}
     roofline = {"bound": "alu", "kernel": "k_tile", "achieved": achieved / 1e9 if achieved else None,
                 "peak": peak_rate / 1e9, "unit": "Gupdates/s", "frac": (achieved / peak_rate) if achieved else None,
                 "traffic": traffic,
@@ -338,6 +339,12 @@ def run_ours(args, world, rank, local_rank):
                               f"f={sm_mhz:.0f} MHz; U={U_band}, E={E_band}; frac at 1965 MHz = "
                               f"{(achieved / peak_max) if achieved else 0:.3f}",
                 "kernel_ms": tile_ms,
+                "issue": ({"kernel": ncu_tile.get("kernel"), "warp_instructions": ncu_tile.get("warp_instructions"),
+                           "issue_active_pct": ncu_tile.get("issue_active_pct"),
+                           "fma_pipe_pct": ncu_tile.get("fma_pipe_pct"),
+                           "note": "what bounds the tile kernel: instruction issue (ncu --set full, "
+                                   "profiles/ncu_tile_traffic.json; DESIGN.md section 9)"}
+                          if ncu_tile.get("warp_instructions") else None),
                 "hbm": {"bytes": 4 * W * (rows if world > 1 else H) + 16 * lf.n,
                         "achieved_GBps": (4 * W * (rows if world > 1 else H) + 16 * lf.n) / (tile_ms * 1e-3) / 1e9,
                         "peak_GBps": peaks.get("hbm_gbs"), "peak_source": peak_src}}

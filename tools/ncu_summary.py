@@ -110,6 +110,12 @@ def traffic(path, cfg):
         rd = float(d["dram__bytes_read.sum"]) * scale.get(u["dram__bytes_read.sum"], 1)
         wr = float(d["dram__bytes_write.sum"]) * scale.get(u["dram__bytes_write.sum"], 1)
         res = {cfg: {"dram_bytes_per_launch": rd + wr, "read": rd, "write": wr,
+                     "kernel": short(d["Kernel Name"]),
+                     "warp_instructions": float(d.get("smsp__inst_executed.sum", "nan").replace(",", "")),
+                     "issue_active_pct": float(d.get("smsp__issue_active.avg.pct_of_peak_sustained_active",
+                                                     "nan").replace(",", "")),
+                     "fma_pipe_pct": float(d.get("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
+                                                 "nan").replace(",", "")),
                      "duration_ns_ncu": float(d["gpu__time_duration.sum"]) *
                      {"us": 1e3, "usecond": 1e3, "ms": 1e6, "msecond": 1e6}.get(u["gpu__time_duration.sum"], 1)}}
     return json.dumps(res, indent=1)
