@@ -29,7 +29,14 @@ namespace starsim {
 constexpr int WS_NSK = NSTRIPS + 1;                  // strip keys 0..16 (0: ROI enters over the left edge)
 constexpr int WS_NBIN = (NBANDS + 1) * WS_NSK;       // 85 corner bins, band-major (band key 0: over the top edge)
 static_assert(WS_NBIN < 128, "bin keys (and the no-bin key WS_NBIN) fit 7 bits");
-constexpr int WS_CHUNK = 256;                        // stars per chunk
+#ifndef WS_CHUNK_OPT
+#define WS_CHUNK_OPT 256
+#endif
+#ifndef WS_CTAS_OPT
+#define WS_CTAS_OPT 1
+#endif
+constexpr int WS_CHUNK = WS_CHUNK_OPT;               // stars per chunk
+constexpr int WS_CTAS = WS_CTAS_OPT;                 // CTAs per SM
 constexpr int WS_PROD = WS_CHUNK / 32;               // producer warps
 constexpr int WS_CONS = 8;                           // consumer warps
 #ifndef WS_PGROUPS
@@ -453,7 +460,7 @@ __device__ __forceinline__ void ws_consumer(WsSmem& S, const FrameParams& fp, vo
 }
 
 template <bool INTEG>
-__global__ void __launch_bounds__(WS_THREADS, 1) k_tile_ws(const uint32_t* __restrict__ ids,
+__global__ void __launch_bounds__(WS_THREADS, WS_CTAS) k_tile_ws(const uint32_t* __restrict__ ids,
                                                            const StarRec* __restrict__ rec, FrameParams fp,
                                                            void* __restrict__ out_, const WorkItem* __restrict__ items,
                                                            const uint2* __restrict__ split_tab,
@@ -503,7 +510,7 @@ void launch_tile_ws(const uint32_t* ids, const StarRec* rec, const FrameParams& 
                     cudaStream_t st) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
-  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)num_sms);  // persistent: one CTA per SM
+  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)WS_CTAS * num_sms);  // persistent CTAs
   if (fp.psf)
     k_tile_ws<true><<<(unsigned)grid, WS_THREADS, sizeof(WsSmem), st>>>(ids, rec, fp, out, items, split_tab,
                                                                          part_buf, done, hdr);
