@@ -42,6 +42,9 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="T")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="N > 1: weak = a W x (H N) frame with N n stars, one H-row band per rank (default); strong = "
+                         "the --config frame itself split into N bands (the north star's C5 target: --config C5)")
     ap.add_argument("--method", default="tiled", choices=["tiled", "atomic"])
     ap.add_argument("--tile-kernel", default="auto", choices=["auto", "lists", "sb", "ws"],
                     help="starsim_set_tile_kernel mode (A/B comparisons; the default is the product path)")
@@ -124,10 +127,10 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------------------------------------ workload
-def workload(cfg_name, world, rank):
+def workload(cfg_name, world, rank, scaling="weak"):
     import synth
     cfg = synth.CONFIGS[cfg_name]
-    if world == 1:
+    if world == 1 or scaling == "strong":
         return cfg, cfg.field(), cfg.H, (0, cfg.H)
     # weak scaling: frame W x (H*world), world*n stars; every rank holds the full catalogue (replicated)
     H = cfg.H * world
@@ -227,7 +230,7 @@ def run_ours(args, world, rank, local_rank):
 
     dev = torch.device(f"cuda:{local_rank}")
     torch.cuda.set_device(dev)
-    cfg, f, H, _ = workload(args.config, world, rank)
+    cfg, f, H, _ = workload(args.config, world, rank, args.scaling)
     W, R, sigma = cfg.W, cfg.R, cfg.sigma
     A = synth.bench_gain(sigma)
     U_frame, E_frame = units_of(f, W, H, R)
@@ -523,7 +526,7 @@ def run_ours(args, world, rank, local_rank):
     if not args.no_cpu_baseline and world == 1:
         cpu = cpu_baseline(cfg, f, W, H)
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": args.scaling,
             "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": f"{cfg.name}: {W}x{H}, {cfg.n} uniform stars, R={R}, sigma={sigma:g}"
                                    + (f"; {world} bands of {prow} rows + NCCL all-gather" if world > 1 else ""),
