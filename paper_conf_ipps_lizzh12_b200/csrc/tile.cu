@@ -72,7 +72,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
 
   // accumulate-phase identity of this lane
   const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
-  const int Q = 8 * wx + q, p = B * NSTRIPS + Q;
+  const int Q = 8 * wx + q;
   const int swz = (Q >> 2) & 1;
   const uint32_t gy_base = (uint32_t)__cvta_generic_to_shared(S.gy) + 16u * hq;
   const uint32_t gxa_base = (uint32_t)__cvta_generic_to_shared(S.gx) + 16u * swz;
