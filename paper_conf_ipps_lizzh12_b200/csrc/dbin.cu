@@ -30,6 +30,7 @@ constexpr int DP_SPT = DB_CTA / DP_THREADS;      // stars per thread (strided by
 constexpr int DCS_THREADS = 256;
 constexpr int DCS_PER = 8;                       // k_dcolscan: consecutive CTA counts per lane
 static_assert(DB_MAXT <= 65536 && DB_CTA <= 65536, "tile ids, slots and star indices are 16-bit in k_dplace");
+static_assert(DP_WARPS == 32, "dp_block_scan scans the warp sums with one warp");
 
 __global__ void __launch_bounds__(DC_THREADS, 2) k_dcount(const float* __restrict__ X, const float* __restrict__ Y,
                                                        const float* __restrict__ M, int64_t n, FrameParams fp,
@@ -112,15 +113,22 @@ __device__ __forceinline__ uint32_t dp_block_scan(uint32_t v, uint32_t* s_w, uin
   }
   if (lane == 31) s_w[warp] = incl;
   __syncthreads();
-  uint32_t pre = 0, tot = 0;
+  if (warp == 0) {  // exclusive scan of the DP_WARPS (= 32) warp sums; the total in slot DP_WARPS
+    const uint32_t u = s_w[lane];
+    uint32_t wi = u;
 #pragma unroll
-  for (int w = 0; w < DP_WARPS; ++w) {
-    const uint32_t u = s_w[w];
-    pre += w < warp ? u : 0u;
-    tot += u;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(0xffffffffu, wi, o);
+      if (lane >= o) wi += t;
+    }
+    __syncwarp();
+    s_w[lane] = wi - u;
+    if (lane == 31) s_w[DP_WARPS] = wi;
   }
   __syncthreads();
-  *total = tot;
+  const uint32_t pre = s_w[warp];
+  *total = s_w[DP_WARPS];
+  __syncthreads();
   return pre + incl - v;
 }
 
@@ -130,7 +138,7 @@ struct DpSmem {
   uint32_t gstart[DB_MAXT + 1];  // per tile: pairs of the CTA, then the first position of the tile's group
   uint32_t cur[DB_MAXT];         // per tile: next free slot of its group; then the tile list position of the group
   uint16_t arr[DP_KEYS];          // the CTA's star indices grouped by tile (in arbitrary order inside a group)
-  uint32_t s_w[DP_WARPS];
+  uint32_t s_w[DP_WARPS + 1];
 };
 
 // the tiles of the star with ROI origin lo, packed: first tile t0 | dx << 16 | dy << 17 (it also covers t0 + 1 if dx,
