@@ -55,7 +55,7 @@ struct starsim_ctx {
   int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto, 1 lists, 2 sorted bins, 3 warp-specialised sorted bins
   int32_t bin_impl = 0;   // starsim_set_binning: 0 auto (dbin.cu when it applies), 1 always bin.cu's pipeline
   std::string err;
-  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat;
+  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat, codes;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
@@ -224,12 +224,12 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
     // (step a2 runs inside k_dplace; an empty catalogue has no k_dplace, so k_scan plans its all-empty tiles)
     uint32_t* C = (uint32_t*)c->cmat.p;
     if (n > 0) {
-      timed(c, 0, st, [&] { launch_dcount(x, y, mag, n, fp, rec, C, (int)ntiles, st); });
+      timed(c, 0, st, [&] { launch_dcount(x, y, mag, n, fp, rec, (uint32_t*)c->codes.p, C, (int)ntiles, st); });
       if ((rc = check_launch(c, "k_dcount"))) return rc;
       timed(c, 2, st, [&] { launch_dcolscan(C, n, (int)ntiles, cnt, 1, st); });  // dense totals for k_dplace
       if ((rc = check_launch(c, "k_dcolscan"))) return rc;
       timed(c, 1, st, [&] {
-        launch_dplace(rec, n, fp, C, (int)ntiles, cnt, tile_off, hdr, (WorkItem*)c->items.p,
+        launch_dplace((const uint32_t*)c->codes.p, n, fp, C, (int)ntiles, cnt, tile_off, hdr, (WorkItem*)c->items.p,
                       (uint2*)c->split_tab.p, part_cap, done, ids, st);
       });
       if ((rc = check_launch(c, "k_dplace"))) return rc;
@@ -323,6 +323,8 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
       (rc = grow(c, c->cmat, sizeof(uint32_t) * (size_t)ntiles * (size_t)(dbin_ctas(n) > 0 ? dbin_ctas(n) : 1),
                  "count matrix")))
     return rc;
+  if (dbin_ok(fp, ntiles) && (rc = grow(c, c->codes, sizeof(uint32_t) * (size_t)(n > 0 ? n : 1), "tile boxes")))
+    return rc;
 
   GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, c->psf, c->tile_impl, c->bin_impl, fp.ndst, {}, sigma, gain, st,
                c->scratch_gen};
@@ -410,7 +412,7 @@ void starsim_destroy(starsim_ctx* c) {
     cudaDeviceSynchronize();
     if (c->have_graph) cudaGraphExecDestroy(c->gexec);
     Buf* bufs[] = {&c->rec, &c->slots, &c->ids, &c->tmp, &c->tile_off, &c->items, &c->split_tab, &c->parts,
-                   &c->partial, &c->zeroed, &c->stage, &c->cmat};
+                   &c->partial, &c->zeroed, &c->stage, &c->cmat, &c->codes};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {

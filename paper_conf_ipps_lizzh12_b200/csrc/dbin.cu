@@ -32,9 +32,14 @@ constexpr int DCS_PER = 8;                       // k_dcolscan: consecutive CTA 
 static_assert(DB_MAXT <= 65536 && DB_CTA <= 65536, "tile ids, slots and star indices are 16-bit in k_dplace");
 static_assert(DP_WARPS == 32, "dp_block_scan scans the warp sums with one warp");
 
+// A star's tile box, packed: first tile t0 | dx << 16 | dy << 17 (it also covers t0 + 1 if dx, t0 + ntx if dy,
+// t0 + ntx + 1 if both); DP_NONE if the star is culled.  Written by k_dcount, read by k_dplace.
+constexpr uint32_t DP_NONE = 0xFFFFFFFFu;
+
 __global__ void __launch_bounds__(DC_THREADS, 2) k_dcount(const float* __restrict__ X, const float* __restrict__ Y,
                                                        const float* __restrict__ M, int64_t n, FrameParams fp,
-                                                       StarRec* __restrict__ rec, uint32_t* __restrict__ C,
+                                                       StarRec* __restrict__ rec, uint32_t* __restrict__ codes,
+                                                       uint32_t* __restrict__ C,
                                                        int nCTA, int ntiles) {
   __shared__ uint32_t cnt[DB_MAXT];
   const int tid = threadIdx.x, cta = blockIdx.x;
@@ -58,12 +63,15 @@ __global__ void __launch_bounds__(DC_THREADS, 2) k_dcount(const float* __restric
     int cx0, cx1, cy0, cy1;
     const StarRec r = prep_star(xs[k], ys[k], ms[k], fp, cx0, cx1, cy0, cy1);
     rec[i] = r;
+    uint32_t code = DP_NONE;
     if (r.lo != LO_CULLED) {
       const int tx0 = cx0 / TILE_W, tx1 = cx1 / TILE_W;
       const int ty0 = (cy0 - fp.row0) / TILE_H, ty1 = (cy1 - fp.row0) / TILE_H;
       for (int ty = ty0; ty <= ty1; ++ty)
         for (int tx = tx0; tx <= tx1; ++tx) atomicAdd(&cnt[ty * fp.ntx + tx], 1u);
+      code = (uint32_t)(ty0 * fp.ntx + tx0) | (uint32_t)(tx1 - tx0) << 16 | (uint32_t)(ty1 - ty0) << 17;
     }
+    codes[i] = code;  // the star's tile box for k_dplace (one coalesced word instead of a record gather)
   }
   __syncthreads();
   for (int t = tid; t < ntiles; t += DC_THREADS) C[(int64_t)t * nCTA + cta] = cnt[t];
@@ -141,18 +149,6 @@ struct DpSmem {
   uint32_t s_w[DP_WARPS + 1];
 };
 
-// the tiles of the star with ROI origin lo, packed: first tile t0 | dx << 16 | dy << 17 (it also covers t0 + 1 if dx,
-// t0 + ntx if dy, t0 + ntx + 1 if both); DP_NONE if the star is culled
-constexpr uint32_t DP_NONE = 0xFFFFFFFFu;
-__device__ __forceinline__ uint32_t star_tiles(const FrameParams& fp, uint32_t lo) {
-  if (lo == LO_CULLED) return DP_NONE;
-  int cx0, cx1, cy0, cy1;
-  clip_roi(fp, lo_x_of(lo), lo_y_of(lo), cx0, cx1, cy0, cy1);  // cx0, cy0 - row0 >= 0: plain shifts
-  const int tx0 = cx0 >> 7, ty0 = (cy0 - fp.row0) >> 6;
-  const uint32_t dx = (uint32_t)((cx1 >> 7) - tx0), dy = (uint32_t)(((cy1 - fp.row0) >> 6) - ty0);
-  return (uint32_t)(ty0 * fp.ntx + tx0) | dx << 16 | dy << 17;
-}
-
 // tiles of a packed box (0 if the star is culled) and its e-th tile, e < box_n (row-major order inside the box)
 __device__ __forceinline__ int box_n(uint32_t code) {
   return code == DP_NONE ? 0 : (1 + (int)((code >> 16) & 1u)) << (int)((code >> 17) & 1u);
@@ -228,13 +224,13 @@ __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restr
   __syncthreads();
 }
 
-__global__ void __launch_bounds__(DP_THREADS, 2) k_dplace(const StarRec* __restrict__ rec, int64_t n, FrameParams fp,
+__global__ void __launch_bounds__(DP_THREADS, 2) k_dplace(const uint32_t* __restrict__ codes, int64_t n, FrameParams fp,
                                                        const uint32_t* __restrict__ C, int nCTA, int ntiles,
                                                        const uint32_t* __restrict__ cnt, uint32_t* __restrict__ tile_off,
                                                        Header* hdr, WorkItem* __restrict__ items,
                                                        uint2* __restrict__ split_tab, int part_cap,
                                                        uint32_t* __restrict__ done, uint32_t* __restrict__ ids) {
-  static_assert(TILE_W == 128 && TILE_H == 64, "star_tiles shifts");
+  static_assert(TILE_W == 128 && TILE_H == 64, "tile boxes span at most 2 x 2 tiles for R <= DB_MAXR");
   extern __shared__ __align__(16) unsigned char dsm_raw[];
   DpSmem& S = *reinterpret_cast<DpSmem*>(dsm_raw);
   const int tid = threadIdx.x, cta = blockIdx.x;
@@ -245,10 +241,8 @@ __global__ void __launch_bounds__(DP_THREADS, 2) k_dplace(const StarRec* __restr
 #pragma unroll
   for (int k = 0; k < DP_SPT; ++k) {
     const int64_t i = c0 + tid + k * DP_THREADS;
-    code[k] = i < n ? __ldg(&rec[i].lo) : LO_CULLED;
+    code[k] = i < n ? __ldg(&codes[i]) : DP_NONE;
   }
-#pragma unroll
-  for (int k = 0; k < DP_SPT; ++k) code[k] = star_tiles(fp, code[k]);
   __syncthreads();
   // group sizes
 #pragma unroll
@@ -316,9 +310,9 @@ void init_dbin_kernels() {
 }
 
 void launch_dcount(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
-                   uint32_t* C, int ntiles, cudaStream_t st) {
+                   uint32_t* codes, uint32_t* C, int ntiles, cudaStream_t st) {
   const int nc = dbin_ctas(n);
-  if (nc > 0) k_dcount<<<nc, DC_THREADS, 0, st>>>(x, y, m, n, fp, rec, C, nc, ntiles);
+  if (nc > 0) k_dcount<<<nc, DC_THREADS, 0, st>>>(x, y, m, n, fp, rec, codes, C, nc, ntiles);
 }
 
 void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstride, cudaStream_t st) {
@@ -326,12 +320,12 @@ void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstr
   k_dcolscan<<<(ntiles + wpb - 1) / wpb, DCS_THREADS, 0, st>>>(C, dbin_ctas(n), ntiles, cnt, cstride);
 }
 
-void launch_dplace(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,
+void launch_dplace(const uint32_t* codes, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,
                    const uint32_t* cnt, uint32_t* tile_off, Header* hdr, WorkItem* items, uint2* split_tab,
                    int part_cap, uint32_t* done, uint32_t* ids, cudaStream_t st) {
   const int nc = dbin_ctas(n);
   if (nc > 0)
-    k_dplace<<<nc, DP_THREADS, sizeof(DpSmem), st>>>(rec, n, fp, C, nc, ntiles, cnt, tile_off, hdr, items, split_tab,
+    k_dplace<<<nc, DP_THREADS, sizeof(DpSmem), st>>>(codes, n, fp, C, nc, ntiles, cnt, tile_off, hdr, items, split_tab,
                                                       part_cap, done, ids);
 }
 

@@ -15,9 +15,9 @@ void init_dbin_kernels();
 size_t dbin_smem(int ntiles);
 int dbin_ctas(int64_t n);
 void launch_dcount(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
-                   uint32_t* C, int ntiles, cudaStream_t st);
+                   uint32_t* codes, uint32_t* C, int ntiles, cudaStream_t st);
 void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstride, cudaStream_t st);
-void launch_dplace(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,
+void launch_dplace(const uint32_t* codes, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,
                    const uint32_t* cnt, uint32_t* tile_off, Header* hdr, WorkItem* items, uint2* split_tab,
                    int part_cap, uint32_t* done, uint32_t* ids, cudaStream_t st);
 void launch_prep(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
