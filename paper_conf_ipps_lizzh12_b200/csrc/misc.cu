@@ -14,6 +14,7 @@ namespace starsim {
 // ---------------------------------------------------------------------------------------------------------------
 constexpr int ATOM_WARPS = 8;
 
+template <bool CIRC>  // NEXT-3: the pixel circle (reading R21) instead of the square ROI
 __global__ void __launch_bounds__(ATOM_WARPS * 32) k_atomic(const float* __restrict__ X, const float* __restrict__ Y,
                                                             const float* __restrict__ M, int64_t n, FrameParams fp,
                                                             float* __restrict__ out) {
@@ -64,7 +65,7 @@ __global__ void __launch_bounds__(ATOM_WARPS * 32) k_atomic(const float* __restr
   for (int p = lane; p < w * h; p += 32) {
     const int r = __float2int_rz(((float)p + 0.5f) * inv_w);
     const int c = p - r * w;
-    if (fp.roi && !in_roi_circle(cy0 + r - ly, cx0 + c - lx, fp.R)) continue;  // NEXT-3: the pixel circle
+    if (CIRC && !in_roi_circle(cy0 + r - ly, cx0 + c - lx, fp.R)) continue;  // NEXT-3: the pixel circle
     atomicAdd(o + (int64_t)r * fp.W + c, gy[r] * gx[c]);
   }
 }
@@ -74,7 +75,10 @@ void launch_atomic(const float* x, const float* y, const float* m, int64_t n, co
   if (n <= 0) return;
   const unsigned blocks = (unsigned)((n + ATOM_WARPS - 1) / ATOM_WARPS);
   const size_t smem = sizeof(float) * 2 * fp.R * ATOM_WARPS;
-  k_atomic<<<blocks, ATOM_WARPS * 32, smem, st>>>(x, y, m, n, fp, out);
+  if (fp.roi)
+    k_atomic<true><<<blocks, ATOM_WARPS * 32, smem, st>>>(x, y, m, n, fp, out);
+  else
+    k_atomic<false><<<blocks, ATOM_WARPS * 32, smem, st>>>(x, y, m, n, fp, out);
 }
 
 // ---------------------------------------------------------------------------------------------------------------
@@ -85,6 +89,7 @@ void launch_atomic(const float* x, const float* y, const float* m, int64_t n, co
 // paper's 3-D table exactly), and each warp adds s' * LUT[r][c] into its star's ROI pixels with global fp32
 // reductions (reading R20: the star sits at its ROI's centre -- exact for stars on pixel centres, odd R).
 // ---------------------------------------------------------------------------------------------------------------
+template <bool CIRC>
 __global__ void __launch_bounds__(ATOM_WARPS * 32) k_lut(const float* __restrict__ X, const float* __restrict__ Y,
                                                          const float* __restrict__ M, int64_t n, FrameParams fp,
                                                          float* __restrict__ out) {
@@ -128,7 +133,7 @@ __global__ void __launch_bounds__(ATOM_WARPS * 32) k_lut(const float* __restrict
   for (int p = lane; p < w * h; p += 32) {
     const int r = __float2int_rz(((float)p + 0.5f) * inv_w);
     const int c = p - r * w;
-    if (fp.roi && !in_roi_circle(cy0 + r - ly, cx0 + c - lx, R)) continue;  // NEXT-3: the pixel circle
+    if (CIRC && !in_roi_circle(cy0 + r - ly, cx0 + c - lx, R)) continue;  // NEXT-3: the pixel circle
     atomicAdd(o + (int64_t)r * fp.W + c, s * lut[r * R + c]);
   }
 }
@@ -138,7 +143,10 @@ void launch_lut(const float* x, const float* y, const float* m, int64_t n, const
   if (n <= 0) return;
   const unsigned blocks = (unsigned)((n + ATOM_WARPS - 1) / ATOM_WARPS);
   const size_t smem = sizeof(float) * (size_t)(fp.R * fp.R + fp.R);
-  k_lut<<<blocks, ATOM_WARPS * 32, smem, st>>>(x, y, m, n, fp, out);
+  if (fp.roi)
+    k_lut<true><<<blocks, ATOM_WARPS * 32, smem, st>>>(x, y, m, n, fp, out);
+  else
+    k_lut<false><<<blocks, ATOM_WARPS * 32, smem, st>>>(x, y, m, n, fp, out);
 }
 
 // ---------------------------------------------------------------------------------------------------------------
