@@ -58,6 +58,9 @@ def test_null_ctx_is_einval(lib):
     assert lib.starsim_render_atomic(None, None, None, None, 0, 16, 16, 1.0, 5, 1.0, vp(1), None) == -1
     assert lib.starsim_quantize(None, None, 0, 8, None, None) == -1
     assert lib.starsim_upload_aos(None, None, 0, None, None, None, None) == -1
+    for fn in (lib.starsim_set_psf, lib.starsim_set_roi, lib.starsim_set_tile_kernel, lib.starsim_set_binning):
+        fn.argtypes = [ctypes.c_void_p, ctypes.c_int32]
+        assert fn(None, 0) == -1
     assert lib.starsim_profile(None, 1) == -1
     lib.starsim_destroy(None)   # NULL-safe
 
