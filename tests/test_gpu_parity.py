@@ -622,3 +622,20 @@ def test_unsplit_huge_tile_lists(torch_dev, ctx):
     ma, rl = errors(a.cpu().numpy().astype(np.float64), ref)
     assert ma <= tol and rl <= tol, (ma, rl, tol)
     assert torch.equal(a, ctx.render(*args, W, H, sigma, R, 1.0))
+
+
+def test_circle_roi_with_integrated_psf(torch_dev, ctx):
+    """NEXT-2 and NEXT-3 together on the star-centric kernels: the pixel-integrated PSF over the pixel-circle ROI."""
+    W, H, n, R, sigma = 400, 300, 3000, 15, 2.5
+    f = synth.uniform_field(n, W, H, seed=45, mag_hi=2.0)
+    args = to_dev(torch_dev, f)
+    ctx.set_roi("circle")
+    ctx.set_psf("integrated")
+    try:
+        ref = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0, psf="integrated", roi="circle")
+        assert_parity(ctx.render_atomic(*args, W, H, sigma, R, 1.0).cpu().numpy(), ref, "circle integrated atomic")
+        ref_l = oracle.render_lut(f.x, f.y, f.mag, W, H, sigma, R, 1.0, psf="integrated", roi="circle")
+        assert_parity(ctx.render_lut(*args, W, H, sigma, R, 1.0).cpu().numpy(), ref_l, "circle integrated lut")
+    finally:
+        ctx.set_roi("square")
+        ctx.set_psf("point")

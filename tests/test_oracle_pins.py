@@ -460,3 +460,16 @@ def test_circle_roi_superposition_and_clipping():
     small = oracle.render(x, y, m, 20, 20, 1.5, 11, 1.0, roi="circle")
     big = oracle.render(x + 10, y + 10, m, 40, 40, 1.5, 11, 1.0, roi="circle")
     assert np.array_equal(small, big[10:30, 10:30])
+
+
+def test_circle_roi_integrated_psf_keeps_the_circle_and_the_masses():
+    """psf="integrated" with roi="circle": the circle's pixels carry exactly the integrated square-ROI values (the
+    mask only removes pixels), and a pixel-centred star's image stays dihedrally symmetric."""
+    x, y, m = star(20.0, 20.0)
+    sq = oracle.render(x, y, m, 41, 41, 1.8, 11, 1.0, psf="integrated")
+    ci = oracle.render(x, y, m, 41, 41, 1.8, 11, 1.0, psf="integrated", roi="circle")
+    inside = ci != 0
+    assert int(inside.sum()) == 97  # Gauss circle N(30) = 97 (OEIS A057655) for R = 11: r^2 = 30.25
+    assert np.array_equal(ci[inside], sq[inside])
+    for t in (ci.T, ci[::-1, :], ci[:, ::-1]):
+        assert np.array_equal(t, ci)
