@@ -23,14 +23,18 @@ namespace starsim {
 constexpr int DB_CTA = 4096;                     // stars per CTA (one column of the count matrix)
 constexpr int DC_THREADS = 1024;                 // k_dcount: DB_CTA / DC_THREADS stars per thread
 constexpr int DC_PER = DB_CTA / DC_THREADS;
-constexpr int DP_THREADS = 1024;                 // k_dplace
+#ifndef DP_THREADS_OPT
+#define DP_THREADS_OPT 1024
+#endif
+constexpr int DP_THREADS = DP_THREADS_OPT;        // k_dplace
+constexpr int DP_MINB = 2048 / DP_THREADS;        // CTAs per SM (all 245 CTAs of a 1M-star frame resident)
 constexpr int DP_WARPS = DP_THREADS / 32;
 constexpr int DP_KEYS = DB_CTA * 4;              // at most 2 x 2 tiles per star
 constexpr int DP_SPT = DB_CTA / DP_THREADS;      // stars per thread (strided by DP_THREADS)
 constexpr int DCS_THREADS = 256;
 constexpr int DCS_PER = 8;                       // k_dcolscan: consecutive CTA counts per lane
 static_assert(DB_MAXT <= 65536 && DB_CTA <= 65536, "tile ids, slots and star indices are 16-bit in k_dplace");
-static_assert(DP_WARPS == 32, "dp_block_scan scans the warp sums with one warp");
+static_assert(DP_WARPS <= 32, "dp_block_scan scans the warp sums with one warp");
 
 // A star's tile box, packed: first tile t0 | dx << 16 | dy << 17 (it also covers t0 + 1 if dx, t0 + ntx if dy,
 // t0 + ntx + 1 if both); DP_NONE if the star is culled.  Written by k_dcount, read by k_dplace.
@@ -122,7 +126,7 @@ __device__ __forceinline__ uint32_t dp_block_scan(uint32_t v, uint32_t* s_w, uin
   if (lane == 31) s_w[warp] = incl;
   __syncthreads();
   if (warp == 0) {  // exclusive scan of the DP_WARPS (= 32) warp sums; the total in slot DP_WARPS
-    const uint32_t u = s_w[lane];
+    const uint32_t u = lane < DP_WARPS ? s_w[lane] : 0u;
     uint32_t wi = u;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -130,7 +134,7 @@ __device__ __forceinline__ uint32_t dp_block_scan(uint32_t v, uint32_t* s_w, uin
       if (lane >= o) wi += t;
     }
     __syncwarp();
-    s_w[lane] = wi - u;
+    if (lane < DP_WARPS) s_w[lane] = wi - u;
     if (lane == 31) s_w[DP_WARPS] = wi;
   }
   __syncthreads();
@@ -182,10 +186,10 @@ __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restr
   if (lane == 31) S.s_w3[warp] = incl;
   __syncthreads();
   if (warp == 0) {  // exclusive scan of the warp sums; the total in the last slot's inclusive value
-    const uint3 v = S.s_w3[lane];
+    const uint3 v = lane < DP_WARPS ? S.s_w3[lane] : make_uint3(0u, 0u, 0u);
     const uint3 wi = warp_incl_scan3(v, lane);
     __syncwarp();
-    S.s_w3[lane] = make_uint3(wi.x - v.x, wi.y - v.y, wi.z - v.z);
+    if (lane < DP_WARPS) S.s_w3[lane] = make_uint3(wi.x - v.x, wi.y - v.y, wi.z - v.z);
     const uint3 ta = make_uint3(__shfl_sync(0xffffffffu, wi.x, 31), __shfl_sync(0xffffffffu, wi.y, 31),
                                 __shfl_sync(0xffffffffu, wi.z, 31));
     if (lane == 0) {
@@ -224,7 +228,7 @@ __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restr
   __syncthreads();
 }
 
-__global__ void __launch_bounds__(DP_THREADS, 2) k_dplace(const uint32_t* __restrict__ codes, int64_t n, FrameParams fp,
+__global__ void __launch_bounds__(DP_THREADS, DP_MINB) k_dplace(const uint32_t* __restrict__ codes, int64_t n, FrameParams fp,
                                                        const uint32_t* __restrict__ C, int nCTA, int ntiles,
                                                        const uint32_t* __restrict__ cnt, uint32_t* __restrict__ tile_off,
                                                        Header* hdr, WorkItem* __restrict__ items,
