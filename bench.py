@@ -356,91 +356,97 @@ def run_ours(args, world, rank, local_rank):
 
     # NEXT-1 variant (1 GPU, tiled): the same frame with the output stage fused -- u8 gray image written by k_tile
     variants = {}
-    if world == 1 and args.method == "tiled":
-        gray = torch.empty((H, W), dtype=torch.uint8, device=dev)
-        Ag = synth.bench_gain(sigma, 8)
+    try:  # the variants are diagnostics: a failure is recorded in the line, not fatal to the headline
+        if world == 1 and args.method == "tiled":
+            gray = torch.empty((H, W), dtype=torch.uint8, device=dev)
+            Ag = synth.bench_gain(sigma, 8)
 
-        def gstep():
-            with torch.cuda.stream(stream):
-                ctx.render_gray(x, y, m, W, H, sigma, R, Ag, bits=8, out=gray, stream=stream)
+            def gstep():
+                with torch.cuda.stream(stream):
+                    ctx.render_gray(x, y, m, W, H, sigma, R, Ag, bits=8, out=gray, stream=stream)
 
-        for _ in range(max(3, args.warmup)):
-            gstep()
-        barrier()
-        g_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-                for _ in range(args.steps)]
-        for i in range(args.steps):
-            with torch.cuda.stream(stream):
-                flush.fill_(float(i))
-                g_ev[i][0].record(stream)
-            gstep()
-            g_ev[i][1].record(stream)
-        barrier()
-        g_ms = sum(a.elapsed_time(b) for a, b in g_ev) / args.steps
-        variants["gray_u8"] = {"ms_per_step": g_ms, "frames_per_s": 1e3 / g_ms, "updates_per_s": U_frame / (g_ms * 1e-3),
-                               "note": "starsim_render_gray (output stage fused into k_tile, u8 image)"}
-        # NEXT-2 variant: the same fp32 frame with the pixel-integrated PSF (erf profiles instead of exp)
-        ctx.set_psf("integrated")
-        for _ in range(max(3, args.warmup)):
-            step(x, y, m)
-        barrier()
-        i_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-                for _ in range(args.steps)]
-        for i in range(args.steps):
-            with torch.cuda.stream(stream):
-                flush.fill_(float(i))
-                i_ev[i][0].record(stream)
-            step(x, y, m)
-            i_ev[i][1].record(stream)
-        barrier()
-        ctx.set_psf("point")
-        i_ms = sum(a.elapsed_time(b) for a, b in i_ev) / args.steps
-        variants["integrated_psf"] = {"ms_per_step": i_ms, "frames_per_s": 1e3 / i_ms,
-                                      "updates_per_s": U_frame / (i_ms * 1e-3),
-                                      "note": "starsim_set_psf(INTEGRATED): Eq. 2 integrated over each pixel (NEXT-2)"}
-
-        # the paper's two star-centric designs on the same frame: the atomic simulator and its lookup-table variant
-        for name, fn_, note in (("atomic", ctx.render_atomic, "starsim_render_atomic: the paper's parallel simulator "
-                                 "(Fig. 6), red.global.add per ROI pixel, nondeterministic order"),
-                                ("lut", ctx.render_lut, "starsim_render_lut: the paper's adaptive simulator "
-                                 "(PAPER.md:158-168), table at the ROI centre (reading R20, approximate off-centre)")):
-            if world > 1:
-                break
-            a_out = torch.empty((H, W), dtype=torch.float32, device=dev)
-            for _ in range(2):
-                fn_(x, y, m, W, H, sigma, R, A, out=a_out, stream=stream)
-            torch.cuda.synchronize()
-            a_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+            for _ in range(max(3, args.warmup)):
+                gstep()
+            barrier()
+            g_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                     for _ in range(args.steps)]
             for i in range(args.steps):
                 with torch.cuda.stream(stream):
                     flush.fill_(float(i))
-                    a_ev[i][0].record(stream)
+                    g_ev[i][0].record(stream)
+                gstep()
+                g_ev[i][1].record(stream)
+            barrier()
+            g_ms = sum(a.elapsed_time(b) for a, b in g_ev) / args.steps
+            variants["gray_u8"] = {"ms_per_step": g_ms, "frames_per_s": 1e3 / g_ms, "updates_per_s": U_frame / (g_ms * 1e-3),
+                                   "note": "starsim_render_gray (output stage fused into k_tile, u8 image)"}
+            # NEXT-2 variant: the same fp32 frame with the pixel-integrated PSF (erf profiles instead of exp)
+            ctx.set_psf("integrated")
+            for _ in range(max(3, args.warmup)):
+                step(x, y, m)
+            barrier()
+            i_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                    for _ in range(args.steps)]
+            for i in range(args.steps):
+                with torch.cuda.stream(stream):
+                    flush.fill_(float(i))
+                    i_ev[i][0].record(stream)
+                step(x, y, m)
+                i_ev[i][1].record(stream)
+            barrier()
+            ctx.set_psf("point")
+            i_ms = sum(a.elapsed_time(b) for a, b in i_ev) / args.steps
+            variants["integrated_psf"] = {"ms_per_step": i_ms, "frames_per_s": 1e3 / i_ms,
+                                          "updates_per_s": U_frame / (i_ms * 1e-3),
+                                          "note": "starsim_set_psf(INTEGRATED): Eq. 2 integrated over each pixel (NEXT-2)"}
+
+            # the paper's two star-centric designs on the same frame: the atomic simulator and its lookup-table variant
+            for name, fn_, note in (("atomic", ctx.render_atomic, "starsim_render_atomic: the paper's parallel simulator "
+                                     "(Fig. 6), red.global.add per ROI pixel, nondeterministic order"),
+                                    ("lut", ctx.render_lut, "starsim_render_lut: the paper's adaptive simulator "
+                                     "(PAPER.md:158-168), table at the ROI centre (reading R20, approximate off-centre)")):
+                if world > 1:
+                    break
+                a_out = torch.empty((H, W), dtype=torch.float32, device=dev)
+                for _ in range(2):
                     fn_(x, y, m, W, H, sigma, R, A, out=a_out, stream=stream)
-                    a_ev[i][1].record(stream)
-            torch.cuda.synchronize()
-            a_ms = sum(a.elapsed_time(b) for a, b in a_ev) / args.steps
-            variants[name] = {"ms_per_step": a_ms, "frames_per_s": 1e3 / a_ms, "updates_per_s": U_frame / (a_ms * 1e-3),
-                              "note": note}
-            if name == "atomic":  # NEXT-3: the same star-centric kernel with the pixel-circle ROI
-                ctx.set_roi("circle")
-                fn_(x, y, m, W, H, sigma, R, A, out=a_out, stream=stream)
                 torch.cuda.synchronize()
-                c_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                a_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                         for _ in range(args.steps)]
                 for i in range(args.steps):
                     with torch.cuda.stream(stream):
                         flush.fill_(float(i))
-                        c_ev[i][0].record(stream)
+                        a_ev[i][0].record(stream)
                         fn_(x, y, m, W, H, sigma, R, A, out=a_out, stream=stream)
-                        c_ev[i][1].record(stream)
+                        a_ev[i][1].record(stream)
                 torch.cuda.synchronize()
-                ctx.set_roi("square")
-                c_ms = sum(a.elapsed_time(b) for a, b in c_ev) / args.steps
-                variants["atomic_circle"] = {"ms_per_step": c_ms, "frames_per_s": 1e3 / c_ms,
-                                             "note": "starsim_set_roi(CIRCLE) + starsim_render_atomic: the paper's "
-                                                     "'pixel circle' ROI (NEXT-3, reading R21)"}
-            del a_out
+                a_ms = sum(a.elapsed_time(b) for a, b in a_ev) / args.steps
+                variants[name] = {"ms_per_step": a_ms, "frames_per_s": 1e3 / a_ms, "updates_per_s": U_frame / (a_ms * 1e-3),
+                                  "note": note}
+                if name == "atomic":  # NEXT-3: the same star-centric kernel with the pixel-circle ROI
+                    ctx.set_roi("circle")
+                    fn_(x, y, m, W, H, sigma, R, A, out=a_out, stream=stream)
+                    torch.cuda.synchronize()
+                    c_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                            for _ in range(args.steps)]
+                    for i in range(args.steps):
+                        with torch.cuda.stream(stream):
+                            flush.fill_(float(i))
+                            c_ev[i][0].record(stream)
+                            fn_(x, y, m, W, H, sigma, R, A, out=a_out, stream=stream)
+                            c_ev[i][1].record(stream)
+                    torch.cuda.synchronize()
+                    ctx.set_roi("square")
+                    c_ms = sum(a.elapsed_time(b) for a, b in c_ev) / args.steps
+                    variants["atomic_circle"] = {"ms_per_step": c_ms, "frames_per_s": 1e3 / c_ms,
+                                                 "note": "starsim_set_roi(CIRCLE) + starsim_render_atomic: the paper's "
+                                                         "'pixel circle' ROI (NEXT-3, reading R21)"}
+                del a_out
+    except Exception as e:  # noqa: BLE001
+        variants["error"] = f"{type(e).__name__}: {e}"
+        torch.cuda.synchronize()
+        ctx.set_psf("point")
+        ctx.set_roi("square")
 
     # e2e: the same C-ABI call with host (pinned) catalogue in and image out, copies inside the timed region
     e2e = None
