@@ -399,6 +399,25 @@ def run_ours(args, world, rank, local_rank):
             variants["integrated_psf"] = {"ms_per_step": i_ms, "frames_per_s": 1e3 / i_ms,
                                           "updates_per_s": U_frame / (i_ms * 1e-3),
                                           "note": "starsim_set_psf(INTEGRATED): Eq. 2 integrated over each pixel (NEXT-2)"}
+            # NEXT-3 variant: the same fp32 frame with the pixel-circle ROI (k_tile_sb masks the circle in its walk)
+            ctx.set_roi("circle")
+            for _ in range(max(3, args.warmup)):
+                step(x, y, m)
+            barrier()
+            r_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                    for _ in range(args.steps)]
+            for i in range(args.steps):
+                with torch.cuda.stream(stream):
+                    flush.fill_(float(i))
+                    r_ev[i][0].record(stream)
+                step(x, y, m)
+                r_ev[i][1].record(stream)
+            barrier()
+            ctx.set_roi("square")
+            r_ms = sum(a.elapsed_time(b) for a, b in r_ev) / args.steps
+            variants["circle_roi"] = {"ms_per_step": r_ms, "frames_per_s": 1e3 / r_ms,
+                                      "note": "starsim_set_roi(CIRCLE): the paper's 'pixel circle' ROI through the tiled "
+                                              "path (NEXT-3, reading R21)"}
 
             # the paper's two star-centric designs on the same frame: the atomic simulator and its lookup-table variant
             for name, fn_, note in (("atomic", ctx.render_atomic, "starsim_render_atomic: the paper's parallel simulator "

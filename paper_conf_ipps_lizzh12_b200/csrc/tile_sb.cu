@@ -57,9 +57,13 @@ struct SbSmem {
   uint32_t hist[TILE_WARPS][SB_NBIN];      // per warp: stars of each corner bin
   uint32_t binoff[TILE_WARPS][SB_NBIN];    // per warp, per bin: stars of the bin in the warps before
   uint32_t binstart[SB_NBIN + 1];          // exclusive scan of the bin totals (bin-major)
+  uint32_t lo2[SB_CHUNK + 1];              // CIRC: sorted star j's ROI origin (tile-relative, int16 x | int16 y << 16)
 };
 
-template <bool INTEG>
+// NEXT-3 in the tiled path (CIRC): the walk masks every ROI pixel outside the pixel circle of reading R21 --
+// (2 (col - lo_x) - (R-1))^2 + (2 (row - lo_y) - (R-1))^2 <= R^2 per (row, column) of the lane's 4 x 8 block, with
+// the star's ROI origin read from its slot.  The profiles, slots and summation order are unchanged.
+template <bool INTEG, bool CIRC>
 __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_t* __restrict__ ids,
                                                              const StarRec* __restrict__ rec, FrameParams fp,
                                                              void* __restrict__ out_,
@@ -122,9 +126,10 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
     const int nvalid = (int)min((uint32_t)SB_CHUNK, j1 - base);
     const StarRec r = rnext;
     int c0 = 0, c1 = -1, r0 = 0, r1 = -1;
-    uint32_t key = SB_NBIN;
+    uint32_t key = SB_NBIN, lo2 = 0u;
     if (tid < nvalid) {
       const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
+      lo2 = (uint32_t)(lx & 0xFFFF) | (uint32_t)ly << 16;
       c0 = max(lx, 0);
       c1 = min(lx + fp.R - 1, TWe - 1);
       r0 = max(ly, 0);
@@ -185,6 +190,7 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
       const uint32_t j = S.binstart[key] + S.binoff[warp][key] + rank;
       const float yr = r.y - (float)IY0, xr = r.x - (float)X0;  // exact
       const float2 sk2 = make_float2(sk, sk), s2 = make_float2(r.s, r.s);
+      if (CIRC) S.lo2[j] = lo2;
       // first band / strip of the slots: the corner bin's (-1 for an ROI that comes in over the top / left edge)
       const int b0 = (int)(key / SB_NSK) - 1, q0 = (int)(key % SB_NSK) - 1;
       // band slots (lane hq reads rows 4 hq .. 4 hq + 3 of a band): the two bands b0, b0+1 are 8 row quads w = 0..7
@@ -304,13 +310,38 @@ __global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_
       asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "r"(xa));
       asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(c.x), "=f"(c.y), "=f"(c.z), "=f"(c.w) : "r"(xa + 16u));
       const float gi[4] = {g.x, g.y, g.z, g.w};
+      if (!CIRC) {
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const float2 gg = make_float2(gi[i], gi[i]);
-        acc[i][0] = __ffma2_rn(gg, make_float2(a.x, a.y), acc[i][0]);
-        acc[i][1] = __ffma2_rn(gg, make_float2(a.z, a.w), acc[i][1]);
-        acc[i][2] = __ffma2_rn(gg, make_float2(c.x, c.y), acc[i][2]);
-        acc[i][3] = __ffma2_rn(gg, make_float2(c.z, c.w), acc[i][3]);
+        for (int i = 0; i < 4; ++i) {
+          const float2 gg = make_float2(gi[i], gi[i]);
+          acc[i][0] = __ffma2_rn(gg, make_float2(a.x, a.y), acc[i][0]);
+          acc[i][1] = __ffma2_rn(gg, make_float2(a.z, a.w), acc[i][1]);
+          acc[i][2] = __ffma2_rn(gg, make_float2(c.x, c.y), acc[i][2]);
+          acc[i][3] = __ffma2_rn(gg, make_float2(c.z, c.w), acc[i][3]);
+        }
+      } else {
+        // the star's ROI origin (its slot's), then per row the largest squared column offset inside the circle
+        const uint32_t jj = in ? t + (in1 ? c1v : c2v) : SB_ZJ;
+        const uint32_t lo = S.lo2[jj];
+        const int lx = (int)(int16_t)(lo & 0xFFFFu), ly = (int)(int16_t)(lo >> 16);
+        const float gx[8] = {a.x, a.y, a.z, a.w, c.x, c.y, c.z, c.w};  // columns 8 Q + ((p + 4 swz) & 7)
+        const int RR = fp.R * fp.R, R1 = fp.R - 1;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int v = 2 * (16 * B + 4 * hq + i - ly) - R1;
+          const int thr = RR - v * v;
+          float gm[8];
+#pragma unroll
+          for (int p = 0; p < 8; ++p) {
+            const int u = 2 * (8 * Q + ((p + 4 * swz) & 7) - lx) - R1;
+            gm[p] = u * u <= thr ? gx[p] : 0.f;
+          }
+          const float2 gg = make_float2(gi[i], gi[i]);
+          acc[i][0] = __ffma2_rn(gg, make_float2(gm[0], gm[1]), acc[i][0]);
+          acc[i][1] = __ffma2_rn(gg, make_float2(gm[2], gm[3]), acc[i][1]);
+          acc[i][2] = __ffma2_rn(gg, make_float2(gm[4], gm[5]), acc[i][2]);
+          acc[i][3] = __ffma2_rn(gg, make_float2(gm[6], gm[7]), acc[i][3]);
+        }
       }
     };
     uint32_t st = 0;
@@ -378,8 +409,10 @@ extern "C" int starsim_debug_sb_timing(double* out6, int reset) {
 #endif
 
 void init_tile_sb_kernel() {
-  cudaFuncSetAttribute(k_tile_sb<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SbSmem));
-  cudaFuncSetAttribute(k_tile_sb<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SbSmem));
+  cudaFuncSetAttribute(k_tile_sb<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SbSmem));
+  cudaFuncSetAttribute(k_tile_sb<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SbSmem));
+  cudaFuncSetAttribute(k_tile_sb<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SbSmem));
+  cudaFuncSetAttribute(k_tile_sb<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SbSmem));
 }
 
 void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
@@ -388,12 +421,9 @@ void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& 
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
   const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)SB_MINB * num_sms);  // persistent CTAs
-  if (fp.psf)
-    k_tile_sb<true><<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab,
-                                                                          part_buf, done, hdr);
-  else
-    k_tile_sb<false><<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab,
-                                                                           part_buf, done, hdr);
+  auto* k = fp.psf ? (fp.roi ? k_tile_sb<true, true> : k_tile_sb<true, false>)
+                   : (fp.roi ? k_tile_sb<false, true> : k_tile_sb<false, false>);
+  k<<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr);
 }
 
 }  // namespace starsim

@@ -564,8 +564,8 @@ def test_lut_einval(torch_dev, ctx):
 @pytest.mark.parametrize("W,H,n,R,sigma,kind", [(1024, 1024, 1000, 5, 1.0, "uniform"), (700, 530, 5000, 15, 2.5, "adv"),
                                                  (300, 200, 2000, 10, 1.7, "uniform"), (512, 384, 3000, 63, 10.5, "uniform")])
 def test_circle_roi_parity(torch_dev, ctx, W, H, n, R, sigma, kind):
-    """starsim_set_roi(CIRCLE): the atomic and lookup-table renders against the oracle's circle ROI; the tiled renders
-    refuse it (EINVAL) and work again once the square ROI is back."""
+    """starsim_set_roi(CIRCLE): the atomic and lookup-table renders against the oracle's circle ROI, the tiled render
+    too for R <= 17 (bands bitwise the frame), EINVAL above; the square ROI works again once it is back."""
     from paper_conf_ipps_lizzh12_b200 import StarsimError
     f = synth.adversarial_field(n, W, H, R, seed=43) if kind == "adv" else synth.uniform_field(n, W, H, seed=44,
                                                                                                   mag_hi=2.0)
@@ -577,8 +577,15 @@ def test_circle_roi_parity(torch_dev, ctx, W, H, n, R, sigma, kind):
         if R <= 63:
             ref_l = oracle.render_lut(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads(), roi="circle")
             assert_parity(ctx.render_lut(*args, W, H, sigma, R, 1.0).cpu().numpy(), ref_l, f"circle lut R={R}")
-        with pytest.raises(StarsimError):
-            ctx.render(*args, W, H, sigma, R, 1.0)
+        if R <= 17:  # the tiled path masks the circle in k_tile_sb's walk (any tile kernel setting)
+            img = ctx.render(*args, W, H, sigma, R, 1.0)
+            assert_parity(img.cpu().numpy(), ref, f"circle tiled R={R}")
+            bands = [ctx.render_band(*args, W, H, g * 64, min(64, H - g * 64), sigma, R, 1.0)
+                     for g in range(-(-H // 64))]
+            assert torch_dev[0].equal(torch_dev[0].cat(bands, 0), img)
+        else:
+            with pytest.raises(StarsimError):
+                ctx.render(*args, W, H, sigma, R, 1.0)
     finally:
         ctx.set_roi("square")
     ref_sq = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads())
