@@ -49,6 +49,7 @@ constexpr int SB_NSK = NSTRIPS + 1;
 constexpr int SB_NBIN = (NBANDS + 1) * SB_NSK;  // 85
 constexpr int SB_CHUNK = CHUNK;             // stars per chunk (<= TILE_THREADS; 192 with 4 CTAs/SM measured slower: spills)
 constexpr int SB_MINB = 3;                  // CTAs per SM (80 registers, 70 KB shared memory)
+constexpr int SB_MINB_CIRC = 2;             // the circle variant: 2 CTAs per SM, registers for its per-pixel mask
 constexpr uint32_t SB_ZJ = SB_CHUNK;        // the all-zero slot
 
 struct SbSmem {
@@ -64,7 +65,7 @@ struct SbSmem {
 // (2 (col - lo_x) - (R-1))^2 + (2 (row - lo_y) - (R-1))^2 <= R^2 per (row, column) of the lane's 4 x 8 block, with
 // the star's ROI origin read from its slot.  The profiles, slots and summation order are unchanged.
 template <bool INTEG, bool CIRC>
-__global__ void __launch_bounds__(TILE_THREADS, SB_MINB) k_tile_sb(const uint32_t* __restrict__ ids,
+__global__ void __launch_bounds__(TILE_THREADS, CIRC ? SB_MINB_CIRC : SB_MINB) k_tile_sb(const uint32_t* __restrict__ ids,
                                                              const StarRec* __restrict__ rec, FrameParams fp,
                                                              void* __restrict__ out_,
                                                              const WorkItem* __restrict__ items,
@@ -420,7 +421,8 @@ void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& 
                     cudaStream_t st) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
-  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)SB_MINB * num_sms);  // persistent CTAs
+  const int64_t grid =
+      std::min<int64_t>(ntiles + part_cap, (int64_t)(fp.roi ? SB_MINB_CIRC : SB_MINB) * num_sms);  // persistent CTAs
   auto* k = fp.psf ? (fp.roi ? k_tile_sb<true, true> : k_tile_sb<true, false>)
                    : (fp.roi ? k_tile_sb<false, true> : k_tile_sb<false, false>);
   k<<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr);
