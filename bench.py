@@ -353,6 +353,26 @@ def run_ours(args, world, rank, local_rank):
                         "peak_GBps": peaks.get("hbm_gbs"), "peak_source": peak_src}}
     kernels = {k: {"ms_per_step": v[0] / args.steps, "launches_per_step": v[1] / args.steps} for k, v in kt.items()
                if v[1]}
+    # the binning kernels' HBM view (north star: "achieved HBM GB/s for the binning ... passes"): algorithmic bytes per
+    # step over each kernel's live time.  a1 (k_dcount): 12 B catalogue in + 16 B record + 4 B tile box
+    # out per star + the count matrix; a2 column scan: the count matrix read and written; a3/a4 (k_dplace): 4 B tile
+    # box per star + 4 B id per pair + the count matrix column
+    if world == 1 and args.method == "tiled" and "sort" in kernels:
+        ntl = (-(-W // 128)) * (-(-H // 64))
+        try:
+            P_pairs = int(ctx.get_bins()[2][ntl])  # tile_off[ntiles] of the last render = the (tile, star) pairs
+        except Exception:  # noqa: BLE001
+            P_pairs = None
+        ncta = -(-lf.n // 4096)
+        cm = 4 * ntl * ncta
+        alg = {"prep": 32 * lf.n + cm, "csr": 2 * cm, "sort": 4 * lf.n + (4 * P_pairs if P_pairs else 0) + cm}
+        hbm_peak = peaks.get("hbm_gbs")
+        for k_, b_ in alg.items():
+            if k_ in kernels and kernels[k_]["ms_per_step"] > 0:
+                gbs = b_ / (kernels[k_]["ms_per_step"] * 1e-3) / 1e9
+                kernels[k_]["algorithmic_bytes"] = b_
+                kernels[k_]["achieved_GBps"] = gbs
+                kernels[k_]["frac_of_hbm_peak"] = gbs / hbm_peak if hbm_peak else None
 
     # NEXT-1 variant (1 GPU, tiled): the same frame with the output stage fused -- u8 gray image written by k_tile
     variants = {}
