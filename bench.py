@@ -46,7 +46,7 @@ def parse():
                     help="N > 1: weak = a W x (H N) frame with N n stars, one H-row band per rank (default); strong = "
                          "the --config frame itself split into N bands (the north star's C5 target: --config C5)")
     ap.add_argument("--method", default="tiled", choices=["tiled", "atomic"])
-    ap.add_argument("--tile-kernel", default="auto", choices=["auto", "lists", "sb", "ws"],
+    ap.add_argument("--tile-kernel", default="auto", choices=["auto", "lists", "sb", "ws", "t8"],
                     help="starsim_set_tile_kernel mode (A/B comparisons; the default is the product path)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")

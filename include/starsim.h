@@ -154,6 +154,7 @@ int starsim_set_binning(starsim_ctx* ctx, int32_t mode);
 #define STARSIM_TILE_LISTS 1
 #define STARSIM_TILE_SB 2
 #define STARSIM_TILE_WS 3
+#define STARSIM_TILE_T8 4
 int starsim_set_tile_kernel(starsim_ctx* ctx, int32_t mode);
 
 /* The paper's own design, kept as the measured comparison (Fig. 6): zero the image, then one

@@ -55,7 +55,7 @@ struct starsim_ctx {
   int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto, 1 lists, 2 sorted bins, 3 warp-specialised sorted bins
   int32_t bin_impl = 0;   // starsim_set_binning: 0 auto (dbin.cu when it applies), 1 always bin.cu's pipeline
   std::string err;
-  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat, codes;
+  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat, codes, segs, srec, sbin, sext;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
@@ -262,10 +262,24 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
     timed(c, 1, st, [&] { launch_sortlists(ids, (uint32_t*)c->tmp.p, tile_off, ntiles, n, st); });
     if ((rc = check_launch(c, "k_sortlists"))) return rc;
   }
-  timed(c, 3, st, [&] {
-    launch_tile(ids, rec, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p, part_cap, done,
-                hdr, c->num_sms, st);
-  });
+  if (fp.tile_impl == STARSIM_TILE_T8 && fp.R <= SB_MAXR) {
+    // k_t8sort: every tile list segment sorted by ROI corner bin, records written in that order (tile8.cu)
+    timed(c, 1, st, [&] {
+      launch_t8sort(ids, rec, fp, (WorkItem*)c->items.p, part_cap, hdr, (StarRec*)c->srec.p, (uint32_t*)c->sbin.p,
+                    (uint32_t*)c->sext.p, st);
+    });
+    if ((rc = check_launch(c, "k_t8sort"))) return rc;
+    timed(c, 3, st, [&] {
+      launch_tile8((StarRec*)c->srec.p, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p,
+                   part_cap, done, (float*)c->segs.p, hdr, (const uint32_t*)c->sbin.p, (const uint32_t*)c->sext.p,
+                   c->num_sms, st);
+    });
+  } else {
+    timed(c, 3, st, [&] {
+      launch_tile(ids, rec, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p, part_cap,
+                  done, hdr, c->num_sms, st);
+    });
+  }
   if ((rc = check_launch(c, "k_tile"))) return rc;
   return STARSIM_OK;
 }
@@ -286,7 +300,8 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   if (fp.tile_impl == STARSIM_TILE_AUTO) {
     // the warp-specialised kernel wins on dense frames (its per-item pipeline latency and static item order cost
     // more than they save on sparse, clustered and integrated-PSF frames: DESIGN.md §9): expected list length per
-    // tile for a uniform field, n (128 + R - 1)(64 + R - 1) / (W rows)
+    // tile for a uniform field, n (128 + R - 1)(64 + R - 1) / (W rows).  k_tile8 (STARSIM_TILE_T8) is faster in the
+    // tile kernel but needs the k_t8sort pass: a slower frame at T, so it is opt-in.
     const double per_tile = (double)n * (TILE_W + R - 1) * (TILE_H + R - 1) / ((double)W * (rows > 0 ? rows : 1));
     fp.tile_impl = (c->psf == 0 && per_tile >= WS_MIN_PER_TILE) ? STARSIM_TILE_WS : STARSIM_TILE_SB;
   }
@@ -321,6 +336,11 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   if ((rc = grow(c, c->partial, sizeof(uint3) * (size_t)((ntiles + SCAN_TILES - 1) / SCAN_TILES), "scan partials")))
     return rc;
   if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
+  if ((rc = grow(c, c->segs, sizeof(float) * tile8_scratch_floats(c->num_sms), "segment scratch"))) return rc;
+  if ((rc = grow(c, c->srec, sizeof(StarRec) * (size_t)(pmax > 0 ? pmax : 1), "bin-sorted records"))) return rc;
+  if ((rc = grow(c, c->sbin, sizeof(uint32_t) * tile8_sbin_words(ntiles, part_cap, pmax), "segment bin starts")))
+    return rc;
+  if ((rc = grow(c, c->sext, sizeof(uint32_t) * (size_t)(ntiles + part_cap), "segment rows"))) return rc;
   if (dbin_ok(fp, ntiles) &&
       (rc = grow(c, c->cmat, sizeof(uint32_t) * (size_t)ntiles * (size_t)(dbin_ctas(n) > 0 ? dbin_ctas(n) : 1),
                  "count matrix")))
@@ -414,7 +434,7 @@ void starsim_destroy(starsim_ctx* c) {
     cudaDeviceSynchronize();
     if (c->have_graph) cudaGraphExecDestroy(c->gexec);
     Buf* bufs[] = {&c->rec, &c->slots, &c->ids, &c->tmp, &c->tile_off, &c->items, &c->split_tab, &c->parts,
-                   &c->partial, &c->zeroed, &c->stage, &c->cmat, &c->codes};
+                   &c->partial, &c->zeroed, &c->stage, &c->cmat, &c->codes, &c->segs, &c->srec, &c->sbin, &c->sext};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {
@@ -499,8 +519,9 @@ int starsim_set_binning(starsim_ctx* c, int32_t mode) {
 
 int starsim_set_tile_kernel(starsim_ctx* c, int32_t mode) {
   if (!c) return STARSIM_EINVAL;
-  if (mode != STARSIM_TILE_AUTO && mode != STARSIM_TILE_LISTS && mode != STARSIM_TILE_SB && mode != STARSIM_TILE_WS)
-    return fail(c, STARSIM_EINVAL, "tile kernel mode must be STARSIM_TILE_AUTO, _LISTS, _SB or _WS");
+  if (mode != STARSIM_TILE_AUTO && mode != STARSIM_TILE_LISTS && mode != STARSIM_TILE_SB && mode != STARSIM_TILE_WS &&
+      mode != STARSIM_TILE_T8)
+    return fail(c, STARSIM_EINVAL, "tile kernel mode must be STARSIM_TILE_AUTO, _LISTS, _SB, _WS or _T8");
   c->tile_impl = mode;
   c->err.clear();
   return STARSIM_OK;

@@ -120,6 +120,7 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_b(const uint32_t* __restr
     hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
     hdr->nsplit = nsplit;
     hdr->next_item = 0u;
+    hdr->next_seg = 0u;
   }
   const int64_t t0 = (int64_t)blockIdx.x * SCAN_TILES + (int64_t)tid * SCAN_PER;
   uint32_t c[SCAN_PER];
@@ -168,6 +169,7 @@ __global__ void __launch_bounds__(SCAN1_THREADS) k_scan_one(const uint32_t* __re
     hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
     hdr->nsplit = nsplit;
     hdr->next_item = 0u;
+    hdr->next_seg = 0u;
   }
   uint32_t run = pre.x + incl.x - sum.x, pb = pre.y + incl.y - sum.y, si = pre.z + incl.z - sum.z;
 #pragma unroll
@@ -493,6 +495,7 @@ void init_kernels() {
   init_tile_kernel();
   init_tile_sb_kernel();
   init_tile_ws_kernel();
+  init_tile8_kernel();
   init_dbin_kernels();
 }
 

@@ -50,7 +50,8 @@ struct Header {
   uint32_t nitems;                     // k_tile work items (written by k_scan)
   uint32_t nsplit;                     // tiles split into several items
   uint32_t next_item;                  // k_tile_sb: the next work item a persistent CTA takes (k_scan zeroes it)
-  uint32_t pad[28];
+  uint32_t next_seg;                   // k_t8sort: extra-segment slots of its bin-start table taken (zeroed likewise)
+  uint32_t pad[27];
 };
 
 // k_tile work item: stars [jb, je) of tile `tile`'s list; aux = ITEM_WHOLE, or (split index << 12 | part index) for

@@ -210,6 +210,7 @@ __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restr
     hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
     hdr->nsplit = nsplit;
     hdr->next_item = 0u;
+    hdr->next_seg = 0u;
   }
 #pragma unroll
   for (int k = 0; k < TPT; ++k) {

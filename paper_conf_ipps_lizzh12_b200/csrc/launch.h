@@ -11,6 +11,8 @@ void init_kernels();
 void init_tile_kernel();
 void init_tile_sb_kernel();
 void init_tile_ws_kernel();
+void init_tile8_kernel();
+size_t tile8_scratch_floats(int num_sms);
 void init_dbin_kernels();
 size_t dbin_smem(int ntiles);
 int dbin_ctas(int64_t n);
@@ -38,6 +40,12 @@ void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& 
 void launch_tile_ws(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
                     cudaStream_t st);
+size_t tile8_sbin_words(int64_t ntiles, int part_cap, int64_t pairs);
+void launch_t8sort(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, const WorkItem* items,
+                   int part_cap, Header* hdr, StarRec* srec, uint32_t* sbin, uint32_t* sext, cudaStream_t st);
+void launch_tile8(const StarRec* srec, const FrameParams& fp, void* out, const WorkItem* items,
+                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, float* seg_scratch,
+                  Header* hdr, const uint32_t* sbin, const uint32_t* sext, int num_sms, cudaStream_t st);
 void launch_atomic(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, float* out,
                    cudaStream_t st);
 void launch_lut(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, float* out,

@@ -36,9 +36,10 @@ __device__ __forceinline__ void plan_tile(uint32_t t, uint32_t c, uint32_t& run,
   if (np) {
     split_tab[si] = make_uint2(pb, np);
     done[si] = 0u;  // the parts' completion counter (k_tile)
-    const uint32_t per_part = (c + np - 1) / np;
+    // parts start at multiples of SPLIT_LEN from the list start: the same boundaries at which a tile kernel that
+    // processes the whole (unsplit) list cuts it into segments, so split and unsplit give the same sums
     for (uint32_t j = 0; j < np; ++j)
-      items[pb + j] = WorkItem{t, run + j * per_part, min(run + c, run + (j + 1) * per_part), (si << 12) | j};
+      items[pb + j] = WorkItem{t, run + j * SPLIT_LEN, min(run + c, run + (j + 1) * SPLIT_LEN), (si << 12) | j};
     pb += np;
     ++si;
   } else {

@@ -173,7 +173,7 @@ def starsim_set_binning(h, mode) -> None:
     _check(h, lib().starsim_set_binning(h, BINNINGS.get(mode, mode) if isinstance(mode, str) else int(mode)))
 
 
-TILE_KERNELS = {"auto": 0, "lists": 1, "sb": 2, "ws": 3}
+TILE_KERNELS = {"auto": 0, "lists": 1, "sb": 2, "ws": 3, "t8": 4}
 
 
 def starsim_set_tile_kernel(h, mode) -> None:

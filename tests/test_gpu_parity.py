@@ -29,9 +29,10 @@ def torch_dev():
     return torch, torch.device("cuda:0")
 
 
-@pytest.fixture(scope="module", params=["ws", "lists", "sb"])
+@pytest.fixture(scope="module", params=["t8", "ws", "lists", "sb"])
 def ctx(torch_dev, request):
-    """Every test runs against the three tile kernels: "ws" (the warp-specialised sorted-corner-bin kernel for
+    """Every test runs against the four tile kernels: "t8" (the 8 x 8 lane-block kernel, the default for R <= 17),
+    "ws" (the warp-specialised sorted-corner-bin kernel for
     R <= 17, the list kernel above), "lists" (the per-block entry-list kernel for every R) and "sb" (the sorted-bin
     kernel with both roles in every warp; "auto" picks ws or sb by the expected list length, same images)."""
     from paper_conf_ipps_lizzh12_b200 import Context
