@@ -277,7 +277,7 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
   } else {
     timed(c, 3, st, [&] {
       launch_tile(ids, rec, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p, part_cap,
-                  done, hdr, c->num_sms, st);
+                  done, hdr, c->num_sms, st, (float*)c->segs.p);
     });
   }
   if ((rc = check_launch(c, "k_tile"))) return rc;

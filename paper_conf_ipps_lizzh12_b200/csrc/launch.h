@@ -33,13 +33,13 @@ void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, in
                       cudaStream_t st);
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                 cudaStream_t st);
+                 cudaStream_t st, float* seg_scratch);
 void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                    cudaStream_t st);
+                    cudaStream_t st, float* seg_scratch);
 void launch_tile_ws(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                    cudaStream_t st);
+                    cudaStream_t st, float* seg_scratch);
 size_t tile8_sbin_words(int64_t ntiles, int part_cap, int64_t pairs);
 void launch_t8sort(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, const WorkItem* items,
                    int part_cap, Header* hdr, StarRec* srec, uint32_t* sbin, uint32_t* sext, cudaStream_t st);

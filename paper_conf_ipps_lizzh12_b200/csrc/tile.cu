@@ -61,7 +61,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
                                                           void* __restrict__ out_, const WorkItem* __restrict__ items,
                                                           const uint2* __restrict__ split_tab,
                                                           float* __restrict__ part_buf, uint32_t* __restrict__ done,
-                                                          Header* hdr) {
+                                                          Header* hdr, float* __restrict__ seg_scratch) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   TileSmem& S = *reinterpret_cast<TileSmem*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -80,9 +80,10 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
   __shared__ int s_last;
   if (tid < 8) S.gx[ZERO_GX * 8 + tid] = 0.f;
 
-  for (int once = 0; once < 1; ++once) {
-  if (blockIdx.x >= __ldcg(&hdr->nitems)) return;
-  const WorkItem wi = items[blockIdx.x];
+  // persistent CTAs: item blockIdx.x first, then items from the counter the planner zeroed
+  const uint32_t nitems = __ldcg(&hdr->nitems);
+  for (uint32_t item = blockIdx.x; item < nitems;) {
+  const WorkItem wi = items[item];
   const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
   const int X0 = tx * TILE_W;    // first column of the tile
   const int Y0 = ty * TILE_H;    // first row of the tile, relative to the band
@@ -95,13 +96,16 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
     for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
 
   const uint32_t j1 = wi.je;
+  uint32_t segs_done = 0;  // SPLIT_LEN segments of this item already in the scratch (tile_common.cuh)
   // this thread's star record of the current chunk, loaded one chunk ahead (its latency hides behind the
   // accumulation of the previous chunk)
   StarRec rnext = {};
   if (wi.jb + tid < j1) rnext = rec[ids[wi.jb + tid]];
   for (uint32_t base = wi.jb; base < j1;) {
     // ======================= prep: thread = star (base + tid)
-    const int nvalid = (int)min((uint32_t)CHUNK, j1 - base);
+    // chunks never cross a SPLIT_LEN segment boundary of the list (segments are summed like the parts of a split tile)
+    const uint32_t seg_end = min(j1, wi.jb + ((base - wi.jb) / SPLIT_LEN + 1u) * SPLIT_LEN);
+    const int nvalid = (int)min((uint32_t)CHUNK, seg_end - base);
     const bool valid = tid < nvalid;
     const StarRec r = rnext;
     int c0 = 0, c1 = -1, r0 = 0, r1 = -1;
@@ -330,11 +334,21 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
       }
     }
     base += (uint32_t)ns;
+    if (base < j1 && (base - wi.jb) % SPLIT_LEN == 0) {
+      seg_flush(acc, seg_scratch, segs_done == 0);
+      ++segs_done;
+    }
   }
+  if (segs_done) seg_finish(acc, seg_scratch);
 
   // ======================= output: rows 16 B + hq + 4 i, columns 64 wx + 8 q .. +7 of the tile
-  if (!tile_reduce_parts<false>(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last)) continue;
-  tile_store<false>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+  if (tile_reduce_parts<false>(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last))
+    tile_store<false>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+  __shared__ uint32_t s_next;
+  __syncthreads();  // every thread is past this item's shared-memory reads
+  if (tid == 0) s_next = atomicAdd(&hdr->next_item, 1u) + gridDim.x;
+  __syncthreads();
+  item = s_next;
   }  // work loop
 }
 
@@ -345,25 +359,24 @@ void init_tile_kernel() {
 
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                 cudaStream_t st) {
+                 cudaStream_t st, float* seg_scratch) {
   if (fp.R <= SB_MAXR && fp.tile_impl == 3) {
-    launch_tile_ws(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st);
+    launch_tile_ws(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st, seg_scratch);
     return;
   }
   if (fp.R <= SB_MAXR && fp.tile_impl == 2) {
-    launch_tile_sb(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st);
+    launch_tile_sb(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st, seg_scratch);
     return;
   }
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
-  const int64_t maxitems = ntiles + part_cap;
-  const int64_t grid = maxitems;  // one CTA per possible item (parts first); CTAs past the item count exit at once
+  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)3 * num_sms);  // persistent, 3 CTAs per SM
   if (fp.psf)
     k_tile<true><<<(unsigned)grid, TILE_THREADS, sizeof(TileSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf,
-                                                                         done, hdr);
+                                                                         done, hdr, seg_scratch);
   else
     k_tile<false><<<(unsigned)grid, TILE_THREADS, sizeof(TileSmem), st>>>(ids, rec, fp, out, items, split_tab,
-                                                                          part_buf, done, hdr);
+                                                                          part_buf, done, hdr, seg_scratch);
 }
 
 }  // namespace starsim

@@ -892,7 +892,7 @@ extern "C" int starsim_debug_t8_timing(double* out16, int reset) {
 }
 #endif
 
-size_t tile8_scratch_floats(int num_sms) { return (size_t)2 * num_sms * TILE_W * TILE_H; }
+size_t tile8_scratch_floats(int num_sms) { return (size_t)4 * num_sms * TILE_W * TILE_H; }  // a slot per CTA
 
 void init_tile8_kernel() {
   cudaFuncSetAttribute(k_tile8<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)T8_SMEM_LAUNCH);

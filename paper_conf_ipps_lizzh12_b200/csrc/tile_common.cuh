@@ -66,6 +66,46 @@ __device__ __forceinline__ bool tile_reduce_parts(float2 (&acc)[4][4], const Wor
   return true;
 }
 
+// Segments (reading R19): a work item longer than SPLIT_LEN -- a heavy tile left whole because the part pool would
+// overflow -- is summed exactly as its parts would be: the chunks of each SPLIT_LEN segment accumulate from zero, and
+// at the end of every segment but the last the partial sum is added to the thread's slot of the CTA's scratch tile
+// (the first segment writes it) and reset; the last segment adds the scratch in front, (((p0 + p1) + p2) + ...),
+// the order of tile_reduce_parts.  So split and unsplit heavy tiles give the same bits, and the rounding of each
+// sequential fp32 chain is that of <= SPLIT_LEN stars.  The scratch slot is thread-private ([k][tid] float4: the
+// thread reads back only what it wrote), no barrier.
+// (the accumulating threads are threads 0 .. TILE_THREADS - 1 of every kernel that uses this)
+__device__ __forceinline__ float4* seg_slot(float* seg_scratch, int k) {
+  return reinterpret_cast<float4*>(seg_scratch + (size_t)blockIdx.x * (TILE_W * TILE_H)) + k * TILE_THREADS +
+         threadIdx.x;
+}
+__device__ __forceinline__ void seg_flush(float2 (&acc)[4][4], float* seg_scratch, bool first) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int k = 0; k < 4; k += 2) {
+      float4* o = seg_slot(seg_scratch, 2 * i + k / 2);
+      float2 a = acc[i][k], b = acc[i][k + 1];
+      if (!first) {
+        const float4 u = __ldcg(o);
+        a = __fadd2_rn(make_float2(u.x, u.y), a);
+        b = __fadd2_rn(make_float2(u.z, u.w), b);
+      }
+      __stcg(o, make_float4(a.x, a.y, b.x, b.y));
+      acc[i][k] = make_float2(0.f, 0.f);
+      acc[i][k + 1] = make_float2(0.f, 0.f);
+    }
+}
+__device__ __forceinline__ void seg_finish(float2 (&acc)[4][4], float* seg_scratch) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int k = 0; k < 4; k += 2) {
+      const float4 u = __ldcg(seg_slot(seg_scratch, 2 * i + k / 2));
+      acc[i][k] = __fadd2_rn(make_float2(u.x, u.y), acc[i][k]);
+      acc[i][k + 1] = __fadd2_rn(make_float2(u.z, u.w), acc[i][k + 1]);
+    }
+}
+
 // Write the lane's 4 rows x 8 columns of the tile (rows Y0 + lane_row(B, hq, i) of the band, columns col0 .. col0+7):
 // fp32, or (fused output stage, NEXT-1) the gray value of each pixel exactly as k_quantize computes it from the same
 // fp32 sum, as u8 / u16.  Coalesced: the 8 lane groups of a warp store 8 adjacent 8-pixel runs of a row.

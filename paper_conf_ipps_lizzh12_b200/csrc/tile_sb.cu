@@ -71,7 +71,7 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? SB_MINB_CIRC : SB_MINB) k
                                                              const WorkItem* __restrict__ items,
                                                              const uint2* __restrict__ split_tab,
                                                              float* __restrict__ part_buf,
-                                                             uint32_t* __restrict__ done, Header* hdr) {
+                                                             uint32_t* __restrict__ done, Header* hdr, float* __restrict__ seg_scratch) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   SbSmem& S = *reinterpret_cast<SbSmem*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -122,6 +122,8 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? SB_MINB_CIRC : SB_MINB) k
     for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
 
   const uint32_t j1 = wi.je;
+  static_assert(SPLIT_LEN % SB_CHUNK == 0, "segments are whole chunks");
+  uint32_t segs_done = 0;  // SPLIT_LEN segments of this item already in the scratch (tile_common.cuh)
   for (uint32_t base = wi.jb; base < j1; base += SB_CHUNK) {
     // ======================= sort: thread = star (base + tid) of the tile's list
     const int nvalid = (int)min((uint32_t)SB_CHUNK, j1 - base);
@@ -363,9 +365,14 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? SB_MINB_CIRC : SB_MINB) k
       SB_ACC(5, 1);
     }
 #endif
+    if ((base + SB_CHUNK - wi.jb) % SPLIT_LEN == 0 && base + SB_CHUNK < j1) {
+      seg_flush(acc, seg_scratch, segs_done == 0);
+      ++segs_done;
+    }
   }
 
   // ======================= output
+  if (segs_done) seg_finish(acc, seg_scratch);
   if (swz) {
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
@@ -418,14 +425,15 @@ void init_tile_sb_kernel() {
 
 void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                    cudaStream_t st) {
+                    cudaStream_t st, float* seg_scratch) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
   const int64_t grid =
       std::min<int64_t>(ntiles + part_cap, (int64_t)(fp.roi ? SB_MINB_CIRC : SB_MINB) * num_sms);  // persistent CTAs
   auto* k = fp.psf ? (fp.roi ? k_tile_sb<true, true> : k_tile_sb<true, false>)
                    : (fp.roi ? k_tile_sb<false, true> : k_tile_sb<false, false>);
-  k<<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr);
+  k<<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr,
+                                                          seg_scratch);
 }
 
 }  // namespace starsim

@@ -55,7 +55,8 @@ constexpr int WS_THREADS = 32 * (WS_PGROUPS * WS_PROD + WS_CONS);
 constexpr int WS_UNROLL = WS_WALK_UNROLL;              // walk steps per loop iteration (pairs of even/odd)
 constexpr int WS_NSTAGE = WS_NSTAGE_OPT;              // depth of the chunk ring (chunk c in stage c mod WS_NSTAGE)
 constexpr uint32_t WS_ZJ = WS_CHUNK;                 // the all-zero slot of every stage
-constexpr uint32_t WS_LAST = 1u, WS_STOP = 2u;       // chunk flags
+constexpr uint32_t WS_LAST = 1u, WS_STOP = 2u, WS_SEGEND = 4u;  // chunk flags (SEGEND: a SPLIT_LEN segment ends)
+static_assert(SPLIT_LEN % WS_CHUNK == 0, "segments are whole chunks");
 constexpr int WS_RSTAGE = WS_RSTAGE_OPT;             // star records of a work item staged in shared memory
 constexpr int WS_RPT = WS_RSTAGE / WS_CHUNK;         // ... per producer thread
 
@@ -330,7 +331,7 @@ __device__ __forceinline__ void ws_producer(WsSmem& S, const uint32_t* __restric
       if (pt == 0) {
         T.tile = wi.tile;
         T.aux = wi.aux;
-        T.flags = last ? WS_LAST : 0u;
+        T.flags = last ? WS_LAST : (((k + 1) % (SPLIT_LEN / WS_CHUNK)) == 0 ? WS_SEGEND : 0u);
       }
       mbar_arrive(&S.full[s]);
 #ifdef STARSIM_WS_TIMING
@@ -363,7 +364,8 @@ __device__ __forceinline__ void ws_producer(WsSmem& S, const uint32_t* __restric
 
 __device__ __forceinline__ void ws_consumer(WsSmem& S, const FrameParams& fp, void* __restrict__ out_,
                                             const uint2* __restrict__ split_tab, float* __restrict__ part_buf,
-                                            uint32_t* __restrict__ done) {
+                                            uint32_t* __restrict__ done, float* __restrict__ seg_scratch) {
+  uint32_t segs_done = 0;  // SPLIT_LEN segments of the current item already in the scratch (tile_common.cuh)
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
   const int Q = 8 * wx + q;
@@ -434,8 +436,17 @@ __device__ __forceinline__ void ws_consumer(WsSmem& S, const FrameParams& fp, vo
     WS_ACC(6, q1 - q0);
     WS_ACC(7, q2 - q1);
     WS_ACC(9, 1);
+    if (flags & WS_SEGEND) {
+      seg_flush(acc, seg_scratch, segs_done == 0);
+      ++segs_done;
+      continue;
+    }
     if (!(flags & WS_LAST)) continue;
     // ---- the item's last chunk: write the tile (or this part of a split heavy tile)
+    if (segs_done) {
+      seg_finish(acc, seg_scratch);
+      segs_done = 0;
+    }
     if (swz) {
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
@@ -465,7 +476,7 @@ __global__ void __launch_bounds__(WS_THREADS, WS_CTAS) k_tile_ws(const uint32_t*
                                                            void* __restrict__ out_, const WorkItem* __restrict__ items,
                                                            const uint2* __restrict__ split_tab,
                                                            float* __restrict__ part_buf, uint32_t* __restrict__ done,
-                                                           Header* hdr) {
+                                                           Header* hdr, float* __restrict__ seg_scratch) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   WsSmem& S = *reinterpret_cast<WsSmem*>(smem_raw);
   const int tid = threadIdx.x;
@@ -483,7 +494,7 @@ __global__ void __launch_bounds__(WS_THREADS, WS_CTAS) k_tile_ws(const uint32_t*
   if (tid >= 32 * WS_CONS)
     ws_producer<INTEG>(S, ids, rec, fp, items, nitems);
   else
-    ws_consumer(S, fp, out_, split_tab, part_buf, done);
+    ws_consumer(S, fp, out_, split_tab, part_buf, done, seg_scratch);
 }
 
 #ifdef STARSIM_WS_TIMING
@@ -507,16 +518,16 @@ void init_tile_ws_kernel() {
 
 void launch_tile_ws(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                    cudaStream_t st) {
+                    cudaStream_t st, float* seg_scratch) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
   const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)WS_CTAS * num_sms);  // persistent CTAs
   if (fp.psf)
     k_tile_ws<true><<<(unsigned)grid, WS_THREADS, sizeof(WsSmem), st>>>(ids, rec, fp, out, items, split_tab,
-                                                                         part_buf, done, hdr);
+                                                                         part_buf, done, hdr, seg_scratch);
   else
     k_tile_ws<false><<<(unsigned)grid, WS_THREADS, sizeof(WsSmem), st>>>(ids, rec, fp, out, items, split_tab,
-                                                                          part_buf, done, hdr);
+                                                                          part_buf, done, hdr, seg_scratch);
 }
 
 }  // namespace starsim
