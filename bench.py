@@ -3,11 +3,14 @@
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config T] [--method tiled|atomic]
 
-A step is one frame: the whole hot path (per-star prep + binning + per-tile sort + CSR + tile accumulation) over one
-synthetic catalogue resident in HBM, written to a device-resident fp32 image.  N=1 renders the north-star frame T
-(4096x4096, 1M uniform stars, R=15, sigma=2.5).  Under torchrun (N>1) the job is weak-scaled: the frame is
-4096 wide and 4096*N tall with N*1M stars, every rank renders its own 4096-row band and the
-bands are assembled with one NCCL all-gather, included in the step.
+A step is one frame: the whole hot path (per-star prep + binning + CSR + tile accumulation) over one synthetic
+catalogue resident in HBM, written to a device-resident fp32 image.  N=1 renders the north-star frame T (4096x4096,
+1M uniform stars, R=15, sigma=2.5).  Under torchrun (N>1) the job is weak-scaled: the frame is 4096 wide and 4096*N
+tall with N*1M stars replicated on every rank; each step every rank routes the catalogue to its 4096-row band on the
+device (starsim_route_band), renders the band and the bands are assembled with one NCCL
+all-gather (STARSIM_EXCHANGE=fused: the peer-memory exchange fused into the tile epilogue), all inside the step.
+Every line also carries `strong_C5`: the C5 frame (16384^2, 10M stars) on 1 GPU and split over the N ranks (render,
+exchange and frame times, efficiencies, NCCL algbw/busbw, bitwise validation of the assembled frame).
 
 Timing: W untimed warm-up steps; the L2 (126 MB) is flushed by writing a 256 MiB buffer before every step (the frame's
 79 MB of inputs+image would otherwise stay L2-resident); each step is bracketed by CUDA events on the render stream;
@@ -50,6 +53,7 @@ def parse():
                     help="starsim_set_tile_kernel mode (A/B comparisons; the default is the product path)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-strong", action="store_true", help="skip the strong_C5 record (C5 frame split over N bands)")
     return ap.parse_args()
 
 
@@ -158,14 +162,30 @@ def units_of(f, W, H, R):
 
 
 # ------------------------------------------------------------------------------------------------ CPU baseline
-def cpu_baseline(cfg, f, W, H, budget_s=12.0):
-    """The fp64 oracle as it stands on all host cores, on a prefix of the catalogue sized for ~budget_s."""
-    import numpy as np
+def cpu_model():
+    """The host CPU model name (lscpu / /proc/cpuinfo) for the baseline's context."""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.lower().startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    try:
+        import subprocess
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.strip().lower().startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:  # noqa: BLE001
+        pass
+    return None
+
+
+def _oracle_rate(f, W, H, cfg, A, threads, budget_s):
+    """U/s of the fp64 oracle on a prefix of the catalogue sized for ~budget_s on `threads` threads."""
     import oracle
     import synth
-    threads = os.cpu_count() or 1
-    A = synth.bench_gain(cfg.sigma)
-    n_cal = max(1000, f.n // 200)
+    n_cal = max(1000, f.n // 500)
     t0 = time.perf_counter()
     oracle.render(f.x[:n_cal], f.y[:n_cal], f.mag[:n_cal], W, H, cfg.sigma, cfg.R, A, threads=threads)
     dt = time.perf_counter() - t0
@@ -173,12 +193,24 @@ def cpu_baseline(cfg, f, W, H, budget_s=12.0):
     t0 = time.perf_counter()
     oracle.render(f.x[:n_s], f.y[:n_s], f.mag[:n_s], W, H, cfg.sigma, cfg.R, A, threads=threads)
     dt = time.perf_counter() - t0
-    sub = synth.Field(f.x[:n_s], f.y[:n_s], f.mag[:n_s])
-    U, _ = units_of(sub, W, H, cfg.R)
-    return {"value": U / dt, "unit": UNIT, "cores": threads, "kind": "oracle",
+    U, _ = units_of(synth.Field(f.x[:n_s], f.y[:n_s], f.mag[:n_s]), W, H, cfg.R)
+    return U / dt, n_s, dt
+
+
+def cpu_baseline(cfg, f, W, H, budget_s=12.0):
+    """The fp64 oracle as it stands on all host cores, and on one core, each on a prefix of the catalogue sized for
+    ~budget_s."""
+    import synth
+    threads = os.cpu_count() or 1
+    A = synth.bench_gain(cfg.sigma)
+    v, n_s, dt = _oracle_rate(f, W, H, cfg, A, threads, budget_s)
+    v1, n1, dt1 = _oracle_rate(f, W, H, cfg, A, 1, budget_s * 0.75)
+    return {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle", "cpu_model": cpu_model(),
             "sample": f"first {n_s} of {f.n} stars of the same frame ({W}x{H}, R={cfg.R}), fp64 oracle, "
                       f"{threads} pthreads over row bands, {dt:.2f} s wall (includes zeroing the fp64 image)",
-            "seconds": dt}
+            "seconds": dt,
+            "single_thread": {"value": v1, "unit": UNIT, "cores": 1,
+                              "sample": f"first {n1} of {f.n} stars, 1 thread, {dt1:.2f} s wall"}}
 
 
 # ------------------------------------------------------------------------------------------------ reference arm
@@ -214,10 +246,99 @@ def run_reference(args, world, rank):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
             "config": {"workload": f"{cfg.name}: {W}x{H}, {cfg.n} uniform stars, R={cfg.R}, sigma={cfg.sigma:g}",
                        "sample_stars": n_s, "frames_per_s_equiv": value / max(1, units_of(f, W, H, cfg.R)[0])},
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "cpu_model": cpu_model(),
                              "sample": f"first {n_s} of {f.n} stars per step, fp64 oracle, {threads} pthreads"},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------------------------ strong scaling, C5
+def strong_c5(args, world, rank, ctx, stream, flush, dev):
+    """The north star's strong-scaling target on the C5 frame (16384 x 16384, 10M uniform stars, R=15), measured in
+    every run: t_1 = one GPU renders the whole frame (each rank does it alone, max over ranks); for N > 1 t_render =
+    route + render of the rank's band, t_exchange = the NCCL all-gather of the bands alone, t_frame = both (NCCL),
+    t_frame_fused = the fused peer-memory exchange when available; each timed like the headline (K steps, L2 flushed,
+    CUDA events on the render stream, max over ranks).  eff = t_1 / (N t).  The assembled frames are compared with the
+    single-GPU frame on the device, all rows (must be bitwise equal: tile-aligned bands)."""
+    import torch
+    import torch.distributed as dist
+    import synth
+    from paper_conf_ipps_lizzh12_b200 import dist as sdist
+    cfg = synth.CONFIGS["C5"]
+    f = cfg.field()
+    W, H, R, sigma = cfg.W, cfg.H, cfg.R, cfg.sigma
+    A = synth.bench_gain(sigma)
+    U, _ = units_of(f, W, H, R)
+    x, y, m = (torch.from_numpy(a).to(dev) for a in (f.x, f.y, f.mag))
+    K = max(3, min(args.steps, 10))
+
+    def t_of(fn):
+        for _ in range(2):
+            with torch.cuda.stream(stream):
+                fn()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+        for i in range(K):
+            with torch.cuda.stream(stream):
+                flush.fill_(float(i))
+                ev[i][0].record(stream)
+                fn()
+                ev[i][1].record(stream)
+        torch.cuda.synchronize()
+        t = torch.tensor([sum(a.elapsed_time(b) for a, b in ev) / K], device=dev, dtype=torch.float64)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    single = torch.empty((H, W), dtype=torch.float32, device=dev)
+    t1 = t_of(lambda: ctx.render(x, y, m, W, H, sigma, R, A, out=single, stream=stream))
+    rec = {"workload": f"C5: {W}x{H}, {f.n} uniform stars, R={R}, sigma={sigma:g}; N = {world} bands",
+           "n_gpus": world, "steps": K, "t_1gpu_ms": t1, "updates_per_frame": U,
+           "updates_per_s_1gpu": U / (t1 * 1e-3)}
+    if world == 1:
+        rec["note"] = "N = 1: the single-GPU frame time every N > 1 run divides by (eff = t_1 / (N t_N))"
+        del single
+        return rec
+    prow = sdist.padded_band_rows(H, world)
+    row0, rows = sdist.band_rows(H, world, rank)
+    band = torch.zeros((prow, W), dtype=torch.float32, device=dev)
+    full = torch.empty((world * prow, W), dtype=torch.float32, device=dev)
+
+    def render():
+        if rows > 0:
+            ctx.render_band_routed(x, y, m, W, H, row0, rows, sigma, R, A, out=band[:rows], stream=stream)
+
+    def gather():
+        dist.all_gather_into_tensor(full, band)
+
+    t_render = t_of(render)  # (allocates the routed-catalogue buffers the routing-only timing below reuses)
+    t_route = t_of(lambda: ctx.route_band(x, y, m, H, row0, max(rows, 1), R, out=ctx._route_buf, stream=stream))
+    t_x = t_of(gather)
+    t_frame = t_of(lambda: (render(), gather()))
+    ok = sdist.frames_agree(full[:H], single)
+    gbytes = 4 * W * prow * world  # the gathered frame (all_gather_into_tensor output)
+    algbw = gbytes / (t_x * 1e-3) / 1e9
+    rec.update({"t_route_ms": t_route, "t_render_ms": t_render, "t_exchange_ms": t_x, "t_frame_ms": t_frame,
+                "eff_render": t1 / (world * t_render), "eff_frame": t1 / (world * t_frame),
+                "exchange": {"op": "NCCL all_gather_into_tensor", "bytes": gbytes, "algbw_GBps": algbw,
+                             "busbw_GBps": algbw * (world - 1) / world},
+                "updates_per_s": U / (t_frame * 1e-3),
+                "assembled_equals_1gpu": ok, "validation": "every rank's assembled frame vs its own single-GPU frame, "
+                                                          "all pixels, bitwise (dist.frames_agree)"})
+    del full
+    if sdist.FusedFrame.available():
+        try:
+            ff = sdist.FusedFrame(H, W, dev)
+            t_fused = t_of(lambda: ff.render(ctx, x, y, m, sigma, R, A, stream=stream))
+            rec.update({"t_frame_fused_ms": t_fused, "eff_frame_fused": t1 / (world * t_fused),
+                        "fused_equals_1gpu": sdist.frames_agree(ff.frame, single)})
+            del ff
+        except Exception as e:  # noqa: BLE001
+            rec["fused_error"] = f"{type(e).__name__}: {e}"
+    del single, band
+    return rec
 
 
 # ------------------------------------------------------------------------------------------------ our arm
@@ -239,19 +360,17 @@ def run_ours(args, world, rank, local_rank):
     stream = torch.cuda.Stream(dev)
     prow = sdist.padded_band_rows(H, world)
     row0, rows = sdist.band_rows(H, world, rank)
-    # N > 1: each rank holds the stars whose ROI rows meet its band (the per-band catalogue query, done once on the
-    # host before the timed region; same tile lists as the whole catalogue, so the same image bit for bit)
-    lf = f if world == 1 else synth.Field(*(a[sdist.band_star_mask(f.y, row0, rows, R)] for a in (f.x, f.y, f.mag)))
-    x, y, m = (torch.from_numpy(a).to(dev) for a in (lf.x, lf.y, lf.mag))
+    # every rank holds the whole (replicated) catalogue; N > 1 routes it to the rank's band on the device inside every
+    # step (starsim_route_band + a device star count: Context.render_band_routed), so routing is timed with the render
+    x, y, m = (torch.from_numpy(a).to(dev) for a in (f.x, f.y, f.mag))
     band = torch.zeros((prow, W), dtype=torch.float32, device=dev)
     full = torch.empty((world * prow, W), dtype=torch.float32, device=dev) if world > 1 else None
     flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
 
-    # N > 1: the fused band exchange (tile epilogue stores into every rank's symmetric-memory frame over NVLink, then
-    # a device barrier) when available, else render_band + NCCL all-gather (STARSIM_EXCHANGE=allgather forces it)
+    # N > 1: routed band render + NCCL all-gather (default), or the fused band exchange (STARSIM_EXCHANGE=fused: the
+    # tile epilogue stores into every rank's symmetric-memory frame over NVLink between two device barriers)
     fused = None
-    if world > 1 and args.method == "tiled" and os.environ.get("STARSIM_EXCHANGE", "fused") == "fused" \
-            and sdist.FusedFrame.available():
+    if world > 1 and os.environ.get("STARSIM_EXCHANGE", "allgather") == "fused" and sdist.FusedFrame.available():
         try:
             fused = sdist.FusedFrame(H, W, dev)
         except Exception as e:  # noqa: BLE001 -- fall back to the all-gather, say so in the JSON line
@@ -261,13 +380,16 @@ def run_ours(args, world, rank, local_rank):
 
     def step(xx, yy, mm):
         with torch.cuda.stream(stream):
-            if args.method == "atomic":
-                ctx.render_atomic(xx, yy, mm, W, H, sigma, R, A, out=band[:H], stream=stream)
+            if world == 1:
+                if args.method == "atomic":
+                    ctx.render_atomic(xx, yy, mm, W, H, sigma, R, A, out=band[:H], stream=stream)
+                else:
+                    ctx.render_band(xx, yy, mm, W, H, 0, H, sigma, R, A, out=band[:H], stream=stream)
             elif fused is not None:
                 fused.render(ctx, xx, yy, mm, sigma, R, A, stream=stream)
             else:
-                ctx.render_band(xx, yy, mm, W, H, row0, rows, sigma, R, A, out=band[:rows], stream=stream)
-            if world > 1 and fused is None:
+                if rows > 0:
+                    ctx.render_band_routed(xx, yy, mm, W, H, row0, rows, sigma, R, A, out=band[:rows], stream=stream)
                 dist.all_gather_into_tensor(full, band)
 
     def barrier():
@@ -278,6 +400,9 @@ def run_ours(args, world, rank, local_rank):
     for _ in range(max(3, args.warmup)):
         step(x, y, m)
     barrier()
+    # stars this rank renders: the whole catalogue (N = 1) or its band's routed stars (the device count, read once here)
+    n_band = f.n if world == 1 else (int(ctx._route_buf[3].item()) if rows > 0 else 0)
+
     def timed_region(profile):
         ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
               for _ in range(args.steps)]
@@ -348,8 +473,8 @@ def run_ours(args, world, rank, local_rank):
                            "note": "what bounds the tile kernel: instruction issue (ncu --set full, "
                                    "profiles/ncu_tile_traffic.json; DESIGN.md section 9)"}
                           if ncu_tile.get("warp_instructions") else None),
-                "hbm": {"bytes": 4 * W * (rows if world > 1 else H) + 16 * lf.n,
-                        "achieved_GBps": (4 * W * (rows if world > 1 else H) + 16 * lf.n) / (tile_ms * 1e-3) / 1e9,
+                "hbm": {"bytes": 4 * W * (rows if world > 1 else H) + 16 * n_band,
+                        "achieved_GBps": (4 * W * (rows if world > 1 else H) + 16 * n_band) / (tile_ms * 1e-3) / 1e9,
                         "peak_GBps": peaks.get("hbm_gbs"), "peak_source": peak_src}}
     kernels = {k: {"ms_per_step": v[0] / args.steps, "launches_per_step": v[1] / args.steps} for k, v in kt.items()
                if v[1]}
@@ -363,9 +488,9 @@ def run_ours(args, world, rank, local_rank):
             P_pairs = int(ctx.get_bins()[2][ntl])  # tile_off[ntiles] of the last render = the (tile, star) pairs
         except Exception:  # noqa: BLE001
             P_pairs = None
-        ncta = -(-lf.n // 4096)
+        ncta = -(-f.n // 4096)
         cm = 4 * ntl * ncta
-        alg = {"prep": 32 * lf.n + cm, "csr": 2 * cm, "sort": 4 * lf.n + (4 * P_pairs if P_pairs else 0) + cm}
+        alg = {"prep": 32 * f.n + cm, "csr": 2 * cm, "sort": 4 * f.n + (4 * P_pairs if P_pairs else 0) + cm}
         hbm_peak = peaks.get("hbm_gbs")
         for k_, b_ in alg.items():
             if k_ in kernels and kernels[k_]["ms_per_step"] > 0:
@@ -490,7 +615,7 @@ def run_ours(args, world, rank, local_rank):
     # e2e: the same C-ABI call with host (pinned) catalogue in and image out, copies inside the timed region
     e2e = None
     if not args.no_e2e:
-        hx, hy, hm = (torch.from_numpy(a).pin_memory() for a in (lf.x, lf.y, lf.mag))
+        hx, hy, hm = (torch.from_numpy(a).pin_memory() for a in (f.x, f.y, f.mag))
         himg = torch.empty((rows if world > 1 else H, W), dtype=torch.float32).pin_memory()
         dx, dy, dm = (torch.empty_like(x) for _ in range(3))
 
@@ -522,9 +647,10 @@ def run_ours(args, world, rank, local_rank):
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
         e_ms = float(te.item())
         e2e = {"value": U_frame / (e_ms * 1e-3), "unit": UNIT, "ms_per_step": e_ms,
-               "h2d_bytes_per_step": int(3 * 4 * lf.n), "d2h_bytes_per_step": int(himg.numel() * 4),
+               "h2d_bytes_per_step": int(3 * 4 * f.n), "d2h_bytes_per_step": int(himg.numel() * 4),
                "note": "pinned host catalogue -> device, render, image -> pinned host, per step, one stream"
-                       + ("; per rank: its band's catalogue in, its band out (max over ranks)" if world > 1 else "")}
+                       + ("; per rank: the whole catalogue in (routed on the device), its band out (max over ranks)"
+                          if world > 1 else "")}
         if world == 1 and args.method == "tiled":
             # the same steps pipelined over two streams (one ctx, catalogue and image buffers each): step i+1's copy in
             # and render overlap step i's copy out (PCIe is full duplex); every step still moves its own catalogue in
@@ -599,6 +725,13 @@ def run_ours(args, world, rank, local_rank):
                 e2e["gray_u8"] = {"error": f"{type(e).__name__}: {e}"}
             ctxs[1].close()
 
+    strong = None
+    if not args.no_strong and args.method == "tiled":
+        try:
+            strong = strong_c5(args, world, rank, ctx, stream, flush, dev)
+        except Exception as e:  # noqa: BLE001 -- a diagnostic record; the headline stands without it
+            strong = {"error": f"{type(e).__name__}: {e}"}
+        torch.cuda.synchronize()
     if rank != 0:
         ctx.close()
         return
@@ -609,18 +742,18 @@ def run_ours(args, world, rank, local_rank):
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": args.scaling,
             "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": f"{cfg.name}: {W}x{H}, {cfg.n} uniform stars, R={R}, sigma={sigma:g}"
-                                   + (f"; {world} bands of {prow} rows + NCCL all-gather" if world > 1 else ""),
+                                   + (f"; {world} bands of {prow} rows, exchange {exchange}" if world > 1 else ""),
                        "W": W, "H": H, "stars": f.n, "R": R, "sigma": sigma, "gain": A, "method": args.method,
                        "frames_per_s": 1e3 / ms, "updates_per_frame": U_frame, "exps_per_frame": E_frame,
                        "parallelism": f"bands{world}" if world > 1 else "single", "exchange": exchange,
                        "catalogue": "whole frame" if world == 1 else
-                                    f"per rank: the stars whose ROI rows meet its band (rank 0: {lf.n} of {f.n}; "
-                                    "selected on the host before the timed region, dist.band_star_mask)",
+                                    f"replicated on every rank; each step routes it to the rank's band on the device "
+                                    f"(starsim_route_band, timed in the step; rank 0 renders {n_band} of {f.n})",
                        "l2": "flushed before every step (256 MiB write, untimed)"},
             "clocks": clocks, "gpu_launches": int(round(launches * args.steps)),
             "gpu_launches_per_step": launches, "kernels": kernels,
             "ms_per_step_direct_launch": sum(ms_prof_steps) / len(ms_prof_steps),
-            "roofline": roofline, "e2e": e2e, "variants": variants,
+            "roofline": roofline, "e2e": e2e, "variants": variants, "strong_C5": strong,
             "cpu_baseline": cpu}
     print(json.dumps(line), flush=True)
     ctx.close()
@@ -634,6 +767,10 @@ def main():
     if args.impl == "reference":
         run_reference(args, world, rank)
         return
+    if world > 1 and args.method == "atomic":
+        # the star-centric render has no band form: it would write the whole frame into a band buffer
+        print(json.dumps({"error": "--method atomic is single-GPU only (no band decomposition)"}), flush=True)
+        sys.exit(2)
     import __graft_entry__
     if rank == 0 or world == 1:
         __graft_entry__.build()

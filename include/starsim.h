@@ -57,8 +57,9 @@ void starsim_destroy(starsim_ctx* ctx);
  * (then a static description of the last create failure). */
 const char* starsim_last_error(const starsim_ctx* ctx);
 
-/* Render a full frame with the tiled path: per-star prep + binning of the (tile, star) pairs and a
- * stable hand-written radix sort on the tile key (CSR in star order), then one register-accumulating tile kernel,
+/* Render a full frame with the tiled path: per-star prep, binning of the (tile, star) pairs into
+ * per-tile lists in star order (a stable counting sort, or atomic slots + a per-tile sort: starsim_set_binning),
+ * then one register-accumulating tile kernel (starsim_set_tile_kernel),
  * free of atomics on the image, that writes every pixel once.  On a non-default stream the launches are captured
  * once into a CUDA graph and replayed while the arguments repeat (STARSIM_NO_GRAPH=1 disables this).
  *   x, y, mag  (device) float[n]: the star catalogue as SoA -- sub-pixel centre (image coordinates) and magnitude.
@@ -129,17 +130,6 @@ int starsim_set_psf(starsim_ctx* ctx, int32_t mode);
 #define STARSIM_ROI_CIRCLE 1
 int starsim_set_roi(starsim_ctx* ctx, int32_t shape);
 
-/* Tile-accumulation kernel of the tiled renders that follow on this ctx (render, render_band, render_gray).  Both
- * compute Eqs. 2-3 per tile in fp32 registers with the separable PSF and write every pixel once;
- * they differ in how a tile's star list is walked, hence in the (deterministic) per-pixel summation order:
- *   STARSIM_TILE_AUTO (default): for R <= 17, STARSIM_TILE_WS on dense frames (expected list length per 128 x 64
- *     tile n (127 + R)(63 + R) / (width rows) >= 100, point PSF), else STARSIM_TILE_SB; for R > 17 the list kernel;
- *   STARSIM_TILE_LISTS: always the per-block entry-list kernel (the comparison / any R);
- *   STARSIM_TILE_SB: for R <= 17 the sorted-corner-bin kernel with both roles in every warp, else the list kernel;
- *   STARSIM_TILE_WS: for R <= 17 the warp-specialised sorted-corner-bin kernel (producer warps sort and evaluate
- *     profiles into a ring of shared-memory stages while consumer warps accumulate), else the list
- *     kernel.  SB and WS sum every pixel in the same order: the same image bit for bit.
- * EINVAL: ctx NULL or an unknown mode. */
 /* Binning pipeline of the tiled renders that follow on this ctx.  Both produce the same CSR (each tile's list in
  * ascending star index, reading R18 of DESIGN.md), hence the same image bit for bit:
  *   STARSIM_BIN_AUTO (default): the deterministic counting sort (dbin.cu, no global atomics) when the frame or band
@@ -150,12 +140,48 @@ int starsim_set_roi(starsim_ctx* ctx, int32_t shape);
 #define STARSIM_BIN_ATOMIC 1
 int starsim_set_binning(starsim_ctx* ctx, int32_t mode);
 
+/* Tile-accumulation kernel of the tiled renders that follow on this ctx (render, render_band, render_band_to,
+ * render_gray).  All compute Eqs. 2-3 per 128 x 64 tile in fp32 registers with the separable PSF
+ * and write every pixel once; they differ in how a tile's star list is walked, hence in the (deterministic)
+ * per-pixel summation order:
+ *   STARSIM_TILE_AUTO (default): for R <= 17, STARSIM_TILE_WS on dense frames (expected list length per tile
+ *     n (127 + R)(63 + R) / (width rows) >= 100, point PSF), else STARSIM_TILE_SB; for R > 17 the list kernel;
+ *   STARSIM_TILE_LISTS: always the per-block entry-list kernel k_tile (the comparison / any R);
+ *   STARSIM_TILE_SB: for R <= 17 k_tile_sb, sorted corner bins with both roles in every warp, else k_tile;
+ *   STARSIM_TILE_WS: for R <= 17 k_tile_ws, the warp-specialised sorted-corner-bin kernel (producer warps sort and
+ *     evaluate profiles into a ring of shared-memory stages while consumer warps accumulate), else
+ *     k_tile.  SB and WS sum every pixel in the same order: the same image bit for bit;
+ *   STARSIM_TILE_T8: for R <= 17 k_t8sort (every list segment sorted by ROI corner bin into a record array) then
+ *     k_tile8 (8 x 8-pixel lane blocks, profile ring in shared memory, warp-specialised), else k_tile.
+ * Every kernel sums a tile list longer than 1024 stars in 1024-star segments, each segment's sum added in list order
+ * (reading R19), so a tile gives the same bits whether or not it was split across CTAs.
+ * EINVAL: ctx NULL or an unknown mode. */
 #define STARSIM_TILE_AUTO 0
 #define STARSIM_TILE_LISTS 1
 #define STARSIM_TILE_SB 2
 #define STARSIM_TILE_WS 3
 #define STARSIM_TILE_T8 4
 int starsim_set_tile_kernel(starsim_ctx* ctx, int32_t mode);
+
+/* Band routing: of the catalogue x, y, mag (device, float[n]), the stars whose
+ * ROI rows meet rows [row0, row0+rows) of a height-row frame -- first ROI row by reading R7 (the R rows nearest y,
+ * ties at k+1/2 upward), exactly the binning's decision; non-finite y never routed -- are written in catalogue order
+ * to x_out, y_out, mag_out (device, float[n] each, capacity n; must not alias the inputs), and their number to
+ * *n_out (device uint32).  Two kernels (count per 4096-star block, then place), no host synchronisation.  A band
+ * rendered from the routed catalogue is bitwise the band rendered from the whole catalogue.  Pair it with
+ * starsim_set_star_count(ctx, n_out) to render the routed catalogue without reading the count back.
+ * EINVAL: ctx NULL, n < 0 or >= 2^32, a NULL array with n > 0, n_out NULL, height outside [1, 32767], the band not
+ * inside the frame, roi outside [1, 255]. */
+int starsim_route_band(starsim_ctx* ctx, const float* x, const float* y, const float* mag, int64_t n, int32_t height,
+                       int32_t row0, int32_t rows, int32_t roi, float* x_out, float* y_out, float* mag_out,
+                       uint32_t* n_out, starsim_stream_t stream);
+
+/* Device-resident star count of the tiled renders that follow on this ctx (render, render_band, render_band_to,
+ * render_gray): with n_dev (device uint32) set, a render's `n` is the capacity of x, y, mag and the kernels take the
+ * first min(n, *n_dev) stars, reading *n_dev when they run (e.g. the n_out of starsim_route_band on the same
+ * stream).  NULL (the default) restores plain `n`.  render_atomic / render_lut return EINVAL while it is set.
+ * The pointer is kept, not copied: it must stay valid while set.  EINVAL: ctx NULL. */
+int starsim_set_star_count(starsim_ctx* ctx, const uint32_t* n_dev);
 
 /* The paper's own design, kept as the measured comparison (Fig. 6): zero the image, then one
  * warp per star adds g*mu into every ROI pixel with global fp32 reductions (red.global.add.f32).  Same arguments
@@ -204,12 +230,14 @@ int starsim_get_bins(starsim_ctx* ctx, int32_t* tile_w, int32_t* tile_h,
 /* Per-kernel device timing for roofline reporting.  When enabled, every launch of the library records CUDA events
  * on the launching stream around it; starsim_kernel_times() synchronises and returns, per kernel class, the summed
  * elapsed milliseconds and launch counts since the last reset.  Classes (index into the arrays):
- *   0 k_bin (prep + scan + emit + digit histograms), 1 k_radix passes, 2 k_offsets (CSR), 3 k_tile (accumulate),
- *   4 k_atomic, 5 memsets, 6 k_quantize, 7 k_split_aos.
+ *   0 "prep": per-star prep + tile counts (k_dcount, k_prep); 1 "sort": list placement / sorting (k_dplace,
+ *   k_sortlists, k_t8sort); 2 "csr": tile scans + scatter (k_dcolscan, k_scan*, k_scatter); 3 "tile": the tile
+ *   kernel (k_tile, k_tile_sb, k_tile_ws, k_tile8); 4 "atomic": the star-centric renders (k_atomic, k_lut);
+ *   5 memsets; 6 k_quantize; 7 k_split_aos; 8 "route": k_route_count + k_route_place.
  * While profiling is enabled, renders are launched directly (not through the captured CUDA graph) so that every
  * kernel can be bracketed; kernel durations are unaffected, only the launch gaps differ.
  * `ms` and `launches` must hold STARSIM_NUM_KCLASS entries.  enable != 0 turns recording on and resets. */
-#define STARSIM_NUM_KCLASS 8
+#define STARSIM_NUM_KCLASS 9
 int starsim_profile(starsim_ctx* ctx, int enable);
 int starsim_kernel_times(starsim_ctx* ctx, double* ms, int64_t* launches);
 

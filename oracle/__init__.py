@@ -70,6 +70,8 @@ def _load():
         lib.oracle_render_full.restype = None
         lib.oracle_bins.argtypes = [f32p, f32p, f32p, i64, i32, i32, i32, i32, i32, u32p, u32p, i64]
         lib.oracle_bins.restype = i64
+        lib.oracle_route_band.argtypes = [f32p, i64, i32, i32, i32, i64p]
+        lib.oracle_route_band.restype = i64
         lib.oracle_quantize.argtypes = [f64p, i64, i32, ctypes.c_void_p]
         lib.oracle_quantize.restype = None
         _lib = lib
@@ -220,6 +222,16 @@ def bins(x, y, mag, W: int, H: int, R: int, tile_w: int, tile_h: int):
     if P < 0:
         raise RuntimeError(f"oracle_bins failed ({P})")
     return off, ids[:P].copy()
+
+
+def route_band(y, R: int, row0: int, rows: int):
+    """Indices (int64, catalogue order) of the stars routed to rows [row0, row0+rows): ROI rows (reading R7) meet the
+    band, y finite -- the definition of starsim_route_band."""
+    ys = np.ascontiguousarray(y, dtype=np.float32)
+    idx = np.empty(max(1, ys.shape[0]), dtype=np.int64)
+    k = _load().oracle_route_band(ys.ctypes.data_as(ctypes.POINTER(ctypes.c_float)), ys.shape[0], int(R), int(row0),
+                                  int(rows), idx.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)))
+    return idx[:k].copy()
 
 
 def quantize(v, bits: int):

@@ -201,6 +201,21 @@ void oracle_render_full(const float* x, const float* y, const float* mag, int64_
         }
 }
 
+/* Band routing (the definition starsim_route_band computes): the indices, in catalogue order,
+ * of the stars whose ROI rows [ly, ly + R - 1] -- ly the first ROI row of reading R7 -- meet rows
+ * [row0, row0 + rows).  Only y decides; a non-finite y is never routed (reading R11).  Returns the count. */
+int64_t oracle_route_band(const float* y, int64_t n, int32_t R, int32_t row0, int32_t rows, int64_t* idx) {
+    int64_t k = 0;
+    for (int64_t i = 0; i < n; ++i) {
+        if (!isfinite(y[i])) continue;
+        /* far from the band: no ROI row can meet it (and keeps oracle_roi_lo exact) */
+        if ((double)y[i] < (double)row0 - R - 2.0 || (double)y[i] > (double)row0 + rows + R + 2.0) continue;
+        int64_t ly = oracle_roi_lo(y[i], R);
+        if (ly <= (int64_t)row0 + rows - 1 && ly + R - 1 >= (int64_t)row0) idx[k++] = i;
+    }
+    return k;
+}
+
 /* Binning definition (get_bins): image tiles of tw x th pixels, ntx = ceil(W/tw) per row,
  * key = ty*ntx + tx.  For each contributing star in index order, one pair per tile its clipped ROI overlaps, tiles in
  * row-major order; then a stable sort by key, i.e. star-index order inside each tile.  Output: CSR

@@ -24,8 +24,21 @@ def _inputs():
         os.path.join(ROOT, "include", "starsim.h"), os.path.abspath(__file__)]
 
 
+STAMP = LIB + ".flags"  # the extra nvcc flags the library was built with (a flag change forces a rebuild)
+
+
+def _extra() -> list[str]:
+    return os.environ.get("STARSIM_NVCC_EXTRA", "").split()  # e.g. -DT8_TIMING (debug builds only)
+
+
 def up_to_date() -> bool:
     if not os.path.exists(LIB):
+        return False
+    try:
+        with open(STAMP) as fh:
+            if fh.read() != " ".join(_extra()):
+                return False
+    except OSError:
         return False
     t = os.path.getmtime(LIB)
     return all(os.path.getmtime(p) <= t for p in _inputs())
@@ -35,7 +48,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and up_to_date():
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
-    extra = os.environ.get("STARSIM_NVCC_EXTRA", "").split()  # e.g. -DSTARSIM_SB_TIMING (debug builds only)
+    extra = _extra()
     cmd = [NVCC, *ARCH, *FLAGS, *extra, "-o", tmp, *sources(), "-lcudart"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     log = os.path.join(PKG, "build.log")
@@ -44,6 +57,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if r.returncode != 0:
         raise RuntimeError(f"nvcc failed (see {log}):\n{r.stderr[-4000:]}")
     os.replace(tmp, LIB)
+    with open(STAMP, "w") as fh:
+        fh.write(" ".join(extra))
     if verbose:
         print(r.stderr)
     return LIB

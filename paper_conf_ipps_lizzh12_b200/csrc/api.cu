@@ -33,6 +33,7 @@ struct Launch {
 // A captured render (CUDA graph) and the arguments it was captured with: replayed when a call repeats them.
 struct GraphKey {
   const void *x, *y, *mag, *out;
+  const uint32_t* n_dev;
   int64_t n;
   int32_t W, H, row0, rows, R, obits, psf, tile_impl, bin_impl, ndst;
   float* dst[MAX_DST];
@@ -40,7 +41,7 @@ struct GraphKey {
   cudaStream_t st;
   uint64_t scratch_gen;
   bool operator==(const GraphKey& o) const {
-    return x == o.x && y == o.y && mag == o.mag && out == o.out && n == o.n && W == o.W && H == o.H &&
+    return x == o.x && y == o.y && mag == o.mag && out == o.out && n_dev == o.n_dev && n == o.n && W == o.W && H == o.H &&
            row0 == o.row0 && rows == o.rows && R == o.R && obits == o.obits && psf == o.psf && tile_impl == o.tile_impl && bin_impl == o.bin_impl && ndst == o.ndst &&
            std::equal(dst, dst + MAX_DST, o.dst) && sigma == o.sigma && gain == o.gain && st == o.st &&
            scratch_gen == o.scratch_gen;
@@ -55,7 +56,9 @@ struct starsim_ctx {
   int32_t tile_impl = 0;  // starsim_set_tile_kernel: 0 auto, 1 lists, 2 sorted bins, 3 warp-specialised sorted bins
   int32_t bin_impl = 0;   // starsim_set_binning: 0 auto (dbin.cu when it applies), 1 always bin.cu's pipeline
   std::string err;
-  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat, codes, segs, srec, sbin, sext;
+  const uint32_t* n_dev = nullptr;  // starsim_set_star_count: device-resident star count of the tiled renders
+  Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat, codes, segs, srec, sbin, sext,
+      rblk;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
@@ -191,6 +194,7 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   fp.bin_impl = 0;
   fp.ndst = 0;
   for (int i = 0; i < MAX_DST; ++i) fp.dst[i] = nullptr;
+  fp.n_dev = nullptr;
   fp.obits = 0;
   fp.vec = 0;
   fp.kint = (float)(1.0 / (std::sqrt(2.0) * s));
@@ -226,7 +230,7 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
     if (n > 0) {
       timed(c, 0, st, [&] { launch_dcount(x, y, mag, n, fp, rec, (uint32_t*)c->codes.p, C, (int)ntiles, st); });
       if ((rc = check_launch(c, "k_dcount"))) return rc;
-      timed(c, 2, st, [&] { launch_dcolscan(C, n, (int)ntiles, cnt, 1, st); });  // dense totals for k_dplace
+      timed(c, 2, st, [&] { launch_dcolscan(C, n, (int)ntiles, cnt, 1, fp.n_dev, st); });  // dense totals for k_dplace
       if ((rc = check_launch(c, "k_dcolscan"))) return rc;
       timed(c, 1, st, [&] {
         launch_dplace((const uint32_t*)c->codes.p, n, fp, C, (int)ntiles, cnt, tile_off, hdr, (WorkItem*)c->items.p,
@@ -237,7 +241,7 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
       timed(
           c, 2, st,
           [&] {
-            launch_dcolscan(C, n, (int)ntiles, cnt, CNT_STRIDE, st);
+            launch_dcolscan(C, n, (int)ntiles, cnt, CNT_STRIDE, nullptr, st);
             launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap,
                         c->partial.p, done, st);
           },
@@ -306,6 +310,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
     fp.tile_impl = (c->psf == 0 && per_tile >= WS_MIN_PER_TILE) ? STARSIM_TILE_WS : STARSIM_TILE_SB;
   }
   fp.bin_impl = c->bin_impl;
+  fp.n_dev = c->n_dev;
   // one vector store per 8-pixel run: 32 B (fp32) / 8 B (u8) / 16 B (u16); rows must keep that alignment
   const int vb = obits == 8 ? 8 : 16;
   bool aligned = ((uintptr_t)out % vb) == 0;
@@ -337,10 +342,12 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
     return rc;
   if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
   if ((rc = grow(c, c->segs, sizeof(float) * tile8_scratch_floats(c->num_sms), "segment scratch"))) return rc;
-  if ((rc = grow(c, c->srec, sizeof(StarRec) * (size_t)(pmax > 0 ? pmax : 1), "bin-sorted records"))) return rc;
-  if ((rc = grow(c, c->sbin, sizeof(uint32_t) * tile8_sbin_words(ntiles, part_cap, pmax), "segment bin starts")))
-    return rc;
-  if ((rc = grow(c, c->sext, sizeof(uint32_t) * (size_t)(ntiles + part_cap), "segment rows"))) return rc;
+  if (fp.tile_impl == STARSIM_TILE_T8 && R <= SB_MAXR) {  // k_t8sort's outputs (the t8 kernel only)
+    if ((rc = grow(c, c->srec, sizeof(StarRec) * (size_t)(pmax > 0 ? pmax : 1), "bin-sorted records"))) return rc;
+    if ((rc = grow(c, c->sbin, sizeof(uint32_t) * tile8_sbin_words(ntiles, part_cap, pmax), "segment bin starts")))
+      return rc;
+    if ((rc = grow(c, c->sext, sizeof(uint32_t) * (size_t)(ntiles + part_cap), "segment rows"))) return rc;
+  }
   if (dbin_ok(fp, ntiles) &&
       (rc = grow(c, c->cmat, sizeof(uint32_t) * (size_t)ntiles * (size_t)(dbin_ctas(n) > 0 ? dbin_ctas(n) : 1),
                  "count matrix")))
@@ -348,7 +355,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   if (dbin_ok(fp, ntiles) && (rc = grow(c, c->codes, sizeof(uint32_t) * (size_t)(n > 0 ? n : 1), "tile boxes")))
     return rc;
 
-  GraphKey key{x, y, mag, out, n, W, H, row0, rows, R, obits, c->psf | c->roi << 1, c->tile_impl, c->bin_impl, fp.ndst, {}, sigma, gain, st,
+  GraphKey key{x, y, mag, out, fp.n_dev, n, W, H, row0, rows, R, obits, c->psf | c->roi << 1, c->tile_impl, c->bin_impl, fp.ndst, {}, sigma, gain, st,
                c->scratch_gen};
   for (int i = 0; i < MAX_DST; ++i) key.dst[i] = fp.dst[i];
   if (st == nullptr || c->prof || !c->use_graphs) {
@@ -434,7 +441,8 @@ void starsim_destroy(starsim_ctx* c) {
     cudaDeviceSynchronize();
     if (c->have_graph) cudaGraphExecDestroy(c->gexec);
     Buf* bufs[] = {&c->rec, &c->slots, &c->ids, &c->tmp, &c->tile_off, &c->items, &c->split_tab, &c->parts,
-                   &c->partial, &c->zeroed, &c->stage, &c->cmat, &c->codes, &c->segs, &c->srec, &c->sbin, &c->sext};
+                   &c->partial, &c->zeroed, &c->stage, &c->cmat, &c->codes, &c->segs, &c->srec, &c->sbin, &c->sext,
+                   &c->rblk};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {
@@ -517,6 +525,41 @@ int starsim_set_binning(starsim_ctx* c, int32_t mode) {
   return STARSIM_OK;
 }
 
+int starsim_set_star_count(starsim_ctx* c, const uint32_t* n_dev) {
+  if (!c) return STARSIM_EINVAL;
+  c->n_dev = n_dev;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
+int starsim_route_band(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t H,
+                       int32_t row0, int32_t rows, int32_t R, float* x_out, float* y_out, float* mag_out,
+                       uint32_t* n_out, starsim_stream_t stream) {
+  if (!c) return STARSIM_EINVAL;
+  if (n < 0) return fail(c, STARSIM_EINVAL, "n < 0");
+  if (n > 0xFFFFFFFFll) return fail(c, STARSIM_EINVAL, "n >= 2^32 (star indices are 32-bit)");
+  if (n > 0 && (!x || !y || !mag || !x_out || !y_out || !mag_out))
+    return fail(c, STARSIM_EINVAL, "n > 0 with a NULL input or output array");
+  if (!n_out) return fail(c, STARSIM_EINVAL, "n_out is NULL");
+  if (H < 1 || H > STARSIM_MAX_DIM) return fail(c, STARSIM_EINVAL, "height outside [1, 32767]");
+  if (row0 < 0 || rows < 1 || (int64_t)row0 + rows > H) return fail(c, STARSIM_EINVAL, "band not inside the image");
+  if (R < 1 || R > STARSIM_MAX_ROI) return fail(c, STARSIM_EINVAL, "roi outside [1, 255]");
+  DevGuard g(c->dev);
+  cudaStream_t st = (cudaStream_t)stream;
+  int rc;
+  if ((rc = grow(c, c->rblk, sizeof(uint32_t) * (route_blocks(n) > 0 ? route_blocks(n) : 1), "route blocks")))
+    return rc;
+  timed(
+      c, 8, st,
+      [&] {
+        launch_route(x, y, mag, n, row0, rows, R, (uint32_t*)c->rblk.p, x_out, y_out, mag_out, n_out, st);
+      },
+      n > 0 ? 2 : 1);
+  if ((rc = check_launch(c, "k_route"))) return rc;
+  c->err.clear();
+  return STARSIM_OK;
+}
+
 int starsim_set_tile_kernel(starsim_ctx* c, int32_t mode) {
   if (!c) return STARSIM_EINVAL;
   if (mode != STARSIM_TILE_AUTO && mode != STARSIM_TILE_LISTS && mode != STARSIM_TILE_SB && mode != STARSIM_TILE_WS &&
@@ -532,6 +575,7 @@ int starsim_render_atomic(starsim_ctx* c, const float* x, const float* y, const 
   if (!c) return STARSIM_EINVAL;
   int rc = validate_frame(c, x, y, mag, n, W, H, sigma, R, gain, out);
   if (rc) return rc;
+  if (c->n_dev) return fail(c, STARSIM_EINVAL, "a device star count (starsim_set_star_count) is set: tiled renders only");
   DevGuard g(c->dev);
   cudaStream_t st = (cudaStream_t)stream;
   FrameParams fp = make_params(W, H, 0, H, sigma, R, gain, c->psf);
@@ -549,6 +593,7 @@ int starsim_render_lut(starsim_ctx* c, const float* x, const float* y, const flo
   int rc = validate_frame(c, x, y, mag, n, W, H, sigma, R, gain, out);
   if (rc) return rc;
   if (R > STARSIM_MAX_LUT_ROI) return fail(c, STARSIM_EINVAL, "roi > 63 for the lookup-table kernel");
+  if (c->n_dev) return fail(c, STARSIM_EINVAL, "a device star count (starsim_set_star_count) is set: tiled renders only");
   DevGuard g(c->dev);
   cudaStream_t st = (cudaStream_t)stream;
   FrameParams fp = make_params(W, H, 0, H, sigma, R, gain, c->psf);

@@ -29,7 +29,7 @@ __global__ void __launch_bounds__(PREP_THREADS) k_prep(const float* __restrict__
                                                        StarRec* __restrict__ rec, uint32_t* __restrict__ cnt,
                                                        uint32_t* __restrict__ slots, int tps) {
   const int64_t i = (int64_t)blockIdx.x * PREP_THREADS + threadIdx.x;
-  if (i >= n) return;
+  if (i >= frame_n(n, fp)) return;
   int cx0, cx1, cy0, cy1;
   const StarRec r = prep_star(X[i], Y[i], M[i], fp, cx0, cx1, cy0, cy1);
   if (r.lo != LO_CULLED) {
@@ -188,7 +188,7 @@ __global__ void __launch_bounds__(PREP_THREADS) k_scatter(const StarRec* __restr
                                                           const uint32_t* __restrict__ tile_off,
                                                           uint32_t* __restrict__ ids) {
   const int64_t i = (int64_t)blockIdx.x * PREP_THREADS + threadIdx.x;
-  if (i >= n) return;
+  if (i >= frame_n(n, fp)) return;
   const uint32_t lo = rec[i].lo;
   if (lo == LO_CULLED) return;
   int cx0, cx1, cy0, cy1;

@@ -88,10 +88,19 @@ struct FrameParams {
   int32_t bin_impl;      // 0: dbin.cu's deterministic binning when it applies; 1: always bin.cu's atomic-slot pipeline
   int32_t ndst;          // > 0: the tile kernels store every pixel into dst[0..ndst) instead of `out` (fused band exchange)
   float* dst[MAX_DST];   // band origins (row0 of each destination frame) -- local and peer-mapped frames
+  const uint32_t* n_dev; // starsim_set_star_count: the star count in device memory (n is then the capacity), or NULL
   float sk;              // sqrt(log2(e) / (2 sigma^2)):  exp(-d^2/(2 sigma^2)) = ex2(-(d * sk)^2)
   float kint;            // 1 / (sqrt(2) sigma): the erf argument scale of the integrated PSF
   double s_scale;        // A / (2 pi sigma^2), applied in fp64 before rounding s' to fp32
 };
+
+// The number of catalogue entries a kernel takes: n, or the device-resident count of a routed catalogue
+// (starsim_route_band -> starsim_set_star_count), read when the kernel runs (no host round trip).
+__device__ __forceinline__ int64_t frame_n(int64_t n, const FrameParams& fp) {
+  if (!fp.n_dev) return n;
+  const int64_t d = (int64_t)*fp.n_dev;
+  return d < n ? d : n;
+}
 
 // Output stage: q = min(2^bits-1, floor(v + 1/2)), v <= 0 or NaN -> 0.  floor(v + 1/2) is taken
 // exactly as f + (v - f >= 1/2), f = floorf(v) (v - f is exact in fp32 for v >= 0); the rounded v + 0.5f would carry

@@ -33,6 +33,8 @@ constexpr int DP_KEYS = DB_CTA * 4;              // at most 2 x 2 tiles per star
 constexpr int DP_SPT = DB_CTA / DP_THREADS;      // stars per thread (strided by DP_THREADS)
 constexpr int DCS_THREADS = 256;
 constexpr int DCS_PER = 8;                       // k_dcolscan: consecutive CTA counts per lane
+// CTAs that hold stars (at least one: CTA 0 plans the tiles of an empty routed catalogue)
+__device__ __forceinline__ int dbin_live_ctas(int64_t n) { return n > 0 ? (int)((n + DB_CTA - 1) / DB_CTA) : 1; }
 static_assert(DB_MAXT <= 65536 && DB_CTA <= 65536, "tile ids, slots and star indices are 16-bit in k_dplace");
 static_assert(DP_WARPS <= 32, "dp_block_scan scans the warp sums with one warp");
 
@@ -47,6 +49,8 @@ __global__ void __launch_bounds__(DC_THREADS, 2) k_dcount(const float* __restric
                                                        int nCTA, int ntiles) {
   __shared__ uint32_t cnt[DB_MAXT];
   const int tid = threadIdx.x, cta = blockIdx.x;
+  n = frame_n(n, fp);
+  if (cta >= dbin_live_ctas(n)) return;  // beyond a routed catalogue's device count: k_dcolscan skips the column
   for (int t = tid; t < ntiles; t += DC_THREADS) cnt[t] = 0u;
   // all loads of the thread's stars first (one memory latency, not DC_PER)
   const int64_t i0 = (int64_t)cta * DB_CTA + tid;
@@ -81,12 +85,14 @@ __global__ void __launch_bounds__(DC_THREADS, 2) k_dcount(const float* __restric
   for (int t = tid; t < ntiles; t += DC_THREADS) C[(int64_t)t * nCTA + cta] = cnt[t];
 }
 
-__global__ void __launch_bounds__(DCS_THREADS) k_dcolscan(uint32_t* __restrict__ C, int nCTA, int ntiles,
-                                                         uint32_t* __restrict__ cnt, int cstride) {
+__global__ void __launch_bounds__(DCS_THREADS) k_dcolscan(uint32_t* __restrict__ C, int cstrideC, int ntiles,
+                                                         uint32_t* __restrict__ cnt, int cstride, int64_t n,
+                                                         const uint32_t* __restrict__ n_dev) {
   const int lane = threadIdx.x & 31;
   const int t = blockIdx.x * (DCS_THREADS / 32) + (threadIdx.x >> 5);
   if (t >= ntiles) return;
-  uint32_t* row = C + (int64_t)t * nCTA;
+  uint32_t* row = C + (int64_t)t * cstrideC;  // row stride: the CTAs of the capacity n
+  const int nCTA = (n_dev && n > 0) ? dbin_live_ctas(n < (int64_t)*n_dev ? n : (int64_t)*n_dev) : cstrideC;
   // lane l takes the DCS_PER consecutive CTAs [DCS_PER l, DCS_PER (l + 1)): all loads first, one warp scan
   uint32_t run = 0;
   for (int b0 = 0; b0 < nCTA; b0 += 32 * DCS_PER) {
@@ -240,7 +246,10 @@ __global__ void __launch_bounds__(DP_THREADS, DP_MINB) k_dplace(const uint32_t* 
   DpSmem& S = *reinterpret_cast<DpSmem*>(dsm_raw);
   const int tid = threadIdx.x, cta = blockIdx.x;
   const int64_t c0 = (int64_t)cta * DB_CTA;
-  dp_scan_tiles(S, cnt, ntiles, nCTA, tile_off, hdr, items, split_tab, part_cap, done);
+  n = frame_n(n, fp);
+  const int live = dbin_live_ctas(n);
+  if (cta >= live) return;
+  dp_scan_tiles(S, cnt, ntiles, live, tile_off, hdr, items, split_tab, part_cap, done);
   for (int t = tid; t <= ntiles; t += DP_THREADS) S.gstart[t] = 0u;
   uint32_t code[DP_SPT];
 #pragma unroll
@@ -320,9 +329,10 @@ void launch_dcount(const float* x, const float* y, const float* m, int64_t n, co
   if (nc > 0) k_dcount<<<nc, DC_THREADS, 0, st>>>(x, y, m, n, fp, rec, codes, C, nc, ntiles);
 }
 
-void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstride, cudaStream_t st) {
+void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstride, const uint32_t* n_dev,
+                     cudaStream_t st) {
   constexpr int wpb = DCS_THREADS / 32;
-  k_dcolscan<<<(ntiles + wpb - 1) / wpb, DCS_THREADS, 0, st>>>(C, dbin_ctas(n), ntiles, cnt, cstride);
+  k_dcolscan<<<(ntiles + wpb - 1) / wpb, DCS_THREADS, 0, st>>>(C, dbin_ctas(n), ntiles, cnt, cstride, n, n_dev);
 }
 
 void launch_dplace(const uint32_t* codes, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,

@@ -18,7 +18,8 @@ size_t dbin_smem(int ntiles);
 int dbin_ctas(int64_t n);
 void launch_dcount(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
                    uint32_t* codes, uint32_t* C, int ntiles, cudaStream_t st);
-void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstride, cudaStream_t st);
+void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstride, const uint32_t* n_dev,
+                     cudaStream_t st);
 void launch_dplace(const uint32_t* codes, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,
                    const uint32_t* cnt, uint32_t* tile_off, Header* hdr, WorkItem* items, uint2* split_tab,
                    int part_cap, uint32_t* done, uint32_t* ids, cudaStream_t st);
@@ -51,6 +52,9 @@ void launch_atomic(const float* x, const float* y, const float* m, int64_t n, co
 void launch_lut(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, float* out,
                 cudaStream_t st);
 void launch_quantize(const float* img, int64_t npix, int bits, void* out, int num_sms, cudaStream_t st);
+size_t route_blocks(int64_t n);
+void launch_route(const float* x, const float* y, const float* m, int64_t n, int32_t row0, int32_t rows, int32_t R,
+                  uint32_t* blk, float* xo, float* yo, float* mo, uint32_t* n_out, cudaStream_t st);
 void launch_split_aos(const float* aos, int64_t n, float* x, float* y, float* m, int num_sms, cudaStream_t st);
 
 }  // namespace starsim

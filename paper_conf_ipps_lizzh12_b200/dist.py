@@ -1,11 +1,13 @@
 """Multi-GPU frames: horizontal bands, one per rank, assembled with one all-gather.
 
 The paper is single-GPU and names multi-GPU scaling as future work (Sec. V).  Here the image is split
-into G horizontal bands of whole 64-row tiles; every rank renders its band with ``starsim_render_band`` (stars are
-routed to a band iff their ROI rows intersect it: ``band_star_mask`` selects a rank's catalogue, and the library's
-binning pass clips every star to the band), and ``torch.distributed.all_gather_into_tensor`` concatenates the bands: row-major band
-concatenation *is* the frame, so there is no re-layout.  With tile-aligned band edges the assembled frame is bitwise
-equal to the single-GPU render (same per-pixel star order).
+into G horizontal bands of whole 64-row tiles.  Every rank holds the replicated catalogue and, each frame, routes it
+to its band on the device (``starsim_route_band``: the stars whose ROI rows meet the band, compacted in catalogue
+order, the count left in device memory) and renders the band from the routed stars (``starsim_set_star_count`` +
+``starsim_render_band``; ``Context.render_band_routed`` does both) -- there is no ROI arithmetic in this module.
+``torch.distributed.all_gather_into_tensor`` then concatenates the bands (row-major band concatenation *is* the frame,
+no re-layout), or ``FusedFrame`` stores every band pixel straight into every rank's frame from the tile kernel.  With
+tile-aligned band edges the assembled frame is bitwise equal to the single-GPU render (same per-pixel star order).
 
 torch.distributed (NCCL on GPUs, gloo in the CPU tests) is plumbing only; the render runs in libstarsim.so.
 """
@@ -28,23 +30,6 @@ def band_rows(height: int, world: int, rank: int, align: int = TILE_H) -> tuple[
     return row0, row1 - row0
 
 
-def band_star_mask(y, row0: int, rows: int, roi: int):
-    """The stars routed to band [row0, row0 + rows): those whose ROI rows meet it, as a boolean
-    mask over the catalogue (host, numpy).  The ROI's first row is the exact rule of reading R7 (the R rows nearest
-    y, ties at k + 1/2 upward), evaluated exactly in fp64 on the fp32 coordinate; stars with a non-finite y are left
-    out (they contribute nothing).  Keeping the catalogue order, a band rendered from ``catalogue[mask]`` has the same
-    tile lists, in the same relative order, as the band rendered from the whole catalogue: the same image bit for bit.
-    This is the per-band catalogue query of a distributed render (the catalogue retrieval itself is out of scope,
-    SURVEY.md §8f); bench.py applies it before the timed region, so no rank bins stars of other bands."""
-    import numpy as np
-    y64 = np.asarray(y, dtype=np.float32).astype(np.float64)
-    fin = np.isfinite(y64)
-    yc = np.where(fin, y64, 0.0)
-    fy = np.floor(yc)
-    ly = (fy + (yc >= fy + 0.5) - (roi - 1) // 2) if roi % 2 else (fy + 1 - roi // 2)
-    return fin & (ly <= row0 + rows - 1) & (ly + roi - 1 >= row0)
-
-
 def padded_band_rows(height: int, world: int, align: int = TILE_H) -> int:
     """Rows of the equal-size band buffers used by the all-gather (all_gather_into_tensor needs equal chunks)."""
     tiles = -(-height // align)
@@ -55,8 +40,9 @@ def render_frame(render_band, x, y, mag, width: int, height: int, sigma: float, 
                  group=None, full_out=None, band_out=None):
     """Render this rank's band and all-gather the frame.
 
-    ``render_band(x, y, mag, width, height, row0, rows, sigma, roi, gain, out)`` renders rows [row0, row0+rows) into
-    ``out`` (rows x width); for the product it is ``Context.render_band``.  Returns (full_frame, band_view).
+    ``render_band(x, y, mag, width, height, row0, rows, sigma, roi, gain, out)`` renders rows [row0, row0+rows) of the
+    frame of the whole catalogue (x, y, mag) into ``out`` (rows x width); for the product it is
+    ``Context.render_band_routed`` (device routing + band render), in the CPU tests the oracle.  Returns (full_frame, band_view).
     The gathered tensor has world * padded rows; the frame is its first ``height`` rows.
     """
     import torch
@@ -81,14 +67,28 @@ def render_frame(render_band, x, y, mag, width: int, height: int, sigma: float, 
     return full_out[:height], band_out
 
 
+def frames_agree(frame, ref, group=None) -> bool:
+    """True iff this rank's assembled frame equals ``ref`` bitwise on EVERY rank of the group (one MIN all-reduce):
+    the validation of a multi-GPU frame against the single-GPU (or oracle) frame, used by bench.py's strong_C5 record
+    and the gloo tests."""
+    import torch
+    import torch.distributed as dist
+    ok = torch.tensor([1 if (frame.shape == ref.shape and bool(torch.equal(frame, ref))) else 0], dtype=torch.int32,
+                      device=frame.device)
+    if dist.is_initialized():
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN, group=group)
+    return bool(ok.item())
+
+
 class FusedFrame:
     """The fused band exchange (north star: bands assembled over NVLink).
 
     The frame lives in torch symmetric memory: every rank maps every other rank's frame into its address space, and
     ``starsim_render_band_to`` makes the tile kernel's epilogue store each pixel of this rank's band into all of them
-    over NVLink / NVSwitch while the rest of the band is still being rendered.  A device-side barrier on the render
-    stream (the symmetric-memory handle's signal pads) then orders every rank's stores before any rank reads its
-    frame.  There is no all-gather pass: the exchange overlaps the render.  Needs CUDA peer access between the ranks'
+    over NVLink / NVSwitch while the rest of the band is still being rendered.  Two device-side barriers on the render
+    stream (the symmetric-memory handle's signal pads) bracket the stores: the one before keeps a rank from writing
+    frame k+1 into a peer's frame while that peer's stream may still be reading frame k, the one after orders every
+    rank's stores before any rank reads its frame.  There is no all-gather pass: the exchange overlaps the render.  Needs CUDA peer access between the ranks'
     GPUs (one node); ``available()`` says whether this process can use it, otherwise ``render_frame`` (NCCL
     all-gather) is the path.
     """
@@ -119,15 +119,17 @@ class FusedFrame:
         return torch.cuda.is_available() and dist.is_initialized() and dist.get_backend() == "nccl"
 
     def render(self, ctx, x, y, mag, sigma: float, roi: int, gain: float, stream=None):
-        """This rank's band into every rank's frame, then the cross-GPU barrier (all on `stream`); returns the local
-        frame, complete once the stream reaches the barrier."""
+        """Barrier, this rank's band (device-routed from the whole catalogue x, y, mag) into every rank's frame,
+        barrier -- all on `stream`.  Returns the local frame, complete once the stream passes the second barrier and
+        valid until the next ``render`` (readers on other streams must be ordered before it)."""
         import torch
 
         row0, rows = band_rows(self.height, self.world, self.rank)
         st = stream if stream is not None else torch.cuda.current_stream()
         with torch.cuda.stream(st):
+            self.handle.barrier(channel=0)  # every peer is done with the previous frame before anyone overwrites it
             if rows > 0:
-                ctx.render_band_to(x, y, mag, self.width, self.height, row0, rows, sigma, roi, gain, self.ptrs,
-                                   stream=st)
+                ctx.render_band_routed(x, y, mag, self.width, self.height, row0, rows, sigma, roi, gain,
+                                       frames=self.ptrs, stream=st)
             self.handle.barrier(channel=0)
         return self.frame

@@ -4,9 +4,13 @@ Every step of the render runs in the library's sm_100a kernels; this module only
 device pointers and the current torch stream to a ``cudaStream_t``.  There is no CPU fallback: if the library is not
 built, or the device is not an sm_100 GPU, the calls raise.  torch is used for device memory and streams only.
 
-Names mirror the C ABI: ``starsim_create``, ``starsim_render``, ``starsim_render_band``, ``starsim_render_atomic``,
-``starsim_upload_aos``, ``starsim_quantize``, ``starsim_get_bins``, ``starsim_profile``, ``starsim_kernel_times``,
-``starsim_destroy``; :class:`Context` wraps a handle with the same methods.
+Names mirror the C ABI (one Python function per entry point of include/starsim.h, same name and argument order,
+``n`` taken from the tensors): ``starsim_create``, ``starsim_render``, ``starsim_render_band``,
+``starsim_render_band_to``, ``starsim_render_gray``, ``starsim_render_atomic``, ``starsim_render_lut``,
+``starsim_route_band``, ``starsim_set_star_count``, ``starsim_set_psf``, ``starsim_set_roi``, ``starsim_set_binning``,
+``starsim_set_tile_kernel``, ``starsim_upload_aos``, ``starsim_quantize``, ``starsim_get_bins``, ``starsim_profile``,
+``starsim_kernel_times``, ``starsim_destroy``; :class:`Context` wraps a handle with the same methods.  Output
+tensors are checked for dtype, contiguity and size here, so a too-small buffer raises instead of being overrun.
 """
 from __future__ import annotations
 
@@ -20,7 +24,7 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("STARSIM_LIB") or os.path.join(_PKG, "libstarsim.so")  # override: A/B tooling only
 
 STARSIM_OK, STARSIM_EINVAL, STARSIM_ENOMEM, STARSIM_ECUDA, STARSIM_ENODEV = 0, -1, -2, -3, -4
-KCLASSES = ("prep", "sort", "csr", "tile", "atomic", "memset", "quantize", "aos")
+KCLASSES = ("prep", "sort", "csr", "tile", "atomic", "memset", "quantize", "aos", "route")
 NUM_KCLASS = len(KCLASSES)
 
 _lock = threading.Lock()
@@ -66,6 +70,10 @@ def lib():
         L.starsim_set_binning.restype = ctypes.c_int
         L.starsim_set_tile_kernel.argtypes = [vp, i32]
         L.starsim_set_tile_kernel.restype = ctypes.c_int
+        L.starsim_route_band.argtypes = [vp, vp, vp, vp, i64, i32, i32, i32, i32, vp, vp, vp, vp, vp]
+        L.starsim_route_band.restype = ctypes.c_int
+        L.starsim_set_star_count.argtypes = [vp, vp]
+        L.starsim_set_star_count.restype = ctypes.c_int
         L.starsim_render_atomic.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
         L.starsim_render_atomic.restype = ctypes.c_int
         L.starsim_render_lut.argtypes = [vp, vp, vp, vp, i64, i32, i32, f32, i32, f32, vp, vp]
@@ -97,8 +105,11 @@ def _stream(stream):
     return ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
 
 
-def _ptr(t, dtype=None, name="tensor"):
+def _ptr(t, dtype=None, name="tensor", numel=None):
+    """Device pointer of a contiguous CUDA tensor; numel: the elements the library will access (checked >=)."""
     if t is None:
+        if numel:
+            raise ValueError(f"{name} is None")
         return None
     if not t.is_cuda:
         raise ValueError(f"{name} must be a CUDA tensor")
@@ -106,7 +117,19 @@ def _ptr(t, dtype=None, name="tensor"):
         raise ValueError(f"{name} must be contiguous")
     if dtype is not None and t.dtype != dtype:
         raise ValueError(f"{name} must be {dtype}, got {t.dtype}")
+    if numel is not None and t.numel() < numel:
+        raise ValueError(f"{name} has {t.numel()} elements, the call writes / reads {numel}")
     return ctypes.c_void_p(t.data_ptr())
+
+
+def _cat(x, y, mag):
+    """Pointers and n of a SoA catalogue (x, y, mag float32, same length; None for an empty catalogue)."""
+    import torch
+    n = int(x.numel()) if x is not None else 0
+    for t, nm in ((y, "y"), (mag, "mag")):
+        if (t.numel() if t is not None else 0) != n:
+            raise ValueError(f"{nm} has a different length than x")
+    return (_ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"), _ptr(mag, torch.float32, "mag"), n)
 
 
 # ------------------------------------------------------------------ C-named functions
@@ -119,6 +142,11 @@ def starsim_create(device: int = 0):
     return h
 
 
+def starsim_last_error(h=None) -> str:
+    """Text of the last error on context h (or of the last create failure when h is None)."""
+    return lib().starsim_last_error(h).decode(errors="replace")
+
+
 def starsim_destroy(h) -> None:
     if h:
         lib().starsim_destroy(h)
@@ -126,30 +154,27 @@ def starsim_destroy(h) -> None:
 
 def starsim_render(h, x, y, mag, width, height, sigma, roi, gain, out, stream=None) -> None:
     import torch
-    n = int(x.numel()) if x is not None else 0
-    _check(h, lib().starsim_render(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
-                                   _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
-                                   int(roi), float(gain), _ptr(out, torch.float32, "out"), _stream(stream)))
+    px, py, pm, n = _cat(x, y, mag)
+    _check(h, lib().starsim_render(h, px, py, pm, n, int(width), int(height), float(sigma), int(roi), float(gain),
+                                   _ptr(out, torch.float32, "out", int(width) * int(height)), _stream(stream)))
 
 
 def starsim_render_band_to(h, x, y, mag, width, height, row0, rows, sigma, roi, gain, dst_ptrs, stream=None) -> None:
     """dst_ptrs: device addresses (ints) of ndst full float32 frames (height x width), local or peer-mapped."""
-    import torch
-    n = int(x.numel()) if x is not None else 0
+    px, py, pm, n = _cat(x, y, mag)
     arr = (ctypes.c_void_p * max(1, len(dst_ptrs)))(*[ctypes.c_void_p(int(p)) for p in dst_ptrs])
-    _check(h, lib().starsim_render_band_to(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
-                                           _ptr(mag, torch.float32, "mag"), n, int(width), int(height), int(row0),
+    _check(h, lib().starsim_render_band_to(h, px, py, pm, n, int(width), int(height), int(row0),
                                            int(rows), float(sigma), int(roi), float(gain), arr, len(dst_ptrs),
                                            _stream(stream)))
 
 
 def starsim_render_gray(h, x, y, mag, width, height, sigma, roi, gain, bits, out, stream=None) -> None:
     import torch
-    n = int(x.numel()) if x is not None else 0
+    px, py, pm, n = _cat(x, y, mag)
     dt = torch.uint8 if int(bits) == 8 else torch.uint16
-    _check(h, lib().starsim_render_gray(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
-                                        _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
-                                        int(roi), float(gain), int(bits), _ptr(out, dt, "out"), _stream(stream)))
+    _check(h, lib().starsim_render_gray(h, px, py, pm, n, int(width), int(height), float(sigma), int(roi),
+                                        float(gain), int(bits), _ptr(out, dt, "out", int(width) * int(height)),
+                                        _stream(stream)))
 
 
 PSF_MODES = {"point": 0, "integrated": 1}
@@ -182,27 +207,43 @@ def starsim_set_tile_kernel(h, mode) -> None:
 
 def starsim_render_band(h, x, y, mag, width, height, row0, rows, sigma, roi, gain, out_band, stream=None) -> None:
     import torch
-    n = int(x.numel()) if x is not None else 0
-    _check(h, lib().starsim_render_band(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
-                                        _ptr(mag, torch.float32, "mag"), n, int(width), int(height), int(row0),
-                                        int(rows), float(sigma), int(roi), float(gain),
-                                        _ptr(out_band, torch.float32, "out_band"), _stream(stream)))
+    px, py, pm, n = _cat(x, y, mag)
+    _check(h, lib().starsim_render_band(h, px, py, pm, n, int(width), int(height), int(row0), int(rows), float(sigma),
+                                        int(roi), float(gain),
+                                        _ptr(out_band, torch.float32, "out_band", int(rows) * int(width)),
+                                        _stream(stream)))
+
+
+def starsim_route_band(h, x, y, mag, height, row0, rows, roi, x_out, y_out, mag_out, n_out, stream=None) -> None:
+    """The stars of (x, y, mag) routed to rows [row0, row0+rows) -> (x_out, y_out, mag_out)[:*n_out] (device)."""
+    import torch
+    px, py, pm, n = _cat(x, y, mag)
+    _check(h, lib().starsim_route_band(h, px, py, pm, n, int(height), int(row0), int(rows), int(roi),
+                                       _ptr(x_out, torch.float32, "x_out", n), _ptr(y_out, torch.float32, "y_out", n),
+                                       _ptr(mag_out, torch.float32, "mag_out", n),
+                                       _ptr(n_out, torch.int32, "n_out", 1), _stream(stream)))
+
+
+def starsim_set_star_count(h, n_dev) -> None:
+    """n_dev: a CUDA int32 tensor holding the star count (read as uint32 by the kernels), or None to clear."""
+    import torch
+    _check(h, lib().starsim_set_star_count(h, None if n_dev is None else _ptr(n_dev, torch.int32, "n_dev", 1)))
 
 
 def starsim_render_atomic(h, x, y, mag, width, height, sigma, roi, gain, out, stream=None) -> None:
     import torch
-    n = int(x.numel()) if x is not None else 0
-    _check(h, lib().starsim_render_atomic(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
-                                          _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
-                                          int(roi), float(gain), _ptr(out, torch.float32, "out"), _stream(stream)))
+    px, py, pm, n = _cat(x, y, mag)
+    _check(h, lib().starsim_render_atomic(h, px, py, pm, n, int(width), int(height), float(sigma), int(roi),
+                                          float(gain), _ptr(out, torch.float32, "out", int(width) * int(height)),
+                                          _stream(stream)))
 
 
 def starsim_render_lut(h, x, y, mag, width, height, sigma, roi, gain, out, stream=None) -> None:
     import torch
-    n = int(x.numel()) if x is not None else 0
-    _check(h, lib().starsim_render_lut(h, _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
-                                          _ptr(mag, torch.float32, "mag"), n, int(width), int(height), float(sigma),
-                                          int(roi), float(gain), _ptr(out, torch.float32, "out"), _stream(stream)))
+    px, py, pm, n = _cat(x, y, mag)
+    _check(h, lib().starsim_render_lut(h, px, py, pm, n, int(width), int(height), float(sigma), int(roi),
+                                       float(gain), _ptr(out, torch.float32, "out", int(width) * int(height)),
+                                       _stream(stream)))
 
 
 def starsim_upload_aos(h, host_aos: np.ndarray, x, y, mag, stream=None) -> None:
@@ -210,16 +251,18 @@ def starsim_upload_aos(h, host_aos: np.ndarray, x, y, mag, stream=None) -> None:
     a = np.ascontiguousarray(host_aos, dtype=np.float32)
     if a.ndim != 2 or a.shape[1] != 3:
         raise ValueError("host_aos must be (n, 3) float32 {mag, posX, posY}")
-    _check(h, lib().starsim_upload_aos(h, a.ctypes.data_as(ctypes.c_void_p), a.shape[0],
-                                       _ptr(x, torch.float32, "x"), _ptr(y, torch.float32, "y"),
-                                       _ptr(mag, torch.float32, "mag"), _stream(stream)))
+    n = a.shape[0]
+    _check(h, lib().starsim_upload_aos(h, a.ctypes.data_as(ctypes.c_void_p), n,
+                                       _ptr(x, torch.float32, "x", n), _ptr(y, torch.float32, "y", n),
+                                       _ptr(mag, torch.float32, "mag", n), _stream(stream)))
 
 
 def starsim_quantize(h, img, bits, out, stream=None) -> None:
     import torch
     want = torch.uint8 if bits == 8 else torch.uint16 if bits == 16 else None
-    _check(h, lib().starsim_quantize(h, _ptr(img, torch.float32, "img"), int(img.numel()), int(bits),
-                                     _ptr(out, want, "out") if want is not None else ctypes.c_void_p(out.data_ptr()),
+    npix = int(img.numel())
+    _check(h, lib().starsim_quantize(h, _ptr(img, torch.float32, "img"), npix, int(bits),
+                                     _ptr(out, want, "out", npix) if want is not None else ctypes.c_void_p(out.data_ptr()),
                                      _stream(stream)))
 
 
@@ -314,7 +357,8 @@ class Context:
         starsim_set_binning(self.h, mode)
 
     def set_tile_kernel(self, mode="auto"):
-        """"auto" (sorted-corner-bin kernel for R <= 17, else the list kernel) or "lists" (always the list kernel)."""
+        """"auto" (R <= 17: "ws" on dense frames, else "sb"; R > 17: "lists"), "lists" (k_tile, any R), "sb" (k_tile_sb),
+        "ws" (k_tile_ws) or "t8" (k_t8sort + k_tile8); include/starsim.h, starsim_set_tile_kernel."""
         starsim_set_tile_kernel(self.h, mode)
 
     def render_band(self, x, y, mag, width, height, row0, rows, sigma, roi, gain, out=None, stream=None):
@@ -331,6 +375,48 @@ class Context:
                                            f.numel() != width * height):
                 raise ValueError("frames must be contiguous float32 tensors of height x width")
         starsim_render_band_to(self.h, x, y, mag, width, height, row0, rows, sigma, roi, gain, ptrs, stream)
+
+    def route_band(self, x, y, mag, height, row0, rows, roi, out=None, stream=None):
+        """Device band routing (starsim_route_band): returns (x_r, y_r, mag_r, n_dev) -- capacity len(x) arrays whose
+        first n_dev[0] entries are the stars routed to rows [row0, row0+rows), in catalogue order, and the count as a
+        one-element int32 CUDA tensor (not read back)."""
+        import torch
+        n = int(x.numel())
+        if out is None:
+            out = tuple(torch.empty(max(n, 1), dtype=torch.float32, device=x.device) for _ in range(3)) + (
+                torch.empty(1, dtype=torch.int32, device=x.device),)
+        xo, yo, mo, nd = out
+        starsim_route_band(self.h, x, y, mag, height, row0, rows, roi, xo, yo, mo, nd, stream)
+        return xo, yo, mo, nd
+
+    def set_star_count(self, n_dev=None):
+        """Tiled renders take the first n_dev[0] stars (device int32 tensor) of their catalogue; None clears."""
+        starsim_set_star_count(self.h, n_dev)
+        self._n_dev = n_dev  # the library keeps the pointer: hold the tensor
+
+    def render_band_routed(self, x, y, mag, width, height, row0, rows, sigma, roi, gain, out=None, frames=None,
+                           stream=None):
+        """Route the catalogue to the band on the device, then render the band from the routed stars (the device
+        count is read by the kernels: no host round trip).  Into `out` (rows x width), or -- with `frames` -- into
+        every full frame of `frames` (the fused exchange, as render_band_to).  Bitwise the band of render_band on the
+        whole catalogue.  The routed buffers are cached per capacity so repeated calls replay one CUDA graph."""
+        import torch
+        n = int(x.numel())
+        key = (n, x.device)
+        if getattr(self, "_route_key", None) != key:
+            self._route_buf = tuple(torch.empty(max(n, 1), dtype=torch.float32, device=x.device) for _ in range(3)) + (
+                torch.empty(1, dtype=torch.int32, device=x.device),)
+            self._route_key = key
+        xo, yo, mo, nd = self.route_band(x, y, mag, height, row0, rows, roi, out=self._route_buf, stream=stream)
+        xo, yo, mo = xo[:n], yo[:n], mo[:n]
+        self.set_star_count(nd)
+        try:
+            if frames is not None:
+                self.render_band_to(xo, yo, mo, width, height, row0, rows, sigma, roi, gain, frames, stream)
+                return None
+            return self.render_band(xo, yo, mo, width, height, row0, rows, sigma, roi, gain, out, stream)
+        finally:
+            self.set_star_count(None)
 
     def render_atomic(self, x, y, mag, width, height, sigma, roi, gain, out=None, stream=None):
         out = self._out(height, width, out)

@@ -1,6 +1,7 @@
 """Multi-GPU band decomposition, host logic on CPU: world_size-2 (and 3) gloo process groups render bands with the fp64
 oracle standing in for the per-rank renderer and assemble them with all_gather_into_tensor; the result must equal the
-single-process frame bitwise."""
+single-process frame bitwise.  Band routing: oracle.route_band, the definition the library's
+starsim_route_band is compared with on the GPU (tests/test_gpu_parity.py), pinned here against exact arithmetic."""
 import os
 import socket
 
@@ -28,23 +29,38 @@ def test_band_rows_partition_every_row():
 
 
 @pytest.mark.parametrize("R", [1, 4, 9, 15])
-def test_band_star_mask_routes_exactly_the_stars_whose_roi_meets_the_band(R):
-    """band_star_mask against the oracle's clipped ROI rows (reading R7, exact) on adversarial coordinates: a star is
-    routed to a band iff its clipped ROI rows meet it; every contributing star reaches at least one band."""
+def test_oracle_route_band_is_the_exact_roi_row_rule(R):
+    """oracle.route_band (the definition starsim_route_band computes) pinned against exact rational arithmetic: a star
+    is routed to a band iff y is finite and its ROI rows [lo, lo + R - 1], lo = floor(y + 1 - R/2) in exact arithmetic
+    (reading R7: the R rows nearest y, ties upward), meet the band; indices ascending.  Adversarial coordinates
+    (half-integers and their fp32 neighbours, band edges, non-finite values, far-off stars); every star whose clipped
+    ROI is non-empty reaches the band(s) its clipped rows meet."""
+    import math
+    from fractions import Fraction
     import oracle
     import synth
     W, H, G = 70, 256, 4
     f = synth.adversarial_field(3000, W, H, R, seed=7)
-    masks = [sdist.band_star_mask(f.y, *sdist.band_rows(H, G, g), R) for g in range(G)]
+    for g in range(G):
+        r0, n = sdist.band_rows(H, G, g)
+        got = oracle.route_band(f.y, R, r0, n)
+        want = []
+        for i, yv in enumerate(f.y.tolist()):
+            if not math.isfinite(yv):
+                continue
+            lo = math.floor(Fraction(yv) + 1 - Fraction(R, 2))
+            if lo <= r0 + n - 1 and lo + R - 1 >= r0:
+                want.append(i)
+        assert got.tolist() == want, g
+    sel = [set(oracle.route_band(f.y, R, *sdist.band_rows(H, G, g)).tolist()) for g in range(G)]
     for i in range(f.n):
         roi = oracle.star_roi(float(f.x[i]), float(f.y[i]), float(f.mag[i]), W, H, R)
         if roi is None:
             continue
-        y0, y1 = roi[2], roi[3]
         for g in range(G):
             r0, n = sdist.band_rows(H, G, g)
-            assert bool(masks[g][i]) == (y0 <= r0 + n - 1 and y1 >= r0), (i, g)
-        assert any(m[i] for m in masks)
+            if roi[2] <= r0 + n - 1 and roi[3] >= r0:
+                assert i in sel[g], (i, g)
 
 
 def _free_port():
@@ -64,15 +80,25 @@ def _worker(rank, world, port, W, H, q):
     f = synth.uniform_field(600, W, H, seed=3)
 
     def render_band(x, y, mag, width, height, row0, rows, sigma, roi, gain, out):
-        # the rank's own catalogue: the stars routed to its band (bench.py does the same before its timed region)
-        sel = sdist.band_star_mask(f.y, row0, rows, roi)
-        img = oracle.render_band(f.x[sel], f.y[sel], f.mag[sel], width, height, row0, rows, sigma, roi, gain)
+        # stand-in for Context.render_band_routed on CPU: route the whole catalogue to the band (the oracle's
+        # definition of starsim_route_band), render the band from the routed stars
+        sel = oracle.route_band(y.numpy(), roi, row0, rows)
+        xs, ys, ms = (t.numpy()[sel] for t in (x, y, mag))
+        img = oracle.render_band(xs, ys, ms, width, height, row0, rows, sigma, roi, gain)
         out.copy_(torch.from_numpy(img.astype(np.float32)))
 
-    x = torch.zeros(1)
-    frame, band = sdist.render_frame(render_band, x, x, x, W, H, 1.7, 9, 1.0)
+    x, y, m = (torch.from_numpy(a) for a in (f.x, f.y, f.mag))
+    frame, band = sdist.render_frame(render_band, x, y, m, W, H, 1.7, 9, 1.0)
+    # the bench's validation (dist.frames_agree): every rank compares its assembled frame with the single-process
+    # frame; a corrupted frame on any one rank must make it fail on all ranks
+    ref = torch.from_numpy(oracle.render(f.x, f.y, f.mag, W, H, 1.7, 9, 1.0).astype(np.float32))
+    ok = sdist.frames_agree(frame, ref)
+    bad = frame.clone()
+    if rank == world - 1:
+        bad[H - 1, W - 1] += 1.0
+    ok_bad = sdist.frames_agree(bad, ref)
     if rank == 0:
-        q.put(frame.numpy().copy())
+        q.put((frame.numpy().copy(), ok, ok_bad))
     dist.barrier()
     dist.destroy_process_group()
 
@@ -88,7 +114,7 @@ def test_gloo_bands_assemble_the_frame(world):
     procs = [ctx.Process(target=_worker, args=(r, world, port, W, H, q)) for r in range(world)]
     for p in procs:
         p.start()
-    frame = q.get(timeout=120)
+    frame, ok, ok_bad = q.get(timeout=120)
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0
@@ -96,3 +122,4 @@ def test_gloo_bands_assemble_the_frame(world):
     ref = oracle.render(f.x, f.y, f.mag, W, H, 1.7, 9, 1.0).astype(np.float32)
     assert frame.shape == (H, W)
     assert np.array_equal(frame, ref)
+    assert ok and not ok_bad

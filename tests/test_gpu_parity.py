@@ -12,6 +12,7 @@ import pytest
 
 import oracle
 import synth
+from paper_conf_ipps_lizzh12_b200 import StarsimError
 
 pytestmark = pytest.mark.gpu
 
@@ -31,10 +32,10 @@ def torch_dev():
 
 @pytest.fixture(scope="module", params=["t8", "ws", "lists", "sb"])
 def ctx(torch_dev, request):
-    """Every test runs against the four tile kernels: "t8" (the 8 x 8 lane-block kernel, the default for R <= 17),
-    "ws" (the warp-specialised sorted-corner-bin kernel for
-    R <= 17, the list kernel above), "lists" (the per-block entry-list kernel for every R) and "sb" (the sorted-bin
-    kernel with both roles in every warp; "auto" picks ws or sb by the expected list length, same images)."""
+    """Every test runs against the four tile kernels: "t8" (k_t8sort + the 8 x 8 lane-block kernel k_tile8, opt-in,
+    R <= 17), "ws" (the warp-specialised sorted-corner-bin kernel for R <= 17, the list kernel above), "lists" (the
+    per-block entry-list kernel for every R) and "sb" (the sorted-bin kernel with both roles in every warp; "auto"
+    picks ws or sb by the expected list length, same images)."""
     from paper_conf_ipps_lizzh12_b200 import Context
     c = Context(0)
     c.set_tile_kernel(request.param)
@@ -310,6 +311,12 @@ def test_kernel_times_recorded(torch_dev, ctx):
     # the t8 mode adds its corner-bin sort (k_t8sort) to the sort class
     assert t["tile"][1] == 1 and t["tile"][0] > 0 and t["prep"][1] == 1 and t["sort"][1] in (1, 2)
     assert t["csr"][1] in (1, 2, 3)
+    assert t["route"][1] == 0
+    ctx.profile(True)
+    ctx.route_band(*args, cfg.H, 0, 64, cfg.R)
+    t = ctx.kernel_times()
+    ctx.profile(False)
+    assert t["route"][1] == 2 and t["route"][0] > 0
 
 
 # ---------------------------------------------------------------- B200-scale frames (full images, threaded oracle)
@@ -620,21 +627,91 @@ def test_circle_roi_parity(torch_dev, ctx, W, H, n, R, sigma, kind):
     assert_parity(ctx.render(*args, W, H, sigma, R, 1.0).cpu().numpy(), ref_sq, f"square after circle R={R}")
 
 
-def test_band_from_routed_catalogue_is_bitwise_the_band(torch_dev, ctx):
-    """A band rendered from its routed catalogue (dist.band_star_mask, what each rank holds in bench.py for N > 1)
-    equals the band rendered from the whole catalogue bit for bit: same tile lists in the same relative order."""
+@pytest.mark.parametrize("n,W,H,R,G,kind", [(0, 64, 64, 5, 1, "uniform"), (1, 64, 64, 5, 1, "uniform"),
+                                             (20001, 700, 530, 9, 3, "adv"), (50000, 640, 1024, 15, 4, "uniform"),
+                                             (1000000, 4096, 4096, 15, 8, "uniform")])
+def test_route_band_parity(torch_dev, ctx, n, W, H, R, G, kind):
+    """starsim_route_band against oracle.route_band (the exact ROI-row rule, pinned in test_dist_cpu.py): the routed
+    count and the compacted x, y, mag bit for bit, in catalogue order, for every band -- ragged 4096-star blocks,
+    non-finite and far-off coordinates (adversarial field), an empty catalogue, and the full 1M-star T catalogue."""
     torch, dev = torch_dev
     from paper_conf_ipps_lizzh12_b200 import dist as sdist
-    W, H, R, G = 640, 1024, 15, 4
-    f = synth.uniform_field(40000, W, H, seed=77, mag_hi=15.0)
-    full = to_dev(torch_dev, f)
+    f = synth.adversarial_field(n, W, H, R, seed=12) if kind == "adv" else synth.uniform_field(n, W, H, seed=12)
+    args = to_dev(torch_dev, f) if n else (torch.empty(0, device=dev),) * 3
     for g in range(G):
         row0, rows = sdist.band_rows(H, G, g)
-        sel = sdist.band_star_mask(f.y, row0, rows, R)
-        local = to_dev(torch_dev, synth.Field(f.x[sel], f.y[sel], f.mag[sel]))
-        a = ctx.render_band(*full, W, H, row0, rows, 2.5, R, 1.0)
-        b = ctx.render_band(*local, W, H, row0, rows, 2.5, R, 1.0)
-        assert torch.equal(a, b), g
+        if rows == 0:
+            continue
+        xo, yo, mo, nd = ctx.route_band(*args, H, row0, rows, R)
+        torch.cuda.synchronize()
+        idx = oracle.route_band(f.y, R, row0, rows)
+        k = int(nd.item())
+        assert k == idx.size, (g, k, idx.size)
+        for got, ref in ((xo, f.x), (yo, f.y), (mo, f.mag)):
+            assert np.array_equal(got[:k].cpu().numpy().view(np.uint32), ref[idx].view(np.uint32)), g
+
+
+@pytest.mark.parametrize("W,H,n,R,G", [(640, 1024, 40000, 15, 4),      # bands of <= 2048 tiles: dbin.cu binning
+                                       (16384, 2176, 200000, 15, 2)])  # 2176 tiles per band: bin.cu's pipeline
+def test_band_from_routed_catalogue_is_bitwise_the_band(torch_dev, ctx, W, H, n, R, G):
+    """A band rendered from the device-routed catalogue (starsim_route_band + starsim_set_star_count:
+    Context.render_band_routed, what every rank does per frame for N > 1) equals the band rendered from the whole
+    catalogue bit for bit -- same tile lists in the same relative order -- for every tile kernel and both binning
+    pipelines; the CUDA graph of the routed render replays with a count that changes between frames."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import dist as sdist
+    f = synth.uniform_field(n, W, H, seed=77, mag_hi=15.0)
+    full = to_dev(torch_dev, f)
+    st = torch.cuda.Stream(dev)  # a non-default stream: the renders go through the captured CUDA graph
+    with torch.cuda.stream(st):
+        for g in range(G):
+            row0, rows = sdist.band_rows(H, G, g)
+            a = ctx.render_band(*full, W, H, row0, rows, 2.5, R, 1.0, stream=st)
+            b = ctx.render_band_routed(*full, W, H, row0, rows, 2.5, R, 1.0, stream=st)
+            st.synchronize()
+            assert torch.equal(a, b), g
+        # same buffers, new content and a different routed count: the replayed graph reads the new device count
+        row0, rows = sdist.band_rows(H, G, 0)
+        out = torch.empty((rows, W), dtype=torch.float32, device=dev)
+        ctx.render_band_routed(*full, W, H, row0, rows, 2.5, R, 1.0, out=out, stream=st)
+        full[1][: n // 2] = full[1][: n // 2] * 0.5  # move half the stars towards row 0: more of them in band 0
+        ctx.render_band_routed(*full, W, H, row0, rows, 2.5, R, 1.0, out=out, stream=st)
+        a = ctx.render_band(*full, W, H, row0, rows, 2.5, R, 1.0, stream=st)
+        st.synchronize()
+        assert torch.equal(a, out)
+        # a band no star reaches: a zero image from a zero device count
+        far = tuple(t.clone() for t in full)
+        far[1].fill_(float(H + 1000))
+        z = ctx.render_band_routed(*far, W, H, row0, rows, 2.5, R, 1.0, stream=st)
+        st.synchronize()
+        assert int(ctx._route_buf[3].item()) == 0 and not z.any()
+
+
+def test_set_star_count_semantics_and_einval(torch_dev, ctx):
+    """With a device count set, tiled renders take the first min(n, count) stars; the star-centric renders refuse."""
+    torch, dev = torch_dev
+    W, H, R = 300, 200, 9
+    f = synth.uniform_field(5000, W, H, seed=5)
+    args = to_dev(torch_dev, f)
+    cnt = torch.tensor([1234], dtype=torch.int32, device=dev)
+    ctx.set_star_count(cnt)
+    try:
+        a = ctx.render(*args, W, H, 1.5, R, 1.0)
+        with pytest.raises(StarsimError):
+            ctx.render_atomic(*args, W, H, 1.5, R, 1.0)
+        with pytest.raises(StarsimError):
+            ctx.render_lut(*args, W, H, 1.5, R, 1.0)
+        cnt.fill_(10 ** 6)  # larger than n: all n stars
+        c = ctx.render(*args, W, H, 1.5, R, 1.0)
+    finally:
+        ctx.set_star_count(None)
+    b = ctx.render(*(t[:1234] for t in args), W, H, 1.5, R, 1.0)
+    assert torch.equal(a, b)
+    assert torch.equal(c, ctx.render(*args, W, H, 1.5, R, 1.0))
+    with pytest.raises(ValueError):  # the binding checks output sizes before the library is called
+        ctx.render(*args, W, H, 1.5, R, 1.0, out=torch.empty((H - 1, W), dtype=torch.float32, device=dev))
+    with pytest.raises(ValueError):
+        ctx.render_band(*args, W, H, 0, 64, 1.5, R, 1.0, out=torch.empty((63, W), dtype=torch.float32, device=dev))
 
 
 def test_unsplit_huge_tile_lists(torch_dev, ctx):
