@@ -24,6 +24,7 @@
 // tile whatever the band decomposition.  The tile is written once, coalesced (each lane stores 2 x 16 B per row).
 // No atomics on the image.
 #include <algorithm>
+#include <cstddef>
 
 #include "common.cuh"
 #include "launch.h"
@@ -44,8 +45,56 @@ struct TileSmem {
   float2 px[CHUNK];                      // per star: (x - X0, c0 | c1 << 8)
   uint16_t gyown[GY_CAP];                // band slot -> star | band << 8
   uint32_t gxown[GX_PAIRS];              // (star, strip) pair j -> strip slot | star << 16
+  StarRec rn[CHUNK];                     // per thread: its star record of the next chunk (cp.async, one chunk ahead)
   int ns, ngy, ngx;
 };
+
+// thread tid's record of the chunk starting at list position jb -> S.rn[tid], asynchronously (no registers held
+// across the accumulation; the thread alone reads its slot, after cp.async.wait_all)
+__device__ __forceinline__ void prefetch_rec(StarRec* slot, const StarRec* __restrict__ rec, uint32_t id) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((uint32_t)__cvta_generic_to_shared(slot)),
+               "l"(rec + id)
+               : "memory");
+  asm volatile("cp.async.commit_group;\n" ::: "memory");
+}
+
+static_assert(sizeof(float) * (GY_CAP * 16 + (RCAP * NSTRIPS + 1) * 8) >= sizeof(float) * TILE_W * TILE_H &&
+                  offsetof(TileSmem, gx) == sizeof(float) * GY_CAP * 16,
+              "the gray epilogue stages the tile in gy + gx");
+
+// The fused output stage of k_tile from the staged fp32 tile (row-major TILE_W floats per row): thread t quantises
+// 4 consecutive pixels of a row (exactly as k_quantize, quant1) and stores them as one u8x4 / u16x4 word when the
+// row run is whole and aligned, else pixel by pixel.
+__device__ __forceinline__ void tile_store_gray_staged(const float* __restrict__ buf, const FrameParams& fp,
+                                                    void* __restrict__ out_, int Y0, int X0, int TWe, int THe) {
+  const float qmax = fp.obits == 8 ? 255.f : 65535.f;
+  for (int p = threadIdx.x * 4; p < TILE_W * TILE_H; p += TILE_THREADS * 4) {
+    const int r = p / TILE_W, c = p % TILE_W;
+    if (r >= THe || c >= TWe) continue;
+    const float4 v = *reinterpret_cast<const float4*>(buf + p);
+    const uint32_t g0 = quant1(v.x, qmax), g1 = quant1(v.y, qmax), g2 = quant1(v.z, qmax), g3 = quant1(v.w, qmax);
+    const int64_t pix = (int64_t)(Y0 + r) * fp.W + X0 + c;
+    if (fp.obits == 8) {
+      uint8_t* o = reinterpret_cast<uint8_t*>(out_) + pix;
+      if (fp.vec && c + 4 <= TWe) {
+        *reinterpret_cast<uint32_t*>(o) = g0 | g1 << 8 | g2 << 16 | g3 << 24;
+      } else {
+        if (c < TWe) o[0] = (uint8_t)g0;
+        if (c + 1 < TWe) o[1] = (uint8_t)g1;
+        if (c + 2 < TWe) o[2] = (uint8_t)g2;
+      }
+    } else {
+      uint16_t* o = reinterpret_cast<uint16_t*>(out_) + pix;
+      if (fp.vec && c + 4 <= TWe) {
+        *reinterpret_cast<uint2*>(o) = make_uint2(g0 | g1 << 16, g2 | g3 << 16);
+      } else {
+        if (c < TWe) o[0] = (uint16_t)g0;
+        if (c + 1 < TWe) o[1] = (uint16_t)g1;
+        if (c + 2 < TWe) o[2] = (uint16_t)g2;
+      }
+    }
+  }
+}
 
 constexpr uint32_t ZERO_GX = RCAP * NSTRIPS;
 constexpr uint32_t ZERO_ENT = ZERO_GX * 32u << 16;  // gy byte offset 0, all-zero strip slot
@@ -56,7 +105,10 @@ constexpr uint32_t ZERO_ENT = ZERO_GX * 32u << 16;  // gy byte offset 0, all-zer
 // parts in part order -- a fixed order, so the image stays deterministic.
 // ---------------------------------------------------------------------------------------------------------------
 template <bool INTEG>  // INTEG: the pixel-integrated PSF (NEXT-2) instead of the paper's point-sampled Eq. 2
-__global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __restrict__ ids,
+#ifndef TILE_MINB_OPT
+#define TILE_MINB_OPT 3
+#endif
+__global__ void __launch_bounds__(TILE_THREADS, TILE_MINB_OPT) k_tile(const uint32_t* __restrict__ ids,
                                                           const StarRec* __restrict__ rec, FrameParams fp,
                                                           void* __restrict__ out_, const WorkItem* __restrict__ items,
                                                           const uint2* __restrict__ split_tab,
@@ -81,8 +133,9 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
   if (tid < 8) S.gx[ZERO_GX * 8 + tid] = 0.f;
 
   // persistent CTAs: item blockIdx.x first, then items from the counter the planner zeroed
-  const uint32_t nitems = __ldcg(&hdr->nitems);
-  for (uint32_t item = blockIdx.x; item < nitems;) {
+  // (the item count and an item's fields are re-read where needed rather than held across the accumulation:
+  // registers are the limit at 3 CTAs per SM)
+  for (uint32_t item = blockIdx.x; item < ld_volatile_u32(&hdr->nitems);) {
   const WorkItem wi = items[item];
   const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
   const int X0 = tx * TILE_W;    // first column of the tile
@@ -99,15 +152,16 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
   uint32_t segs_done = 0;  // SPLIT_LEN segments of this item already in the scratch (tile_common.cuh)
   // this thread's star record of the current chunk, loaded one chunk ahead (its latency hides behind the
   // accumulation of the previous chunk)
-  StarRec rnext = {};
-  if (wi.jb + tid < j1) rnext = rec[ids[wi.jb + tid]];
+  if (wi.jb + tid < j1) prefetch_rec(&S.rn[tid], rec, ids[wi.jb + tid]);
   for (uint32_t base = wi.jb; base < j1;) {
     // ======================= prep: thread = star (base + tid)
     // chunks never cross a SPLIT_LEN segment boundary of the list (segments are summed like the parts of a split tile)
     const uint32_t seg_end = min(j1, wi.jb + ((base - wi.jb) / SPLIT_LEN + 1u) * SPLIT_LEN);
     const int nvalid = (int)min((uint32_t)CHUNK, seg_end - base);
     const bool valid = tid < nvalid;
-    const StarRec r = rnext;
+    StarRec r = {};
+    asm volatile("cp.async.wait_all;\n" ::: "memory");
+    if (valid) r = S.rn[tid];
     int c0 = 0, c1 = -1, r0 = 0, r1 = -1;
     if (valid) {
       const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
@@ -311,7 +365,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
       for (uint32_t st = len; st < steps; ++st) ent[st * (NBANDS * NSTRIPS)] = ZERO_ENT;
     __syncthreads();
 
-    if (nb + tid < j1) rnext = rec[nid];
+    if (nb + tid < j1) prefetch_rec(&S.rn[tid], rec, nid);
     // ======================= accumulate: lane group q walks the (padded) list of block (B, Q)
     {
 #pragma unroll 4
@@ -342,8 +396,24 @@ __global__ void __launch_bounds__(TILE_THREADS, 3) k_tile(const uint32_t* __rest
   if (segs_done) seg_finish(acc, seg_scratch);
 
   // ======================= output: rows 16 B + hq + 4 i, columns 64 wx + 8 q .. +7 of the tile
-  if (tile_reduce_parts<false>(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &s_last))
-    tile_store<false>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+  if (tile_reduce_parts<false>(acc, ld_volatile_item(items + item), split_tab, part_buf, done, B, wx, q, hq, &s_last)) {
+    if (fp.obits == 0) {
+      tile_store<false>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+    } else {
+      // fused output stage: the fp32 tile is staged in shared memory (the profile slots are free now) and quantised
+      // from there by all threads, 4 pixels each -- the register-resident form would spill at 3 CTAs per SM
+      float* buf = S.gy;  // gy + gx: >= TILE_W * TILE_H floats
+      __syncthreads();
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        float4* d = reinterpret_cast<float4*>(buf + lane_row<false>(B, hq, i) * TILE_W + 64 * wx + 8 * q);
+        d[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
+        d[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
+      }
+      __syncthreads();
+      tile_store_gray_staged(buf, fp, out_, Y0, X0, TWe, THe);
+    }
+  }
   __shared__ uint32_t s_next;
   __syncthreads();  // every thread is past this item's shared-memory reads
   if (tid == 0) s_next = atomicAdd(&hdr->next_item, 1u) + gridDim.x;

@@ -106,6 +106,17 @@ __device__ __forceinline__ void seg_finish(float2 (&acc)[4][4], float* seg_scrat
     }
 }
 
+__device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ WorkItem ld_volatile_item(const WorkItem* p) {
+  WorkItem w;
+  asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(w.tile), "=r"(w.jb), "=r"(w.je), "=r"(w.aux) : "l"(p));
+  return w;
+}
+
 // Write the lane's 4 rows x 8 columns of the tile (rows Y0 + lane_row(B, hq, i) of the band, columns col0 .. col0+7):
 // fp32, or (fused output stage, NEXT-1) the gray value of each pixel exactly as k_quantize computes it from the same
 // fp32 sum, as u8 / u16.  Coalesced: the 8 lane groups of a warp store 8 adjacent 8-pixel runs of a row.

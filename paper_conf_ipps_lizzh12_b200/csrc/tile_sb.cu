@@ -48,7 +48,10 @@ __device__ unsigned long long g_sb_prof[6];
 constexpr int SB_NSK = NSTRIPS + 1;
 constexpr int SB_NBIN = (NBANDS + 1) * SB_NSK;  // 85
 constexpr int SB_CHUNK = CHUNK;             // stars per chunk (<= TILE_THREADS; 192 with 4 CTAs/SM measured slower: spills)
-constexpr int SB_MINB = 3;                  // CTAs per SM (80 registers, 70 KB shared memory)
+#ifndef SB_MINB_OPT
+#define SB_MINB_OPT 2
+#endif
+constexpr int SB_MINB = SB_MINB_OPT;         // CTAs per SM: 2 (128 registers, no spills; 3 CTAs at 80 registers spilled and measured 4-20 % slower, profiles/r2_ab_minb.txt)
 constexpr int SB_MINB_CIRC = 2;             // the circle variant: 2 CTAs per SM, registers for its per-pixel mask
 constexpr uint32_t SB_ZJ = SB_CHUNK;        // the all-zero slot
 

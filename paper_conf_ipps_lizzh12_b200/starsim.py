@@ -37,6 +37,13 @@ class StarsimError(RuntimeError):
         self.code = code
 
 
+class StarsimSizeError(StarsimError, ValueError):
+    """A buffer smaller than the call would access: rejected by the binding (EINVAL) before the library runs."""
+
+    def __init__(self, msg: str):
+        super().__init__(STARSIM_EINVAL, msg)
+
+
 def lib():
     """Load libstarsim.so (fails loudly if it has not been built)."""
     global _lib
@@ -118,7 +125,7 @@ def _ptr(t, dtype=None, name="tensor", numel=None):
     if dtype is not None and t.dtype != dtype:
         raise ValueError(f"{name} must be {dtype}, got {t.dtype}")
     if numel is not None and t.numel() < numel:
-        raise ValueError(f"{name} has {t.numel()} elements, the call writes / reads {numel}")
+        raise StarsimSizeError(f"{name} has {t.numel()} elements, the call writes / reads {numel}")
     return ctypes.c_void_p(t.data_ptr())
 
 

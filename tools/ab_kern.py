@@ -21,9 +21,10 @@ def main():
     ap.add_argument("--R", type=int, default=0)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--mode", default="t8")
+    ap.add_argument("--n", type=int, default=0, help="override the config's star count")
     a = ap.parse_args()
     cfg = synth.with_R(synth.CONFIGS[a.config], a.R) if a.R else synth.CONFIGS[a.config]
-    f = cfg.field()
+    f = cfg.field(a.n) if a.n else cfg.field()
     dev = torch.device("cuda:0")
     x, y, m = (torch.from_numpy(v).to(dev) for v in (f.x, f.y, f.mag))
     out = torch.empty((cfg.H, cfg.W), dtype=torch.float32, device=dev)
@@ -42,7 +43,7 @@ def main():
         names = list(per[0].keys())
         med = {k: sorted(p[k] for p in per)[len(per) // 2] * 1e3 for k in names}
     lib = os.path.basename(os.environ.get("STARSIM_LIB", "cur"))
-    print(lib, a.config, a.mode, " ".join(f"{k}={v:.1f}us" for k, v in med.items() if v > 0))
+    print(lib, a.config + (f"/R{a.R}" if a.R else "") + (f"/n{a.n}" if a.n else ""), a.mode, " ".join(f"{k}={v:.1f}us" for k, v in med.items() if v > 0))
 
 
 if __name__ == "__main__":
