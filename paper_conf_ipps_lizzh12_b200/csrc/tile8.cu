@@ -107,12 +107,20 @@ __device__ __forceinline__ void mbar_init(unsigned long long* b, uint32_t count)
 __device__ __forceinline__ void mbar_arrive(unsigned long long* b) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
 }
-// one arrival per warp: the warp's lanes' shared-memory writes are ordered before lane 0's (release) arrive by the
-// __syncwarp, and release is cumulative -- 1 instead of 32 serialised arrivals per warp
+// T8_WARP_ARRIVE: one arrival per warp -- the lanes' shared-memory writes are ordered before lane 0's (release)
+// arrive by the __syncwarp, and release is cumulative; 1 instead of 32 arrivals per warp, but compute-sanitizer's
+// racecheck does not model it (it reports the hand-offs as hazards).  Default: every thread arrives (the counts below
+// are threads), the form racecheck verifies.
+#ifdef T8_WARP_ARRIVE
+constexpr uint32_t T8_ARRIVALS_PER_WARP = 1;
 __device__ __forceinline__ void mbar_arrive_warp(unsigned long long* b) {
   __syncwarp();
   if ((threadIdx.x & 31) == 0) mbar_arrive(b);
 }
+#else
+constexpr uint32_t T8_ARRIVALS_PER_WARP = 32;
+__device__ __forceinline__ void mbar_arrive_warp(unsigned long long* b) { mbar_arrive(b); }
+#endif
 __device__ __forceinline__ void mbar_wait(unsigned long long* b, uint32_t parity) {
   const uint32_t a = smem_u32(b);
   uint32_t ok;
@@ -846,8 +854,8 @@ __global__ void __launch_bounds__(T8_THREADS, 2)
 #endif
   for (int i = tid; i < T8_NS * 16; i += T8_THREADS) S.st[i / 16].zero[i % 16] = make_float4(0.f, 0.f, 0.f, 0.f);
   if (tid < T8_NS) {
-    mbar_init(&S.full[tid], T8_PROD);
-    mbar_init(&S.empty[tid], T8_CONS);
+    mbar_init(&S.full[tid], T8_PROD * T8_ARRIVALS_PER_WARP);
+    mbar_init(&S.empty[tid], T8_CONS * T8_ARRIVALS_PER_WARP);
   }
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();

@@ -27,19 +27,22 @@ def heavy(n, W, H, seed):
 
 def main():
     quick = "--quick" in sys.argv  # racecheck: fewer frames
+    only = next((a.split("=", 1)[1].split(",") for a in sys.argv if a.startswith("--kernels=")), None)
     dev = torch.device("cuda:0")
     c1 = synth.CONFIGS["C1"]
     cases = [("C1", c1.field(), c1.W, c1.H, c1.R, c1.sigma), ("heavy", heavy(30000, 256, 256, 3), 256, 256, 15, 2.5)]
     with Context(0) as ctx:
         for name, f, W, H, R, sigma in cases:
             x, y, m = (torch.from_numpy(a).to(dev) for a in (f.x, f.y, f.mag))
-            for tk in (["ws", "t8"] if quick else ["lists", "sb", "ws", "t8"]):
+            for tk in (only or (["ws", "t8"] if quick else ["lists", "sb", "ws", "t8"])):
                 for binning in (["auto"] if quick else ["auto", "atomic"]):
                     ctx.set_tile_kernel(tk)
                     ctx.set_binning(binning)
                     ctx.render(x, y, m, W, H, sigma, R, 1.0)
             ctx.set_tile_kernel("auto")
             ctx.set_binning("auto")
+            if only:
+                continue
             ctx.render_band(x, y, m, W, H, 64, 64, sigma, R, 1.0)
             ctx.render_band_routed(x, y, m, W, H, 64, 64, sigma, R, 1.0)
             if not quick:
