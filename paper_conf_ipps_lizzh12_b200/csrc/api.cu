@@ -195,6 +195,7 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   fp.ndst = 0;
   for (int i = 0; i < MAX_DST; ++i) fp.dst[i] = nullptr;
   fp.n_dev = nullptr;
+  fp.lite = 0;
   fp.obits = 0;
   fp.vec = 0;
   fp.kint = (float)(1.0 / (std::sqrt(2.0) * s));
@@ -279,10 +280,13 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
                    c->num_sms, st);
     });
   } else {
-    timed(c, 3, st, [&] {
-      launch_tile(ids, rec, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p, part_cap,
-                  done, hdr, c->num_sms, st, (float*)c->segs.p);
-    });
+    timed(
+        c, 3, st,
+        [&] {
+          launch_tile(ids, rec, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p, part_cap,
+                      done, hdr, c->num_sms, st, (float*)c->segs.p);
+        },
+        fp.lite ? 2 : 1);
   }
   if ((rc = check_launch(c, "k_tile"))) return rc;
   return STARSIM_OK;
@@ -311,6 +315,8 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   }
   fp.bin_impl = c->bin_impl;
   fp.n_dev = c->n_dev;
+  // k_tile_sb hands the light tiles to k_tile_lite (same bits; tile_sb.cu)
+  fp.lite = (fp.tile_impl == STARSIM_TILE_SB && R <= SB_MAXR && LITE_MAX > 0) ? 1 : 0;
   // one vector store per 8-pixel run: 32 B (fp32) / 8 B (u8) / 16 B (u16); rows must keep that alignment
   const int vb = obits == 8 ? 8 : 16;
   bool aligned = ((uintptr_t)out % vb) == 0;
@@ -338,7 +344,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   if ((rc = grow(c, c->zeroed, zbytes, "header+counters"))) return rc;
   if ((rc = grow(c, c->items, sizeof(WorkItem) * (size_t)(ntiles + part_cap), "work items"))) return rc;
   if ((rc = grow(c, c->split_tab, sizeof(uint2) * (size_t)ntiles, "split table"))) return rc;
-  if ((rc = grow(c, c->partial, sizeof(uint3) * (size_t)((ntiles + SCAN_TILES - 1) / SCAN_TILES), "scan partials")))
+  if ((rc = grow(c, c->partial, sizeof(uint4) * (size_t)((ntiles + SCAN_TILES - 1) / SCAN_TILES), "scan partials")))
     return rc;
   if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
   if ((rc = grow(c, c->segs, sizeof(float) * tile8_scratch_floats(c->num_sms), "segment scratch"))) return rc;

@@ -54,85 +54,76 @@ __global__ void __launch_bounds__(PREP_THREADS) k_prep(const float* __restrict__
 // Two kernels, SCAN_TILES tiles per CTA (SCAN_PER per thread): k_scan_a writes each CTA's sums (pairs, parts, split
 // tiles); k_scan_b re-reduces the sums of the CTAs before it and of all CTAs (a few hundred at most), scans its own
 // tiles and writes tile_off and the work items.
-// block-wide exclusive scan of uint3 (SCAN_THREADS threads); *total receives the block sum
-__device__ __forceinline__ uint3 block_excl_scan3(uint3 v, uint3* s_w, uint3* total) {
+// block-wide exclusive scan of uint4 (SCAN_THREADS threads); *total receives the block sum
+__device__ __forceinline__ uint4 block_excl_scan4(uint4 v, uint4* s_w, uint4* total) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint3 incl = warp_incl_scan3(v, lane);
+  const uint4 incl = warp_incl_scan4(v, lane);
   if (lane == 31) s_w[warp] = incl;
   __syncthreads();
-  uint3 pre = make_uint3(0, 0, 0), tot = make_uint3(0, 0, 0);
+  uint4 pre = make_uint4(0, 0, 0, 0), tot = make_uint4(0, 0, 0, 0);
 #pragma unroll
   for (int w = 0; w < SCAN_THREADS / 32; ++w) {
-    const uint3 u = s_w[w];
-    if (w < warp) pre = add3(pre, u);
-    tot = add3(tot, u);
+    const uint4 u = s_w[w];
+    if (w < warp) pre = add4(pre, u);
+    tot = add4(tot, u);
   }
   __syncthreads();
   *total = tot;
-  return make_uint3(pre.x + incl.x - v.x, pre.y + incl.y - v.y, pre.z + incl.z - v.z);
+  return sub4(add4(pre, incl), v);
 }
 
-__device__ __forceinline__ void load_counts(const uint32_t* cnt, int64_t ntiles, int64_t t0, uint32_t* c, uint3& sum) {
-  sum = make_uint3(0, 0, 0);
+__device__ __forceinline__ void load_counts(const uint32_t* cnt, int64_t ntiles, int64_t t0, uint32_t* c, uint4& sum) {
+  sum = make_uint4(0, 0, 0, 0);
 #pragma unroll
   for (int k = 0; k < SCAN_PER; ++k) c[k] = t0 + k < ntiles ? __ldcg(&cnt[(t0 + k) * CNT_STRIDE]) : 0u;
 #pragma unroll
-  for (int k = 0; k < SCAN_PER; ++k) {
-    const uint32_t np = parts_of(c[k]);
-    sum = add3(sum, make_uint3(c[k], np, np ? 1u : 0u));
-  }
+  for (int k = 0; k < SCAN_PER; ++k) sum = add4(sum, t0 + k < ntiles ? tile_counts(c[k]) : make_uint4(0, 0, 0, 0));
 }
 
 __global__ void __launch_bounds__(SCAN_THREADS) k_scan_a(const uint32_t* __restrict__ cnt, int64_t ntiles,
-                                                         uint3* __restrict__ partial) {
-  __shared__ uint3 s_w[SCAN_THREADS / 32];
+                                                         uint4* __restrict__ partial) {
+  __shared__ uint4 s_w[SCAN_THREADS / 32];
   const int64_t t0 = (int64_t)blockIdx.x * SCAN_TILES + (int64_t)threadIdx.x * SCAN_PER;
   uint32_t c[SCAN_PER];
-  uint3 sum, tot;
+  uint4 sum, tot;
   load_counts(cnt, ntiles, t0, c, sum);
-  block_excl_scan3(sum, s_w, &tot);
+  block_excl_scan4(sum, s_w, &tot);
   if (threadIdx.x == 0) partial[blockIdx.x] = tot;
 }
 
 __global__ void __launch_bounds__(SCAN_THREADS) k_scan_b(const uint32_t* __restrict__ cnt, int64_t ntiles,
-                                                         const uint3* __restrict__ partial, int nblk,
+                                                         const uint4* __restrict__ partial, int nblk,
                                                          uint32_t* __restrict__ tile_off, Header* hdr,
                                                          WorkItem* __restrict__ items,
                                                          uint2* __restrict__ split_tab, int part_cap,
                                                          uint32_t* __restrict__ done) {
-  __shared__ uint3 s_w[SCAN_THREADS / 32];
+  __shared__ uint4 s_w[SCAN_THREADS / 32];
   const int tid = threadIdx.x;
   // sums of the CTAs before this one, and of all CTAs
-  uint3 before = make_uint3(0, 0, 0), all = make_uint3(0, 0, 0);
+  uint4 before = make_uint4(0, 0, 0, 0), all = make_uint4(0, 0, 0, 0);
   for (int k = tid; k < nblk; k += SCAN_THREADS) {
-    const uint3 u = partial[k];
-    if (k < (int)blockIdx.x) before = add3(before, u);
-    all = add3(all, u);
+    const uint4 u = partial[k];
+    if (k < (int)blockIdx.x) before = add4(before, u);
+    all = add4(all, u);
   }
-  uint3 tb, ta;
-  block_excl_scan3(before, s_w, &tb);
-  block_excl_scan3(all, s_w, &ta);
+  uint4 tb, ta;
+  block_excl_scan4(before, s_w, &tb);
+  block_excl_scan4(all, s_w, &ta);
   const bool split_on = ta.y <= (uint32_t)part_cap;
   const uint32_t nparts = split_on ? ta.y : 0u, nsplit = split_on ? ta.z : 0u;
-  if (blockIdx.x == 0 && tid == 0) {
-    hdr->P = ta.x;
-    tile_off[ntiles] = ta.x;
-    hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
-    hdr->nsplit = nsplit;
-    hdr->next_item = 0u;
-    hdr->next_seg = 0u;
-  }
+  const uint32_t lite0 = nparts + (uint32_t)ntiles - nsplit - ta.w;
+  if (blockIdx.x == 0 && tid == 0) plan_header(hdr, tile_off, ntiles, ta, part_cap);
   const int64_t t0 = (int64_t)blockIdx.x * SCAN_TILES + (int64_t)tid * SCAN_PER;
   uint32_t c[SCAN_PER];
-  uint3 sum, tot;
+  uint4 sum, tot;
   load_counts(cnt, ntiles, t0, c, sum);
-  const uint3 ex = add3(tb, block_excl_scan3(sum, s_w, &tot));
-  uint32_t run = ex.x, pb = ex.y, si = ex.z;
+  const uint4 ex = add4(tb, block_excl_scan4(sum, s_w, &tot));
+  uint32_t run = ex.x, pb = ex.y, si = ex.z, li = ex.w;
 #pragma unroll
   for (int k = 0; k < SCAN_PER; ++k) {
     const int64_t t = t0 + k;
     if (t >= ntiles) break;
-    plan_tile((uint32_t)t, c[k], run, pb, si, nparts, split_on, tile_off, items, split_tab, done);
+    plan_tile((uint32_t)t, c[k], run, pb, si, li, nparts, lite0, split_on, tile_off, items, split_tab, done);
   }
 }
 
@@ -146,37 +137,36 @@ __global__ void __launch_bounds__(SCAN1_THREADS) k_scan_one(const uint32_t* __re
                                                              WorkItem* __restrict__ items,
                                                              uint2* __restrict__ split_tab, int part_cap,
                                                              uint32_t* __restrict__ done) {
-  __shared__ uint3 s_w[SCAN1_THREADS / 32];
+  __shared__ uint4 s_w[SCAN1_THREADS / 32];
+  __shared__ uint4 s_tot;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t t0 = (int64_t)tid * SCAN_PER;
   uint32_t c[SCAN_PER];
-  uint3 sum;
+  uint4 sum;
   load_counts(cnt, ntiles, t0, c, sum);
-  const uint3 incl = warp_incl_scan3(sum, lane);
+  const uint4 incl = warp_incl_scan4(sum, lane);
   if (lane == 31) s_w[warp] = incl;
   __syncthreads();
-  uint3 pre = make_uint3(0, 0, 0), ta = make_uint3(0, 0, 0);
-  for (int w = 0; w < SCAN1_THREADS / 32; ++w) {
-    const uint3 u = s_w[w];
-    if (w < warp) pre = add3(pre, u);
-    ta = add3(ta, u);
+  if (warp == 0) {  // exclusive scan of the warp sums in place; the total
+    const uint4 v = s_w[lane];
+    const uint4 wi = warp_incl_scan4(v, lane);
+    __syncwarp();
+    s_w[lane] = sub4(wi, v);
+    if (lane == 31) s_tot = wi;
   }
+  __syncthreads();
+  const uint4 pre = s_w[warp], ta = s_tot;
   const bool split_on = ta.y <= (uint32_t)part_cap;
   const uint32_t nparts = split_on ? ta.y : 0u, nsplit = split_on ? ta.z : 0u;
-  if (tid == 0) {
-    hdr->P = ta.x;
-    tile_off[ntiles] = ta.x;
-    hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
-    hdr->nsplit = nsplit;
-    hdr->next_item = 0u;
-    hdr->next_seg = 0u;
-  }
-  uint32_t run = pre.x + incl.x - sum.x, pb = pre.y + incl.y - sum.y, si = pre.z + incl.z - sum.z;
+  const uint32_t lite0 = nparts + (uint32_t)ntiles - nsplit - ta.w;
+  if (tid == 0) plan_header(hdr, tile_off, ntiles, ta, part_cap);
+  const uint4 ex = sub4(add4(pre, incl), sum);
+  uint32_t run = ex.x, pb = ex.y, si = ex.z, li = ex.w;
 #pragma unroll
   for (int k = 0; k < SCAN_PER; ++k) {
     const int64_t t = t0 + k;
     if (t >= ntiles) break;
-    plan_tile((uint32_t)t, c[k], run, pb, si, nparts, split_on, tile_off, items, split_tab, done);
+    plan_tile((uint32_t)t, c[k], run, pb, si, li, nparts, lite0, split_on, tile_off, items, split_tab, done);
   }
 }
 
@@ -470,8 +460,8 @@ void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header
     return;
   }
   const int nblk = (int)((ntiles + SCAN_TILES - 1) / SCAN_TILES);
-  k_scan_a<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (uint3*)partial);
-  k_scan_b<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (const uint3*)partial, nblk, tile_off, hdr, items, split_tab,
+  k_scan_a<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (uint4*)partial);
+  k_scan_b<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (const uint4*)partial, nblk, tile_off, hdr, items, split_tab,
                                          part_cap, done);
 }
 

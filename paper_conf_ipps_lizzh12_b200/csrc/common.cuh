@@ -51,7 +51,8 @@ struct Header {
   uint32_t nsplit;                     // tiles split into several items
   uint32_t next_item;                  // k_tile_sb: the next work item a persistent CTA takes (k_scan zeroes it)
   uint32_t next_seg;                   // k_t8sort: extra-segment slots of its bin-start table taken (zeroed likewise)
-  uint32_t pad[27];
+  uint32_t lite0;                      // first light item (whole tiles of <= LITE_MAX stars come last, plan.cuh)
+  uint32_t pad[26];
 };
 
 // k_tile work item: stars [jb, je) of tile `tile`'s list; aux = ITEM_WHOLE, or (split index << 12 | part index) for
@@ -60,6 +61,12 @@ struct WorkItem {
   uint32_t tile, jb, je, aux;
 };
 constexpr uint32_t ITEM_WHOLE = 0xFFFFFFFFu;
+// light tiles: a whole tile list of at most LITE_MAX stars (empty included).  The planner puts their items last
+// (Header::lite0 on); with k_tile_sb they go to k_tile_lite instead (tile_sb.cu).
+#ifndef SB_LITE_MAX
+#define SB_LITE_MAX 32
+#endif
+constexpr int LITE_MAX = SB_LITE_MAX;
 constexpr int SPLIT_LEN = 1024;        // a tile list longer than this is split into parts of <= SPLIT_LEN stars
 constexpr int PART_CAP = 512;          // partial-tile buffers (128 x 64 fp32 each, 16 MB) available per render
 
@@ -86,6 +93,7 @@ struct FrameParams {
   int32_t roi;           // 0: square ROI (reading R5); 1: the pixel circle inscribed in it (NEXT-3, reading R21)
   int32_t tile_impl;     // resolved by render_tiled: 1 the list kernel (tile.cu); 2 tile_sb.cu, 3 tile_ws.cu when R <= SB_MAXR (else tile.cu)
   int32_t bin_impl;      // 0: dbin.cu's deterministic binning when it applies; 1: always bin.cu's atomic-slot pipeline
+  int32_t lite;          // 1: k_tile_sb takes items [0, lite0) and k_tile_lite the light items [lite0, nitems)
   int32_t ndst;          // > 0: the tile kernels store every pixel into dst[0..ndst) instead of `out` (fused band exchange)
   float* dst[MAX_DST];   // band origins (row0 of each destination frame) -- local and peer-mapped frames
   const uint32_t* n_dev; // starsim_set_star_count: the star count in device memory (n is then the capacity), or NULL

@@ -13,6 +13,8 @@
 //                index, and it goes to tile_off[t] + C[t][c] + rank: every tile list holds its stars in ascending
 //                star index -- the unique CSR (reading R18), bit-exact, with no sort pass over the lists and no
 //                atomics on global memory.  (Groups are (tile, 2048-star block) pairs: a few stars each.)
+#include <algorithm>
+
 #include "common.cuh"
 #include "launch.h"
 #include "plan.cuh"
@@ -152,7 +154,8 @@ __device__ __forceinline__ uint32_t dp_block_scan(uint32_t v, uint32_t* s_w, uin
 
 struct DpSmem {
   uint32_t toff[DB_MAXT];        // step a2, computed by every CTA: the first list position of every tile
-  uint3 s_w3[DP_WARPS];
+  uint4 s_w4[DP_WARPS];
+  uint4 s_tot;
   uint32_t gstart[DB_MAXT + 1];  // per tile: pairs of the CTA, then the first position of the tile's group
   uint32_t cur[DB_MAXT];         // per tile: next free slot of its group; then the tile list position of the group
   uint16_t arr[DP_KEYS];          // the CTA's star indices grouped by tile (in arbitrary order inside a group)
@@ -180,56 +183,45 @@ __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restr
   static_assert(TPT * DP_THREADS == DB_MAXT, "tiles per thread");
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, cta = blockIdx.x;
   uint32_t c[TPT];
-  uint3 sum = make_uint3(0u, 0u, 0u);
+  uint4 sum = make_uint4(0u, 0u, 0u, 0u);
 #pragma unroll
   for (int k = 0; k < TPT; ++k) {
     const int t = tid * TPT + k;
     c[k] = t < ntiles ? __ldcg(&cnt[t]) : 0u;  // dense totals (k_dcolscan with cstride 1)
-    const uint32_t np = parts_of(c[k]);
-    sum = add3(sum, make_uint3(c[k], np, np ? 1u : 0u));
+    if (t < ntiles) sum = add4(sum, tile_counts(c[k]));
   }
-  const uint3 incl = warp_incl_scan3(sum, lane);
-  if (lane == 31) S.s_w3[warp] = incl;
+  const uint4 incl = warp_incl_scan4(sum, lane);
+  if (lane == 31) S.s_w4[warp] = incl;
   __syncthreads();
-  if (warp == 0) {  // exclusive scan of the warp sums; the total in the last slot's inclusive value
-    const uint3 v = lane < DP_WARPS ? S.s_w3[lane] : make_uint3(0u, 0u, 0u);
-    const uint3 wi = warp_incl_scan3(v, lane);
+  if (warp == 0) {  // exclusive scan of the warp sums; the total
+    const uint4 v = lane < DP_WARPS ? S.s_w4[lane] : make_uint4(0u, 0u, 0u, 0u);
+    const uint4 wi = warp_incl_scan4(v, lane);
     __syncwarp();
-    if (lane < DP_WARPS) S.s_w3[lane] = make_uint3(wi.x - v.x, wi.y - v.y, wi.z - v.z);
-    const uint3 ta = make_uint3(__shfl_sync(0xffffffffu, wi.x, 31), __shfl_sync(0xffffffffu, wi.y, 31),
-                                __shfl_sync(0xffffffffu, wi.z, 31));
-    if (lane == 0) {
-      S.gstart[0] = ta.x;  // borrowed for the totals until gstart is cleared after the next barrier
-      S.gstart[1] = ta.y;
-      S.gstart[2] = ta.z;
-    }
+    if (lane < DP_WARPS) S.s_w4[lane] = sub4(wi, v);
+    if (lane == 31) S.s_tot = wi;
   }
   __syncthreads();
-  const uint3 pre = S.s_w3[warp];
-  const uint3 ta = make_uint3(S.gstart[0], S.gstart[1], S.gstart[2]);
+  const uint4 pre = S.s_w4[warp];
+  const uint4 ta = S.s_tot;
   const bool split_on = ta.y <= (uint32_t)part_cap;
   const uint32_t nparts = split_on ? ta.y : 0u, nsplit = split_on ? ta.z : 0u;
-  uint32_t run = pre.x + incl.x - sum.x, pb = pre.y + incl.y - sum.y, si = pre.z + incl.z - sum.z;
-  if (cta == 0 && tid == 0) {
-    hdr->P = ta.x;
-    tile_off[ntiles] = ta.x;
-    hdr->nitems = nparts + (uint32_t)ntiles - nsplit;
-    hdr->nsplit = nsplit;
-    hdr->next_item = 0u;
-    hdr->next_seg = 0u;
-  }
+  const uint32_t lite0 = nparts + (uint32_t)ntiles - nsplit - ta.w;
+  const uint4 ex = sub4(add4(pre, incl), sum);
+  uint32_t run = ex.x, pb = ex.y, si = ex.z, li = ex.w;
+  if (cta == 0 && tid == 0) plan_header(hdr, tile_off, ntiles, ta, part_cap);
 #pragma unroll
   for (int k = 0; k < TPT; ++k) {
     const int t = tid * TPT + k;
     if (t >= ntiles) break;
     S.toff[t] = run;
     if (t % nCTA == cta) {
-      plan_tile((uint32_t)t, c[k], run, pb, si, nparts, split_on, tile_off, items, split_tab, done);
-    } else {
-      const uint32_t np = split_on ? parts_of(c[k]) : 0u;
-      run += c[k];
-      pb += np;
-      si += np ? 1u : 0u;
+      plan_tile((uint32_t)t, c[k], run, pb, si, li, nparts, lite0, split_on, tile_off, items, split_tab, done);
+    } else {  // the same prefix updates as plan_tile
+      const uint4 u = tile_counts(c[k]);
+      run += u.x;
+      pb += split_on ? u.y : 0u;
+      si += split_on ? u.z : 0u;
+      li += u.w;
     }
   }
   __syncthreads();
@@ -247,9 +239,10 @@ __global__ void __launch_bounds__(DP_THREADS, DP_MINB) k_dplace(const uint32_t* 
   const int tid = threadIdx.x, cta = blockIdx.x;
   const int64_t c0 = (int64_t)cta * DB_CTA;
   n = frame_n(n, fp);
-  const int live = dbin_live_ctas(n);
-  if (cta >= live) return;
-  dp_scan_tiles(S, cnt, ntiles, live, tile_off, hdr, items, split_tab, part_cap, done);
+  // step a2 is spread over every CTA of the grid (CTA c plans the tiles t = c mod gridDim.x; the grid has at least
+  // ntiles / 256 CTAs, so a sparse frame's plan is not one CTA's serial work); only the CTAs that hold stars go on
+  dp_scan_tiles(S, cnt, ntiles, (int)gridDim.x, tile_off, hdr, items, split_tab, part_cap, done);
+  if (cta >= dbin_live_ctas(n)) return;
   for (int t = tid; t <= ntiles; t += DP_THREADS) S.gstart[t] = 0u;
   uint32_t code[DP_SPT];
 #pragma unroll
@@ -339,9 +332,10 @@ void launch_dplace(const uint32_t* codes, int64_t n, const FrameParams& fp, cons
                    const uint32_t* cnt, uint32_t* tile_off, Header* hdr, WorkItem* items, uint2* split_tab,
                    int part_cap, uint32_t* done, uint32_t* ids, cudaStream_t st) {
   const int nc = dbin_ctas(n);
+  const int grid = std::max(nc, (ntiles + 255) / 256);  // planning CTAs (k_dplace)
   if (nc > 0)
-    k_dplace<<<nc, DP_THREADS, sizeof(DpSmem), st>>>(codes, n, fp, C, nc, ntiles, cnt, tile_off, hdr, items, split_tab,
-                                                      part_cap, done, ids);
+    k_dplace<<<grid, DP_THREADS, sizeof(DpSmem), st>>>(codes, n, fp, C, nc, ntiles, cnt, tile_off, hdr, items,
+                                                        split_tab, part_cap, done, ids);
 }
 
 }  // namespace starsim

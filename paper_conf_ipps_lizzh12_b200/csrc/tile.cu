@@ -62,40 +62,6 @@ static_assert(sizeof(float) * (GY_CAP * 16 + (RCAP * NSTRIPS + 1) * 8) >= sizeof
                   offsetof(TileSmem, gx) == sizeof(float) * GY_CAP * 16,
               "the gray epilogue stages the tile in gy + gx");
 
-// The fused output stage of k_tile from the staged fp32 tile (row-major TILE_W floats per row): thread t quantises
-// 4 consecutive pixels of a row (exactly as k_quantize, quant1) and stores them as one u8x4 / u16x4 word when the
-// row run is whole and aligned, else pixel by pixel.
-__device__ __forceinline__ void tile_store_gray_staged(const float* __restrict__ buf, const FrameParams& fp,
-                                                    void* __restrict__ out_, int Y0, int X0, int TWe, int THe) {
-  const float qmax = fp.obits == 8 ? 255.f : 65535.f;
-  for (int p = threadIdx.x * 4; p < TILE_W * TILE_H; p += TILE_THREADS * 4) {
-    const int r = p / TILE_W, c = p % TILE_W;
-    if (r >= THe || c >= TWe) continue;
-    const float4 v = *reinterpret_cast<const float4*>(buf + p);
-    const uint32_t g0 = quant1(v.x, qmax), g1 = quant1(v.y, qmax), g2 = quant1(v.z, qmax), g3 = quant1(v.w, qmax);
-    const int64_t pix = (int64_t)(Y0 + r) * fp.W + X0 + c;
-    if (fp.obits == 8) {
-      uint8_t* o = reinterpret_cast<uint8_t*>(out_) + pix;
-      if (fp.vec && c + 4 <= TWe) {
-        *reinterpret_cast<uint32_t*>(o) = g0 | g1 << 8 | g2 << 16 | g3 << 24;
-      } else {
-        if (c < TWe) o[0] = (uint8_t)g0;
-        if (c + 1 < TWe) o[1] = (uint8_t)g1;
-        if (c + 2 < TWe) o[2] = (uint8_t)g2;
-      }
-    } else {
-      uint16_t* o = reinterpret_cast<uint16_t*>(out_) + pix;
-      if (fp.vec && c + 4 <= TWe) {
-        *reinterpret_cast<uint2*>(o) = make_uint2(g0 | g1 << 16, g2 | g3 << 16);
-      } else {
-        if (c < TWe) o[0] = (uint16_t)g0;
-        if (c + 1 < TWe) o[1] = (uint16_t)g1;
-        if (c + 2 < TWe) o[2] = (uint16_t)g2;
-      }
-    }
-  }
-}
-
 constexpr uint32_t ZERO_GX = RCAP * NSTRIPS;
 constexpr uint32_t ZERO_ENT = ZERO_GX * 32u << 16;  // gy byte offset 0, all-zero strip slot
 
@@ -104,7 +70,9 @@ constexpr uint32_t ZERO_ENT = ZERO_GX * 32u << 16;  // gy byte offset 0, all-zer
 // directly; a part writes its 128 x 64 partial to part_buf, and the last part to finish (per-tile counter) sums the
 // parts in part order -- a fixed order, so the image stays deterministic.
 // ---------------------------------------------------------------------------------------------------------------
-template <bool INTEG>  // INTEG: the pixel-integrated PSF (NEXT-2) instead of the paper's point-sampled Eq. 2
+// INTEG: the pixel-integrated PSF (NEXT-2) instead of the paper's point-sampled Eq. 2; GRAY: the fused output stage
+// (u8 / u16 image) instead of the fp32 image
+template <bool INTEG, bool GRAY>
 #ifndef TILE_MINB_OPT
 #define TILE_MINB_OPT 3
 #endif
@@ -397,8 +365,8 @@ __global__ void __launch_bounds__(TILE_THREADS, TILE_MINB_OPT) k_tile(const uint
 
   // ======================= output: rows 16 B + hq + 4 i, columns 64 wx + 8 q .. +7 of the tile
   if (tile_reduce_parts<false>(acc, ld_volatile_item(items + item), split_tab, part_buf, done, B, wx, q, hq, &s_last)) {
-    if (fp.obits == 0) {
-      tile_store<false>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+    if (!GRAY) {
+      tile_store<false, 0>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
     } else {
       // fused output stage: the fp32 tile is staged in shared memory (the profile slots are free now) and quantised
       // from there by all threads, 4 pixels each -- the register-resident form would spill at 3 CTAs per SM
@@ -411,7 +379,10 @@ __global__ void __launch_bounds__(TILE_THREADS, TILE_MINB_OPT) k_tile(const uint
         d[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
       }
       __syncthreads();
-      tile_store_gray_staged(buf, fp, out_, Y0, X0, TWe, THe);
+      // the tile geometry again from the item (not held in registers across the accumulation)
+      const uint32_t t2 = ld_volatile_item(items + item).tile;
+      const int X2 = (int)(t2 % (uint32_t)fp.ntx) * TILE_W, Y2 = (int)(t2 / (uint32_t)fp.ntx) * TILE_H;
+      tile_store_gray_staged(buf, fp, out_, Y2, X2, min(TILE_W, fp.W - X2), min(TILE_H, fp.rows - Y2));
     }
   }
   __shared__ uint32_t s_next;
@@ -423,8 +394,10 @@ __global__ void __launch_bounds__(TILE_THREADS, TILE_MINB_OPT) k_tile(const uint
 }
 
 void init_tile_kernel() {
-  cudaFuncSetAttribute(k_tile<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
-  cudaFuncSetAttribute(k_tile<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
+  cudaFuncSetAttribute(k_tile<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
+  cudaFuncSetAttribute(k_tile<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
+  cudaFuncSetAttribute(k_tile<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
+  cudaFuncSetAttribute(k_tile<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
 }
 
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
@@ -441,12 +414,10 @@ void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp,
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
   const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)3 * num_sms);  // persistent, 3 CTAs per SM
-  if (fp.psf)
-    k_tile<true><<<(unsigned)grid, TILE_THREADS, sizeof(TileSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf,
-                                                                         done, hdr, seg_scratch);
-  else
-    k_tile<false><<<(unsigned)grid, TILE_THREADS, sizeof(TileSmem), st>>>(ids, rec, fp, out, items, split_tab,
-                                                                          part_buf, done, hdr, seg_scratch);
+  auto* k = fp.psf ? (fp.obits ? k_tile<true, true> : k_tile<true, false>)
+                   : (fp.obits ? k_tile<false, true> : k_tile<false, false>);
+  k<<<(unsigned)grid, TILE_THREADS, sizeof(TileSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr,
+                                                            seg_scratch);
 }
 
 }  // namespace starsim

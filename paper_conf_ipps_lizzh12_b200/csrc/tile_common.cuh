@@ -120,10 +120,11 @@ __device__ __forceinline__ WorkItem ld_volatile_item(const WorkItem* p) {
 // Write the lane's 4 rows x 8 columns of the tile (rows Y0 + lane_row(B, hq, i) of the band, columns col0 .. col0+7):
 // fp32, or (fused output stage, NEXT-1) the gray value of each pixel exactly as k_quantize computes it from the same
 // fp32 sum, as u8 / u16.  Coalesced: the 8 lane groups of a warp store 8 adjacent 8-pixel runs of a row.
-template <bool CONTIG>
+template <bool CONTIG, int OB = -1>  // OB: the output bits when fixed at compile time (0, 8, 16), -1: fp.obits
 __device__ __forceinline__ void tile_store_one(const float2 (&acc)[4][4], const FrameParams& fp, void* __restrict__ out_,
                                            int Y0, int col0, int B, int hq) {
-  if (fp.obits == 0) {
+  const int obits = OB >= 0 ? OB : fp.obits;
+  if (obits == 0) {
     float* out = reinterpret_cast<float*>(out_);
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
@@ -142,7 +143,7 @@ __device__ __forceinline__ void tile_store_one(const float2 (&acc)[4][4], const 
       }
     }
   } else {
-    const float qmax = fp.obits == 8 ? 255.f : 65535.f;
+    const float qmax = obits == 8 ? 255.f : 65535.f;
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
       const int row = Y0 + lane_row<CONTIG>(B, hq, i);
@@ -154,7 +155,7 @@ __device__ __forceinline__ void tile_store_one(const float2 (&acc)[4][4], const 
         g[2 * k + 1] = quant1(acc[i][k].y, qmax);
       }
       const int64_t pix = (int64_t)row * fp.W + col0;
-      if (fp.obits == 8) {
+      if (obits == 8) {
         uint8_t* o = reinterpret_cast<uint8_t*>(out_) + pix;
         if (fp.vec && col0 + 8 <= fp.W) {
           *reinterpret_cast<uint2*>(o) = make_uint2(g[0] | g[1] << 8 | g[2] << 16 | g[3] << 24,
@@ -180,15 +181,49 @@ __device__ __forceinline__ void tile_store_one(const float2 (&acc)[4][4], const 
 }
 
 
+// The fused output stage (NEXT-1) from an fp32 tile staged in shared memory (row-major TILE_W floats per row): thread t quantises
+// 4 consecutive pixels of a row (exactly as k_quantize, quant1) and stores them as one u8x4 / u16x4 word when the
+// row run is whole and aligned, else pixel by pixel.
+__device__ __forceinline__ void tile_store_gray_staged(const float* __restrict__ buf, const FrameParams& fp,
+                                                    void* __restrict__ out_, int Y0, int X0, int TWe, int THe) {
+  const float qmax = fp.obits == 8 ? 255.f : 65535.f;
+  for (int p = threadIdx.x * 4; p < TILE_W * TILE_H; p += TILE_THREADS * 4) {
+    const int r = p / TILE_W, c = p % TILE_W;
+    if (r >= THe || c >= TWe) continue;
+    const float4 v = *reinterpret_cast<const float4*>(buf + p);
+    const uint32_t g0 = quant1(v.x, qmax), g1 = quant1(v.y, qmax), g2 = quant1(v.z, qmax), g3 = quant1(v.w, qmax);
+    const int64_t pix = (int64_t)(Y0 + r) * fp.W + X0 + c;
+    if (fp.obits == 8) {
+      uint8_t* o = reinterpret_cast<uint8_t*>(out_) + pix;
+      if (fp.vec && c + 4 <= TWe) {
+        *reinterpret_cast<uint32_t*>(o) = g0 | g1 << 8 | g2 << 16 | g3 << 24;
+      } else {
+        if (c < TWe) o[0] = (uint8_t)g0;
+        if (c + 1 < TWe) o[1] = (uint8_t)g1;
+        if (c + 2 < TWe) o[2] = (uint8_t)g2;
+      }
+    } else {
+      uint16_t* o = reinterpret_cast<uint16_t*>(out_) + pix;
+      if (fp.vec && c + 4 <= TWe) {
+        *reinterpret_cast<uint2*>(o) = make_uint2(g0 | g1 << 16, g2 | g3 << 16);
+      } else {
+        if (c < TWe) o[0] = (uint16_t)g0;
+        if (c + 1 < TWe) o[1] = (uint16_t)g1;
+        if (c + 2 < TWe) o[2] = (uint16_t)g2;
+      }
+    }
+  }
+}
+
 // The epilogue: into `out_`, or (fused band exchange) into each of the fp.ndst destination frames.
-template <bool CONTIG>
+template <bool CONTIG, int OB = -1>
 __device__ __forceinline__ void tile_store(const float2 (&acc)[4][4], const FrameParams& fp, void* __restrict__ out_,
                                            int Y0, int col0, int B, int hq) {
   if (fp.ndst == 0) {
-    tile_store_one<CONTIG>(acc, fp, out_, Y0, col0, B, hq);
+    tile_store_one<CONTIG, OB>(acc, fp, out_, Y0, col0, B, hq);
     return;
   }
-  for (int g = 0; g < fp.ndst; ++g) tile_store_one<CONTIG>(acc, fp, fp.dst[g], Y0, col0, B, hq);
+  for (int g = 0; g < fp.ndst; ++g) tile_store_one<CONTIG, OB>(acc, fp, fp.dst[g], Y0, col0, B, hq);
 }
 
 }  // namespace starsim

@@ -101,7 +101,8 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? SB_MINB_CIRC : SB_MINB) k
   // profiles are done, its first star ids before the last chunk's accumulation and its records after it: the
   // latency of starting a tile hides behind the previous tile's work.
   __shared__ uint32_t s_next;
-  const uint32_t nitems = __ldcg(&hdr->nitems);
+  // with k_tile_lite (fp.lite) this kernel takes the items before the light ones
+  const uint32_t nitems = fp.lite ? __ldcg(&hdr->lite0) : __ldcg(&hdr->nitems);
   uint32_t item = blockIdx.x;
   if (item >= nitems) return;
   WorkItem wi = items[item];
@@ -405,6 +406,199 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? SB_MINB_CIRC : SB_MINB) k
   }  // work loop
 }
 
+
+// ---------------------------------------------------------------------------------------------------------------
+// k_tile_lite: the light items (whole tiles of at most LITE_MAX stars, empty ones included: the planner puts them
+// last, from Header::lite0 on), one CTA per item, many CTAs per SM -- with k_tile_sb, whose persistent CTAs take the
+// items before lite0.  No slots and no per-block ranges: the tile's stars, sorted by corner bin exactly as a chunk of
+// k_tile_sb is (stable: corner bin, then list order), are walked by every warp whose 64 x 16 region the ROI meets,
+// and each lane evaluates its own 4 row and 8 column factors with the very operations of k_tile_sb's slot
+// preparation (same roundings, same zero masks, same circle mask) and adds them in that order: the same per-pixel
+// sums, bit for bit, as k_tile_sb (and k_tile_ws) give the tile -- only cheaper to start (the sparse-frame floor,
+// DESIGN.md §9).  Same lane layout and epilogue (tile_store<true>).
+// ---------------------------------------------------------------------------------------------------------------
+#ifndef LITE_MINB
+#define LITE_MINB 3
+#endif
+template <bool INTEG, bool CIRC, int OB>  // OB: output bits (0: fp32 image, 8 / 16: the fused output stage)
+__global__ void __launch_bounds__(TILE_THREADS, LITE_MINB) k_tile_lite(const uint32_t* __restrict__ ids,
+                                                                      const StarRec* __restrict__ rec, FrameParams fp,
+                                                                      void* __restrict__ out_,
+                                                                      const WorkItem* __restrict__ items,
+                                                                      const Header* __restrict__ hdr) {
+  __shared__ uint32_t lkey[LITE_MAX > 0 ? LITE_MAX : 1];
+  __shared__ float4 lrec[LITE_MAX > 0 ? LITE_MAX : 1];
+  __shared__ uint32_t llo[LITE_MAX > 0 ? LITE_MAX : 1];
+  const uint32_t item = __ldcg(&hdr->lite0) + blockIdx.x;
+  if (item >= __ldcg(&hdr->nitems)) return;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
+  const int Q = 8 * wx + q;
+  const int swz = (Q >> 2) & 1;
+  const float sk = fp.sk;
+  const WorkItem wi = items[item];
+  const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
+  const int X0 = tx * TILE_W, Y0 = ty * TILE_H, IY0 = fp.row0 + Y0;
+  const int TWe = min(TILE_W, fp.W - X0), THe = min(TILE_H, fp.rows - Y0);
+  const int n = (int)(wi.je - wi.jb);  // <= LITE_MAX
+  float2 acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
+  if (n > 0) {
+    // sort: thread t = list star t; its corner bin (k_tile_sb's key) and its rank (corner bin, then list order)
+    StarRec r = {};
+    if (tid < n) r = rec[__ldg(&ids[wi.jb + tid])];
+    uint32_t key = SB_NBIN, lo2 = 0u;
+    if (tid < n) {
+      const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
+      lo2 = (uint32_t)(lx & 0xFFFF) | (uint32_t)ly << 16;
+      const int c0 = max(lx, 0), c1 = min(lx + fp.R - 1, TWe - 1);
+      const int r0 = max(ly, 0), r1 = min(ly + fp.R - 1, THe - 1);
+      if (c0 <= c1 && r0 <= r1) key = (uint32_t)((ly < 0 ? 0 : 1 + (r0 >> 4)) * SB_NSK + (lx < 0 ? 0 : 1 + (c0 >> 3)));
+      lkey[tid] = key;
+    }
+    __syncthreads();
+    if (tid < n) {
+      uint32_t rank = 0;
+      for (int u = 0; u < n; ++u) {
+        const uint32_t ku = lkey[u];
+        rank += (ku < key || (ku == key && u < tid)) ? 1u : 0u;
+      }
+      lrec[rank] = make_float4(r.x - (float)X0, r.y - (float)IY0, r.s, __uint_as_float(key));  // exact
+      llo[rank] = lo2;
+    }
+    __syncthreads();
+    const float2 sk2 = make_float2(sk, sk);
+    for (int k = 0; k < n; ++k) {
+      const float4 st = lrec[k];
+      const uint32_t sk_key = __float_as_uint(st.w);
+      if (sk_key >= (uint32_t)SB_NBIN) continue;
+      const uint32_t lo = llo[k];
+      const int lx = (int)(int16_t)(lo & 0xFFFFu), ly = (int)(int16_t)(lo >> 16);
+      const int c0 = max(lx, 0), c1 = min(lx + fp.R - 1, TWe - 1);
+      const int r0 = max(ly, 0), r1 = min(ly + fp.R - 1, THe - 1);
+      // the warp's 64 x 16 region (uniform branch)
+      if (r1 < 16 * B || r0 > 16 * B + 15 || c1 < 64 * wx || c0 > 64 * wx + 63) continue;
+      const int b0 = (int)(sk_key / SB_NSK) - 1, q0 = (int)(sk_key % SB_NSK) - 1;
+      const float xr = st.x, yr = st.y;
+      // row factors of rows 16 B + 4 hq + i: quad w = 4 (B - b0) + hq of the star's two bands (slot preparation)
+      float gyv[4];
+      {
+        const int ra0 = r0 - 16 * b0, rb0 = r1 - 16 * b0;
+        const uint32_t m0 = (0xFFFFFFFFu >> (31 - min(rb0, 31))) & (0xFFFFFFFFu << ra0);
+        const int w = 4 * (B - b0) + hq;
+        const uint32_t m = (w >= 0 && w < 8) ? m0 >> (4 * w) : 0u;
+        const float bf0 = (float)(16 * b0) - yr;
+        const float bf = bf0 + (float)(4 * w);
+        if (!INTEG) {
+          const float2 s2 = make_float2(st.z, st.z);
+          const float2 bb = make_float2(bf, bf);
+#pragma unroll
+          for (int i = 0; i < 4; i += 2) {
+            float2 d = __fadd2_rn(bb, make_float2((float)i, (float)(i + 1)));
+            d = __fmul2_rn(d, sk2);
+            d = __fmul2_rn(d, make_float2(-d.x, -d.y));
+            const float2 e = __fmul2_rn(make_float2(ex2_approx(d.x), ex2_approx(d.y)), s2);
+            gyv[i] = (m >> i) & 1u ? e.x : 0.f;
+            gyv[i + 1] = (m >> (i + 1)) & 1u ? e.y : 0.f;
+          }
+        } else {
+          float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const float tn = (bf + (float)i + 0.5f) * fp.kint, en = edge_erfc(tn);
+            gyv[i] = (m >> i) & 1u ? st.z * pix_mass(t, e, tn, en) : 0.f;
+            t = tn;
+            e = en;
+          }
+        }
+      }
+      // column factors of strip Q (one of the star's strips q0 .. q0 + 2, else zero) in the lane's load order:
+      // slot p holds column 8 Q + pp, pp = (p + 4 swz) & 7 (the same operations on the same operands as k_tile_sb)
+      float gxv[8];
+      {
+        const int rel = 8 * Q;
+        const int lo_ = max(c0 - rel, 0), hi = min(c1 - rel, 7);
+        const uint32_t m = (Q >= q0 && Q <= q0 + 2 && hi >= lo_) ? ((0xFFu >> (7 - hi)) & (0xFFu << lo_)) : 0u;
+        const float bf = (float)rel - xr;
+        if (!INTEG) {
+#pragma unroll
+          for (int p = 0; p < 8; p += 2) {
+            const int pp = (p + 4 * swz) & 7;
+            float2 d = __fmul2_rn(__fadd2_rn(make_float2(bf, bf), make_float2((float)pp, (float)(pp + 1))), sk2);
+            d = __fmul2_rn(d, make_float2(-d.x, -d.y));
+            gxv[p] = (m >> pp) & 1u ? ex2_approx(d.x) : 0.f;
+            gxv[p + 1] = (m >> (pp + 1)) & 1u ? ex2_approx(d.y) : 0.f;
+          }
+        } else {
+          float v[8];
+          float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
+#pragma unroll
+          for (int p = 0; p < 8; ++p) {
+            const float tn = (bf + (float)p + 0.5f) * fp.kint, en = edge_erfc(tn);
+            v[p] = (m >> p) & 1u ? pix_mass(t, e, tn, en) : 0.f;
+            t = tn;
+            e = en;
+          }
+#pragma unroll
+          for (int p = 0; p < 8; ++p) gxv[p] = swz ? v[(p + 4) & 7] : v[p];
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const float2 gg = make_float2(gyv[i], gyv[i]);
+        if (CIRC) {
+          const int RR = fp.R * fp.R, R1 = fp.R - 1;
+          const int v = 2 * (16 * B + 4 * hq + i - ly) - R1;
+          const int thr = RR - v * v;
+          float gm[8];
+#pragma unroll
+          for (int p = 0; p < 8; ++p) {
+            const int u = 2 * (8 * Q + ((p + 4 * swz) & 7) - lx) - R1;
+            gm[p] = u * u <= thr ? gxv[p] : 0.f;
+          }
+          acc[i][0] = __ffma2_rn(gg, make_float2(gm[0], gm[1]), acc[i][0]);
+          acc[i][1] = __ffma2_rn(gg, make_float2(gm[2], gm[3]), acc[i][1]);
+          acc[i][2] = __ffma2_rn(gg, make_float2(gm[4], gm[5]), acc[i][2]);
+          acc[i][3] = __ffma2_rn(gg, make_float2(gm[6], gm[7]), acc[i][3]);
+        } else {
+          acc[i][0] = __ffma2_rn(gg, make_float2(gxv[0], gxv[1]), acc[i][0]);
+          acc[i][1] = __ffma2_rn(gg, make_float2(gxv[2], gxv[3]), acc[i][1]);
+          acc[i][2] = __ffma2_rn(gg, make_float2(gxv[4], gxv[5]), acc[i][2]);
+          acc[i][3] = __ffma2_rn(gg, make_float2(gxv[6], gxv[7]), acc[i][3]);
+        }
+      }
+    }
+  }
+  // the lanes with swz = 1 hold columns 4-7 of their strip in acc[i][0..1] (k_tile_sb's load order)
+  if (swz) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float2 t0 = acc[i][0], t1 = acc[i][1];
+      acc[i][0] = acc[i][2];
+      acc[i][1] = acc[i][3];
+      acc[i][2] = t0;
+      acc[i][3] = t1;
+    }
+  }
+  if (OB == 0) {
+    tile_store<true, 0>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+  } else {
+    // the gray image: staged in shared memory and quantised from there (the register-resident form spills here)
+    __shared__ __align__(16) float gbuf[OB ? TILE_W * TILE_H : 4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      float4* d = reinterpret_cast<float4*>(gbuf + lane_row<true>(B, hq, i) * TILE_W + 64 * wx + 8 * q);
+      d[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
+      d[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
+    }
+    __syncthreads();
+    tile_store_gray_staged(gbuf, fp, out_, Y0, X0, TWe, THe);
+  }
+}
+
 #ifdef STARSIM_SB_TIMING
 extern "C" int starsim_debug_sb_timing(double* out6, int reset) {
   unsigned long long h[6];
@@ -437,6 +631,16 @@ void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& 
                    : (fp.roi ? k_tile_sb<false, true> : k_tile_sb<false, false>);
   k<<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr,
                                                           seg_scratch);
+  if (fp.lite) {  // the light items: one CTA each (at most one per tile; the surplus CTAs return at once)
+    using KL = void (*)(const uint32_t*, const StarRec*, FrameParams, void*, const WorkItem*, const Header*);
+    static const KL kls[2][2][3] = {
+        {{k_tile_lite<false, false, 0>, k_tile_lite<false, false, 8>, k_tile_lite<false, false, 16>},
+         {k_tile_lite<false, true, 0>, k_tile_lite<false, true, 8>, k_tile_lite<false, true, 16>}},
+        {{k_tile_lite<true, false, 0>, k_tile_lite<true, false, 8>, k_tile_lite<true, false, 16>},
+         {k_tile_lite<true, true, 0>, k_tile_lite<true, true, 8>, k_tile_lite<true, true, 16>}}};
+    const KL kl = kls[fp.psf ? 1 : 0][fp.roi ? 1 : 0][fp.obits == 8 ? 1 : fp.obits == 16 ? 2 : 0];
+    kl<<<(unsigned)ntiles, TILE_THREADS, 0, st>>>(ids, rec, fp, out, items, hdr);
+  }
 }
 
 }  // namespace starsim

@@ -470,10 +470,15 @@ def test_tile_kernels_agree_within_rounding(torch_dev):
 
 @pytest.mark.parametrize("psf", ["point", "integrated"])
 @pytest.mark.parametrize("W,H,n,R,seed", [(1000, 700, 60000, 15, 24), (4096, 4096, 1000000, 15, 1),
-                                          (301, 177, 3000, 17, 5), (700, 500, 0, 9, 6)])
+                                          (301, 177, 3000, 17, 5), (700, 500, 0, 9, 6),
+                                          (4096, 4096, 2000, 15, 7), (2048, 2048, 20000, 9, 8),
+                                          (1024, 1024, 1000, 5, 9), (515, 301, 700, 17, 10), (256, 256, 300, 1, 11),
+                                          (640, 384, 2500, 12, 12)])
 def test_ws_equals_sb_bitwise(torch_dev, psf, W, H, n, R, seed):
     """The warp-specialised kernel (auto) sums every pixel in k_tile_sb's order: the images are identical bit for bit,
-    also with heavy tiles split into parts (the clustered field) and with the integrated PSF."""
+    also with heavy tiles split into parts (the clustered field) and with the integrated PSF.  The sparse fields put
+    most tiles on k_tile_sb's light-item path (lists of <= SB_LITE_MAX stars, evaluated per lane without slots),
+    which must give the chunked path's bits exactly (ws has no light path)."""
     torch, dev = torch_dev
     from paper_conf_ipps_lizzh12_b200 import Context
     f = synth.uniform_field(n, W, H, seed=seed, mag_hi=15.0)
