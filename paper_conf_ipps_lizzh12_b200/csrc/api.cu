@@ -198,6 +198,7 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   fp.lite = 0;
   fp.obits = 0;
   fp.vec = 0;
+  fp.vec32 = 0;
   fp.kint = (float)(1.0 / (std::sqrt(2.0) * s));
   if (psf) fp.s_scale = (double)gain;  // the pixel masses of the integrated PSF are already normalised
   return fp;
@@ -284,7 +285,7 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
         c, 3, st,
         [&] {
           launch_tile(ids, rec, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p, part_cap,
-                      done, hdr, c->num_sms, st, (float*)c->segs.p);
+                      done, hdr, c->num_sms, st, (float*)c->segs.p, tile_off);
         },
         fp.lite ? 2 : 1);
   }
@@ -316,7 +317,14 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   fp.bin_impl = c->bin_impl;
   fp.n_dev = c->n_dev;
   // k_tile_sb hands the light tiles to k_tile_lite (same bits; tile_sb.cu)
-  fp.lite = (fp.tile_impl == STARSIM_TILE_SB && R <= SB_MAXR && LITE_MAX > 0) ? 1 : 0;
+  // (worth its second launch on frames of many mostly-light tiles: measured, DESIGN.md §9 -- C3 with 1K / 16K
+  // stars gains 4-6 us; C1, C2 and fig2, with few tiles or ~50 stars per tile, lose 2-8 us)
+  {
+    const double per_tile = (double)n * (TILE_W + R - 1) * (TILE_H + R - 1) / ((double)W * (rows > 0 ? rows : 1));
+    const int64_t nt = (int64_t)fp.ntx * fp.nty;
+    fp.lite = (fp.tile_impl == STARSIM_TILE_SB && R <= SB_MAXR && LITE_MAX > 0 && per_tile <= LITE_AUTO_PER_TILE &&
+               nt >= LITE_AUTO_TILES) ? 1 : 0;
+  }
   // one vector store per 8-pixel run: 32 B (fp32) / 8 B (u8) / 16 B (u16); rows must keep that alignment
   const int vb = obits == 8 ? 8 : 16;
   bool aligned = ((uintptr_t)out % vb) == 0;
@@ -326,6 +334,9 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
     aligned = aligned && ((uintptr_t)fp.dst[i] % vb) == 0;
   }
   fp.vec = ((W * (obits ? obits / 8 : 4)) % vb == 0 && aligned) ? 1 : 0;
+  bool al32 = ((uintptr_t)out % 32) == 0;
+  for (int i = 0; i < ndst; ++i) al32 = al32 && ((uintptr_t)fp.dst[i] % 32) == 0;
+  fp.vec32 = (obits == 0 && (W * 4) % 32 == 0 && al32) ? 1 : 0;
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   const int tps = tiles_per_axis(R, TILE_W, fp.ntx) * tiles_per_axis(R, TILE_H, fp.nty);
   const int64_t pmax = n * (int64_t)tps;

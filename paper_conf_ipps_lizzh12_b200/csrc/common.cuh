@@ -67,6 +67,8 @@ constexpr uint32_t ITEM_WHOLE = 0xFFFFFFFFu;
 #define SB_LITE_MAX 32
 #endif
 constexpr int LITE_MAX = SB_LITE_MAX;
+constexpr double LITE_AUTO_PER_TILE = 16.0;  // k_tile_lite is launched when the expected list per tile is <= this
+constexpr int64_t LITE_AUTO_TILES = 1024;    // ... and the frame / band has at least this many tiles
 constexpr int SPLIT_LEN = 1024;        // a tile list longer than this is split into parts of <= SPLIT_LEN stars
 constexpr int PART_CAP = 512;          // partial-tile buffers (128 x 64 fp32 each, 16 MB) available per render
 
@@ -88,6 +90,7 @@ struct FrameParams {
   int32_t R;
   int32_t ntx, nty;      // tiles over the band
   int32_t vec;           // 1 if every 8-pixel run of an out row is aligned for one vector store
+  int32_t vec32;         // fp32 image: 1 if every 8-pixel run is 32-B aligned (one 256-bit store, st.global.v8)
   int32_t obits;         // 0: fp32 image; 8 / 16: gray values quantised in the epilogue (u8 / u16 image)
   int32_t psf;           // 0: Eq. 2 point-sampled (the paper); 1: Eq. 2 integrated over the pixel square (NEXT-2)
   int32_t roi;           // 0: square ROI (reading R5); 1: the pixel circle inscribed in it (NEXT-3, reading R21)

@@ -34,10 +34,10 @@ void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, in
                       cudaStream_t st);
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                 cudaStream_t st, float* seg_scratch);
+                 cudaStream_t st, float* seg_scratch, const uint32_t* tile_off);
 void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                    cudaStream_t st, float* seg_scratch);
+                    cudaStream_t st, float* seg_scratch, const uint32_t* tile_off);
 void launch_tile_ws(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
                     cudaStream_t st, float* seg_scratch);

@@ -402,13 +402,14 @@ void init_tile_kernel() {
 
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                 cudaStream_t st, float* seg_scratch) {
+                 cudaStream_t st, float* seg_scratch, const uint32_t* tile_off) {
   if (fp.R <= SB_MAXR && fp.tile_impl == 3) {
     launch_tile_ws(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st, seg_scratch);
     return;
   }
   if (fp.R <= SB_MAXR && fp.tile_impl == 2) {
-    launch_tile_sb(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st, seg_scratch);
+    launch_tile_sb(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st, seg_scratch,
+                   tile_off);
     return;
   }
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;

@@ -131,7 +131,13 @@ __device__ __forceinline__ void tile_store_one(const float2 (&acc)[4][4], const 
       const int row = Y0 + lane_row<CONTIG>(B, hq, i);  // band-relative
       if (row >= fp.rows || col0 >= fp.W) continue;
       float* o = out + (int64_t)row * fp.W + col0;
-      if (fp.vec && col0 + 8 <= fp.W) {
+      if (fp.vec32 && col0 + 8 <= fp.W) {
+        // the lane's 8 pixels of the row as one 256-bit store: one whole 32-B sector per lane
+        asm volatile("st.global.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(o), "f"(acc[i][0].x),
+                     "f"(acc[i][0].y), "f"(acc[i][1].x), "f"(acc[i][1].y), "f"(acc[i][2].x), "f"(acc[i][2].y),
+                     "f"(acc[i][3].x), "f"(acc[i][3].y)
+                     : "memory");
+      } else if (fp.vec && col0 + 8 <= fp.W) {
         reinterpret_cast<float4*>(o)[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
         reinterpret_cast<float4*>(o)[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
       } else {

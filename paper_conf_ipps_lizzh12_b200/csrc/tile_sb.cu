@@ -418,29 +418,29 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? SB_MINB_CIRC : SB_MINB) k
 // DESIGN.md §9).  Same lane layout and epilogue (tile_store<true>).
 // ---------------------------------------------------------------------------------------------------------------
 #ifndef LITE_MINB
-#define LITE_MINB 3
+#define LITE_MINB 4
 #endif
 template <bool INTEG, bool CIRC, int OB>  // OB: output bits (0: fp32 image, 8 / 16: the fused output stage)
-__global__ void __launch_bounds__(TILE_THREADS, LITE_MINB) k_tile_lite(const uint32_t* __restrict__ ids,
+__global__ void __launch_bounds__(TILE_THREADS, CIRC ? 3 : LITE_MINB) k_tile_lite(const uint32_t* __restrict__ ids,
                                                                       const StarRec* __restrict__ rec, FrameParams fp,
                                                                       void* __restrict__ out_,
-                                                                      const WorkItem* __restrict__ items,
-                                                                      const Header* __restrict__ hdr) {
+                                                                      const uint32_t* __restrict__ tile_off) {
   __shared__ uint32_t lkey[LITE_MAX > 0 ? LITE_MAX : 1];
   __shared__ float4 lrec[LITE_MAX > 0 ? LITE_MAX : 1];
   __shared__ uint32_t llo[LITE_MAX > 0 ? LITE_MAX : 1];
-  const uint32_t item = __ldcg(&hdr->lite0) + blockIdx.x;
-  if (item >= __ldcg(&hdr->nitems)) return;
+  // CTA b takes tile b if its list is light (heavy tiles are k_tile_sb's items): one load less than the item list
+  const uint32_t tile = blockIdx.x;
+  const uint32_t jb = __ldg(&tile_off[tile]), je = __ldg(&tile_off[tile + 1]);
+  if (je - jb > (uint32_t)LITE_MAX) return;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
   const int Q = 8 * wx + q;
   const int swz = (Q >> 2) & 1;
   const float sk = fp.sk;
-  const WorkItem wi = items[item];
-  const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
+  const int tx = (int)(tile % (uint32_t)fp.ntx), ty = (int)(tile / (uint32_t)fp.ntx);
   const int X0 = tx * TILE_W, Y0 = ty * TILE_H, IY0 = fp.row0 + Y0;
   const int TWe = min(TILE_W, fp.W - X0), THe = min(TILE_H, fp.rows - Y0);
-  const int n = (int)(wi.je - wi.jb);  // <= LITE_MAX
+  const int n = (int)(je - jb);  // <= LITE_MAX
   float2 acc[4][4];
 #pragma unroll
   for (int i = 0; i < 4; ++i)
@@ -449,7 +449,7 @@ __global__ void __launch_bounds__(TILE_THREADS, LITE_MINB) k_tile_lite(const uin
   if (n > 0) {
     // sort: thread t = list star t; its corner bin (k_tile_sb's key) and its rank (corner bin, then list order)
     StarRec r = {};
-    if (tid < n) r = rec[__ldg(&ids[wi.jb + tid])];
+    if (tid < n) r = rec[__ldg(&ids[jb + tid])];
     uint32_t key = SB_NBIN, lo2 = 0u;
     if (tid < n) {
       const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
@@ -622,7 +622,7 @@ void init_tile_sb_kernel() {
 
 void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                    cudaStream_t st, float* seg_scratch) {
+                    cudaStream_t st, float* seg_scratch, const uint32_t* tile_off) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
   const int64_t grid =
@@ -632,14 +632,14 @@ void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& 
   k<<<(unsigned)grid, TILE_THREADS, sizeof(SbSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr,
                                                           seg_scratch);
   if (fp.lite) {  // the light items: one CTA each (at most one per tile; the surplus CTAs return at once)
-    using KL = void (*)(const uint32_t*, const StarRec*, FrameParams, void*, const WorkItem*, const Header*);
+    using KL = void (*)(const uint32_t*, const StarRec*, FrameParams, void*, const uint32_t*);
     static const KL kls[2][2][3] = {
         {{k_tile_lite<false, false, 0>, k_tile_lite<false, false, 8>, k_tile_lite<false, false, 16>},
          {k_tile_lite<false, true, 0>, k_tile_lite<false, true, 8>, k_tile_lite<false, true, 16>}},
         {{k_tile_lite<true, false, 0>, k_tile_lite<true, false, 8>, k_tile_lite<true, false, 16>},
          {k_tile_lite<true, true, 0>, k_tile_lite<true, true, 8>, k_tile_lite<true, true, 16>}}};
     const KL kl = kls[fp.psf ? 1 : 0][fp.roi ? 1 : 0][fp.obits == 8 ? 1 : fp.obits == 16 ? 2 : 0];
-    kl<<<(unsigned)ntiles, TILE_THREADS, 0, st>>>(ids, rec, fp, out, items, hdr);
+    kl<<<(unsigned)ntiles, TILE_THREADS, 0, st>>>(ids, rec, fp, out, tile_off);
   }
 }
 
