@@ -229,7 +229,14 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
     // deterministic counting sort (dbin.cu): no memset, no atomics on global counters, no per-tile sort
     // (step a2 runs inside k_dplace; an empty catalogue has no k_dplace, so k_scan plans its all-empty tiles)
     uint32_t* C = (uint32_t*)c->cmat.p;
-    if (n > 0) {
+    if (n > 0 && dsmall_ok(n)) {
+      // at most DB_CTA stars: the whole binning in one CTA, one launch (k_dsmall)
+      timed(c, 0, st, [&] {
+        launch_dsmall(x, y, mag, n, fp, rec, (int)ntiles, tile_off, hdr, (WorkItem*)c->items.p,
+                      (uint2*)c->split_tab.p, part_cap, done, ids, st);
+      });
+      if ((rc = check_launch(c, "k_dsmall"))) return rc;
+    } else if (n > 0) {
       timed(c, 0, st, [&] { launch_dcount(x, y, mag, n, fp, rec, (uint32_t*)c->codes.p, C, (int)ntiles, st); });
       if ((rc = check_launch(c, "k_dcount"))) return rc;
       timed(c, 2, st, [&] { launch_dcolscan(C, n, (int)ntiles, cnt, 1, fp.n_dev, st); });  // dense totals for k_dplace

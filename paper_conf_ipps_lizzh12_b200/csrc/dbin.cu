@@ -175,6 +175,7 @@ __device__ __forceinline__ int box_tile(uint32_t code, int e, int ntx) {
 // Step a2 inside k_dplace (no separate scan launch): every CTA scans the DB_MAXT tile totals k_dcolscan wrote (2 per
 // thread) into S.toff, and CTA c writes tile_off, the work items, the split table and the header for the tiles
 // t = c mod nCTA -- the same values k_scan_one computes (plan_tile).
+template <bool SMEM_CNT = false>  // counts in shared memory (k_dsmall) instead of k_dcolscan's global totals
 __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restrict__ cnt, int ntiles, int nCTA,
                                               uint32_t* __restrict__ tile_off, Header* hdr,
                                               WorkItem* __restrict__ items, uint2* __restrict__ split_tab,
@@ -187,7 +188,7 @@ __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restr
 #pragma unroll
   for (int k = 0; k < TPT; ++k) {
     const int t = tid * TPT + k;
-    c[k] = t < ntiles ? __ldcg(&cnt[t]) : 0u;  // dense totals (k_dcolscan with cstride 1)
+    c[k] = t < ntiles ? (SMEM_CNT ? cnt[t] : __ldcg(&cnt[t])) : 0u;  // dense totals (k_dcolscan, cstride 1)
     if (t < ntiles) sum = add4(sum, tile_counts(c[k]));
   }
   const uint4 incl = warp_incl_scan4(sum, lane);
@@ -227,29 +228,15 @@ __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restr
   __syncthreads();
 }
 
-__global__ void __launch_bounds__(DP_THREADS, DP_MINB) k_dplace(const uint32_t* __restrict__ codes, int64_t n, FrameParams fp,
-                                                       const uint32_t* __restrict__ C, int nCTA, int ntiles,
-                                                       const uint32_t* __restrict__ cnt, uint32_t* __restrict__ tile_off,
-                                                       Header* hdr, WorkItem* __restrict__ items,
-                                                       uint2* __restrict__ split_tab, int part_cap,
-                                                       uint32_t* __restrict__ done, uint32_t* __restrict__ ids) {
-  static_assert(TILE_W == 128 && TILE_H == 64, "tile boxes span at most 2 x 2 tiles for R <= DB_MAXR");
-  extern __shared__ __align__(16) unsigned char dsm_raw[];
-  DpSmem& S = *reinterpret_cast<DpSmem*>(dsm_raw);
+// Steps a3-a4 of k_dplace for the CTA's stars (codes in registers, star i = blockIdx.x DB_CTA + tid + k DP_THREADS):
+// group the pairs by tile in shared memory, rank each in its group by star index, write it to
+// tile_off[t] + C[t][cta] + rank (C == nullptr: a single CTA, every group starts at its tile's list start).
+__device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SPT], const FrameParams& fp,
+                                         const uint32_t* __restrict__ C, int nCTA, int ntiles,
+                                         uint32_t* __restrict__ ids) {
   const int tid = threadIdx.x, cta = blockIdx.x;
   const int64_t c0 = (int64_t)cta * DB_CTA;
-  n = frame_n(n, fp);
-  // step a2 is spread over every CTA of the grid (CTA c plans the tiles t = c mod gridDim.x; the grid has at least
-  // ntiles / 256 CTAs, so a sparse frame's plan is not one CTA's serial work); only the CTAs that hold stars go on
-  dp_scan_tiles(S, cnt, ntiles, (int)gridDim.x, tile_off, hdr, items, split_tab, part_cap, done);
-  if (cta >= dbin_live_ctas(n)) return;
   for (int t = tid; t <= ntiles; t += DP_THREADS) S.gstart[t] = 0u;
-  uint32_t code[DP_SPT];
-#pragma unroll
-  for (int k = 0; k < DP_SPT; ++k) {
-    const int64_t i = c0 + tid + k * DP_THREADS;
-    code[k] = i < n ? __ldg(&codes[i]) : DP_NONE;
-  }
   __syncthreads();
   // group sizes
 #pragma unroll
@@ -291,7 +278,7 @@ __global__ void __launch_bounds__(DP_THREADS, DP_MINB) k_dplace(const uint32_t* 
   }
   __syncthreads();
   // first list position of every group: tile_off[t] + (pairs of tile t in the CTAs before)
-  for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = S.toff[t] + C[(int64_t)t * nCTA + cta];
+  for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = S.toff[t] + (C ? C[(int64_t)t * nCTA + cta] : 0u);
   __syncthreads();
   // a pair's rank in its group = the group's stars with a smaller index
 #pragma unroll
@@ -308,12 +295,97 @@ __global__ void __launch_bounds__(DP_THREADS, DP_MINB) k_dplace(const uint32_t* 
   }
 }
 
+__global__ void __launch_bounds__(DP_THREADS, DP_MINB) k_dplace(const uint32_t* __restrict__ codes, int64_t n, FrameParams fp,
+                                                       const uint32_t* __restrict__ C, int nCTA, int ntiles,
+                                                       const uint32_t* __restrict__ cnt, uint32_t* __restrict__ tile_off,
+                                                       Header* hdr, WorkItem* __restrict__ items,
+                                                       uint2* __restrict__ split_tab, int part_cap,
+                                                       uint32_t* __restrict__ done, uint32_t* __restrict__ ids) {
+  static_assert(TILE_W == 128 && TILE_H == 64, "tile boxes span at most 2 x 2 tiles for R <= DB_MAXR");
+  extern __shared__ __align__(16) unsigned char dsm_raw[];
+  DpSmem& S = *reinterpret_cast<DpSmem*>(dsm_raw);
+  const int tid = threadIdx.x, cta = blockIdx.x;
+  const int64_t c0 = (int64_t)cta * DB_CTA;
+  n = frame_n(n, fp);
+  // step a2 is spread over every CTA of the grid (CTA c plans the tiles t = c mod gridDim.x; the grid has at least
+  // ntiles / 256 CTAs, so a sparse frame's plan is not one CTA's serial work); only the CTAs that hold stars go on
+  dp_scan_tiles(S, cnt, ntiles, (int)gridDim.x, tile_off, hdr, items, split_tab, part_cap, done);
+  if (cta >= dbin_live_ctas(n)) return;
+  uint32_t code[DP_SPT];
+#pragma unroll
+  for (int k = 0; k < DP_SPT; ++k) {
+    const int64_t i = c0 + tid + k * DP_THREADS;
+    code[k] = i < n ? __ldg(&codes[i]) : DP_NONE;
+  }
+  dp_place(S, code, fp, C, nCTA, ntiles, ids);
+}
+
+// k_dsmall: a catalogue of at most DB_CTA stars binned by ONE CTA in one launch -- k_dcount's step a1 and counts
+// (shared-memory atomics), step a2 over the counts in shared memory (dp_scan_tiles: the CTA plans every tile), and
+// k_dplace's grouping and ranking with no count matrix (one CTA: every group starts at its tile's list start).  The
+// same records, CSR and plan as the three-kernel path, bit for bit; for small frames the launches and the count
+// matrix round trip were the cost.
+__global__ void __launch_bounds__(DP_THREADS, 1) k_dsmall(const float* __restrict__ X, const float* __restrict__ Y,
+                                                          const float* __restrict__ M, int64_t n, FrameParams fp,
+                                                          StarRec* __restrict__ rec, int ntiles,
+                                                          uint32_t* __restrict__ tile_off, Header* hdr,
+                                                          WorkItem* __restrict__ items, uint2* __restrict__ split_tab,
+                                                          int part_cap, uint32_t* __restrict__ done,
+                                                          uint32_t* __restrict__ ids) {
+  static_assert(DP_THREADS == DC_THREADS && DP_SPT == DC_PER, "k_dcount's star-to-thread map");
+  extern __shared__ __align__(16) unsigned char dsm_raw[];
+  DpSmem& S = *reinterpret_cast<DpSmem*>(dsm_raw);
+  const int tid = threadIdx.x;
+  n = frame_n(n, fp);
+  for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = 0u;  // the tile counts
+  float xs[DP_SPT], ys[DP_SPT], ms[DP_SPT];
+#pragma unroll
+  for (int k = 0; k < DP_SPT; ++k) {
+    const int64_t i = tid + (int64_t)k * DP_THREADS;
+    const bool in = i < n;
+    xs[k] = in ? __ldg(&X[i]) : 0.f;
+    ys[k] = in ? __ldg(&Y[i]) : 0.f;
+    ms[k] = in ? __ldg(&M[i]) : 0.f;
+  }
+  __syncthreads();
+  uint32_t code[DP_SPT];
+#pragma unroll
+  for (int k = 0; k < DP_SPT; ++k) {
+    const int64_t i = tid + (int64_t)k * DP_THREADS;
+    code[k] = DP_NONE;
+    if (i >= n) continue;
+    int cx0, cx1, cy0, cy1;
+    const StarRec r = prep_star(xs[k], ys[k], ms[k], fp, cx0, cx1, cy0, cy1);
+    rec[i] = r;
+    if (r.lo != LO_CULLED) {
+      const int tx0 = cx0 / TILE_W, tx1 = cx1 / TILE_W;
+      const int ty0 = (cy0 - fp.row0) / TILE_H, ty1 = (cy1 - fp.row0) / TILE_H;
+      for (int ty = ty0; ty <= ty1; ++ty)
+        for (int tx = tx0; tx <= tx1; ++tx) atomicAdd(&S.cur[ty * fp.ntx + tx], 1u);
+      code[k] = (uint32_t)(ty0 * fp.ntx + tx0) | (uint32_t)(tx1 - tx0) << 16 | (uint32_t)(ty1 - ty0) << 17;
+    }
+  }
+  __syncthreads();
+  dp_scan_tiles<true>(S, S.cur, ntiles, 1, tile_off, hdr, items, split_tab, part_cap, done);
+  dp_place(S, code, fp, nullptr, 1, ntiles, ids);
+}
+
 size_t dbin_smem(int) { return sizeof(DpSmem); }
 
 int dbin_ctas(int64_t n) { return (int)((n + DB_CTA - 1) / DB_CTA); }
 
 void init_dbin_kernels() {
   cudaFuncSetAttribute(k_dplace, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DpSmem));
+  cudaFuncSetAttribute(k_dsmall, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DpSmem));
+}
+
+bool dsmall_ok(int64_t n) { return n <= DB_CTA; }
+
+void launch_dsmall(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
+                   int ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items, uint2* split_tab, int part_cap,
+                   uint32_t* done, uint32_t* ids, cudaStream_t st) {
+  k_dsmall<<<1, DP_THREADS, sizeof(DpSmem), st>>>(x, y, m, n, fp, rec, ntiles, tile_off, hdr, items, split_tab,
+                                                  part_cap, done, ids);
 }
 
 void launch_dcount(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,

@@ -16,6 +16,10 @@ size_t tile8_scratch_floats(int num_sms);
 void init_dbin_kernels();
 size_t dbin_smem(int ntiles);
 int dbin_ctas(int64_t n);
+bool dsmall_ok(int64_t n);  // k_dsmall applies (at most DB_CTA stars)
+void launch_dsmall(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
+                   int ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items, uint2* split_tab, int part_cap,
+                   uint32_t* done, uint32_t* ids, cudaStream_t st);
 void launch_dcount(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
                    uint32_t* codes, uint32_t* C, int ntiles, cudaStream_t st);
 void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstride, const uint32_t* n_dev,

@@ -309,9 +309,10 @@ def test_kernel_times_recorded(torch_dev, ctx):
     t = ctx.kernel_times()
     ctx.profile(False)
     # the t8 mode adds its corner-bin sort (k_t8sort) to the sort class
-    # sb hands the light tiles to k_tile_lite (a second launch)
-    assert t["tile"][1] in (1, 2) and t["tile"][0] > 0 and t["prep"][1] == 1 and t["sort"][1] in (1, 2)
-    assert t["csr"][1] in (1, 2, 3)
+    # sb may hand the light tiles to k_tile_lite (a second launch); C1's 1000 stars are binned by k_dsmall alone
+    # (class "prep"), the t8 mode adds its corner-bin sort (k_t8sort) to the sort class
+    assert t["tile"][1] in (1, 2) and t["tile"][0] > 0 and t["prep"][1] == 1 and t["sort"][1] in (0, 1)
+    assert t["csr"][1] == 0
     assert t["route"][1] == 0
     ctx.profile(True)
     ctx.route_band(*args, cfg.H, 0, 64, cfg.R)
