@@ -34,7 +34,7 @@ constexpr int DP_WARPS = DP_THREADS / 32;
 constexpr int DP_KEYS = DB_CTA * 4;              // at most 2 x 2 tiles per star
 constexpr int DP_SPT = DB_CTA / DP_THREADS;      // stars per thread (strided by DP_THREADS)
 constexpr int DCS_THREADS = 256;
-constexpr int DCS_PER = 8;                       // k_dcolscan: consecutive CTA counts per lane
+
 // CTAs that hold stars (at least one: CTA 0 plans the tiles of an empty routed catalogue)
 __device__ __forceinline__ int dbin_live_ctas(int64_t n) { return n > 0 ? (int)((n + DB_CTA - 1) / DB_CTA) : 1; }
 static_assert(DB_MAXT <= 65536 && DB_CTA <= 65536, "tile ids, slots and star indices are 16-bit in k_dplace");
@@ -84,42 +84,56 @@ __global__ void __launch_bounds__(DC_THREADS, 2) k_dcount(const float* __restric
     codes[i] = code;  // the star's tile box for k_dplace (one coalesced word instead of a record gather)
   }
   __syncthreads();
-  for (int t = tid; t < ntiles; t += DC_THREADS) C[(int64_t)t * nCTA + cta] = cnt[t];
+  for (int t = tid; t < ntiles; t += DC_THREADS) C[(int64_t)cta * ntiles + t] = cnt[t];  // CTA-major row
 }
 
-__global__ void __launch_bounds__(DCS_THREADS) k_dcolscan(uint32_t* __restrict__ C, int cstrideC, int ntiles,
+// C is CTA-major: C[cta][t] (row stride ntiles), so k_dcount's and k_dplace's accesses to their own CTA's row are
+// coalesced.  k_dcolscan takes DCS_TILES tiles per CTA: it stages DCS_ROWS rows of the block in shared memory
+// (coalesced 128-B row reads), scans every tile's column there (lane l holds rows l + 32 k; one warp scan per 32 rows,
+// carried), and writes the exclusive prefixes back in place (coalesced), then the tile totals.
+constexpr int DCS_TILES = 8;   // one tile per warp
+constexpr int DCS_ROWS = 256;
+__global__ void __launch_bounds__(DCS_THREADS) k_dcolscan(uint32_t* __restrict__ C, int nCTA_cap, int ntiles,
                                                          uint32_t* __restrict__ cnt, int cstride, int64_t n,
                                                          const uint32_t* __restrict__ n_dev) {
-  const int lane = threadIdx.x & 31;
-  const int t = blockIdx.x * (DCS_THREADS / 32) + (threadIdx.x >> 5);
-  if (t >= ntiles) return;
-  uint32_t* row = C + (int64_t)t * cstrideC;  // row stride: the CTAs of the capacity n
-  const int nCTA = (n_dev && n > 0) ? dbin_live_ctas(n < (int64_t)*n_dev ? n : (int64_t)*n_dev) : cstrideC;
-  // lane l takes the DCS_PER consecutive CTAs [DCS_PER l, DCS_PER (l + 1)): all loads first, one warp scan
-  uint32_t run = 0;
-  for (int b0 = 0; b0 < nCTA; b0 += 32 * DCS_PER) {
-    const int j0 = b0 + lane * DCS_PER;
-    uint32_t v[DCS_PER], sum = 0;
+  static_assert(DCS_THREADS == 32 * DCS_TILES, "one warp per tile");
+  __shared__ uint32_t sm[DCS_ROWS][DCS_TILES + 1];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int t0 = blockIdx.x * DCS_TILES;
+  const int nCTA = (n_dev && n > 0) ? dbin_live_ctas(n < (int64_t)*n_dev ? n : (int64_t)*n_dev) : nCTA_cap;
+  // staging map: thread -> (row tid / 8 + 32 i, tile tid % 8): 8 consecutive words (one sector) per row
+  const int sr = tid / DCS_TILES, st_ = tid % DCS_TILES;
+  const bool tin = t0 + st_ < ntiles;
+  uint32_t carry = 0;  // warp w: tile t0 + w (uniform across the warp)
+  for (int r0 = 0; r0 < nCTA; r0 += DCS_ROWS) {
+    const int rows = min(DCS_ROWS, nCTA - r0);
 #pragma unroll
-    for (int k = 0; k < DCS_PER; ++k) {
-      v[k] = j0 + k < nCTA ? row[j0 + k] : 0u;
-      sum += v[k];
+    for (int i = 0; i < DCS_ROWS / 32; ++i) {
+      const int r = sr + 32 * i;
+      if (r < rows) sm[r][st_] = tin ? C[(int64_t)(r0 + r) * ntiles + t0 + st_] : 0u;
     }
-    uint32_t incl = sum;
+    __syncthreads();
+    for (int k = 0; k < DCS_ROWS / 32 && 32 * k < rows; ++k) {
+      const int r = 32 * k + lane;
+      const uint32_t v = r < rows ? sm[r][warp] : 0u;
+      uint32_t incl = v;
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
-      if (lane >= o) incl += u;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += u;
+      }
+      if (r < rows) sm[r][warp] = carry + incl - v;
+      carry += __shfl_sync(0xffffffffu, incl, 31);
     }
-    uint32_t ex = run + incl - sum;
+    __syncthreads();
 #pragma unroll
-    for (int k = 0; k < DCS_PER; ++k) {
-      if (j0 + k < nCTA) row[j0 + k] = ex;
-      ex += v[k];
+    for (int i = 0; i < DCS_ROWS / 32; ++i) {
+      const int r = sr + 32 * i;
+      if (r < rows && tin) C[(int64_t)(r0 + r) * ntiles + t0 + st_] = sm[r][st_];
     }
-    run += __shfl_sync(0xffffffffu, incl, 31);
+    __syncthreads();
   }
-  if (lane == 0) cnt[(int64_t)t * cstride] = run;
+  if (lane == 0 && t0 + warp < ntiles) cnt[(int64_t)(t0 + warp) * cstride] = carry;
 }
 
 // block-wide exclusive scan of one value per thread (DP_THREADS); returns the prefix, *total the sum
@@ -278,7 +292,7 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
   }
   __syncthreads();
   // first list position of every group: tile_off[t] + (pairs of tile t in the CTAs before)
-  for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = S.toff[t] + (C ? C[(int64_t)t * nCTA + cta] : 0u);
+  for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = S.toff[t] + (C ? C[(int64_t)cta * ntiles + t] : 0u);
   __syncthreads();
   // a pair's rank in its group = the group's stars with a smaller index
 #pragma unroll
@@ -396,8 +410,8 @@ void launch_dcount(const float* x, const float* y, const float* m, int64_t n, co
 
 void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstride, const uint32_t* n_dev,
                      cudaStream_t st) {
-  constexpr int wpb = DCS_THREADS / 32;
-  k_dcolscan<<<(ntiles + wpb - 1) / wpb, DCS_THREADS, 0, st>>>(C, dbin_ctas(n), ntiles, cnt, cstride, n, n_dev);
+  k_dcolscan<<<(ntiles + DCS_TILES - 1) / DCS_TILES, DCS_THREADS, 0, st>>>(C, dbin_ctas(n), ntiles, cnt, cstride, n,
+                                                                           n_dev);
 }
 
 void launch_dplace(const uint32_t* codes, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,
