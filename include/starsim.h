@@ -121,10 +121,10 @@ int starsim_set_psf(starsim_ctx* ctx, int32_t mode);
  *   STARSIM_ROI_SQUARE (default): the R x R square of reading R5/R7 (Fig. 1 caption PAPER.md:19, Fig. 5);
  *   STARSIM_ROI_CIRCLE: the paper's literal "pixel circle" -- the pixels of that square whose centres lie
  *     in the circle inscribed in it: ROI row / column offsets (i, j) with (2j - (R-1))^2 + (2i - (R-1))^2 <= R^2,
- *     an exact integer test, then clipped to the image.  Supported by starsim_render_atomic and starsim_render_lut
- *     for any roi, and by the tiled renders (render, render_band, render_band_to, render_gray) for roi <= 17: they
- *     then run k_tile_sb whatever starsim_set_tile_kernel says, which masks the circle per pixel in its walk (same
- *     profiles, same deterministic order); a tiled render with roi > 17 returns EINVAL while it is set.
+ *     an exact integer test, then clipped to the image.  Supported by every render: the star-centric ones (atomic,
+ *     lookup table) and the tiled ones (render, render_band, render_band_to, render_gray), which mask the circle per
+ *     pixel in the tile kernel's walk -- k_tile_sb's for roi <= 17 (whatever starsim_set_tile_kernel says) and
+ *     k_tile's for wider ROIs -- with the same profiles and the same deterministic order.
  * EINVAL: ctx NULL or an unknown shape. */
 #define STARSIM_ROI_SQUARE 0
 #define STARSIM_ROI_CIRCLE 1

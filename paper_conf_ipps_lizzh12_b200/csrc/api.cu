@@ -303,16 +303,13 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
 int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, int32_t W, int32_t H,
                  int32_t row0, int32_t rows, float sigma, int32_t R, float gain, int32_t obits, void* out,
                  cudaStream_t st, float* const* dsts = nullptr, int ndst = 0) {
-  if (c->roi != STARSIM_ROI_SQUARE && R > SB_MAXR)
-    return fail(c, STARSIM_EINVAL,
-                "circular ROI (NEXT-3): the tiled renders support roi <= 17 (k_tile_sb masks the circle in its walk); "
-                "use starsim_render_atomic or starsim_render_lut for wider circles");
   DevGuard g(c->dev);
   FrameParams fp = make_params(W, H, row0, rows, sigma, R, gain, c->psf);
   fp.obits = obits;
   fp.tile_impl = c->tile_impl;
   fp.roi = c->roi;
-  if (fp.roi) fp.tile_impl = STARSIM_TILE_SB;  // NEXT-3: the circle mask lives in k_tile_sb's walk
+  // NEXT-3: the circle mask lives in k_tile_sb's walk (R <= SB_MAXR) and in k_tile's (wider ROIs)
+  if (fp.roi) fp.tile_impl = STARSIM_TILE_SB;
   if (fp.tile_impl == STARSIM_TILE_AUTO) {
     // the warp-specialised kernel wins on dense frames (its per-item pipeline latency and static item order cost
     // more than they save on sparse, clustered and integrated-PSF frames: DESIGN.md §9): expected list length per

@@ -41,7 +41,7 @@ struct TileSmem {
   uint32_t lpre[NBANDS * NSTRIPS][TILE_WARPS];  // per (B,Q): entries of the warps before
   uint32_t rpre[NSTRIPS][TILE_WARPS];           // per Q: strip slots of the warps before
   uint32_t wsum[TILE_WARPS];
-  float4 py[CHUNK];                      // per star: (y - IY0, s', r0 | r1 << 8, -)
+  float4 py[CHUNK];                      // per star: (y - IY0, s', r0 | r1 << 8, ROI origin lx | ly << 16 (CIRC))
   float2 px[CHUNK];                      // per star: (x - X0, c0 | c1 << 8)
   uint16_t gyown[GY_CAP];                // band slot -> star | band << 8
   uint32_t gxown[GX_PAIRS];              // (star, strip) pair j -> strip slot | star << 16
@@ -71,12 +71,14 @@ constexpr uint32_t ZERO_ENT = ZERO_GX * 32u << 16;  // gy byte offset 0, all-zer
 // parts in part order -- a fixed order, so the image stays deterministic.
 // ---------------------------------------------------------------------------------------------------------------
 // INTEG: the pixel-integrated PSF (NEXT-2) instead of the paper's point-sampled Eq. 2; GRAY: the fused output stage
-// (u8 / u16 image) instead of the fp32 image
-template <bool INTEG, bool GRAY>
+// (u8 / u16 image) instead of the fp32 image; CIRC: the pixel-circle ROI (NEXT-3, reading R21) -- the walk masks each
+// of the lane's 4 x 8 pixels by the integer disc test against the star's ROI origin (looked up through its band slot),
+// 2 CTAs per SM for the extra registers.  k_tile serves the circle for R > SB_MAXR (k_tile_sb below).
 #ifndef TILE_MINB_OPT
 #define TILE_MINB_OPT 3
 #endif
-__global__ void __launch_bounds__(TILE_THREADS, TILE_MINB_OPT) k_tile(const uint32_t* __restrict__ ids,
+template <bool INTEG, bool GRAY, bool CIRC>
+__global__ void __launch_bounds__(TILE_THREADS, CIRC ? 2 : TILE_MINB_OPT) k_tile(const uint32_t* __restrict__ ids,
                                                           const StarRec* __restrict__ rec, FrameParams fp,
                                                           void* __restrict__ out_, const WorkItem* __restrict__ items,
                                                           const uint2* __restrict__ split_tab,
@@ -217,7 +219,9 @@ __global__ void __launch_bounds__(TILE_THREADS, TILE_MINB_OPT) k_tile(const uint
       } else {
         atomicMin(&S.ns, tid);
       }
-      S.py[tid] = make_float4(r.y - (float)IY0, r.s, __int_as_float(r0 | (r1 << 8)), 0.f);
+      S.py[tid] = make_float4(r.y - (float)IY0, r.s, __int_as_float(r0 | (r1 << 8)),
+                              __uint_as_float((uint32_t)((lo_x_of(r.lo) - X0) & 0xFFFF) |
+                                              (uint32_t)(lo_y_of(r.lo) - IY0) << 16));
       S.px[tid] = make_float2(r.x - (float)X0, __int_as_float(c0 | (c1 << 8)));
     }
     __syncthreads();
@@ -345,13 +349,38 @@ __global__ void __launch_bounds__(TILE_THREADS, TILE_MINB_OPT) k_tile(const uint
         asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "r"(gxa_base + xo));
         asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(c.x), "=f"(c.y), "=f"(c.z), "=f"(c.w) : "r"(gxb_base + xo));
         const float gi[4] = {g.x, g.y, g.z, g.w};
+        if (!CIRC) {
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const float2 gg = make_float2(gi[i], gi[i]);
-          acc[i][0] = __ffma2_rn(gg, make_float2(a.x, a.y), acc[i][0]);
-          acc[i][1] = __ffma2_rn(gg, make_float2(a.z, a.w), acc[i][1]);
-          acc[i][2] = __ffma2_rn(gg, make_float2(c.x, c.y), acc[i][2]);
-          acc[i][3] = __ffma2_rn(gg, make_float2(c.z, c.w), acc[i][3]);
+          for (int i = 0; i < 4; ++i) {
+            const float2 gg = make_float2(gi[i], gi[i]);
+            acc[i][0] = __ffma2_rn(gg, make_float2(a.x, a.y), acc[i][0]);
+            acc[i][1] = __ffma2_rn(gg, make_float2(a.z, a.w), acc[i][1]);
+            acc[i][2] = __ffma2_rn(gg, make_float2(c.x, c.y), acc[i][2]);
+            acc[i][3] = __ffma2_rn(gg, make_float2(c.z, c.w), acc[i][3]);
+          }
+        } else {
+          // the star of the entry's band slot and its ROI origin; pixel (row, col) of the lane's block is inside the
+          // circle iff (2 (col - lx) - (R-1))^2 + (2 (row - ly) - (R-1))^2 <= R^2 (reading R21)
+          const uint32_t lo = __float_as_uint(S.py[S.gyown[go >> 6] & 0xFFu].w);
+          const int lx = (int)(int16_t)(lo & 0xFFFFu), ly = (int)(int16_t)(lo >> 16);
+          const int RR = fp.R * fp.R, R1 = fp.R - 1;
+          const float gx[8] = {a.x, a.y, a.z, a.w, c.x, c.y, c.z, c.w};
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const int v = 2 * (16 * B + hq + 4 * i - ly) - R1;
+            const int thr = RR - v * v;
+            float gm[8];
+#pragma unroll
+            for (int p = 0; p < 8; ++p) {
+              const int u = 2 * (8 * Q + p - lx) - R1;
+              gm[p] = u * u <= thr ? gx[p] : 0.f;
+            }
+            const float2 gg = make_float2(gi[i], gi[i]);
+            acc[i][0] = __ffma2_rn(gg, make_float2(gm[0], gm[1]), acc[i][0]);
+            acc[i][1] = __ffma2_rn(gg, make_float2(gm[2], gm[3]), acc[i][1]);
+            acc[i][2] = __ffma2_rn(gg, make_float2(gm[4], gm[5]), acc[i][2]);
+            acc[i][3] = __ffma2_rn(gg, make_float2(gm[6], gm[7]), acc[i][3]);
+          }
         }
       }
     }
@@ -394,10 +423,17 @@ __global__ void __launch_bounds__(TILE_THREADS, TILE_MINB_OPT) k_tile(const uint
 }
 
 void init_tile_kernel() {
-  cudaFuncSetAttribute(k_tile<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
-  cudaFuncSetAttribute(k_tile<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
-  cudaFuncSetAttribute(k_tile<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
-  cudaFuncSetAttribute(k_tile<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem));
+#define STARSIM_KT_ATTR(I, G, C) \
+  cudaFuncSetAttribute(k_tile<I, G, C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))
+  STARSIM_KT_ATTR(false, false, false);
+  STARSIM_KT_ATTR(true, false, false);
+  STARSIM_KT_ATTR(false, true, false);
+  STARSIM_KT_ATTR(true, true, false);
+  STARSIM_KT_ATTR(false, false, true);
+  STARSIM_KT_ATTR(true, false, true);
+  STARSIM_KT_ATTR(false, true, true);
+  STARSIM_KT_ATTR(true, true, true);
+#undef STARSIM_KT_ATTR
 }
 
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
@@ -414,9 +450,14 @@ void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp,
   }
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
-  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)3 * num_sms);  // persistent, 3 CTAs per SM
-  auto* k = fp.psf ? (fp.obits ? k_tile<true, true> : k_tile<true, false>)
-                   : (fp.obits ? k_tile<false, true> : k_tile<false, false>);
+  // persistent, 3 CTAs per SM (2 for the circle ROI)
+  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)(fp.roi ? 2 : TILE_MINB_OPT) * num_sms);
+  using KT = void (*)(const uint32_t*, const StarRec*, FrameParams, void*, const WorkItem*, const uint2*, float*,
+                      uint32_t*, Header*, float*);
+  static const KT kts[2][2][2] = {
+      {{k_tile<false, false, false>, k_tile<false, false, true>}, {k_tile<false, true, false>, k_tile<false, true, true>}},
+      {{k_tile<true, false, false>, k_tile<true, false, true>}, {k_tile<true, true, false>, k_tile<true, true, true>}}};
+  const KT k = kts[fp.psf ? 1 : 0][fp.obits ? 1 : 0][fp.roi ? 1 : 0];
   k<<<(unsigned)grid, TILE_THREADS, sizeof(TileSmem), st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr,
                                                             seg_scratch);
 }

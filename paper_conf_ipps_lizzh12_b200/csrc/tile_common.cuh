@@ -207,6 +207,7 @@ __device__ __forceinline__ void tile_store_gray_staged(const float* __restrict__
         if (c < TWe) o[0] = (uint8_t)g0;
         if (c + 1 < TWe) o[1] = (uint8_t)g1;
         if (c + 2 < TWe) o[2] = (uint8_t)g2;
+        if (c + 3 < TWe) o[3] = (uint8_t)g3;
       }
     } else {
       uint16_t* o = reinterpret_cast<uint16_t*>(out_) + pix;
@@ -216,6 +217,7 @@ __device__ __forceinline__ void tile_store_gray_staged(const float* __restrict__
         if (c < TWe) o[0] = (uint16_t)g0;
         if (c + 1 < TWe) o[1] = (uint16_t)g1;
         if (c + 2 < TWe) o[2] = (uint16_t)g2;
+        if (c + 3 < TWe) o[3] = (uint16_t)g3;
       }
     }
   }

@@ -355,8 +355,8 @@ class Context:
         starsim_set_psf(self.h, mode)
 
     def set_roi(self, shape="square"):
-        """"square" (the R x R ROI, reading R5) or "circle" (the pixel circle inscribed in it, NEXT-3: the atomic and
-        lookup-table renders for any R, the tiled renders for R <= 17 -- EINVAL above)."""
+        """"square" (the R x R ROI, reading R5) or "circle" (the pixel circle inscribed in it, NEXT-3, reading R21: every
+        render; the tiled ones mask it in k_tile_sb's walk for R <= 17 and in k_tile's above)."""
         starsim_set_roi(self.h, shape)
 
     def set_binning(self, mode="auto"):

@@ -224,7 +224,9 @@ def test_render_gray_is_quantize_of_render(torch_dev, ctx, bits, W, H):
     args = to_dev(torch_dev, f)
     img = ctx.render(*args, W, H, 1.5, 9, A)
     q_two_pass = ctx.quantize(img, bits).cpu().numpy()
-    q_fused = ctx.render_gray(*args, W, H, 1.5, 9, A, bits=bits).cpu().numpy()
+    # into a buffer prefilled with a sentinel: every pixel must be written
+    pre = torch.full((H, W), 0xAB, dtype=torch.uint8 if bits == 8 else torch.uint16, device=dev)
+    q_fused = ctx.render_gray(*args, W, H, 1.5, 9, A, bits=bits, out=pre).cpu().numpy()
     assert q_fused.dtype == (np.uint8 if bits == 8 else np.uint16)
     assert np.array_equal(q_fused, q_two_pass)
     ref = oracle.quantize(oracle.render(f.x, f.y, f.mag, W, H, 1.5, 9, A, threads=_threads()), bits)
@@ -606,11 +608,13 @@ def test_lut_einval(torch_dev, ctx):
 
 @pytest.mark.parametrize("W,H,n,R,sigma,kind", [(1024, 1024, 1000, 5, 1.0, "uniform"), (700, 530, 5000, 15, 2.5, "adv"),
                                                  (300, 200, 2000, 10, 1.7, "uniform"), (512, 384, 3000, 63, 10.5, "uniform"),
-                                                 (4096, 2048, 6000, 15, 2.5, "adv")])  # sparse: k_tile_lite
+                                                 (4096, 2048, 6000, 15, 2.5, "adv"),  # sparse: k_tile_lite
+                                                 (700, 530, 6000, 21, 3.5, "adv"), (640, 520, 8000, 31, 5.2, "uniform"),
+                                                 (600, 500, 4000, 41, 6.8, "adv")])    # R > 17: k_tile's masked walk
 def test_circle_roi_parity(torch_dev, ctx, W, H, n, R, sigma, kind):
-    """starsim_set_roi(CIRCLE): the atomic and lookup-table renders against the oracle's circle ROI, the tiled render
-    too for R <= 17 (bands bitwise the frame), EINVAL above; the square ROI works again once it is back."""
-    from paper_conf_ipps_lizzh12_b200 import StarsimError
+    """starsim_set_roi(CIRCLE): the atomic, lookup-table and tiled renders against the oracle's circle ROI (the tiled
+    path masks the circle in k_tile_sb's walk for R <= 17 and in k_tile's above; bands bitwise the frame); the square
+    ROI works again once it is back."""
     f = synth.adversarial_field(n, W, H, R, seed=43) if kind == "adv" else synth.uniform_field(n, W, H, seed=44,
                                                                                                   mag_hi=2.0)
     args = to_dev(torch_dev, f)
@@ -621,15 +625,13 @@ def test_circle_roi_parity(torch_dev, ctx, W, H, n, R, sigma, kind):
         if R <= 63:
             ref_l = oracle.render_lut(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads(), roi="circle")
             assert_parity(ctx.render_lut(*args, W, H, sigma, R, 1.0).cpu().numpy(), ref_l, f"circle lut R={R}")
-        if R <= 17:  # the tiled path masks the circle in k_tile_sb's walk (any tile kernel setting)
-            img = ctx.render(*args, W, H, sigma, R, 1.0)
-            assert_parity(img.cpu().numpy(), ref, f"circle tiled R={R}")
-            bands = [ctx.render_band(*args, W, H, g * 64, min(64, H - g * 64), sigma, R, 1.0)
-                     for g in range(-(-H // 64))]
-            assert torch_dev[0].equal(torch_dev[0].cat(bands, 0), img)
-        else:
-            with pytest.raises(StarsimError):
-                ctx.render(*args, W, H, sigma, R, 1.0)
+        img = ctx.render(*args, W, H, sigma, R, 1.0)
+        assert_parity(img.cpu().numpy(), ref, f"circle tiled R={R}")
+        bands = [ctx.render_band(*args, W, H, g * 64, min(64, H - g * 64), sigma, R, 1.0)
+                 for g in range(-(-H // 64))]
+        assert torch_dev[0].equal(torch_dev[0].cat(bands, 0), img)
+        g8 = ctx.render_gray(*args, W, H, sigma, R, 1.0, bits=8)
+        assert torch_dev[0].equal(g8, ctx.quantize(img, 8))
     finally:
         ctx.set_roi("square")
     ref_sq = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads())
