@@ -57,8 +57,9 @@ struct starsim_ctx {
   int32_t bin_impl = 0;   // starsim_set_binning: 0 auto (dbin.cu when it applies), 1 always bin.cu's pipeline
   std::string err;
   const uint32_t* n_dev = nullptr;  // starsim_set_star_count: device-resident star count of the tiled renders
+  bool ws_presort = false;          // k_tile_ws reads chunks presorted by k_chsort (env STARSIM_WS_PRESORT=1; slower)
   Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat, codes, segs, srec, sbin, sext,
-      rblk;
+      rblk, cbin;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
@@ -212,6 +213,12 @@ int tiles_per_axis(int R, int tile, int ntiles_axis) {
   return t < ntiles_axis ? t : ntiles_axis;
 }
 
+// k_tile_ws with its chunks presorted by k_chsort (STARSIM_WS_PRESORT=1 at context creation; measured slower at T:
+// k_chsort 21 us against 6 us saved in k_tile_ws)
+bool ws_presort(const starsim_ctx* c, const FrameParams& fp) {
+  return c->ws_presort && fp.tile_impl == STARSIM_TILE_WS && fp.R <= SB_MAXR;
+}
+
 // Enqueue the tiled render on stream st: memset of the header + tile counters, k_prep, k_scan, k_scatter,
 // k_sortlists, k_tile.
 int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, const FrameParams& fp,
@@ -288,11 +295,21 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
                    c->num_sms, st);
     });
   } else {
+    const bool pre = ws_presort(c, fp);
+    if (pre) {
+      // k_chsort: k_tile_ws's per-chunk corner-bin sort done ahead (records in walk order, bin starts per chunk)
+      timed(c, 1, st, [&] {
+        launch_chsort(ids, rec, fp, (WorkItem*)c->items.p, part_cap, hdr, (StarRec*)c->srec.p, (uint16_t*)c->cbin.p,
+                      st);
+      });
+      if ((rc = check_launch(c, "k_chsort"))) return rc;
+    }
     timed(
         c, 3, st,
         [&] {
           launch_tile(ids, rec, fp, out, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, (float*)c->parts.p, part_cap,
-                      done, hdr, c->num_sms, st, (float*)c->segs.p, tile_off);
+                      done, hdr, c->num_sms, st, (float*)c->segs.p, tile_off, pre ? (StarRec*)c->srec.p : nullptr,
+                      pre ? (uint16_t*)c->cbin.p : nullptr);
         },
         fp.lite ? 2 : 1);
   }
@@ -363,6 +380,11 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
     return rc;
   if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
   if ((rc = grow(c, c->segs, sizeof(float) * tile8_scratch_floats(c->num_sms), "segment scratch"))) return rc;
+  if (ws_presort(c, fp)) {  // k_chsort's outputs
+    if ((rc = grow(c, c->srec, sizeof(StarRec) * (size_t)(pmax > 0 ? pmax : 1), "bin-sorted records"))) return rc;
+    if ((rc = grow(c, c->cbin, sizeof(uint16_t) * chsort_slots(ntiles, pmax) * chsort_words16(), "chunk bin starts")))
+      return rc;
+  }
   if (fp.tile_impl == STARSIM_TILE_T8 && R <= SB_MAXR) {  // k_t8sort's outputs (the t8 kernel only)
     if ((rc = grow(c, c->srec, sizeof(StarRec) * (size_t)(pmax > 0 ? pmax : 1), "bin-sorted records"))) return rc;
     if ((rc = grow(c, c->sbin, sizeof(uint32_t) * tile8_sbin_words(ntiles, part_cap, pmax), "segment bin starts")))
@@ -448,6 +470,8 @@ int starsim_create(starsim_ctx** out, int cuda_device) {
   c->dev = cuda_device;
   c->num_sms = prop.multiProcessorCount;
   init_kernels();
+  const char* wp = getenv("STARSIM_WS_PRESORT");
+  c->ws_presort = wp && wp[0] == '1';
   const char* ng = getenv("STARSIM_NO_GRAPH");
   c->use_graphs = !(ng && ng[0] == '1');
   *out = c;
@@ -463,7 +487,7 @@ void starsim_destroy(starsim_ctx* c) {
     if (c->have_graph) cudaGraphExecDestroy(c->gexec);
     Buf* bufs[] = {&c->rec, &c->slots, &c->ids, &c->tmp, &c->tile_off, &c->items, &c->split_tab, &c->parts,
                    &c->partial, &c->zeroed, &c->stage, &c->cmat, &c->codes, &c->segs, &c->srec, &c->sbin, &c->sext,
-                   &c->rblk};
+                   &c->rblk, &c->cbin};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {

@@ -4,15 +4,17 @@
 //
 //   k_dcount     a1 + counts: CTA c takes stars [c*DB_CTA, (c+1)*DB_CTA); per star the record of step a1
 //                (prep_star); per tile the number of pairs of the CTA (shared-memory atomics -- counts do not depend
-//                on order) -> C[tile][c].
-//   k_dcolscan   per tile (one warp): exclusive scan of C[tile][0..nCTA) in CTA order (in place) and the tile's
-//                total -> cnt[tile].
-//   k_dplace     CTA c again: step a2 first (every CTA scans the tile totals; CTA c writes tile_off and the work
-//                items of the tiles t = c mod nCTA -- no scan launch between the two), then its pairs are grouped by tile in shared memory (slots from shared-memory atomics, in
-//                arbitrary order); a pair's rank in its group is the number of the group's stars with a smaller
-//                index, and it goes to tile_off[t] + C[t][c] + rank: every tile list holds its stars in ascending
-//                star index -- the unique CSR (reading R18), bit-exact, with no sort pass over the lists and no
-//                atomics on global memory.  (Groups are (tile, 2048-star block) pairs: a few stars each.)
+//                on order) -> row c of the block-major count matrix C[c][tile] (coalesced).
+//   k_dcolscan   per 8-tile column block: the rows staged in shared memory, exclusive scan of every tile's column
+//                C[0..nCTA)[tile] in CTA order (in place) and the tile's total -> cnt[tile].
+//   k_dplace     step a2 first on every CTA of the grid (each scans the tile totals; CTA c writes tile_off and the
+//                work items of the tiles t = c mod gridDim -- no scan launch between the two; the grid has at least
+//                ntiles / 256 CTAs), then CTA c's pairs are grouped by tile in shared memory (slots from
+//                shared-memory atomics, in arbitrary order); a pair's rank in its group is the number of the group's
+//                stars with a smaller index, and it goes to tile_off[t] + C[c][t] + rank: every tile list holds its
+//                stars in ascending star index -- the unique CSR (reading R18), bit-exact, with no sort pass over the
+//                lists and no atomics on global memory.  (Groups are (4096-star block, tile) pairs: a few stars each.)
+//   k_dsmall     a catalogue of at most DB_CTA stars: all of the above in one CTA and one launch.
 #include <algorithm>
 
 #include "common.cuh"

@@ -38,13 +38,18 @@ void launch_sortlists(uint32_t* ids, uint32_t* tmp, const uint32_t* tile_off, in
                       cudaStream_t st);
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                 cudaStream_t st, float* seg_scratch, const uint32_t* tile_off);
+                 cudaStream_t st, float* seg_scratch, const uint32_t* tile_off, const StarRec* ws_srec,
+                 const uint16_t* ws_cbin);
 void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
                     cudaStream_t st, float* seg_scratch, const uint32_t* tile_off);
 void launch_tile_ws(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                    cudaStream_t st, float* seg_scratch);
+                    cudaStream_t st, float* seg_scratch, const StarRec* srec, const uint16_t* cbin);
+size_t chsort_slots(int64_t ntiles, int64_t pmax);  // rows of k_chsort's bin-start table
+size_t chsort_words16();                            // u16 per row
+void launch_chsort(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, const WorkItem* items, int part_cap,
+                   const Header* hdr, StarRec* srec, uint16_t* cbin, cudaStream_t st);
 size_t tile8_sbin_words(int64_t ntiles, int part_cap, int64_t pairs);
 void launch_t8sort(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, const WorkItem* items,
                    int part_cap, Header* hdr, StarRec* srec, uint32_t* sbin, uint32_t* sext, cudaStream_t st);

@@ -438,9 +438,11 @@ void init_tile_kernel() {
 
 void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                  const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                 cudaStream_t st, float* seg_scratch, const uint32_t* tile_off) {
+                 cudaStream_t st, float* seg_scratch, const uint32_t* tile_off, const StarRec* ws_srec,
+                 const uint16_t* ws_cbin) {
   if (fp.R <= SB_MAXR && fp.tile_impl == 3) {
-    launch_tile_ws(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st, seg_scratch);
+    launch_tile_ws(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st, seg_scratch,
+                   ws_srec, ws_cbin);
     return;
   }
   if (fp.R <= SB_MAXR && fp.tile_impl == 2) {

@@ -116,8 +116,10 @@ __device__ __forceinline__ uint32_t item_chunks(const WorkItem& w) {
 }
 // The ids of the stars of work item w that producer thread pt of group g reads: star e = pt + WS_CHUNK k sits in
 // chunk k, which group g produces iff (cb + k) % WS_PGROUPS == g (cb: the CTA's index of the item's first chunk).
+template <bool PRE>
 __device__ __forceinline__ void load_ids(uint32_t (&id)[WS_RPT], const uint32_t* __restrict__ ids, const WorkItem& w,
                                          uint32_t cb, int g, int pt) {
+  if (PRE) return;  // presorted records are read in list order: no ids
   const uint32_t len = w.je - w.jb;
 #pragma unroll
   for (int k = 0; k < WS_RPT; ++k) {
@@ -127,22 +129,28 @@ __device__ __forceinline__ void load_ids(uint32_t (&id)[WS_RPT], const uint32_t*
 }
 // ... and their records, copied into the group's record stage at the same places: thread pt is the only reader of
 // its slots, so cp.async + wait_all needs no barrier.
+template <bool PRE>
 __device__ __forceinline__ void stage_records(StarRec* dst, const StarRec* __restrict__ rec, const uint32_t (&id)[WS_RPT],
                                               const WorkItem& w, uint32_t cb, int g, int pt) {
   const uint32_t len = w.je - w.jb;
 #pragma unroll
   for (int k = 0; k < WS_RPT; ++k) {
     const uint32_t e = (uint32_t)pt + (uint32_t)(k * WS_CHUNK);
+    // PRE: rec is the presorted record array (list order within each chunk sorted by corner bin, k_chsort)
+    const StarRec* src = PRE ? rec + w.jb + e : rec + id[k];
     if (e < len && (cb + (uint32_t)k) % WS_PGROUPS == (uint32_t)g)
-      asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst + e)), "l"(rec + id[k]) : "memory");
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst + e)), "l"(src) : "memory");
   }
   asm volatile("cp.async.commit_group;" ::: "memory");
 }
 
-template <bool INTEG>
+// PRE: the chunks come presorted by k_chsort (records in sorted order, bin starts per chunk): the producers skip the
+// sort, its two barriers and the record gather through the ids, and only evaluate the profiles (sorted star j = pt).
+template <bool INTEG, bool PRE>
 __device__ __forceinline__ void ws_producer(WsSmem& S, const uint32_t* __restrict__ ids,
                                             const StarRec* __restrict__ rec, const FrameParams& fp,
-                                            const WorkItem* __restrict__ items, uint32_t nitems) {
+                                            const WorkItem* __restrict__ items, uint32_t nitems,
+                                            const uint16_t* __restrict__ cbin) {
   const int pq = threadIdx.x - 32 * WS_CONS;
   const int g = pq / WS_CHUNK, pt = pq % WS_CHUNK, lane = pt & 31, pw = pt >> 5;
   const uint32_t lt = (1u << lane) - 1u;
@@ -159,14 +167,14 @@ __device__ __forceinline__ void ws_producer(WsSmem& S, const uint32_t* __restric
   WorkItem wn = it + G < nitems ? items[it + G] : none;
   WorkItem wnn = it + 2 * G < nitems ? items[it + 2 * G] : none;
   uint32_t idn[WS_RPT];
-  load_ids(idn, ids, wi, 0u, g, pt);
-  stage_records(S.rst[g][0], rec, idn, wi, 0u, g, pt);
-  load_ids(idn, ids, wn, item_chunks(wi), g, pt);
+  load_ids<PRE>(idn, ids, wi, 0u, g, pt);
+  stage_records<PRE>(S.rst[g][0], rec, idn, wi, 0u, g, pt);
+  load_ids<PRE>(idn, ids, wn, item_chunks(wi), g, pt);
   while (it < nitems) {
     const uint32_t nch = item_chunks(wi), cbn = cb + nch;
     asm volatile("cp.async.wait_all;" ::: "memory");
-    stage_records(S.rst[g][p ^ 1u], rec, idn, wn, cbn, g, pt);
-    load_ids(idn, ids, wnn, cbn + item_chunks(wn), g, pt);
+    stage_records<PRE>(S.rst[g][p ^ 1u], rec, idn, wn, cbn, g, pt);
+    load_ids<PRE>(idn, ids, wnn, cbn + item_chunks(wn), g, pt);
     const WorkItem w3 = it + 3 * G < nitems ? items[it + 3 * G] : none;
     const StarRec* rs = S.rst[g][p];
     const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
@@ -183,7 +191,7 @@ __device__ __forceinline__ void ws_producer(WsSmem& S, const uint32_t* __restric
       StarRec r = {};
       if (pt < nvalid) {
         const uint32_t off = base - wi.jb + (uint32_t)pt;
-        r = off < (uint32_t)WS_RSTAGE ? rs[off] : rec[__ldg(&ids[base + pt])];
+        r = off < (uint32_t)WS_RSTAGE ? rs[off] : (PRE ? rec[base + pt] : rec[__ldg(&ids[base + pt])]);
       }
       int c0 = 0, c1 = -1, r0 = 0, r1 = -1;
       uint32_t key = WS_NBIN;
@@ -196,29 +204,37 @@ __device__ __forceinline__ void ws_producer(WsSmem& S, const uint32_t* __restric
         if (c0 <= c1 && r0 <= r1)
           key = (uint32_t)((ly < 0 ? 0 : 1 + (r0 >> 4)) * WS_NSK + (lx < 0 ? 0 : 1 + (c0 >> 3)));
       }
+      // PRE: this chunk's bin starts (k_chsort), loaded ahead of the stage wait
+      uint32_t cbv = 0u;
+      if (PRE && pt <= WS_NBIN && nvalid > 0)
+        cbv = __ldg(&cbin[(size_t)((base >> 8) + wi.tile) * (WS_NBIN + 1) + pt]);
       // stars of the warp with the same key (what __match_any_sync gives, from 7 ballots: MATCH.ANY costs a loop over
       // the distinct keys of the warp)
-      uint32_t peers = 0xffffffffu;
+      uint32_t peers = 0xffffffffu, rank = 0u;
+      if (!PRE) {
 #pragma unroll
       for (int b = 0; b < 7; ++b) {
         const uint32_t kb = (key >> b) & 1u;
         const uint32_t m = __ballot_sync(0xffffffffu, kb);
         peers &= kb ? m : ~m;
       }
-      const uint32_t rank = __popc(peers & lt);
+      rank = __popc(peers & lt);
       // hist was last read by producer warp 0's scan of the previous chunk, before its second producer barrier
       hist[pw][lane] = 0u;
       hist[pw][lane + 32] = 0u;
       if (lane < WS_NBIN - 64) hist[pw][lane + 64] = 0u;
       __syncwarp();
       if (rank == 0 && key < WS_NBIN) hist[pw][key] = __popc(peers);
+      }
       WS_T(p1);
-      prod_barrier(g);
+      if (!PRE) prod_barrier(g);
       WS_T(p2);
       // stage s is free once every consumer warp has walked the chunk it held WS_NSTAGE chunks ago
       mbar_wait(&S.empty[s], ph ^ 1u);
       WS_T(p3);
-      if (pw == 0) {
+      if (PRE) {
+        if (pt <= WS_NBIN) T.binstart[pt] = cbv;
+      } else if (pw == 0) {
         uint32_t tot[3], sum = 0;
 #pragma unroll
         for (int h = 0; h < 3; ++h) {
@@ -249,7 +265,7 @@ __device__ __forceinline__ void ws_producer(WsSmem& S, const uint32_t* __restric
           ex += tot[h];
         }
       }
-      prod_barrier(g);
+      if (!PRE) prod_barrier(g);
       WS_T(p4);
       // ---- the star's profiles at its sorted place j (exactly k_tile_sb's values and slots)
 #ifdef WS_NOPROF
@@ -257,7 +273,7 @@ __device__ __forceinline__ void ws_producer(WsSmem& S, const uint32_t* __restric
 #else
       if (key < WS_NBIN) {
 #endif
-        const uint32_t j = T.binstart[key] + binoff[pw][key] + rank;
+        const uint32_t j = PRE ? (uint32_t)pt : T.binstart[key] + binoff[pw][key] + rank;
         const float yr = r.y - (float)IY0, xr = r.x - (float)X0;  // exact
         const float2 sk2 = make_float2(sk, sk), s2 = make_float2(r.s, r.s);
         const int b0 = (int)(key / WS_NSK) - 1, q0 = (int)(key % WS_NSK) - 1;
@@ -470,13 +486,14 @@ __device__ __forceinline__ void ws_consumer(WsSmem& S, const FrameParams& fp, vo
   }
 }
 
-template <bool INTEG>
+template <bool INTEG, bool PRE>
 __global__ void __launch_bounds__(WS_THREADS, WS_CTAS) k_tile_ws(const uint32_t* __restrict__ ids,
                                                            const StarRec* __restrict__ rec, FrameParams fp,
                                                            void* __restrict__ out_, const WorkItem* __restrict__ items,
                                                            const uint2* __restrict__ split_tab,
                                                            float* __restrict__ part_buf, uint32_t* __restrict__ done,
-                                                           Header* hdr, float* __restrict__ seg_scratch) {
+                                                           Header* hdr, float* __restrict__ seg_scratch,
+                                                           const uint16_t* __restrict__ cbin) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   WsSmem& S = *reinterpret_cast<WsSmem*>(smem_raw);
   const int tid = threadIdx.x;
@@ -492,9 +509,122 @@ __global__ void __launch_bounds__(WS_THREADS, WS_CTAS) k_tile_ws(const uint32_t*
   __syncthreads();
   const uint32_t nitems = __ldcg(&hdr->nitems);
   if (tid >= 32 * WS_CONS)
-    ws_producer<INTEG>(S, ids, rec, fp, items, nitems);
+    ws_producer<INTEG, PRE>(S, ids, rec, fp, items, nitems, cbin);
   else
     ws_consumer(S, fp, out_, split_tab, part_buf, done, seg_scratch);
+}
+
+
+// ---------------------------------------------------------------------------------------------------------------
+// k_chsort: the producers' per-chunk sort, done ahead for the whole frame.  One warp per (work item, chunk k mod 4):
+// the chunk's <= 256 stars (list positions base + 32 r + lane, r = 0..7) get their corner bin exactly as a producer
+// computes it, the chunk's bin starts go to cbin[(base >> 8) + tile] (86 u16: bins 0..84 and the total), and every
+// record is written to srec[base + its stable rank by (bin, list position)] -- the order k_tile_sb / k_tile_ws walk
+// (reading R12): k_tile_ws<PRE> then reads each chunk's records contiguously and only evaluates profiles.  The slot
+// index (base >> 8) + tile is unique: chunks of one tile start 256 apart, and a later tile's first chunk starts at a
+// later list position.
+// ---------------------------------------------------------------------------------------------------------------
+constexpr int CHS_WARPS = 8;
+__global__ void __launch_bounds__(32 * CHS_WARPS) k_chsort(const uint32_t* __restrict__ ids,
+                                                           const StarRec* __restrict__ rec, FrameParams fp,
+                                                           const WorkItem* __restrict__ items,
+                                                           const Header* __restrict__ hdr, StarRec* __restrict__ srec,
+                                                           uint16_t* __restrict__ cbin) {
+  static_assert(WS_CHUNK == 256, "k_chsort sorts 256-star chunks (8 rounds of 32)");
+  __shared__ uint32_t cnt[CHS_WARPS][WS_NBIN + 1];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  const uint32_t gw = blockIdx.x * CHS_WARPS + (uint32_t)w;
+  const uint32_t item = gw >> 2;
+  if (item >= __ldcg(&hdr->nitems)) return;
+  const WorkItem wi = items[item];
+  const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
+  const int X0 = tx * TILE_W, Y0 = ty * TILE_H, IY0 = fp.row0 + Y0;
+  const int TWe = min(TILE_W, fp.W - X0), THe = min(TILE_H, fp.rows - Y0);
+  uint32_t* c = cnt[w];
+  for (uint32_t base = wi.jb + (gw & 3u) * WS_CHUNK; base < wi.je; base += 4u * WS_CHUNK) {
+    const uint32_t n = min((uint32_t)WS_CHUNK, wi.je - base);
+    StarRec r[8];
+    uint32_t key[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const uint32_t e = (uint32_t)(32 * k + lane);
+      r[k] = e < n ? rec[__ldg(&ids[base + e])] : StarRec{0.f, 0.f, 0.f, LO_CULLED};
+    }
+    for (int b = lane; b <= WS_NBIN; b += 32) c[b] = 0u;
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      key[k] = WS_NBIN;
+      if ((uint32_t)(32 * k + lane) < n) {
+        const int lx = lo_x_of(r[k].lo) - X0, ly = lo_y_of(r[k].lo) - IY0;
+        const int c0 = max(lx, 0), c1 = min(lx + fp.R - 1, TWe - 1);
+        const int r0 = max(ly, 0), r1 = min(ly + fp.R - 1, THe - 1);
+        if (c0 <= c1 && r0 <= r1)
+          key[k] = (uint32_t)((ly < 0 ? 0 : 1 + (r0 >> 4)) * WS_NSK + (lx < 0 ? 0 : 1 + (c0 >> 3)));
+        atomicAdd(&c[key[k]], 1u);  // bin WS_NBIN collects the stars that miss the tile (placed last)
+      }
+    }
+    __syncwarp();
+    // exclusive scan of the 86 bin counts (3 per lane) -> bin starts; the chunk's row of cbin
+    uint32_t v[3], sum = 0;
+#pragma unroll
+    for (int h = 0; h < 3; ++h) {
+      const int bin = 3 * lane + h;
+      v[h] = bin <= WS_NBIN ? c[bin] : 0u;
+      sum += v[h];
+    }
+    uint32_t incl = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += u;
+    }
+    uint32_t ex = incl - sum;
+    uint16_t* row = cbin + (size_t)((base >> 8) + wi.tile) * (WS_NBIN + 1);
+    __syncwarp();
+#pragma unroll
+    for (int h = 0; h < 3; ++h) {
+      const int bin = 3 * lane + h;
+      if (bin <= WS_NBIN) {
+        c[bin] = ex;                // running position of the bin
+        row[bin] = (uint16_t)ex;    // bin starts; row[WS_NBIN] = the stars that meet the tile
+      }
+      ex += v[h];
+    }
+    __syncwarp();
+    // stable placement, round by round (list order): rank among the round's equal keys, then the bin's cursor
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const bool in = (uint32_t)(32 * k + lane) < n;
+      const uint32_t mi = __ballot_sync(0xffffffffu, in);
+      uint32_t peers = mi;  // the round's lanes with the same key
+#pragma unroll
+      for (int b = 0; b < 7; ++b) {
+        const uint32_t kb = (key[k] >> b) & 1u;
+        const uint32_t m = __ballot_sync(0xffffffffu, kb && in);
+        peers &= kb ? m : ~m;
+      }
+      const uint32_t rank = __popc(peers & lt);
+      const uint32_t pos = in ? c[key[k]] + rank : 0u;
+      __syncwarp();
+      if (in && rank == 0) c[key[k]] += __popc(peers);
+      __syncwarp();
+      if (in) srec[base + pos] = r[k];
+    }
+    __syncwarp();
+  }
+}
+
+size_t chsort_slots(int64_t ntiles, int64_t pmax) { return (size_t)(pmax / WS_CHUNK + ntiles + 2); }
+size_t chsort_words16() { return WS_NBIN + 1; }
+
+void launch_chsort(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, const WorkItem* items, int part_cap,
+                   const Header* hdr, StarRec* srec, uint16_t* cbin, cudaStream_t st) {
+  const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
+  const int64_t warps = 4 * (ntiles + part_cap);
+  k_chsort<<<(unsigned)((warps + CHS_WARPS - 1) / CHS_WARPS), 32 * CHS_WARPS, 0, st>>>(ids, rec, fp, items, hdr, srec,
+                                                                                      cbin);
 }
 
 #ifdef STARSIM_WS_TIMING
@@ -512,22 +642,23 @@ extern "C" int starsim_debug_ws_timing(double* out10, int reset) {
 #endif
 
 void init_tile_ws_kernel() {
-  cudaFuncSetAttribute(k_tile_ws<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WsSmem));
-  cudaFuncSetAttribute(k_tile_ws<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WsSmem));
+  cudaFuncSetAttribute(k_tile_ws<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WsSmem));
+  cudaFuncSetAttribute(k_tile_ws<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WsSmem));
+  cudaFuncSetAttribute(k_tile_ws<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WsSmem));
+  cudaFuncSetAttribute(k_tile_ws<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WsSmem));
 }
 
 void launch_tile_ws(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
-                    cudaStream_t st, float* seg_scratch) {
+                    cudaStream_t st, float* seg_scratch, const StarRec* srec, const uint16_t* cbin) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
   const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)WS_CTAS * num_sms);  // persistent CTAs
-  if (fp.psf)
-    k_tile_ws<true><<<(unsigned)grid, WS_THREADS, sizeof(WsSmem), st>>>(ids, rec, fp, out, items, split_tab,
-                                                                         part_buf, done, hdr, seg_scratch);
-  else
-    k_tile_ws<false><<<(unsigned)grid, WS_THREADS, sizeof(WsSmem), st>>>(ids, rec, fp, out, items, split_tab,
-                                                                          part_buf, done, hdr, seg_scratch);
+  // srec != nullptr: the chunks were presorted by k_chsort (srec, cbin)
+  auto* k = srec ? (fp.psf ? k_tile_ws<true, true> : k_tile_ws<false, true>)
+                 : (fp.psf ? k_tile_ws<true, false> : k_tile_ws<false, false>);
+  k<<<(unsigned)grid, WS_THREADS, sizeof(WsSmem), st>>>(ids, srec ? srec : rec, fp, out, items, split_tab, part_buf,
+                                                         done, hdr, seg_scratch, cbin);
 }
 
 }  // namespace starsim
