@@ -74,8 +74,10 @@ constexpr uint32_t ZERO_ENT = ZERO_GX * 32u << 16;  // gy byte offset 0, all-zer
 // (u8 / u16 image) instead of the fp32 image; CIRC: the pixel-circle ROI (NEXT-3, reading R21) -- the walk masks each
 // of the lane's 4 x 8 pixels by the integer disc test against the star's ROI origin (looked up through its band slot),
 // 2 CTAs per SM for the extra registers.  k_tile serves the circle for R > SB_MAXR (k_tile_sb below).
+// CTAs per SM: 2 (128 registers) -- measured 1.2-1.35x faster than 3 at 80 registers on the clustered C4 frames at
+// R = 21 / 31 / 63 (profiles/r2_ktile_ab.txt), and spill-free
 #ifndef TILE_MINB_OPT
-#define TILE_MINB_OPT 3
+#define TILE_MINB_OPT 2
 #endif
 template <bool INTEG, bool GRAY, bool CIRC>
 __global__ void __launch_bounds__(TILE_THREADS, CIRC ? 2 : TILE_MINB_OPT) k_tile(const uint32_t* __restrict__ ids,
@@ -122,7 +124,12 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? 2 : TILE_MINB_OPT) k_tile
   uint32_t segs_done = 0;  // SPLIT_LEN segments of this item already in the scratch (tile_common.cuh)
   // this thread's star record of the current chunk, loaded one chunk ahead (its latency hides behind the
   // accumulation of the previous chunk)
+#ifdef KT_REG_PREFETCH
+  StarRec rnext = {};
+  if (wi.jb + tid < j1) rnext = rec[ids[wi.jb + tid]];
+#else
   if (wi.jb + tid < j1) prefetch_rec(&S.rn[tid], rec, ids[wi.jb + tid]);
+#endif
   for (uint32_t base = wi.jb; base < j1;) {
     // ======================= prep: thread = star (base + tid)
     // chunks never cross a SPLIT_LEN segment boundary of the list (segments are summed like the parts of a split tile)
@@ -130,8 +137,12 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? 2 : TILE_MINB_OPT) k_tile
     const int nvalid = (int)min((uint32_t)CHUNK, seg_end - base);
     const bool valid = tid < nvalid;
     StarRec r = {};
+#ifdef KT_REG_PREFETCH
+    r = rnext;
+#else
     asm volatile("cp.async.wait_all;\n" ::: "memory");
     if (valid) r = S.rn[tid];
+#endif
     int c0 = 0, c1 = -1, r0 = 0, r1 = -1;
     if (valid) {
       const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
@@ -337,7 +348,11 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? 2 : TILE_MINB_OPT) k_tile
       for (uint32_t st = len; st < steps; ++st) ent[st * (NBANDS * NSTRIPS)] = ZERO_ENT;
     __syncthreads();
 
+#ifdef KT_REG_PREFETCH
+    if (nb + tid < j1) rnext = rec[nid];
+#else
     if (nb + tid < j1) prefetch_rec(&S.rn[tid], rec, nid);
+#endif
     // ======================= accumulate: lane group q walks the (padded) list of block (B, Q)
     {
 #pragma unroll 4

@@ -499,6 +499,28 @@ def test_ws_equals_sb_bitwise(torch_dev, psf, W, H, n, R, seed):
     assert torch.equal(out["ws"], out["sb"])
 
 
+@pytest.mark.parametrize("W,H,n,R,seed", [(1000, 700, 60000, 15, 24), (4096, 4096, 1000000, 15, 1),
+                                          (515, 301, 700, 17, 10), (700, 500, 0, 9, 6)])
+def test_ws_presorted_equals_sb_bitwise(torch_dev, monkeypatch, W, H, n, R, seed):
+    """k_tile_ws fed by k_chsort (STARSIM_WS_PRESORT=1: every 256-star chunk presorted by corner bin, records in walk
+    order) gives k_tile_sb's image bit for bit -- split heavy tiles, empty frames and R = 17 included."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context
+    f = synth.uniform_field(n, W, H, seed=seed, mag_hi=15.0)
+    if n == 60000:
+        f = _dense_field(n, W, H, 500.0, 350.0, 120.0, seed=seed)
+    args = to_dev(torch_dev, f)
+    monkeypatch.setenv("STARSIM_WS_PRESORT", "1")
+    with Context(0) as c:
+        c.set_tile_kernel("ws")
+        pre = c.render(*args, W, H, R / 6, R, 1.0)
+    monkeypatch.delenv("STARSIM_WS_PRESORT")
+    with Context(0) as c:
+        c.set_tile_kernel("sb")
+        ref = c.render(*args, W, H, R / 6, R, 1.0)
+    assert torch.equal(pre, ref)
+
+
 def test_mode_setters_einval(torch_dev):
     from paper_conf_ipps_lizzh12_b200 import Context, StarsimError
     with Context(0) as c:

@@ -20,6 +20,8 @@ S=/usr/local/cuda/bin/compute-sanitizer
 for t in memcheck synccheck initcheck; do
   timeout 900 $S --tool $t --print-limit 20 python tools/sanitize_run.py > gpurun_out/${TAG}_sanitize_$t.log 2>&1
 done
+timeout 900 $S --tool racecheck --racecheck-report all --print-limit 20 python tools/sanitize_run.py --quick \
+  > gpurun_out/${TAG}_sanitize_racecheck_all.log 2>&1
 for k in lists sb ws t8; do
   timeout 600 $S --tool racecheck --racecheck-report all --print-limit 20 python tools/sanitize_run.py --quick \
     --kernels=$k > gpurun_out/${TAG}_sanitize_racecheck_$k.log 2>&1

@@ -3,7 +3,8 @@
 initcheck):  compute-sanitizer --tool racecheck python tools/sanitize_run.py
 C1 (1024^2, 1000 stars, R=5) and a heavy-tile field (256^2, 30K stars in a 40-px disc: split tiles, partial buffers,
 1024-star segments) through every tile kernel (lists, sb, ws, t8; both binning pipelines), a band, the gray epilogue,
-the integrated PSF, the circle ROI, the star-centric kernels, quantize, upload_aos and the band routing."""
+the integrated PSF, the circle ROI, the star-centric kernels, quantize, upload_aos and the band routing; a sparse 4096 x 2048
+frame (2,000 stars) for k_tile_lite; k_tile_ws fed by k_chsort."""
 import os
 import sys
 
@@ -30,7 +31,8 @@ def main():
     only = next((a.split("=", 1)[1].split(",") for a in sys.argv if a.startswith("--kernels=")), None)
     dev = torch.device("cuda:0")
     c1 = synth.CONFIGS["C1"]
-    cases = [("C1", c1.field(), c1.W, c1.H, c1.R, c1.sigma), ("heavy", heavy(30000, 256, 256, 3), 256, 256, 15, 2.5)]
+    cases = [("C1", c1.field(), c1.W, c1.H, c1.R, c1.sigma), ("heavy", heavy(30000, 256, 256, 3), 256, 256, 15, 2.5),
+             ("sparse", synth.uniform_field(2000, 4096, 2048, seed=5), 4096, 2048, 15, 2.5)]  # k_tile_lite
     with Context(0) as ctx:
         for name, f, W, H, R, sigma in cases:
             x, y, m = (torch.from_numpy(a).to(dev) for a in (f.x, f.y, f.mag))
@@ -62,6 +64,13 @@ def main():
                 img = ctx.render(x, y, m, W, H, sigma, R, 1.0)
                 ctx.quantize(img, 8)
                 ctx.upload_aos(f.aos()[:1000])
+            if not quick or name != "sparse":
+                # k_tile_ws fed by k_chsort (a context created with STARSIM_WS_PRESORT=1)
+                os.environ["STARSIM_WS_PRESORT"] = "1"
+                with Context(0) as cpre:
+                    cpre.set_tile_kernel("ws")
+                    cpre.render(x, y, m, W, H, sigma, R, 1.0)
+                del os.environ["STARSIM_WS_PRESORT"]
             torch.cuda.synchronize()
             print(name, "ok", flush=True)
 
