@@ -31,7 +31,13 @@ constexpr int DC_PER = DB_CTA / DC_THREADS;
 #define DP_THREADS_OPT 1024
 #endif
 constexpr int DP_THREADS = DP_THREADS_OPT;        // k_dplace
-constexpr int DP_MINB = 2048 / DP_THREADS;        // CTAs per SM (all 245 CTAs of a 1M-star frame resident)
+#ifndef DP_MINB_OPT
+#define DP_MINB_OPT (2048 / DP_THREADS_OPT)
+#endif
+#ifndef DC_MINB_OPT
+#define DC_MINB_OPT 2
+#endif
+constexpr int DP_MINB = DP_MINB_OPT;              // CTAs per SM (all 245 CTAs of a 1M-star frame resident)
 constexpr int DP_WARPS = DP_THREADS / 32;
 constexpr int DP_KEYS = DB_CTA * 4;              // at most 2 x 2 tiles per star
 constexpr int DP_SPT = DB_CTA / DP_THREADS;      // stars per thread (strided by DP_THREADS)
@@ -46,7 +52,7 @@ static_assert(DP_WARPS <= 32, "dp_block_scan scans the warp sums with one warp")
 // t0 + ntx + 1 if both); DP_NONE if the star is culled.  Written by k_dcount, read by k_dplace.
 constexpr uint32_t DP_NONE = 0xFFFFFFFFu;
 
-__global__ void __launch_bounds__(DC_THREADS, 2) k_dcount(const float* __restrict__ X, const float* __restrict__ Y,
+__global__ void __launch_bounds__(DC_THREADS, DC_MINB_OPT) k_dcount(const float* __restrict__ X, const float* __restrict__ Y,
                                                        const float* __restrict__ M, int64_t n, FrameParams fp,
                                                        StarRec* __restrict__ rec, uint32_t* __restrict__ codes,
                                                        uint32_t* __restrict__ C,
