@@ -57,9 +57,10 @@ struct starsim_ctx {
   int32_t bin_impl = 0;   // starsim_set_binning: 0 auto (dbin.cu when it applies), 1 always bin.cu's pipeline
   std::string err;
   const uint32_t* n_dev = nullptr;  // starsim_set_star_count: device-resident star count of the tiled renders
+  int dfused_grid = 0;              // largest co-resident k_dfused grid (0: the three-kernel binning only)
   bool ws_presort = false;          // k_tile_ws reads chunks presorted by k_chsort (env STARSIM_WS_PRESORT=1; slower)
   Buf rec, slots, ids, tmp, tile_off, items, split_tab, parts, partial, zeroed, stage, cmat, codes, segs, srec, sbin, sext,
-      rblk, cbin;
+      rblk, cbin, gbar;
   uint64_t scratch_gen = 0;  // bumped whenever a scratch buffer moves (invalidates the captured graph)
   // last tiled render, for starsim_get_bins
   bool have_bins = false;
@@ -243,6 +244,15 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
                       (uint2*)c->split_tab.p, part_cap, done, ids, st);
       });
       if ((rc = check_launch(c, "k_dsmall"))) return rc;
+    } else if (n > 0 && c->dfused_grid > 0 && dbin_ctas(n) <= c->dfused_grid) {
+      // every CTA of the catalogue resident: count, column scan and placement in one cooperative launch (k_dfused)
+      cudaError_t le = cudaSuccess;
+      timed(c, 0, st, [&] {
+        le = launch_dfused(x, y, mag, n, fp, rec, C, cnt, (int)ntiles, tile_off, hdr, (WorkItem*)c->items.p,
+                           (uint2*)c->split_tab.p, part_cap, done, ids, (uint32_t*)c->gbar.p, st);
+      });
+      if (le != cudaSuccess) return cuda_fail(c, le, "k_dfused (cooperative launch)");
+      if ((rc = check_launch(c, "k_dfused"))) return rc;
     } else if (n > 0) {
       timed(c, 0, st, [&] { launch_dcount(x, y, mag, n, fp, rec, (uint32_t*)c->codes.p, C, (int)ntiles, st); });
       if ((rc = check_launch(c, "k_dcount"))) return rc;
@@ -397,6 +407,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
     return rc;
   if (dbin_ok(fp, ntiles) && (rc = grow(c, c->codes, sizeof(uint32_t) * (size_t)(n > 0 ? n : 1), "tile boxes")))
     return rc;
+  if ((rc = grow(c, c->gbar, 64, "grid barrier"))) return rc;
 
   GraphKey key{x, y, mag, out, fp.n_dev, n, W, H, row0, rows, R, obits, c->psf | c->roi << 1, c->tile_impl, c->bin_impl, fp.ndst, {}, sigma, gain, st,
                c->scratch_gen};
@@ -470,6 +481,10 @@ int starsim_create(starsim_ctx** out, int cuda_device) {
   c->dev = cuda_device;
   c->num_sms = prop.multiProcessorCount;
   init_kernels();
+  // k_dfused (one cooperative launch for the three binning kernels) is opt-in: STARSIM_DFUSED=1 at context creation
+  // (same CSR; measured 2-6 us slower per frame than the three graph-replayed kernels)
+  const char* df = getenv("STARSIM_DFUSED");
+  c->dfused_grid = (df && df[0] == '1') ? dfused_max_grid(c->num_sms) : 0;
   const char* wp = getenv("STARSIM_WS_PRESORT");
   c->ws_presort = wp && wp[0] == '1';
   const char* ng = getenv("STARSIM_NO_GRAPH");
@@ -487,7 +502,7 @@ void starsim_destroy(starsim_ctx* c) {
     if (c->have_graph) cudaGraphExecDestroy(c->gexec);
     Buf* bufs[] = {&c->rec, &c->slots, &c->ids, &c->tmp, &c->tile_off, &c->items, &c->split_tab, &c->parts,
                    &c->partial, &c->zeroed, &c->stage, &c->cmat, &c->codes, &c->segs, &c->srec, &c->sbin, &c->sext,
-                   &c->rblk, &c->cbin};
+                   &c->rblk, &c->cbin, &c->gbar};
     for (Buf* b : bufs)
       if (b->p) cudaFree(b->p);
     for (auto& l : c->pending) {

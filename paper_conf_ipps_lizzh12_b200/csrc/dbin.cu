@@ -300,7 +300,7 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
   }
   __syncthreads();
   // first list position of every group: tile_off[t] + (pairs of tile t in the CTAs before)
-  for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = S.toff[t] + (C ? C[(int64_t)cta * ntiles + t] : 0u);
+  for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = S.toff[t] + (C ? __ldcg(&C[(int64_t)cta * ntiles + t]) : 0u);
   __syncthreads();
   // a pair's rank in its group = the group's stars with a smaller index
 #pragma unroll
@@ -392,6 +392,134 @@ __global__ void __launch_bounds__(DP_THREADS, 1) k_dsmall(const float* __restric
   dp_place(S, code, fp, nullptr, 1, ntiles, ids);
 }
 
+
+// ---------------------------------------------------------------------------------------------------------------
+// k_dfused: k_dcount, k_dcolscan and k_dplace in ONE cooperative launch (every CTA resident: the driver refuses the
+// launch otherwise), separated by two grid barriers -- no launch gaps, and each CTA keeps its stars' tile boxes in
+// registers from the count to the placement.  Same records, count matrix, plan and CSR, bit for bit.
+//   phase 1 (CTA c < live): step a1 + the CTA's pair counts -> row c of C;
+//   barrier;
+//   phase 2: 32-tile column blocks b = c, c + gridDim, ...: the live rows staged in shared memory, every tile's
+//            column scanned (exclusive, in place) and its total -> cnt;
+//   barrier;
+//   phase 3: step a2 (every CTA, the tiles t = c mod gridDim) and, for the live CTAs, the placement.
+// The barrier counter is zeroed by a memset node before every launch (api.cu), so no state survives a frame.
+// ---------------------------------------------------------------------------------------------------------------
+constexpr int DF_ROWS = 256;
+struct DfSmem {
+  union {
+    uint32_t cnt[DB_MAXT];
+    uint32_t sm[DF_ROWS][33];
+    DpSmem dp;
+  };
+};
+
+__device__ __forceinline__ void grid_barrier(uint32_t* bar, uint32_t target) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(bar, 1u);
+    uint32_t v;
+    do {
+      asm volatile("ld.acquire.gpu.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
+    } while (v < target);
+  }
+  __syncthreads();
+}
+
+__global__ void __launch_bounds__(DP_THREADS, 2) k_dfused(const float* __restrict__ X, const float* __restrict__ Y,
+                                                          const float* __restrict__ M, int64_t n, FrameParams fp,
+                                                          StarRec* __restrict__ rec, uint32_t* __restrict__ C,
+                                                          uint32_t* __restrict__ cntg, int ntiles,
+                                                          uint32_t* __restrict__ tile_off, Header* hdr,
+                                                          WorkItem* __restrict__ items, uint2* __restrict__ split_tab,
+                                                          int part_cap, uint32_t* __restrict__ done,
+                                                          uint32_t* __restrict__ ids, uint32_t* bar) {
+  static_assert(DP_THREADS == DC_THREADS && DP_SPT == DC_PER, "k_dcount's star-to-thread map");
+  static_assert(DP_THREADS == 1024, "phase 2: 32 warps, one per tile of a 32-tile block");
+  extern __shared__ __align__(16) unsigned char dsm_raw[];
+  DfSmem& F = *reinterpret_cast<DfSmem*>(dsm_raw);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, cta = blockIdx.x;
+  const uint32_t nC = gridDim.x;
+  n = frame_n(n, fp);
+  const int live = dbin_live_ctas(n);
+  // ---- phase 1 (k_dcount)
+  uint32_t code[DP_SPT];
+#pragma unroll
+  for (int k = 0; k < DP_SPT; ++k) code[k] = DP_NONE;
+  if (cta < live) {
+    for (int t = tid; t < ntiles; t += DP_THREADS) F.cnt[t] = 0u;
+    const int64_t i0 = (int64_t)cta * DB_CTA + tid;
+    float xs[DP_SPT], ys[DP_SPT], ms[DP_SPT];
+#pragma unroll
+    for (int k = 0; k < DP_SPT; ++k) {
+      const int64_t i = i0 + (int64_t)k * DP_THREADS;
+      const bool in = i < n;
+      xs[k] = in ? __ldg(&X[i]) : 0.f;
+      ys[k] = in ? __ldg(&Y[i]) : 0.f;
+      ms[k] = in ? __ldg(&M[i]) : 0.f;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < DP_SPT; ++k) {
+      const int64_t i = i0 + (int64_t)k * DP_THREADS;
+      if (i >= n) break;
+      int cx0, cx1, cy0, cy1;
+      const StarRec r = prep_star(xs[k], ys[k], ms[k], fp, cx0, cx1, cy0, cy1);
+      rec[i] = r;
+      if (r.lo != LO_CULLED) {
+        const int tx0 = cx0 / TILE_W, tx1 = cx1 / TILE_W;
+        const int ty0 = (cy0 - fp.row0) / TILE_H, ty1 = (cy1 - fp.row0) / TILE_H;
+        for (int ty = ty0; ty <= ty1; ++ty)
+          for (int tx = tx0; tx <= tx1; ++tx) atomicAdd(&F.cnt[ty * fp.ntx + tx], 1u);
+        code[k] = (uint32_t)(ty0 * fp.ntx + tx0) | (uint32_t)(tx1 - tx0) << 16 | (uint32_t)(ty1 - ty0) << 17;
+      }
+    }
+    __syncthreads();
+    for (int t = tid; t < ntiles; t += DP_THREADS) C[(int64_t)cta * ntiles + t] = F.cnt[t];
+  }
+  grid_barrier(bar, nC);
+  // ---- phase 2 (k_dcolscan): 32-tile column blocks, warp w = tile t0 + w, lane l = rows l + 32 k
+  for (int t0 = cta * 32; t0 < ntiles; t0 += (int)nC * 32) {
+    const bool tin = t0 + lane < ntiles;
+    uint32_t carry = 0;
+    for (int r0 = 0; r0 < live; r0 += DF_ROWS) {
+      const int rows = min(DF_ROWS, live - r0);
+#pragma unroll
+      for (int i = 0; i < DF_ROWS / 32; ++i) {
+        const int r = warp + 32 * i;
+        if (r < rows) F.sm[r][lane] = tin ? __ldcg(&C[(int64_t)(r0 + r) * ntiles + t0 + lane]) : 0u;
+      }
+      __syncthreads();
+      for (int k = 0; k < DF_ROWS / 32 && 32 * k < rows; ++k) {
+        const int r = 32 * k + lane;
+        const uint32_t v = r < rows ? F.sm[r][warp] : 0u;
+        uint32_t incl = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
+          if (lane >= o) incl += u;
+        }
+        if (r < rows) F.sm[r][warp] = carry + incl - v;
+        carry += __shfl_sync(0xffffffffu, incl, 31);
+      }
+      __syncthreads();
+#pragma unroll
+      for (int i = 0; i < DF_ROWS / 32; ++i) {
+        const int r = warp + 32 * i;
+        if (r < rows && tin) C[(int64_t)(r0 + r) * ntiles + t0 + lane] = F.sm[r][lane];
+      }
+      __syncthreads();
+    }
+    if (lane == 0 && t0 + warp < ntiles) cntg[t0 + warp] = carry;
+  }
+  grid_barrier(bar, 2u * nC);
+  // ---- phase 3 (k_dplace)
+  dp_scan_tiles(F.dp, cntg, ntiles, (int)nC, tile_off, hdr, items, split_tab, part_cap, done);
+  if (cta >= live) return;
+  dp_place(F.dp, code, fp, C, (int)nC, ntiles, ids);
+}
+
 size_t dbin_smem(int) { return sizeof(DpSmem); }
 
 int dbin_ctas(int64_t n) { return (int)((n + DB_CTA - 1) / DB_CTA); }
@@ -399,9 +527,40 @@ int dbin_ctas(int64_t n) { return (int)((n + DB_CTA - 1) / DB_CTA); }
 void init_dbin_kernels() {
   cudaFuncSetAttribute(k_dplace, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DpSmem));
   cudaFuncSetAttribute(k_dsmall, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DpSmem));
+  cudaFuncSetAttribute(k_dfused, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DfSmem));
 }
 
 bool dsmall_ok(int64_t n) { return n <= DB_CTA; }
+
+// the largest co-resident k_dfused grid on this device (0: none); the fused binning applies when the catalogue's
+// CTAs fit it (and the cooperative launch re-checks)
+int dfused_max_grid(int num_sms) {
+  int nb = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_dfused, DP_THREADS, sizeof(DfSmem)) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return nb * num_sms;
+}
+
+cudaError_t launch_dfused(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp,
+                          StarRec* rec, uint32_t* C, uint32_t* cnt, int ntiles, uint32_t* tile_off, Header* hdr,
+                          WorkItem* items, uint2* split_tab, int part_cap, uint32_t* done, uint32_t* ids,
+                          uint32_t* bar, cudaStream_t st) {
+  cudaMemsetAsync(bar, 0, sizeof(uint32_t), st);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)dbin_ctas(n));
+  cfg.blockDim = dim3(DP_THREADS);
+  cfg.dynamicSmemBytes = sizeof(DfSmem);
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, k_dfused, x, y, m, n, fp, rec, C, cnt, ntiles, tile_off, hdr, items, split_tab,
+                            part_cap, done, ids, bar);
+}
 
 void launch_dsmall(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
                    int ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items, uint2* split_tab, int part_cap,

@@ -17,6 +17,11 @@ void init_dbin_kernels();
 size_t dbin_smem(int ntiles);
 int dbin_ctas(int64_t n);
 bool dsmall_ok(int64_t n);  // k_dsmall applies (at most DB_CTA stars)
+int dfused_max_grid(int num_sms);
+cudaError_t launch_dfused(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp,
+                          StarRec* rec, uint32_t* C, uint32_t* cnt, int ntiles, uint32_t* tile_off, Header* hdr,
+                          WorkItem* items, uint2* split_tab, int part_cap, uint32_t* done, uint32_t* ids,
+                          uint32_t* bar, cudaStream_t st);
 void launch_dsmall(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
                    int ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items, uint2* split_tab, int part_cap,
                    uint32_t* done, uint32_t* ids, cudaStream_t st);

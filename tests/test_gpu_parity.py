@@ -521,6 +521,28 @@ def test_ws_presorted_equals_sb_bitwise(torch_dev, monkeypatch, W, H, n, R, seed
     assert torch.equal(pre, ref)
 
 
+@pytest.mark.parametrize("W,H,n,R,seed", [(4096, 4096, 1000000, 15, 3), (700, 530, 20000, 9, 4),
+                                          (1000, 700, 60000, 15, 24), (640, 1024, 5000, 31, 5)])
+def test_fused_binning_same_csr_and_image(torch_dev, monkeypatch, W, H, n, R, seed):
+    """k_dfused (STARSIM_DFUSED=1: count, column scan and placement in one cooperative launch with two grid barriers)
+    writes the CSR of the oracle's bins bit for bit and the same image as the three-kernel binning."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context
+    f = synth.uniform_field(n, W, H, seed=seed, mag_hi=15.0)
+    if n == 60000:
+        f = _dense_field(n, W, H, 500.0, 350.0, 120.0, seed=seed)
+    args = to_dev(torch_dev, f)
+    with Context(0) as c:
+        ref = c.render(*args, W, H, 2.5, R, 1.0)
+    monkeypatch.setenv("STARSIM_DFUSED", "1")
+    with Context(0) as c:
+        img = c.render(*args, W, H, 2.5, R, 1.0)
+        tw, th, off, ids = c.get_bins()
+    assert torch.equal(img, ref)
+    ro, ri = oracle.bins(f.x, f.y, f.mag, W, H, R, tw, th)
+    assert np.array_equal(off[:ro.size], ro) and np.array_equal(ids, ri)
+
+
 def test_mode_setters_einval(torch_dev):
     from paper_conf_ipps_lizzh12_b200 import Context, StarsimError
     with Context(0) as c:
