@@ -66,6 +66,14 @@ struct starsim_ctx {
   bool have_bins = false;
   cudaStream_t last_stream = nullptr;
   int64_t last_ntiles = 0;
+  // the last tiled render took the sparse path (no CSR built): starsim_get_bins bins these arrays on demand
+  bool last_sparse = false;
+  struct {
+    const float *x, *y, *m;
+    int64_t n;
+    FrameParams fp;
+    int tps, part_cap;
+  } sp{};
   // CUDA graph of the last render signature (non-default streams only; STARSIM_NO_GRAPH=1 disables)
   bool use_graphs = true;
   bool have_graph = false;
@@ -222,8 +230,8 @@ bool ws_presort(const starsim_ctx* c, const FrameParams& fp) {
 
 // Enqueue the tiled render on stream st: memset of the header + tile counters, k_prep, k_scan, k_scatter,
 // k_sortlists, k_tile.
-int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, const FrameParams& fp,
-                  int64_t ntiles, int tps, int part_cap, void* out, cudaStream_t st) {
+int enqueue_binning(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n,
+                    const FrameParams& fp, int64_t ntiles, int tps, int part_cap, cudaStream_t st) {
   Header* hdr = (Header*)c->zeroed.p;
   uint32_t* cnt = (uint32_t*)(hdr + 1);
   const size_t zbytes = sizeof(Header) + sizeof(uint32_t) * (CNT_STRIDE + 1) * (size_t)ntiles;
@@ -292,6 +300,27 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
     timed(c, 1, st, [&] { launch_sortlists(ids, (uint32_t*)c->tmp.p, tile_off, ntiles, n, st); });
     if ((rc = check_launch(c, "k_sortlists"))) return rc;
   }
+  return STARSIM_OK;
+}
+
+int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* mag, int64_t n, const FrameParams& fp,
+                  int64_t ntiles, int tps, int part_cap, void* out, cudaStream_t st, bool sparse) {
+  int rc;
+  if (sparse) {
+    // the sparse path (tile_sb.cu): records, then one CTA per tile that builds its own list -- no binning launches
+    timed(c, 0, st, [&] { launch_srec(x, y, mag, n, fp, (StarRec*)c->rec.p, st); });
+    if ((rc = check_launch(c, "k_srec"))) return rc;
+    timed(c, 3, st, [&] { launch_tile_sparse((const StarRec*)c->rec.p, n, fp, out, (float*)c->segs.p, st); });
+    return check_launch(c, "k_tile_sparse");
+  }
+  if ((rc = enqueue_binning(c, x, y, mag, n, fp, ntiles, tps, part_cap, st))) return rc;
+  Header* hdr = (Header*)c->zeroed.p;
+  uint32_t* cnt = (uint32_t*)(hdr + 1);
+  uint32_t* done = cnt + CNT_STRIDE * ntiles;
+  uint32_t* ids = (uint32_t*)c->ids.p;
+  uint32_t* tile_off = (uint32_t*)c->tile_off.p;
+  StarRec* rec = (StarRec*)c->rec.p;
+  (void)cnt;
   if (fp.tile_impl == STARSIM_TILE_T8 && fp.R <= SB_MAXR) {
     // k_t8sort: every tile list segment sorted by ROI corner bin, records written in that order (tile8.cu)
     timed(c, 1, st, [&] {
@@ -356,6 +385,10 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
     fp.lite = (fp.tile_impl == STARSIM_TILE_SB && R <= SB_MAXR && LITE_MAX > 0 && per_tile <= LITE_AUTO_PER_TILE &&
                nt >= LITE_AUTO_TILES) ? 1 : 0;
   }
+  // the sparse path (AUTO, <= SPARSE_MAX stars): no binning launches, the same image bit for bit (tile_sb.cu)
+  const bool sparse = c->tile_impl == STARSIM_TILE_AUTO && c->bin_impl == STARSIM_BIN_AUTO &&
+                      fp.tile_impl == STARSIM_TILE_SB && R <= SB_MAXR &&
+                      sparse_ok(n, (int64_t)fp.ntx * fp.nty);
   // one vector store per 8-pixel run: 32 B (fp32) / 8 B (u8) / 16 B (u16); rows must keep that alignment
   const int vb = obits == 8 ? 8 : 16;
   bool aligned = ((uintptr_t)out % vb) == 0;
@@ -389,7 +422,12 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   if ((rc = grow(c, c->partial, sizeof(uint4) * (size_t)((ntiles + SCAN_TILES - 1) / SCAN_TILES), "scan partials")))
     return rc;
   if ((rc = grow(c, c->parts, sizeof(float) * TILE_W * TILE_H * (size_t)part_cap, "partial tiles"))) return rc;
-  if ((rc = grow(c, c->segs, sizeof(float) * tile8_scratch_floats(c->num_sms), "segment scratch"))) return rc;
+  // segment scratch: one tile per persistent CTA of the tile kernels, one per tile for the sparse path
+  if ((rc = grow(c, c->segs,
+                 sizeof(float) * std::max<size_t>(tile8_scratch_floats(c->num_sms),
+                                                  sparse ? (size_t)ntiles * TILE_W * TILE_H : 0),
+                 "segment scratch")))
+    return rc;
   if (ws_presort(c, fp)) {  // k_chsort's outputs
     if ((rc = grow(c, c->srec, sizeof(StarRec) * (size_t)(pmax > 0 ? pmax : 1), "bin-sorted records"))) return rc;
     if ((rc = grow(c, c->cbin, sizeof(uint16_t) * chsort_slots(ntiles, pmax) * chsort_words16(), "chunk bin starts")))
@@ -413,7 +451,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
                c->scratch_gen};
   for (int i = 0; i < MAX_DST; ++i) key.dst[i] = fp.dst[i];
   if (st == nullptr || c->prof || !c->use_graphs) {
-    if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st))) return rc;
+    if ((rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st, sparse))) return rc;
   } else {
     if (!(c->have_graph && c->gkey == key)) {
       if (c->have_graph) {
@@ -422,7 +460,7 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
       }
       cudaError_t e = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal);
       if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamBeginCapture");
-      rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st);
+      rc = enqueue_tiled(c, x, y, mag, n, fp, ntiles, tps, part_cap, out, st, sparse);
       cudaGraph_t graph = nullptr;
       e = cudaStreamEndCapture(st, &graph);
       if (rc) {
@@ -442,6 +480,8 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
   c->have_bins = true;
   c->last_stream = st;
   c->last_ntiles = ntiles;
+  c->last_sparse = sparse;
+  if (sparse) c->sp = {x, y, mag, n, fp, tps, part_cap};
   c->err.clear();
   return STARSIM_OK;
 }
@@ -704,6 +744,16 @@ int starsim_get_bins(starsim_ctx* c, int32_t* tile_w, int32_t* tile_h, uint32_t*
   if (!c) return STARSIM_EINVAL;
   if (!c->have_bins) return fail(c, STARSIM_EINVAL, "no tiled render on this ctx yet");
   DevGuard g(c->dev);
+  if (c->last_sparse) {
+    // the last render took the sparse path: bin its (still caller-owned) arrays now, on its stream
+    const bool prof = c->prof;
+    c->prof = false;
+    const int rc = enqueue_binning(c, c->sp.x, c->sp.y, c->sp.m, c->sp.n, c->sp.fp, c->last_ntiles, c->sp.tps,
+                                   c->sp.part_cap, c->last_stream);
+    c->prof = prof;
+    if (rc) return rc;
+    c->last_sparse = false;
+  }
   cudaError_t e = cudaStreamSynchronize(c->last_stream);
   if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamSynchronize");
   Header h;

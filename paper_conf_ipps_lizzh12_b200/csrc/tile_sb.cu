@@ -29,6 +29,7 @@
 
 #include "common.cuh"
 #include "launch.h"
+#include "prep.cuh"
 #include "tile_common.cuh"
 
 namespace starsim {
@@ -407,6 +408,143 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? SB_MINB_CIRC : SB_MINB) k
 }
 
 
+// One chunk of <= CAP stars of a tile's list, given in list order (thread t < n holds star t's record r): the stars
+// ranked by corner bin (stable: then list order) exactly as a k_tile_sb chunk is sorted, and walked by every warp whose
+// 64 x 16 region the ROI meets, each lane evaluating its own 4 row and 8 column factors with the very operations of
+// k_tile_sb's slot preparation and adding them in that order (same per-pixel sums, bit for bit).  Two barriers; the
+// arrays are the caller's shared memory.
+template <bool INTEG, bool CIRC, int CAP>
+__device__ __forceinline__ void lite_chunk(float2 (&acc)[4][4], uint32_t* lkey, float4* lrec, uint32_t* llo,
+                                           const StarRec& r, int n, const FrameParams& fp, int X0, int IY0,
+                                           int TWe, int THe) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
+  const int Q = 8 * wx + q;
+  const int swz = (Q >> 2) & 1;
+  const float sk = fp.sk;
+  uint32_t key = SB_NBIN, lo2 = 0u;
+  if (tid < n) {
+    const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
+    lo2 = (uint32_t)(lx & 0xFFFF) | (uint32_t)ly << 16;
+    const int c0 = max(lx, 0), c1 = min(lx + fp.R - 1, TWe - 1);
+    const int r0 = max(ly, 0), r1 = min(ly + fp.R - 1, THe - 1);
+    if (c0 <= c1 && r0 <= r1) key = (uint32_t)((ly < 0 ? 0 : 1 + (r0 >> 4)) * SB_NSK + (lx < 0 ? 0 : 1 + (c0 >> 3)));
+    lkey[tid] = key;
+  }
+  __syncthreads();
+  if (tid < n) {
+    uint32_t rank = 0;
+    for (int u = 0; u < n; ++u) {
+      const uint32_t ku = lkey[u];
+      rank += (ku < key || (ku == key && u < tid)) ? 1u : 0u;
+    }
+    lrec[rank] = make_float4(r.x - (float)X0, r.y - (float)IY0, r.s, __uint_as_float(key));  // exact
+    llo[rank] = lo2;
+  }
+  __syncthreads();
+  const float2 sk2 = make_float2(sk, sk);
+  for (int k = 0; k < n; ++k) {
+    const float4 st = lrec[k];
+    const uint32_t sk_key = __float_as_uint(st.w);
+    if (sk_key >= (uint32_t)SB_NBIN) continue;
+    const uint32_t lo = llo[k];
+    const int lx = (int)(int16_t)(lo & 0xFFFFu), ly = (int)(int16_t)(lo >> 16);
+    const int c0 = max(lx, 0), c1 = min(lx + fp.R - 1, TWe - 1);
+    const int r0 = max(ly, 0), r1 = min(ly + fp.R - 1, THe - 1);
+    // the warp's 64 x 16 region (uniform branch)
+    if (r1 < 16 * B || r0 > 16 * B + 15 || c1 < 64 * wx || c0 > 64 * wx + 63) continue;
+    const int b0 = (int)(sk_key / SB_NSK) - 1, q0 = (int)(sk_key % SB_NSK) - 1;
+    const float xr = st.x, yr = st.y;
+    // row factors of rows 16 B + 4 hq + i: quad w = 4 (B - b0) + hq of the star's two bands (slot preparation)
+    float gyv[4];
+    {
+      const int ra0 = r0 - 16 * b0, rb0 = r1 - 16 * b0;
+      const uint32_t m0 = (0xFFFFFFFFu >> (31 - min(rb0, 31))) & (0xFFFFFFFFu << ra0);
+      const int w = 4 * (B - b0) + hq;
+      const uint32_t m = (w >= 0 && w < 8) ? m0 >> (4 * w) : 0u;
+      const float bf0 = (float)(16 * b0) - yr;
+      const float bf = bf0 + (float)(4 * w);
+      if (!INTEG) {
+        const float2 s2 = make_float2(st.z, st.z);
+        const float2 bb = make_float2(bf, bf);
+#pragma unroll
+        for (int i = 0; i < 4; i += 2) {
+          float2 d = __fadd2_rn(bb, make_float2((float)i, (float)(i + 1)));
+          d = __fmul2_rn(d, sk2);
+          d = __fmul2_rn(d, make_float2(-d.x, -d.y));
+          const float2 e = __fmul2_rn(make_float2(ex2_approx(d.x), ex2_approx(d.y)), s2);
+          gyv[i] = (m >> i) & 1u ? e.x : 0.f;
+          gyv[i + 1] = (m >> (i + 1)) & 1u ? e.y : 0.f;
+        }
+      } else {
+        float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const float tn = (bf + (float)i + 0.5f) * fp.kint, en = edge_erfc(tn);
+          gyv[i] = (m >> i) & 1u ? st.z * pix_mass(t, e, tn, en) : 0.f;
+          t = tn;
+          e = en;
+        }
+      }
+    }
+    // column factors of strip Q (one of the star's strips q0 .. q0 + 2, else zero) in the lane's load order:
+    // slot p holds column 8 Q + pp, pp = (p + 4 swz) & 7 (the same operations on the same operands as k_tile_sb)
+    float gxv[8];
+    {
+      const int rel = 8 * Q;
+      const int lo_ = max(c0 - rel, 0), hi = min(c1 - rel, 7);
+      const uint32_t m = (Q >= q0 && Q <= q0 + 2 && hi >= lo_) ? ((0xFFu >> (7 - hi)) & (0xFFu << lo_)) : 0u;
+      const float bf = (float)rel - xr;
+      if (!INTEG) {
+#pragma unroll
+        for (int p = 0; p < 8; p += 2) {
+          const int pp = (p + 4 * swz) & 7;
+          float2 d = __fmul2_rn(__fadd2_rn(make_float2(bf, bf), make_float2((float)pp, (float)(pp + 1))), sk2);
+          d = __fmul2_rn(d, make_float2(-d.x, -d.y));
+          gxv[p] = (m >> pp) & 1u ? ex2_approx(d.x) : 0.f;
+          gxv[p + 1] = (m >> (pp + 1)) & 1u ? ex2_approx(d.y) : 0.f;
+        }
+      } else {
+        float v[8];
+        float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
+#pragma unroll
+        for (int p = 0; p < 8; ++p) {
+          const float tn = (bf + (float)p + 0.5f) * fp.kint, en = edge_erfc(tn);
+          v[p] = (m >> p) & 1u ? pix_mass(t, e, tn, en) : 0.f;
+          t = tn;
+          e = en;
+        }
+#pragma unroll
+        for (int p = 0; p < 8; ++p) gxv[p] = swz ? v[(p + 4) & 7] : v[p];
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float2 gg = make_float2(gyv[i], gyv[i]);
+      if (CIRC) {
+        const int RR = fp.R * fp.R, R1 = fp.R - 1;
+        const int v = 2 * (16 * B + 4 * hq + i - ly) - R1;
+        const int thr = RR - v * v;
+        float gm[8];
+#pragma unroll
+        for (int p = 0; p < 8; ++p) {
+          const int u = 2 * (8 * Q + ((p + 4 * swz) & 7) - lx) - R1;
+          gm[p] = u * u <= thr ? gxv[p] : 0.f;
+        }
+        acc[i][0] = __ffma2_rn(gg, make_float2(gm[0], gm[1]), acc[i][0]);
+        acc[i][1] = __ffma2_rn(gg, make_float2(gm[2], gm[3]), acc[i][1]);
+        acc[i][2] = __ffma2_rn(gg, make_float2(gm[4], gm[5]), acc[i][2]);
+        acc[i][3] = __ffma2_rn(gg, make_float2(gm[6], gm[7]), acc[i][3]);
+      } else {
+        acc[i][0] = __ffma2_rn(gg, make_float2(gxv[0], gxv[1]), acc[i][0]);
+        acc[i][1] = __ffma2_rn(gg, make_float2(gxv[2], gxv[3]), acc[i][1]);
+        acc[i][2] = __ffma2_rn(gg, make_float2(gxv[4], gxv[5]), acc[i][2]);
+        acc[i][3] = __ffma2_rn(gg, make_float2(gxv[6], gxv[7]), acc[i][3]);
+      }
+    }
+  }
+  }
+
 // ---------------------------------------------------------------------------------------------------------------
 // k_tile_lite: the light items (whole tiles of at most LITE_MAX stars, empty ones included: the planner puts them
 // last, from Header::lite0 on), one CTA per item, many CTAs per SM -- with k_tile_sb, whose persistent CTAs take the
@@ -447,130 +585,9 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? 3 : LITE_MINB) k_tile_lit
 #pragma unroll
     for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
   if (n > 0) {
-    // sort: thread t = list star t; its corner bin (k_tile_sb's key) and its rank (corner bin, then list order)
     StarRec r = {};
     if (tid < n) r = rec[__ldg(&ids[jb + tid])];
-    uint32_t key = SB_NBIN, lo2 = 0u;
-    if (tid < n) {
-      const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
-      lo2 = (uint32_t)(lx & 0xFFFF) | (uint32_t)ly << 16;
-      const int c0 = max(lx, 0), c1 = min(lx + fp.R - 1, TWe - 1);
-      const int r0 = max(ly, 0), r1 = min(ly + fp.R - 1, THe - 1);
-      if (c0 <= c1 && r0 <= r1) key = (uint32_t)((ly < 0 ? 0 : 1 + (r0 >> 4)) * SB_NSK + (lx < 0 ? 0 : 1 + (c0 >> 3)));
-      lkey[tid] = key;
-    }
-    __syncthreads();
-    if (tid < n) {
-      uint32_t rank = 0;
-      for (int u = 0; u < n; ++u) {
-        const uint32_t ku = lkey[u];
-        rank += (ku < key || (ku == key && u < tid)) ? 1u : 0u;
-      }
-      lrec[rank] = make_float4(r.x - (float)X0, r.y - (float)IY0, r.s, __uint_as_float(key));  // exact
-      llo[rank] = lo2;
-    }
-    __syncthreads();
-    const float2 sk2 = make_float2(sk, sk);
-    for (int k = 0; k < n; ++k) {
-      const float4 st = lrec[k];
-      const uint32_t sk_key = __float_as_uint(st.w);
-      if (sk_key >= (uint32_t)SB_NBIN) continue;
-      const uint32_t lo = llo[k];
-      const int lx = (int)(int16_t)(lo & 0xFFFFu), ly = (int)(int16_t)(lo >> 16);
-      const int c0 = max(lx, 0), c1 = min(lx + fp.R - 1, TWe - 1);
-      const int r0 = max(ly, 0), r1 = min(ly + fp.R - 1, THe - 1);
-      // the warp's 64 x 16 region (uniform branch)
-      if (r1 < 16 * B || r0 > 16 * B + 15 || c1 < 64 * wx || c0 > 64 * wx + 63) continue;
-      const int b0 = (int)(sk_key / SB_NSK) - 1, q0 = (int)(sk_key % SB_NSK) - 1;
-      const float xr = st.x, yr = st.y;
-      // row factors of rows 16 B + 4 hq + i: quad w = 4 (B - b0) + hq of the star's two bands (slot preparation)
-      float gyv[4];
-      {
-        const int ra0 = r0 - 16 * b0, rb0 = r1 - 16 * b0;
-        const uint32_t m0 = (0xFFFFFFFFu >> (31 - min(rb0, 31))) & (0xFFFFFFFFu << ra0);
-        const int w = 4 * (B - b0) + hq;
-        const uint32_t m = (w >= 0 && w < 8) ? m0 >> (4 * w) : 0u;
-        const float bf0 = (float)(16 * b0) - yr;
-        const float bf = bf0 + (float)(4 * w);
-        if (!INTEG) {
-          const float2 s2 = make_float2(st.z, st.z);
-          const float2 bb = make_float2(bf, bf);
-#pragma unroll
-          for (int i = 0; i < 4; i += 2) {
-            float2 d = __fadd2_rn(bb, make_float2((float)i, (float)(i + 1)));
-            d = __fmul2_rn(d, sk2);
-            d = __fmul2_rn(d, make_float2(-d.x, -d.y));
-            const float2 e = __fmul2_rn(make_float2(ex2_approx(d.x), ex2_approx(d.y)), s2);
-            gyv[i] = (m >> i) & 1u ? e.x : 0.f;
-            gyv[i + 1] = (m >> (i + 1)) & 1u ? e.y : 0.f;
-          }
-        } else {
-          float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const float tn = (bf + (float)i + 0.5f) * fp.kint, en = edge_erfc(tn);
-            gyv[i] = (m >> i) & 1u ? st.z * pix_mass(t, e, tn, en) : 0.f;
-            t = tn;
-            e = en;
-          }
-        }
-      }
-      // column factors of strip Q (one of the star's strips q0 .. q0 + 2, else zero) in the lane's load order:
-      // slot p holds column 8 Q + pp, pp = (p + 4 swz) & 7 (the same operations on the same operands as k_tile_sb)
-      float gxv[8];
-      {
-        const int rel = 8 * Q;
-        const int lo_ = max(c0 - rel, 0), hi = min(c1 - rel, 7);
-        const uint32_t m = (Q >= q0 && Q <= q0 + 2 && hi >= lo_) ? ((0xFFu >> (7 - hi)) & (0xFFu << lo_)) : 0u;
-        const float bf = (float)rel - xr;
-        if (!INTEG) {
-#pragma unroll
-          for (int p = 0; p < 8; p += 2) {
-            const int pp = (p + 4 * swz) & 7;
-            float2 d = __fmul2_rn(__fadd2_rn(make_float2(bf, bf), make_float2((float)pp, (float)(pp + 1))), sk2);
-            d = __fmul2_rn(d, make_float2(-d.x, -d.y));
-            gxv[p] = (m >> pp) & 1u ? ex2_approx(d.x) : 0.f;
-            gxv[p + 1] = (m >> (pp + 1)) & 1u ? ex2_approx(d.y) : 0.f;
-          }
-        } else {
-          float v[8];
-          float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
-#pragma unroll
-          for (int p = 0; p < 8; ++p) {
-            const float tn = (bf + (float)p + 0.5f) * fp.kint, en = edge_erfc(tn);
-            v[p] = (m >> p) & 1u ? pix_mass(t, e, tn, en) : 0.f;
-            t = tn;
-            e = en;
-          }
-#pragma unroll
-          for (int p = 0; p < 8; ++p) gxv[p] = swz ? v[(p + 4) & 7] : v[p];
-        }
-      }
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const float2 gg = make_float2(gyv[i], gyv[i]);
-        if (CIRC) {
-          const int RR = fp.R * fp.R, R1 = fp.R - 1;
-          const int v = 2 * (16 * B + 4 * hq + i - ly) - R1;
-          const int thr = RR - v * v;
-          float gm[8];
-#pragma unroll
-          for (int p = 0; p < 8; ++p) {
-            const int u = 2 * (8 * Q + ((p + 4 * swz) & 7) - lx) - R1;
-            gm[p] = u * u <= thr ? gxv[p] : 0.f;
-          }
-          acc[i][0] = __ffma2_rn(gg, make_float2(gm[0], gm[1]), acc[i][0]);
-          acc[i][1] = __ffma2_rn(gg, make_float2(gm[2], gm[3]), acc[i][1]);
-          acc[i][2] = __ffma2_rn(gg, make_float2(gm[4], gm[5]), acc[i][2]);
-          acc[i][3] = __ffma2_rn(gg, make_float2(gm[6], gm[7]), acc[i][3]);
-        } else {
-          acc[i][0] = __ffma2_rn(gg, make_float2(gxv[0], gxv[1]), acc[i][0]);
-          acc[i][1] = __ffma2_rn(gg, make_float2(gxv[2], gxv[3]), acc[i][1]);
-          acc[i][2] = __ffma2_rn(gg, make_float2(gxv[4], gxv[5]), acc[i][2]);
-          acc[i][3] = __ffma2_rn(gg, make_float2(gxv[6], gxv[7]), acc[i][3]);
-        }
-      }
-    }
+    lite_chunk<INTEG, CIRC, LITE_MAX>(acc, lkey, lrec, llo, r, n, fp, X0, IY0, TWe, THe);
   }
   // the lanes with swz = 1 hold columns 4-7 of their strip in acc[i][0..1] (k_tile_sb's load order)
   if (swz) {
@@ -597,6 +614,147 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? 3 : LITE_MINB) k_tile_lit
     __syncthreads();
     tile_store_gray_staged(gbuf, fp, out_, Y0, X0, TWe, THe);
   }
+}
+
+
+// ---------------------------------------------------------------------------------------------------------------
+// The sparse path (STARSIM_TILE_AUTO, catalogues of <= SPARSE_MAX stars, R <= SB_MAXR): no binning.  k_srec writes
+// the star records (step a1); k_tile_sparse runs one CTA per tile that scans the whole (L2-resident) record array,
+// compacts the stars whose clipped ROI meets its tile in ascending star index -- exactly the tile's CSR list -- and
+// renders it chunk by chunk with lite_chunk: the same per-pixel sums as k_tile_sb / k_tile_ws, bit for bit, in two
+// launches instead of four.  starsim_get_bins after a sparse render bins the same arrays on demand (api.cu).
+// ---------------------------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_srec(const float* __restrict__ X, const float* __restrict__ Y,
+                                              const float* __restrict__ M, int64_t n, FrameParams fp,
+                                              StarRec* __restrict__ rec) {
+  const int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x;
+  if (i >= frame_n(n, fp)) return;
+  int cx0, cx1, cy0, cy1;
+  rec[i] = prep_star(__ldg(&X[i]), __ldg(&Y[i]), __ldg(&M[i]), fp, cx0, cx1, cy0, cy1);
+}
+
+template <bool INTEG, bool CIRC, int OB>
+__global__ void __launch_bounds__(TILE_THREADS, (CIRC && INTEG) ? 2 : (CIRC || INTEG) ? 3 : LITE_MINB) k_tile_sparse(const StarRec* __restrict__ rec,
+                                                                                    int64_t n, FrameParams fp,
+                                                                                    void* __restrict__ out_,
+                                                                                    float* __restrict__ seg_scratch) {
+  // the list and the chunk arrays, and (gray output) the staged tile afterwards, share one buffer
+  struct Lists {
+    uint32_t lidx[SPARSE_MAX];
+    uint32_t lkey[SB_CHUNK];
+    float4 lrec[SB_CHUNK];
+    uint32_t llo[SB_CHUNK];
+  };
+  __shared__ __align__(16) unsigned char sraw[OB && sizeof(float) * TILE_W * TILE_H > sizeof(Lists)
+                                                  ? sizeof(float) * TILE_W * TILE_H
+                                                  : sizeof(Lists)];
+  Lists& L = *reinterpret_cast<Lists*>(sraw);
+  uint32_t* lidx = L.lidx;
+  uint32_t* lkey = L.lkey;
+  float4* lrec = L.lrec;
+  uint32_t* llo = L.llo;
+  __shared__ uint32_t wcnt[TILE_WARPS];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
+  const int Q = 8 * wx + q;
+  const int swz = (Q >> 2) & 1;
+  const uint32_t tile = blockIdx.x;
+  const int tx = (int)(tile % (uint32_t)fp.ntx), ty = (int)(tile / (uint32_t)fp.ntx);
+  const int X0 = tx * TILE_W, Y0 = ty * TILE_H, IY0 = fp.row0 + Y0;
+  const int TWe = min(TILE_W, fp.W - X0), THe = min(TILE_H, fp.rows - Y0);
+  n = frame_n(n, fp);
+  // the tile's list: stars whose clipped ROI meets it (the binning's pair rule), ascending star index
+  uint32_t len = 0;
+  const uint32_t lt = (1u << lane) - 1u;
+  for (int64_t base = 0; base < n; base += TILE_THREADS) {
+    const int64_t i = base + tid;
+    bool hit = false;
+    if (i < n) {
+      const uint32_t lo = __ldg(&rec[i].lo);
+      if (lo != LO_CULLED) {
+        const int lx = lo_x_of(lo) - X0, ly = lo_y_of(lo) - IY0;
+        hit = lx <= TWe - 1 && lx + fp.R - 1 >= 0 && ly <= THe - 1 && ly + fp.R - 1 >= 0;
+      }
+    }
+    const uint32_t wm = __ballot_sync(0xffffffffu, hit);
+    if (lane == 0) wcnt[warp] = __popc(wm);
+    __syncthreads();
+    uint32_t pre = 0, tot = 0;
+#pragma unroll
+    for (int w = 0; w < TILE_WARPS; ++w) {
+      const uint32_t cw = wcnt[w];
+      pre += w < warp ? cw : 0u;
+      tot += cw;
+    }
+    if (hit) lidx[len + pre + __popc(wm & lt)] = (uint32_t)i;
+    len += tot;
+    __syncthreads();
+  }
+  float2 acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
+  // chunks of SB_CHUNK from the list start, as k_tile_sb cuts them; a list longer than SPLIT_LEN is summed in
+  // segments (reading R19) through the tile's own slot of the segment scratch (one CTA per tile)
+  uint32_t segs_done = 0;
+  for (uint32_t c0 = 0; c0 < len; c0 += SB_CHUNK) {
+    const int nn = (int)min((uint32_t)SB_CHUNK, len - c0);
+    StarRec r = {};
+    if (tid < nn) r = rec[lidx[c0 + tid]];
+    lite_chunk<INTEG, CIRC, SB_CHUNK>(acc, lkey, lrec, llo, r, nn, fp, X0, IY0, TWe, THe);
+    if ((c0 + SB_CHUNK) % SPLIT_LEN == 0 && c0 + SB_CHUNK < len) {
+      seg_flush(acc, seg_scratch, segs_done == 0);
+      ++segs_done;
+    }
+  }
+  if (segs_done) seg_finish(acc, seg_scratch);
+  if (swz) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float2 t0 = acc[i][0], t1 = acc[i][1];
+      acc[i][0] = acc[i][2];
+      acc[i][1] = acc[i][3];
+      acc[i][2] = t0;
+      acc[i][3] = t1;
+    }
+  }
+  if (OB == 0) {
+    tile_store<true, 0>(acc, fp, out_, Y0, X0 + 64 * wx + 8 * q, B, hq);
+  } else {
+    float* gbuf = reinterpret_cast<float*>(sraw);
+    __syncthreads();  // the last chunk's walk is done with the list arrays
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      float4* d = reinterpret_cast<float4*>(gbuf + lane_row<true>(B, hq, i) * TILE_W + 64 * wx + 8 * q);
+      d[0] = make_float4(acc[i][0].x, acc[i][0].y, acc[i][1].x, acc[i][1].y);
+      d[1] = make_float4(acc[i][2].x, acc[i][2].y, acc[i][3].x, acc[i][3].y);
+    }
+    __syncthreads();
+    tile_store_gray_staged(gbuf, fp, out_, Y0, X0, TWe, THe);
+  }
+}
+
+// every tile CTA tests every star: worth it while stars x tiles stays small (measured: C1 64 K, fig2 288 K, C3 with
+// 1 K stars 2 M pair tests win; C3 with 4 K stars, 8 M, loses to the binning path)
+bool sparse_ok(int64_t n, int64_t ntiles) { return n <= SPARSE_MAX && n * ntiles <= SPARSE_TESTS; }
+
+void launch_srec(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
+                 cudaStream_t st) {
+  if (n > 0) k_srec<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(x, y, m, n, fp, rec);
+}
+
+void launch_tile_sparse(const StarRec* rec, int64_t n, const FrameParams& fp, void* out, float* seg_scratch,
+                        cudaStream_t st) {
+  const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
+  using KS = void (*)(const StarRec*, int64_t, FrameParams, void*, float*);
+  static const KS ks[2][2][3] = {
+      {{k_tile_sparse<false, false, 0>, k_tile_sparse<false, false, 8>, k_tile_sparse<false, false, 16>},
+       {k_tile_sparse<false, true, 0>, k_tile_sparse<false, true, 8>, k_tile_sparse<false, true, 16>}},
+      {{k_tile_sparse<true, false, 0>, k_tile_sparse<true, false, 8>, k_tile_sparse<true, false, 16>},
+       {k_tile_sparse<true, true, 0>, k_tile_sparse<true, true, 8>, k_tile_sparse<true, true, 16>}}};
+  const KS k = ks[fp.psf ? 1 : 0][fp.roi ? 1 : 0][fp.obits == 8 ? 1 : fp.obits == 16 ? 2 : 0];
+  k<<<(unsigned)ntiles, TILE_THREADS, 0, st>>>(rec, n, fp, out, seg_scratch);
 }
 
 #ifdef STARSIM_SB_TIMING

@@ -543,6 +543,52 @@ def test_fused_binning_same_csr_and_image(torch_dev, monkeypatch, W, H, n, R, se
     assert np.array_equal(off[:ro.size], ro) and np.array_equal(ids, ri)
 
 
+@pytest.mark.parametrize("W,H,n,R,seed,kind", [(1024, 1024, 1000, 5, 1, "uniform"), (4096, 4096, 1000, 11, 2, "uniform"),
+                                               (700, 530, 1024, 15, 3, "adv"), (300, 200, 900, 17, 4, "dense"),
+                                               (129, 65, 1, 9, 5, "uniform"), (256, 256, 0, 7, 6, "uniform"),
+                                               (1024, 1024, 2252, 11, 7, "uniform"), (4096, 2048, 4096, 15, 8, "adv"),
+                                               (300, 200, 4000, 15, 9, "dense")])  # > 1,024 stars in a tile
+def test_sparse_path_is_bitwise_sb(torch_dev, W, H, n, R, seed, kind):
+    """STARSIM_TILE_AUTO renders catalogues of <= 4,096 stars through the sparse path (k_srec + k_tile_sparse: no
+    binning launches, every tile CTA builds its own list; lists over 1,024 stars summed in segments, reading R19):
+    the same image as k_tile_sb bit for bit -- point and
+    integrated PSF, square and circle ROI, fp32 and u8 -- at parity with the oracle, bands bitwise the frame, and
+    starsim_get_bins afterwards (binned on demand) the oracle's CSR."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context
+    if kind == "adv":
+        f = synth.adversarial_field(n, W, H, R, seed=seed)
+    elif kind == "dense":
+        f = _dense_field(n, W, H, 150.0, 100.0, 20.0, seed=seed)
+    else:
+        f = synth.uniform_field(n, W, H, seed=seed, mag_hi=15.0)
+    args = to_dev(torch_dev, f) if n else (torch.empty(0, device=dev),) * 3
+    sigma = R / 6
+    with Context(0) as a, Context(0) as b:
+        b.set_tile_kernel("sb")
+        for psf in ("point", "integrated"):
+            for roi in ("square", "circle"):
+                for c in (a, b):
+                    c.set_psf(psf)
+                    c.set_roi(roi)
+                ia = a.render(*args, W, H, sigma, R, 1.0)
+                assert torch.equal(ia, b.render(*args, W, H, sigma, R, 1.0)), (psf, roi)
+                ga = a.render_gray(*args, W, H, sigma, R, 1.0, bits=8)
+                assert torch.equal(ga, b.render_gray(*args, W, H, sigma, R, 1.0, bits=8)), (psf, roi)
+        for c in (a, b):
+            c.set_psf("point")
+            c.set_roi("square")
+        img = a.render(*args, W, H, sigma, R, 1.0)
+        if n:
+            assert_parity(img.cpu().numpy(), oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0), f"sparse {W}x{H}")
+        bands = [a.render_band(*args, W, H, g * 64, min(64, H - g * 64), sigma, R, 1.0) for g in range(-(-H // 64))]
+        assert torch.equal(torch.cat(bands, 0), img)
+        a.render(*args, W, H, sigma, R, 1.0)
+        tw, th, off, ids = a.get_bins()
+        ro, ri = oracle.bins(f.x, f.y, f.mag, W, H, R, tw, th)
+        assert np.array_equal(off[:ro.size], ro) and np.array_equal(ids, ri)
+
+
 def test_mode_setters_einval(torch_dev):
     from paper_conf_ipps_lizzh12_b200 import Context, StarsimError
     with Context(0) as c:
