@@ -308,9 +308,11 @@ int enqueue_tiled(starsim_ctx* c, const float* x, const float* y, const float* m
   int rc;
   if (sparse) {
     // the sparse path (tile_sb.cu): records, then one CTA per tile that builds its own list -- no binning launches
-    timed(c, 0, st, [&] { launch_srec(x, y, mag, n, fp, (StarRec*)c->rec.p, st); });
+    timed(c, 0, st, [&] { launch_srec(x, y, mag, n, fp, (StarRec*)c->rec.p, (uint32_t*)c->codes.p, st); });
     if ((rc = check_launch(c, "k_srec"))) return rc;
-    timed(c, 3, st, [&] { launch_tile_sparse((const StarRec*)c->rec.p, n, fp, out, (float*)c->segs.p, st); });
+    timed(c, 3, st, [&] {
+      launch_tile_sparse((const StarRec*)c->rec.p, (const uint32_t*)c->codes.p, n, fp, out, (float*)c->segs.p, st);
+    });
     return check_launch(c, "k_tile_sparse");
   }
   if ((rc = enqueue_binning(c, x, y, mag, n, fp, ntiles, tps, part_cap, st))) return rc;
@@ -443,7 +445,8 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
       (rc = grow(c, c->cmat, sizeof(uint32_t) * (size_t)ntiles * (size_t)(dbin_ctas(n) > 0 ? dbin_ctas(n) : 1),
                  "count matrix")))
     return rc;
-  if (dbin_ok(fp, ntiles) && (rc = grow(c, c->codes, sizeof(uint32_t) * (size_t)(n > 0 ? n : 1), "tile boxes")))
+  if ((dbin_ok(fp, ntiles) || sparse) &&
+      (rc = grow(c, c->codes, sizeof(uint32_t) * (size_t)(n > 0 ? n : 1), "tile boxes")))
     return rc;
   if ((rc = grow(c, c->gbar, 64, "grid barrier"))) return rc;
 

@@ -71,9 +71,9 @@ void launch_route(const float* x, const float* y, const float* m, int64_t n, int
                   uint32_t* blk, float* xo, float* yo, float* mo, uint32_t* n_out, cudaStream_t st);
 bool sparse_ok(int64_t n, int64_t ntiles);
 void launch_srec(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
-                 cudaStream_t st);
-void launch_tile_sparse(const StarRec* rec, int64_t n, const FrameParams& fp, void* out, float* seg_scratch,
-                        cudaStream_t st);
+                 uint32_t* box, cudaStream_t st);
+void launch_tile_sparse(const StarRec* rec, const uint32_t* box, int64_t n, const FrameParams& fp, void* out,
+                        float* seg_scratch, cudaStream_t st);
 void launch_split_aos(const float* aos, int64_t n, float* x, float* y, float* m, int num_sms, cudaStream_t st);
 
 }  // namespace starsim

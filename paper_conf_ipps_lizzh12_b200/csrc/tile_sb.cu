@@ -618,29 +618,44 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? 3 : LITE_MINB) k_tile_lit
 
 
 // ---------------------------------------------------------------------------------------------------------------
-// The sparse path (STARSIM_TILE_AUTO, catalogues of <= SPARSE_MAX stars, R <= SB_MAXR): no binning.  k_srec writes
-// the star records (step a1); k_tile_sparse runs one CTA per tile that scans the whole (L2-resident) record array,
-// compacts the stars whose clipped ROI meets its tile in ascending star index -- exactly the tile's CSR list -- and
-// renders it chunk by chunk with lite_chunk: the same per-pixel sums as k_tile_sb / k_tile_ws, bit for bit, in two
-// launches instead of four.  starsim_get_bins after a sparse render bins the same arrays on demand (api.cu).
+// The sparse path (STARSIM_TILE_AUTO, catalogues of <= SPARSE_MAX stars with stars x tiles <= SPARSE_TESTS,
+// R <= SB_MAXR): no binning.  k_srec writes the star records (step a1) and each star's packed tile box (the tiles its
+// clipped ROI meets: at most 2 x 2); k_tile_sparse runs one CTA per tile that streams the box array in star order,
+// keeps the stars whose box holds its tile -- exactly the tile's CSR list, in the same order -- and renders every
+// 256 list entries as one chunk with lite_chunk (the remainder at the end), summing lists longer than SPLIT_LEN in
+// segments through its own slot of the segment scratch (reading R19): the same per-pixel sums as k_tile_sb /
+// k_tile_ws, bit for bit, in two launches instead of four.  starsim_get_bins after a sparse render bins the same
+// arrays on demand (api.cu).
 // ---------------------------------------------------------------------------------------------------------------
+constexpr uint32_t SP_NONE = 0xFFFFFFFFu;
+__device__ __forceinline__ uint32_t sp_box(int tx0, int ty0, int dx, int dy) {  // 8 + 9 + 1 + 1 bits
+  return (uint32_t)tx0 | (uint32_t)ty0 << 8 | (uint32_t)dx << 17 | (uint32_t)dy << 18;
+}
+
 __global__ void __launch_bounds__(256) k_srec(const float* __restrict__ X, const float* __restrict__ Y,
                                               const float* __restrict__ M, int64_t n, FrameParams fp,
-                                              StarRec* __restrict__ rec) {
+                                              StarRec* __restrict__ rec, uint32_t* __restrict__ box) {
   const int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x;
   if (i >= frame_n(n, fp)) return;
   int cx0, cx1, cy0, cy1;
-  rec[i] = prep_star(__ldg(&X[i]), __ldg(&Y[i]), __ldg(&M[i]), fp, cx0, cx1, cy0, cy1);
+  const StarRec r = prep_star(__ldg(&X[i]), __ldg(&Y[i]), __ldg(&M[i]), fp, cx0, cx1, cy0, cy1);
+  rec[i] = r;
+  uint32_t b = SP_NONE;
+  if (r.lo != LO_CULLED) {
+    const int tx0 = cx0 / TILE_W, ty0 = (cy0 - fp.row0) / TILE_H;
+    b = sp_box(tx0, ty0, cx1 / TILE_W - tx0, (cy1 - fp.row0) / TILE_H - ty0);
+  }
+  box[i] = b;
 }
 
+constexpr int SP_BUF = SB_CHUNK + TILE_THREADS * 4;  // pending list entries: < one chunk + one round's hits
 template <bool INTEG, bool CIRC, int OB>
-__global__ void __launch_bounds__(TILE_THREADS, (CIRC && INTEG) ? 2 : (CIRC || INTEG) ? 3 : LITE_MINB) k_tile_sparse(const StarRec* __restrict__ rec,
-                                                                                    int64_t n, FrameParams fp,
-                                                                                    void* __restrict__ out_,
-                                                                                    float* __restrict__ seg_scratch) {
-  // the list and the chunk arrays, and (gray output) the staged tile afterwards, share one buffer
+__global__ void __launch_bounds__(TILE_THREADS, (CIRC && INTEG) ? 2 : (CIRC || INTEG) ? 3 : LITE_MINB) k_tile_sparse(
+    const StarRec* __restrict__ rec, const uint32_t* __restrict__ box, int64_t n, FrameParams fp,
+    void* __restrict__ out_, float* __restrict__ seg_scratch) {
+  // the pending list and the chunk arrays, and (gray output) the staged tile afterwards, share one buffer
   struct Lists {
-    uint32_t lidx[SPARSE_MAX];
+    uint32_t lidx[SP_BUF];
     uint32_t lkey[SB_CHUNK];
     float4 lrec[SB_CHUNK];
     uint32_t llo[SB_CHUNK];
@@ -649,10 +664,6 @@ __global__ void __launch_bounds__(TILE_THREADS, (CIRC && INTEG) ? 2 : (CIRC || I
                                                   ? sizeof(float) * TILE_W * TILE_H
                                                   : sizeof(Lists)];
   Lists& L = *reinterpret_cast<Lists*>(sraw);
-  uint32_t* lidx = L.lidx;
-  uint32_t* lkey = L.lkey;
-  float4* lrec = L.lrec;
-  uint32_t* llo = L.llo;
   __shared__ uint32_t wcnt[TILE_WARPS];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
@@ -663,51 +674,89 @@ __global__ void __launch_bounds__(TILE_THREADS, (CIRC && INTEG) ? 2 : (CIRC || I
   const int X0 = tx * TILE_W, Y0 = ty * TILE_H, IY0 = fp.row0 + Y0;
   const int TWe = min(TILE_W, fp.W - X0), THe = min(TILE_H, fp.rows - Y0);
   n = frame_n(n, fp);
-  // the tile's list: stars whose clipped ROI meets it (the binning's pair rule), ascending star index
-  uint32_t len = 0;
-  const uint32_t lt = (1u << lane) - 1u;
-  for (int64_t base = 0; base < n; base += TILE_THREADS) {
-    const int64_t i = base + tid;
-    bool hit = false;
-    if (i < n) {
-      const uint32_t lo = __ldg(&rec[i].lo);
-      if (lo != LO_CULLED) {
-        const int lx = lo_x_of(lo) - X0, ly = lo_y_of(lo) - IY0;
-        hit = lx <= TWe - 1 && lx + fp.R - 1 >= 0 && ly <= THe - 1 && ly + fp.R - 1 >= 0;
-      }
-    }
-    const uint32_t wm = __ballot_sync(0xffffffffu, hit);
-    if (lane == 0) wcnt[warp] = __popc(wm);
-    __syncthreads();
-    uint32_t pre = 0, tot = 0;
-#pragma unroll
-    for (int w = 0; w < TILE_WARPS; ++w) {
-      const uint32_t cw = wcnt[w];
-      pre += w < warp ? cw : 0u;
-      tot += cw;
-    }
-    if (hit) lidx[len + pre + __popc(wm & lt)] = (uint32_t)i;
-    len += tot;
-    __syncthreads();
-  }
   float2 acc[4][4];
 #pragma unroll
   for (int i = 0; i < 4; ++i)
 #pragma unroll
     for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
-  // chunks of SB_CHUNK from the list start, as k_tile_sb cuts them; a list longer than SPLIT_LEN is summed in
-  // segments (reading R19) through the tile's own slot of the segment scratch (one CTA per tile)
-  uint32_t segs_done = 0;
-  for (uint32_t c0 = 0; c0 < len; c0 += SB_CHUNK) {
-    const int nn = (int)min((uint32_t)SB_CHUNK, len - c0);
+  const uint32_t lt = (1u << lane) - 1u;
+  uint32_t pending = 0, done_chunks = 0, segs_done = 0;
+  // a round: warp w takes the 128 consecutive stars base + 128 w .. (4 x 32), so the hits come out in star order
+  // as (warp, sub-round, lane); one block prefix over the warps places them after the pending entries
+  auto render_chunk = [&](int nn) {
     StarRec r = {};
-    if (tid < nn) r = rec[lidx[c0 + tid]];
-    lite_chunk<INTEG, CIRC, SB_CHUNK>(acc, lkey, lrec, llo, r, nn, fp, X0, IY0, TWe, THe);
-    if ((c0 + SB_CHUNK) % SPLIT_LEN == 0 && c0 + SB_CHUNK < len) {
-      seg_flush(acc, seg_scratch, segs_done == 0);
-      ++segs_done;
+    if (tid < nn) r = rec[L.lidx[tid]];
+    lite_chunk<INTEG, CIRC, SB_CHUNK>(acc, L.lkey, L.lrec, L.llo, r, nn, fp, X0, IY0, TWe, THe);
+    ++done_chunks;
+  };
+  for (int64_t base = 0; base < n; base += (int64_t)TILE_THREADS * 4) {
+    uint32_t hm[4];
+    uint32_t cw = 0;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int64_t i = base + 128 * warp + 32 * j + lane;
+      bool hit = false;
+      if (i < n) {
+        const uint32_t b = __ldg(&box[i]);
+        if (b != SP_NONE) {
+          const int btx = (int)(b & 0xFFu), bty = (int)((b >> 8) & 0x1FFu);
+          hit = tx >= btx && tx <= btx + (int)((b >> 17) & 1u) && ty >= bty && ty <= bty + (int)((b >> 18) & 1u);
+        }
+      }
+      hm[j] = __ballot_sync(0xffffffffu, hit);
+      cw += __popc(hm[j]);
+    }
+    if (lane == 0) wcnt[warp] = cw;
+    __syncthreads();
+    uint32_t pre = 0, tot = 0;
+#pragma unroll
+    for (int w = 0; w < TILE_WARPS; ++w) {
+      const uint32_t c = wcnt[w];
+      pre += w < warp ? c : 0u;
+      tot += c;
+    }
+    uint32_t pos = pending + pre;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      if ((hm[j] >> lane) & 1u) L.lidx[pos + __popc(hm[j] & lt)] = (uint32_t)(base + 128 * warp + 32 * j + lane);
+      pos += __popc(hm[j]);
+    }
+    pending += tot;
+    __syncthreads();
+    // whole chunks: render them in list order, then move the remainder to the front
+    uint32_t off = 0;
+    while (pending - off >= (uint32_t)SB_CHUNK) {
+      if (off) {  // bring the next chunk's entries to the front of the list buffer
+        uint32_t v = tid < SB_CHUNK ? L.lidx[off + tid] : 0u;
+        __syncthreads();
+        if (tid < SB_CHUNK) L.lidx[tid] = v;
+        __syncthreads();
+        // (the entries after it stay where they are; off counts from the moved chunk)
+        for (uint32_t k = SB_CHUNK + tid; k < pending - off; k += TILE_THREADS) L.lidx[k] = L.lidx[off + k];
+        __syncthreads();
+        pending -= off;
+        off = 0;
+      }
+      render_chunk(SB_CHUNK);
+      if (((done_chunks * SB_CHUNK) % SPLIT_LEN) == 0) {
+        seg_flush(acc, seg_scratch, segs_done == 0);  // a full segment: more list entries may follow
+        ++segs_done;
+      }
+      off = SB_CHUNK;
+      __syncthreads();
+    }
+    if (off) {  // keep the remainder (< one chunk) at the front
+      const uint32_t rem = pending - off;
+      uint32_t v = tid < (int)rem ? L.lidx[off + tid] : 0u;
+      __syncthreads();
+      if ((uint32_t)tid < rem) L.lidx[tid] = v;
+      pending = rem;
+      __syncthreads();
     }
   }
+  if (pending) render_chunk((int)pending);
+  // a segment flushed right at the list's end holds the whole last segment: fold it back (the order of R19 is kept:
+  // the flushed partial sums come first, the empty rest adds zeros)
   if (segs_done) seg_finish(acc, seg_scratch);
   if (swz) {
 #pragma unroll
@@ -735,26 +784,25 @@ __global__ void __launch_bounds__(TILE_THREADS, (CIRC && INTEG) ? 2 : (CIRC || I
   }
 }
 
-// every tile CTA tests every star: worth it while stars x tiles stays small (measured: C1 64 K, fig2 288 K, C3 with
-// 1 K stars 2 M pair tests win; C3 with 4 K stars, 8 M, loses to the binning path)
+// every tile CTA streams every star's 4-B tile box: worth it while stars x tiles stays small (measured)
 bool sparse_ok(int64_t n, int64_t ntiles) { return n <= SPARSE_MAX && n * ntiles <= SPARSE_TESTS; }
 
 void launch_srec(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
-                 cudaStream_t st) {
-  if (n > 0) k_srec<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(x, y, m, n, fp, rec);
+                 uint32_t* box, cudaStream_t st) {
+  if (n > 0) k_srec<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(x, y, m, n, fp, rec, box);
 }
 
-void launch_tile_sparse(const StarRec* rec, int64_t n, const FrameParams& fp, void* out, float* seg_scratch,
-                        cudaStream_t st) {
+void launch_tile_sparse(const StarRec* rec, const uint32_t* box, int64_t n, const FrameParams& fp, void* out,
+                        float* seg_scratch, cudaStream_t st) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
-  using KS = void (*)(const StarRec*, int64_t, FrameParams, void*, float*);
+  using KS = void (*)(const StarRec*, const uint32_t*, int64_t, FrameParams, void*, float*);
   static const KS ks[2][2][3] = {
       {{k_tile_sparse<false, false, 0>, k_tile_sparse<false, false, 8>, k_tile_sparse<false, false, 16>},
        {k_tile_sparse<false, true, 0>, k_tile_sparse<false, true, 8>, k_tile_sparse<false, true, 16>}},
       {{k_tile_sparse<true, false, 0>, k_tile_sparse<true, false, 8>, k_tile_sparse<true, false, 16>},
        {k_tile_sparse<true, true, 0>, k_tile_sparse<true, true, 8>, k_tile_sparse<true, true, 16>}}};
   const KS k = ks[fp.psf ? 1 : 0][fp.roi ? 1 : 0][fp.obits == 8 ? 1 : fp.obits == 16 ? 2 : 0];
-  k<<<(unsigned)ntiles, TILE_THREADS, 0, st>>>(rec, n, fp, out, seg_scratch);
+  k<<<(unsigned)ntiles, TILE_THREADS, 0, st>>>(rec, box, n, fp, out, seg_scratch);
 }
 
 #ifdef STARSIM_SB_TIMING

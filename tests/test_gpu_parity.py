@@ -547,9 +547,11 @@ def test_fused_binning_same_csr_and_image(torch_dev, monkeypatch, W, H, n, R, se
                                                (700, 530, 1024, 15, 3, "adv"), (300, 200, 900, 17, 4, "dense"),
                                                (129, 65, 1, 9, 5, "uniform"), (256, 256, 0, 7, 6, "uniform"),
                                                (1024, 1024, 2252, 11, 7, "uniform"), (4096, 2048, 4096, 15, 8, "adv"),
-                                               (300, 200, 4000, 15, 9, "dense")])  # > 1,024 stars in a tile
+                                               (300, 200, 4000, 15, 9, "dense"),  # > 1,024 stars in a tile
+                                               (4096, 2048, 8000, 11, 10, "uniform"), (1024, 1024, 30000, 9, 11, "uniform"),
+                                               (256, 192, 9000, 13, 12, "dense")])
 def test_sparse_path_is_bitwise_sb(torch_dev, W, H, n, R, seed, kind):
-    """STARSIM_TILE_AUTO renders catalogues of <= 4,096 stars through the sparse path (k_srec + k_tile_sparse: no
+    """STARSIM_TILE_AUTO renders small catalogues (<= 32,768 stars, stars x tiles <= 8 M) through the sparse path (k_srec + k_tile_sparse: no
     binning launches, every tile CTA builds its own list; lists over 1,024 stars summed in segments, reading R19):
     the same image as k_tile_sb bit for bit -- point and
     integrated PSF, square and circle ROI, fp32 and u8 -- at parity with the oracle, bands bitwise the frame, and
