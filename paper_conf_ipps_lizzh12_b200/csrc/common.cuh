@@ -68,7 +68,10 @@ constexpr uint32_t ITEM_WHOLE = 0xFFFFFFFFu;
 #endif
 constexpr int LITE_MAX = SB_LITE_MAX;
 constexpr int SPARSE_MAX = 32768;            // catalogues of at most this many stars take the sparse path (AUTO)
-constexpr int64_t SPARSE_TESTS = 8 << 20;    // ... when stars x tiles (the star tests of its tile CTAs) is at most this
+#ifndef SPARSE_TESTS_OPT
+#define SPARSE_TESTS_OPT (8 << 20)
+#endif
+constexpr int64_t SPARSE_TESTS = SPARSE_TESTS_OPT;  // ... when stars x tiles (the tile CTAs' star tests) is at most this
 constexpr double LITE_AUTO_PER_TILE = 16.0;  // k_tile_lite is launched when the expected list per tile is <= this
 constexpr int64_t LITE_AUTO_TILES = 1024;    // ... and the frame / band has at least this many tiles
 constexpr int SPLIT_LEN = 1024;        // a tile list longer than this is split into parts of <= SPLIT_LEN stars

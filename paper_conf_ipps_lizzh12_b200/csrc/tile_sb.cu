@@ -648,7 +648,11 @@ __global__ void __launch_bounds__(256) k_srec(const float* __restrict__ X, const
   box[i] = b;
 }
 
-constexpr int SP_BUF = SB_CHUNK + TILE_THREADS * 4;  // pending list entries: < one chunk + one round's hits
+#ifndef SP_PER_OPT
+#define SP_PER_OPT 8
+#endif
+constexpr int SP_PER = SP_PER_OPT;                        // stars per thread and round (loads issued together)
+constexpr int SP_BUF = SB_CHUNK + TILE_THREADS * SP_PER;  // pending list entries: < one chunk + one round's hits
 template <bool INTEG, bool CIRC, int OB>
 __global__ void __launch_bounds__(TILE_THREADS, (CIRC && INTEG) ? 2 : (CIRC || INTEG) ? 3 : LITE_MINB) k_tile_sparse(
     const StarRec* __restrict__ rec, const uint32_t* __restrict__ box, int64_t n, FrameParams fp,
@@ -681,7 +685,7 @@ __global__ void __launch_bounds__(TILE_THREADS, (CIRC && INTEG) ? 2 : (CIRC || I
     for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
   const uint32_t lt = (1u << lane) - 1u;
   uint32_t pending = 0, done_chunks = 0, segs_done = 0;
-  // a round: warp w takes the 128 consecutive stars base + 128 w .. (4 x 32), so the hits come out in star order
+  // a round: warp w takes the 32 SP_PER consecutive stars from base + 32 SP_PER w, so the hits come out in star order
   // as (warp, sub-round, lane); one block prefix over the warps places them after the pending entries
   auto render_chunk = [&](int nn) {
     StarRec r = {};
@@ -689,19 +693,20 @@ __global__ void __launch_bounds__(TILE_THREADS, (CIRC && INTEG) ? 2 : (CIRC || I
     lite_chunk<INTEG, CIRC, SB_CHUNK>(acc, L.lkey, L.lrec, L.llo, r, nn, fp, X0, IY0, TWe, THe);
     ++done_chunks;
   };
-  for (int64_t base = 0; base < n; base += (int64_t)TILE_THREADS * 4) {
-    uint32_t hm[4];
+  for (int64_t base = 0; base < n; base += (int64_t)TILE_THREADS * SP_PER) {
+    uint32_t hm[SP_PER];
+    uint32_t bx[SP_PER];
     uint32_t cw = 0;
+    const int64_t wb = base + (int64_t)(32 * SP_PER) * warp + lane;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int64_t i = base + 128 * warp + 32 * j + lane;
+    for (int j = 0; j < SP_PER; ++j) bx[j] = wb + 32 * j < n ? __ldg(&box[wb + 32 * j]) : SP_NONE;
+#pragma unroll
+    for (int j = 0; j < SP_PER; ++j) {
       bool hit = false;
-      if (i < n) {
-        const uint32_t b = __ldg(&box[i]);
-        if (b != SP_NONE) {
-          const int btx = (int)(b & 0xFFu), bty = (int)((b >> 8) & 0x1FFu);
-          hit = tx >= btx && tx <= btx + (int)((b >> 17) & 1u) && ty >= bty && ty <= bty + (int)((b >> 18) & 1u);
-        }
+      const uint32_t b = bx[j];
+      if (b != SP_NONE) {
+        const int btx = (int)(b & 0xFFu), bty = (int)((b >> 8) & 0x1FFu);
+        hit = tx >= btx && tx <= btx + (int)((b >> 17) & 1u) && ty >= bty && ty <= bty + (int)((b >> 18) & 1u);
       }
       hm[j] = __ballot_sync(0xffffffffu, hit);
       cw += __popc(hm[j]);
@@ -717,8 +722,8 @@ __global__ void __launch_bounds__(TILE_THREADS, (CIRC && INTEG) ? 2 : (CIRC || I
     }
     uint32_t pos = pending + pre;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      if ((hm[j] >> lane) & 1u) L.lidx[pos + __popc(hm[j] & lt)] = (uint32_t)(base + 128 * warp + 32 * j + lane);
+    for (int j = 0; j < SP_PER; ++j) {
+      if ((hm[j] >> lane) & 1u) L.lidx[pos + __popc(hm[j] & lt)] = (uint32_t)(wb + 32 * j);
       pos += __popc(hm[j]);
     }
     pending += tot;
