@@ -87,12 +87,21 @@ def _worker(rank, world, port, W, H, q):
         img = oracle.render_band(xs, ys, ms, width, height, row0, rows, sigma, roi, gain)
         out.copy_(torch.from_numpy(img.astype(np.float32)))
 
+    # back-to-back frames through the same band buffer (different catalogues): each assembled frame checked
+    band_out = None
+    ok = True
+    for k, seed in enumerate((11, 12, 13)):
+        fk = synth.uniform_field(400 + 50 * k, W, H, seed=seed)
+        xk, yk, mk = (torch.from_numpy(a) for a in (fk.x, fk.y, fk.mag))
+        fr, band_out = sdist.render_frame(render_band, xk, yk, mk, W, H, 1.7, 9, 1.0, band_out=band_out)
+        refk = torch.from_numpy(oracle.render(fk.x, fk.y, fk.mag, W, H, 1.7, 9, 1.0).astype(np.float32))
+        ok = ok and sdist.frames_agree(fr, refk)
     x, y, m = (torch.from_numpy(a) for a in (f.x, f.y, f.mag))
     frame, band = sdist.render_frame(render_band, x, y, m, W, H, 1.7, 9, 1.0)
     # the bench's validation (dist.frames_agree): every rank compares its assembled frame with the single-process
     # frame; a corrupted frame on any one rank must make it fail on all ranks
     ref = torch.from_numpy(oracle.render(f.x, f.y, f.mag, W, H, 1.7, 9, 1.0).astype(np.float32))
-    ok = sdist.frames_agree(frame, ref)
+    ok = ok and sdist.frames_agree(frame, ref)
     bad = frame.clone()
     if rank == world - 1:
         bad[H - 1, W - 1] += 1.0
