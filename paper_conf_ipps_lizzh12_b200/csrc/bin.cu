@@ -485,6 +485,7 @@ void init_kernels() {
   init_tile_kernel();
   init_tile_sb_kernel();
   init_tile_ws_kernel();
+  init_tile_wide_kernel();
   init_tile8_kernel();
   init_dbin_kernels();
 }

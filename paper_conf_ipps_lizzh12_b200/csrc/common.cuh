@@ -24,6 +24,7 @@ constexpr int LCAP = 32;                         // entries per (band, strip) li
 constexpr int GX_PAIRS = 768;                    // (star, strip) pairs per chunk
 constexpr int WS_MIN_PER_TILE = 100;            // STARSIM_TILE_AUTO picks tile_ws.cu from this expected list length
 constexpr int SB_MAXR = 17;                      // tile_sb.cu: an ROI of side <= 17 spans <= 2 bands and <= 3 strips
+constexpr int WIDE_MAXR = 65;                    // tile_wide.cu: 17 < R <= 65 (<= 5 bands and <= 9 strips)
 
 // k_prep: one star per thread; per-tile counters CNT_STRIDE words apart (one 128-B line each, so that the
 // atomics of different tiles never serialise on one L2 line)

@@ -182,7 +182,9 @@ struct DpSmem {
   uint32_t cur[DB_MAXT];         // per tile: next free slot of its group; then the tile list position of the group
   uint16_t arr[DP_KEYS];          // the CTA's star indices grouped by tile (in arbitrary order inside a group)
   uint32_t s_w[DP_WARPS + 1];
+  uint32_t bmap[DP_WARPS][DB_CTA / 32];  // per warp: a large group's members as a bitmap of star indices
 };
+constexpr uint32_t DP_BIG = 32;  // groups of more pairs are placed through a bitmap, not the rank loop
 
 // tiles of a packed box (0 if the star is culled) and its e-th tile, e < box_n (row-major order inside the box)
 __device__ __forceinline__ int box_n(uint32_t code) {
@@ -302,7 +304,8 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
   // first list position of every group: tile_off[t] + (pairs of tile t in the CTAs before)
   for (int t = tid; t < ntiles; t += DP_THREADS) S.cur[t] = S.toff[t] + (C ? __ldcg(&C[(int64_t)cta * ntiles + t]) : 0u);
   __syncthreads();
-  // a pair's rank in its group = the group's stars with a smaller index
+  // a pair's rank in its group = the group's stars with a smaller index (groups of at most DP_BIG pairs: the common
+  // case of uniform fields)
 #pragma unroll
   for (int k = 0; k < DP_SPT; ++k) {
     const uint32_t idx = (uint32_t)(tid + k * DP_THREADS);
@@ -310,10 +313,52 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
     for (int e = 0; e < nb; ++e) {
       const int t = box_tile(code[k], e, fp.ntx);
       const uint32_t g0 = S.gstart[t], g1 = S.gstart[t + 1];
+      if (g1 - g0 > DP_BIG) continue;
       uint32_t rank = 0;
       for (uint32_t u = g0; u < g1; ++u) rank += S.arr[u] < idx ? 1u : 0u;
       ids[S.cur[t] + rank] = (uint32_t)c0 + idx;
     }
+  }
+  // larger groups (clustered fields: the rank loop would cost O(group^2)): one warp per group sets the members' bits
+  // in a bitmap of the CTA's star indices, then writes the set bits in ascending order (a warp scan of the per-lane
+  // counts) -- the same ascending-index list
+  const int lane = tid & 31, warp = tid >> 5;
+  uint32_t* bm = S.bmap[warp];
+  for (int t = warp; t < ntiles; t += DP_WARPS) {
+    const uint32_t g0 = S.gstart[t], g1 = S.gstart[t + 1];
+    if (g1 - g0 <= DP_BIG) continue;  // warp-uniform
+    constexpr int WPL = DB_CTA / 32 / 32;  // bitmap words per lane
+#pragma unroll
+    for (int w = 0; w < WPL; ++w) bm[lane * WPL + w] = 0u;
+    __syncwarp();
+    for (uint32_t u = g0 + lane; u < g1; u += 32) {
+      const uint32_t v = S.arr[u];
+      atomicOr(&bm[v >> 5], 1u << (v & 31u));
+    }
+    __syncwarp();
+    uint32_t wv[WPL], cntl = 0;
+#pragma unroll
+    for (int w = 0; w < WPL; ++w) {
+      wv[w] = bm[lane * WPL + w];
+      cntl += __popc(wv[w]);
+    }
+    uint32_t incl = cntl;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t q = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += q;
+    }
+    uint32_t pos = S.cur[t] + incl - cntl;
+#pragma unroll
+    for (int w = 0; w < WPL; ++w) {
+      uint32_t m = wv[w];
+      while (m) {
+        const int b = __ffs(m) - 1;
+        m &= m - 1u;
+        ids[pos++] = (uint32_t)c0 + (uint32_t)((lane * WPL + w) * 32 + b);
+      }
+    }
+    __syncwarp();
   }
 }
 

@@ -11,6 +11,8 @@ void init_kernels();
 void init_tile_kernel();
 void init_tile_sb_kernel();
 void init_tile_ws_kernel();
+void init_tile_wide_kernel();
+bool wide_ok(int R);  // k_tile_wide serves this ROI side (SB_MAXR < R <= WIDE_MAXR)
 void init_tile8_kernel();
 size_t tile8_scratch_floats(int num_sms);
 void init_dbin_kernels();
@@ -51,6 +53,9 @@ void launch_tile_sb(const uint32_t* ids, const StarRec* rec, const FrameParams& 
 void launch_tile_ws(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
                     const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
                     cudaStream_t st, float* seg_scratch, const StarRec* srec, const uint16_t* cbin);
+void launch_tile_wide(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, void* out, const WorkItem* items,
+                      const uint2* split_tab, float* part_buf, int part_cap, uint32_t* done, Header* hdr, int num_sms,
+                      cudaStream_t st, float* seg_scratch);
 size_t chsort_slots(int64_t ntiles, int64_t pmax);  // rows of k_chsort's bin-start table
 size_t chsort_words16();                            // u16 per row
 void launch_chsort(const uint32_t* ids, const StarRec* rec, const FrameParams& fp, const WorkItem* items, int part_cap,

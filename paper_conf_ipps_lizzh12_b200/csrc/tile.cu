@@ -465,6 +465,10 @@ void launch_tile(const uint32_t* ids, const StarRec* rec, const FrameParams& fp,
                    tile_off);
     return;
   }
+  if (wide_ok(fp.R) && fp.tile_impl != 1) {  // every mode but STARSIM_TILE_LISTS: the sorted-bin kernel for wide ROIs
+    launch_tile_wide(ids, rec, fp, out, items, split_tab, part_buf, part_cap, done, hdr, num_sms, st, seg_scratch);
+    return;
+  }
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
   // persistent, 3 CTAs per SM (2 for the circle ROI)

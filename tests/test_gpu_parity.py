@@ -340,7 +340,7 @@ def test_full_frame_parity(torch_dev, ctx, name):
     assert_parity(img, ref, name)
 
 
-@pytest.mark.parametrize("R", [3, 15, 63])
+@pytest.mark.parametrize("R", [3, 15, 21, 31, 47, 63])
 def test_c4_clustered_parity(torch_dev, ctx, R):
     cfg = synth.with_R(synth.CONFIGS["C4"], R)
     f = cfg.field()
@@ -452,6 +452,53 @@ def test_binning_pipelines_identical(torch_dev, name, W, H, n, R, kind):
     assert torch.equal(ia, ib)
     ref_off, ref_ids = oracle.bins(f.x, f.y, f.mag, W, H, R, tw, th)
     assert np.array_equal(oa[:ntiles + 1], ref_off) and np.array_equal(da, ref_ids)
+
+
+@pytest.mark.parametrize("R,psf", [(18, "point"), (25, "integrated"), (33, "point"), (34, "point"), (49, "point"),
+                                   (50, "integrated"), (65, "point")])
+def test_wide_roi_kernel(torch_dev, R, psf):
+    """k_tile_wide (17 < R <= 65, sorted corner bins over <= 5 bands x 9 strips) at each band-slot count's edges:
+    parity against the oracle, within rounding of the list kernel k_tile (a different fixed order), deterministic,
+    and tile-aligned bands bitwise the frame -- on a 537 x 411 frame (ragged tiles) with stars off every border."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context
+    W, H, sigma = 537, 411, R / 6.0
+    f = synth.adversarial_field(4000, W, H, R, seed=R)
+    args = to_dev(torch_dev, f)
+    ref = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads(), psf=psf)
+    out = {}
+    for mode in ("auto", "lists"):
+        with Context(0) as c:
+            c.set_tile_kernel(mode)
+            c.set_psf(psf)
+            a = c.render(*args, W, H, sigma, R, 1.0)
+            assert_parity(a.cpu().numpy(), ref, f"wide R={R} {psf} {mode}")
+            if mode == "auto":
+                assert torch.equal(a, c.render(*args, W, H, sigma, R, 1.0))
+                bands = [c.render_band(*args, W, H, g * 64, min(64, H - g * 64), sigma, R, 1.0)
+                         for g in range(-(-H // 64))]
+                assert torch.equal(torch.cat(bands, 0), a)
+            out[mode] = a.double().cpu().numpy()
+    peak = float(np.abs(ref).max())
+    assert float(np.abs(out["auto"] - out["lists"]).max()) <= 1e-5 * peak
+
+
+@pytest.mark.parametrize("R", [31, 63])
+def test_wide_roi_heavy_tiles(torch_dev, ctx, R):
+    """Clustered wide-ROI field with tiles of > 4 x SPLIT_LEN stars (split into parts): parity, determinism, bands
+    bitwise the frame -- for k_tile_wide (auto / sb / ws / t8 modes) and k_tile (lists)."""
+    torch, dev = torch_dev
+    W, H, sigma = 512, 384, R / 6.0
+    f = _dense_field(9000, W, H, 200.0, 150.0, 40.0, seed=33)
+    args = to_dev(torch_dev, f)
+    a = ctx.render(*args, W, H, sigma, R, 1.0)
+    tw, th, off, ids = ctx.get_bins()
+    assert int(np.diff(off).max()) > 4 * 1024
+    ref = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads())
+    assert_parity(a.cpu().numpy(), ref, f"wide heavy R={R}")
+    assert torch.equal(a, ctx.render(*args, W, H, sigma, R, 1.0))
+    bands = [ctx.render_band(*args, W, H, g * 64, 64, sigma, R, 1.0) for g in range(H // 64)]
+    assert torch.equal(torch.cat(bands, 0), a)
 
 
 def test_tile_kernels_agree_within_rounding(torch_dev):
