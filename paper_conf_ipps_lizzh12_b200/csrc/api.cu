@@ -10,6 +10,7 @@
 #include "../../include/starsim.h"
 #include "common.cuh"
 #include "launch.h"
+#include "plan.cuh"
 
 using namespace starsim;
 
@@ -210,6 +211,9 @@ FrameParams make_params(int32_t W, int32_t H, int32_t row0, int32_t rows, float 
   fp.vec = 0;
   fp.vec32 = 0;
   fp.kint = (float)(1.0 / (std::sqrt(2.0) * s));
+  // the part / segment length of long tile lists (reading R19): shorter for the wide-ROI kernel, whose stars cost
+  // R^2 FMAs each (a heavy tile then spreads over more CTAs)
+  fp.split = wide_ok(R) ? WIDE_SPLIT : SPLIT_LEN;
   if (psf) fp.s_scale = (double)gain;  // the pixel masses of the integrated PSF are already normalised
   return fp;
 }
@@ -240,6 +244,7 @@ int enqueue_binning(starsim_ctx* c, const float* x, const float* y, const float*
   uint32_t* tile_off = (uint32_t*)c->tile_off.p;
   uint32_t* slots = (uint32_t*)c->slots.p;
   StarRec* rec = (StarRec*)c->rec.p;
+  const int plan = plan_word(part_cap, fp.split);  // the planner's pool size and part length (plan.cuh)
   int rc;
   if (dbin_ok(fp, ntiles)) {
     // deterministic counting sort (dbin.cu): no memset, no atomics on global counters, no per-tile sort
@@ -249,7 +254,7 @@ int enqueue_binning(starsim_ctx* c, const float* x, const float* y, const float*
       // at most DB_CTA stars: the whole binning in one CTA, one launch (k_dsmall)
       timed(c, 0, st, [&] {
         launch_dsmall(x, y, mag, n, fp, rec, (int)ntiles, tile_off, hdr, (WorkItem*)c->items.p,
-                      (uint2*)c->split_tab.p, part_cap, done, ids, st);
+                      (uint2*)c->split_tab.p, plan, done, ids, st);
       });
       if ((rc = check_launch(c, "k_dsmall"))) return rc;
     } else if (n > 0 && c->dfused_grid > 0 && dbin_ctas(n) <= c->dfused_grid) {
@@ -257,7 +262,7 @@ int enqueue_binning(starsim_ctx* c, const float* x, const float* y, const float*
       cudaError_t le = cudaSuccess;
       timed(c, 0, st, [&] {
         le = launch_dfused(x, y, mag, n, fp, rec, C, cnt, (int)ntiles, tile_off, hdr, (WorkItem*)c->items.p,
-                           (uint2*)c->split_tab.p, part_cap, done, ids, (uint32_t*)c->gbar.p, st);
+                           (uint2*)c->split_tab.p, plan, done, ids, (uint32_t*)c->gbar.p, st);
       });
       if (le != cudaSuccess) return cuda_fail(c, le, "k_dfused (cooperative launch)");
       if ((rc = check_launch(c, "k_dfused"))) return rc;
@@ -268,7 +273,7 @@ int enqueue_binning(starsim_ctx* c, const float* x, const float* y, const float*
       if ((rc = check_launch(c, "k_dcolscan"))) return rc;
       timed(c, 1, st, [&] {
         launch_dplace((const uint32_t*)c->codes.p, n, fp, C, (int)ntiles, cnt, tile_off, hdr, (WorkItem*)c->items.p,
-                      (uint2*)c->split_tab.p, part_cap, done, ids, st);
+                      (uint2*)c->split_tab.p, plan, done, ids, st);
       });
       if ((rc = check_launch(c, "k_dplace"))) return rc;
     } else {
@@ -276,7 +281,7 @@ int enqueue_binning(starsim_ctx* c, const float* x, const float* y, const float*
           c, 2, st,
           [&] {
             launch_dcolscan(C, n, (int)ntiles, cnt, CNT_STRIDE, nullptr, st);
-            launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap,
+            launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, plan,
                         c->partial.p, done, st);
           },
           1 + scan_launches(ntiles));
@@ -291,7 +296,7 @@ int enqueue_binning(starsim_ctx* c, const float* x, const float* y, const float*
     timed(
         c, 2, st,
         [&] {
-          launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, part_cap,
+          launch_scan(cnt, ntiles, tile_off, hdr, (WorkItem*)c->items.p, (uint2*)c->split_tab.p, plan,
                       c->partial.p, done, st);
           launch_scatter(rec, n, fp, slots, tps, tile_off, ids, st);
         },
@@ -374,7 +379,8 @@ int render_tiled(starsim_ctx* c, const float* x, const float* y, const float* ma
     // tile for a uniform field, n (128 + R - 1)(64 + R - 1) / (W rows).  k_tile8 (STARSIM_TILE_T8) is faster in the
     // tile kernel but needs the k_t8sort pass: a slower frame at T, so it is opt-in.
     const double per_tile = (double)n * (TILE_W + R - 1) * (TILE_H + R - 1) / ((double)W * (rows > 0 ? rows : 1));
-    fp.tile_impl = (c->psf == 0 && per_tile >= WS_MIN_PER_TILE) ? STARSIM_TILE_WS : STARSIM_TILE_SB;
+    // (wide ROIs: STARSIM_TILE_SB = k_tile_wide, measured faster than its warp-specialised form k_tile_wws)
+    fp.tile_impl = (c->psf == 0 && per_tile >= WS_MIN_PER_TILE && !wide_ok(R)) ? STARSIM_TILE_WS : STARSIM_TILE_SB;
   }
   fp.bin_impl = c->bin_impl;
   fp.n_dev = c->n_dev;

@@ -72,21 +72,22 @@ __device__ __forceinline__ uint4 block_excl_scan4(uint4 v, uint4* s_w, uint4* to
   return sub4(add4(pre, incl), v);
 }
 
-__device__ __forceinline__ void load_counts(const uint32_t* cnt, int64_t ntiles, int64_t t0, uint32_t* c, uint4& sum) {
+__device__ __forceinline__ void load_counts(const uint32_t* cnt, int64_t ntiles, int64_t t0, uint32_t* c, uint4& sum,
+                                            uint32_t split) {
   sum = make_uint4(0, 0, 0, 0);
 #pragma unroll
   for (int k = 0; k < SCAN_PER; ++k) c[k] = t0 + k < ntiles ? __ldcg(&cnt[(t0 + k) * CNT_STRIDE]) : 0u;
 #pragma unroll
-  for (int k = 0; k < SCAN_PER; ++k) sum = add4(sum, t0 + k < ntiles ? tile_counts(c[k]) : make_uint4(0, 0, 0, 0));
+  for (int k = 0; k < SCAN_PER; ++k) sum = add4(sum, t0 + k < ntiles ? tile_counts(c[k], split) : make_uint4(0, 0, 0, 0));
 }
 
 __global__ void __launch_bounds__(SCAN_THREADS) k_scan_a(const uint32_t* __restrict__ cnt, int64_t ntiles,
-                                                         uint4* __restrict__ partial) {
+                                                         uint4* __restrict__ partial, int plan) {
   __shared__ uint4 s_w[SCAN_THREADS / 32];
   const int64_t t0 = (int64_t)blockIdx.x * SCAN_TILES + (int64_t)threadIdx.x * SCAN_PER;
   uint32_t c[SCAN_PER];
   uint4 sum, tot;
-  load_counts(cnt, ntiles, t0, c, sum);
+  load_counts(cnt, ntiles, t0, c, sum, plan_split(plan));
   block_excl_scan4(sum, s_w, &tot);
   if (threadIdx.x == 0) partial[blockIdx.x] = tot;
 }
@@ -95,10 +96,12 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_b(const uint32_t* __restr
                                                          const uint4* __restrict__ partial, int nblk,
                                                          uint32_t* __restrict__ tile_off, Header* hdr,
                                                          WorkItem* __restrict__ items,
-                                                         uint2* __restrict__ split_tab, int part_cap,
+                                                         uint2* __restrict__ split_tab, int plan,
                                                          uint32_t* __restrict__ done) {
   __shared__ uint4 s_w[SCAN_THREADS / 32];
   const int tid = threadIdx.x;
+  const int part_cap = plan_cap(plan);
+  const uint32_t split = plan_split(plan);
   // sums of the CTAs before this one, and of all CTAs
   uint4 before = make_uint4(0, 0, 0, 0), all = make_uint4(0, 0, 0, 0);
   for (int k = tid; k < nblk; k += SCAN_THREADS) {
@@ -116,14 +119,14 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_b(const uint32_t* __restr
   const int64_t t0 = (int64_t)blockIdx.x * SCAN_TILES + (int64_t)tid * SCAN_PER;
   uint32_t c[SCAN_PER];
   uint4 sum, tot;
-  load_counts(cnt, ntiles, t0, c, sum);
+  load_counts(cnt, ntiles, t0, c, sum, split);
   const uint4 ex = add4(tb, block_excl_scan4(sum, s_w, &tot));
   uint32_t run = ex.x, pb = ex.y, si = ex.z, li = ex.w;
 #pragma unroll
   for (int k = 0; k < SCAN_PER; ++k) {
     const int64_t t = t0 + k;
     if (t >= ntiles) break;
-    plan_tile((uint32_t)t, c[k], run, pb, si, li, nparts, lite0, split_on, tile_off, items, split_tab, done);
+    plan_tile((uint32_t)t, c[k], run, pb, si, li, nparts, lite0, split_on, tile_off, items, split_tab, done, split);
   }
 }
 
@@ -135,15 +138,17 @@ constexpr int SCAN1_TILES = SCAN1_THREADS * SCAN_PER;
 __global__ void __launch_bounds__(SCAN1_THREADS) k_scan_one(const uint32_t* __restrict__ cnt, int64_t ntiles,
                                                              uint32_t* __restrict__ tile_off, Header* hdr,
                                                              WorkItem* __restrict__ items,
-                                                             uint2* __restrict__ split_tab, int part_cap,
+                                                             uint2* __restrict__ split_tab, int plan,
                                                              uint32_t* __restrict__ done) {
+  const int part_cap = plan_cap(plan);
+  const uint32_t split = plan_split(plan);
   __shared__ uint4 s_w[SCAN1_THREADS / 32];
   __shared__ uint4 s_tot;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t t0 = (int64_t)tid * SCAN_PER;
   uint32_t c[SCAN_PER];
   uint4 sum;
-  load_counts(cnt, ntiles, t0, c, sum);
+  load_counts(cnt, ntiles, t0, c, sum, split);
   const uint4 incl = warp_incl_scan4(sum, lane);
   if (lane == 31) s_w[warp] = incl;
   __syncthreads();
@@ -166,7 +171,7 @@ __global__ void __launch_bounds__(SCAN1_THREADS) k_scan_one(const uint32_t* __re
   for (int k = 0; k < SCAN_PER; ++k) {
     const int64_t t = t0 + k;
     if (t >= ntiles) break;
-    plan_tile((uint32_t)t, c[k], run, pb, si, li, nparts, lite0, split_on, tile_off, items, split_tab, done);
+    plan_tile((uint32_t)t, c[k], run, pb, si, li, nparts, lite0, split_on, tile_off, items, split_tab, done, split);
   }
 }
 
@@ -454,15 +459,15 @@ void launch_prep(const float* x, const float* y, const float* m, int64_t n, cons
 int scan_launches(int64_t ntiles) { return ntiles <= SCAN1_TILES ? 1 : 2; }
 
 void launch_scan(const uint32_t* cnt, int64_t ntiles, uint32_t* tile_off, Header* hdr, WorkItem* items,
-                 uint2* split_tab, int part_cap, void* partial, uint32_t* done, cudaStream_t st) {
+                 uint2* split_tab, int plan, void* partial, uint32_t* done, cudaStream_t st) {
   if (ntiles <= SCAN1_TILES) {
-    k_scan_one<<<1, SCAN1_THREADS, 0, st>>>(cnt, ntiles, tile_off, hdr, items, split_tab, part_cap, done);
+    k_scan_one<<<1, SCAN1_THREADS, 0, st>>>(cnt, ntiles, tile_off, hdr, items, split_tab, plan, done);
     return;
   }
   const int nblk = (int)((ntiles + SCAN_TILES - 1) / SCAN_TILES);
-  k_scan_a<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (uint4*)partial);
+  k_scan_a<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (uint4*)partial, plan);
   k_scan_b<<<nblk, SCAN_THREADS, 0, st>>>(cnt, ntiles, (const uint4*)partial, nblk, tile_off, hdr, items, split_tab,
-                                         part_cap, done);
+                                         plan, done);
 }
 
 void launch_scatter(const StarRec* rec, int64_t n, const FrameParams& fp, const uint32_t* slots, int tps,

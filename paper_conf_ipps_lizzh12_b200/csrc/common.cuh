@@ -76,7 +76,11 @@ constexpr int64_t SPARSE_TESTS = SPARSE_TESTS_OPT;  // ... when stars x tiles (t
 constexpr double LITE_AUTO_PER_TILE = 16.0;  // k_tile_lite is launched when the expected list per tile is <= this
 constexpr int64_t LITE_AUTO_TILES = 1024;    // ... and the frame / band has at least this many tiles
 constexpr int SPLIT_LEN = 1024;        // a tile list longer than this is split into parts of <= SPLIT_LEN stars
-constexpr int PART_CAP = 512;          // partial-tile buffers (128 x 64 fp32 each, 16 MB) available per render
+constexpr int PART_CAP = 2048;         // partial-tile buffers (128 x 64 fp32 each, 64 MB) available per render
+#ifndef WIDE_SPLIT_OPT
+#define WIDE_SPLIT_OPT 256
+#endif
+constexpr int WIDE_SPLIT = WIDE_SPLIT_OPT;  // the part / segment length for the wide-ROI kernels (FrameParams::split)
 
 // Star record written by k_prep, read by k_scatter and k_tile: {x, y, s', lo_x | lo_y << 16}.
 // s' = A * 2.512^-m / (2 pi sigma^2), evaluated in fp64 and rounded once to fp32.
@@ -106,6 +110,7 @@ struct FrameParams {
   int32_t ndst;          // > 0: the tile kernels store every pixel into dst[0..ndst) instead of `out` (fused band exchange)
   float* dst[MAX_DST];   // band origins (row0 of each destination frame) -- local and peer-mapped frames
   const uint32_t* n_dev; // starsim_set_star_count: the star count in device memory (n is then the capacity), or NULL
+  int32_t split;         // part / segment length of long tile lists: SPLIT_LEN, or WIDE_SPLIT for k_tile_wide's ROIs
   float sk;              // sqrt(log2(e) / (2 sigma^2)):  exp(-d^2/(2 sigma^2)) = ex2(-(d * sk)^2)
   float kint;            // 1 / (sqrt(2) sigma): the erf argument scale of the integrated PSF
   double s_scale;        // A / (2 pi sigma^2), applied in fp64 before rounding s' to fp32

@@ -203,7 +203,9 @@ template <bool SMEM_CNT = false>  // counts in shared memory (k_dsmall) instead 
 __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restrict__ cnt, int ntiles, int nCTA,
                                               uint32_t* __restrict__ tile_off, Header* hdr,
                                               WorkItem* __restrict__ items, uint2* __restrict__ split_tab,
-                                              int part_cap, uint32_t* __restrict__ done) {
+                                              int plan, uint32_t* __restrict__ done) {
+  const int part_cap = plan_cap(plan);
+  const uint32_t split = plan_split(plan);
   constexpr int TPT = DB_MAXT / DP_THREADS;
   static_assert(TPT * DP_THREADS == DB_MAXT, "tiles per thread");
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, cta = blockIdx.x;
@@ -213,7 +215,7 @@ __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restr
   for (int k = 0; k < TPT; ++k) {
     const int t = tid * TPT + k;
     c[k] = t < ntiles ? (SMEM_CNT ? cnt[t] : __ldcg(&cnt[t])) : 0u;  // dense totals (k_dcolscan, cstride 1)
-    if (t < ntiles) sum = add4(sum, tile_counts(c[k]));
+    if (t < ntiles) sum = add4(sum, tile_counts(c[k], split));
   }
   const uint4 incl = warp_incl_scan4(sum, lane);
   if (lane == 31) S.s_w4[warp] = incl;
@@ -240,9 +242,9 @@ __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restr
     if (t >= ntiles) break;
     S.toff[t] = run;
     if (t % nCTA == cta) {
-      plan_tile((uint32_t)t, c[k], run, pb, si, li, nparts, lite0, split_on, tile_off, items, split_tab, done);
+      plan_tile((uint32_t)t, c[k], run, pb, si, li, nparts, lite0, split_on, tile_off, items, split_tab, done, split);
     } else {  // the same prefix updates as plan_tile
-      const uint4 u = tile_counts(c[k]);
+      const uint4 u = tile_counts(c[k], split);
       run += u.x;
       pb += split_on ? u.y : 0u;
       si += split_on ? u.z : 0u;

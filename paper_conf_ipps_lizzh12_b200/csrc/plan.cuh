@@ -8,9 +8,14 @@
 
 namespace starsim {
 
-__device__ __forceinline__ uint32_t parts_of(uint32_t len) {
-  if (len <= (uint32_t)SPLIT_LEN) return 0u;
-  return min((len + SPLIT_LEN - 1) / SPLIT_LEN, 4095u);
+// The planner's argument word: the partial-buffer pool size | the part length (FrameParams::split) << 16.
+__host__ __device__ __forceinline__ int plan_word(int part_cap, int split) { return part_cap | split << 16; }
+__device__ __forceinline__ int plan_cap(int plan) { return plan & 0xFFFF; }
+__device__ __forceinline__ uint32_t plan_split(int plan) { return (uint32_t)plan >> 16; }
+
+__device__ __forceinline__ uint32_t parts_of(uint32_t len, uint32_t split) {
+  if (len <= split) return 0u;
+  return min((len + split - 1) / split, 4095u);
 }
 
 // Per-tile planning counts, scanned over the tiles: (pairs, parts, split tiles, light tiles).
@@ -20,8 +25,8 @@ __device__ __forceinline__ uint4 add4(uint4 a, uint4 b) {
 __device__ __forceinline__ uint4 sub4(uint4 a, uint4 b) {
   return make_uint4(a.x - b.x, a.y - b.y, a.z - b.z, a.w - b.w);
 }
-__device__ __forceinline__ uint4 tile_counts(uint32_t c) {
-  const uint32_t np = parts_of(c);
+__device__ __forceinline__ uint4 tile_counts(uint32_t c, uint32_t split) {
+  const uint32_t np = parts_of(c, split);
   return make_uint4(c, np, np ? 1u : 0u, c <= (uint32_t)LITE_MAX ? 1u : 0u);
 }
 
@@ -56,16 +61,17 @@ __device__ __forceinline__ void plan_header(Header* hdr, uint32_t* __restrict__ 
 __device__ __forceinline__ void plan_tile(uint32_t t, uint32_t c, uint32_t& run, uint32_t& pb, uint32_t& si,
                                           uint32_t& li, uint32_t nparts, uint32_t lite0, bool split_on,
                                           uint32_t* __restrict__ tile_off, WorkItem* __restrict__ items,
-                                          uint2* __restrict__ split_tab, uint32_t* __restrict__ done) {
+                                          uint2* __restrict__ split_tab, uint32_t* __restrict__ done,
+                                          uint32_t split) {
   tile_off[t] = run;
-  const uint32_t np = split_on ? parts_of(c) : 0u;
+  const uint32_t np = split_on ? parts_of(c, split) : 0u;
   if (np) {
     split_tab[si] = make_uint2(pb, np);
     done[si] = 0u;  // the parts' completion counter (k_tile)
-    // parts start at multiples of SPLIT_LEN from the list start: the same boundaries at which a tile kernel that
+    // parts start at multiples of split from the list start: the same boundaries at which a tile kernel that
     // processes the whole (unsplit) list cuts it into segments, so split and unsplit give the same sums
     for (uint32_t j = 0; j < np; ++j)
-      items[pb + j] = WorkItem{t, run + j * SPLIT_LEN, min(run + c, run + (j + 1) * SPLIT_LEN), (si << 12) | j};
+      items[pb + j] = WorkItem{t, run + j * split, min(run + c, run + (j + 1) * split), (si << 12) | j};
     pb += np;
     ++si;
   } else if (c <= (uint32_t)LITE_MAX) {

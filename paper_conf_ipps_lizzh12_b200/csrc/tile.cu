@@ -133,7 +133,7 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? 2 : TILE_MINB_OPT) k_tile
   for (uint32_t base = wi.jb; base < j1;) {
     // ======================= prep: thread = star (base + tid)
     // chunks never cross a SPLIT_LEN segment boundary of the list (segments are summed like the parts of a split tile)
-    const uint32_t seg_end = min(j1, wi.jb + ((base - wi.jb) / SPLIT_LEN + 1u) * SPLIT_LEN);
+    const uint32_t seg_end = min(j1, wi.jb + ((base - wi.jb) / (uint32_t)fp.split + 1u) * (uint32_t)fp.split);
     const int nvalid = (int)min((uint32_t)CHUNK, seg_end - base);
     const bool valid = tid < nvalid;
     StarRec r = {};
@@ -400,7 +400,7 @@ __global__ void __launch_bounds__(TILE_THREADS, CIRC ? 2 : TILE_MINB_OPT) k_tile
       }
     }
     base += (uint32_t)ns;
-    if (base < j1 && (base - wi.jb) % SPLIT_LEN == 0) {
+    if (base < j1 && (base - wi.jb) % (uint32_t)fp.split == 0) {
       seg_flush(acc, seg_scratch, segs_done == 0);
       ++segs_done;
     }

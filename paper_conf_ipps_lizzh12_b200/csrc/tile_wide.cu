@@ -37,6 +37,7 @@
 #include "common.cuh"
 #include "launch.h"
 #include "tile_common.cuh"
+#include "tile_wide.cuh"
 
 namespace starsim {
 
@@ -45,24 +46,8 @@ namespace {
 constexpr int WD_CHUNK = 128;                     // stars per chunk (two prep threads per star)
 constexpr int WD_MINB = 2;                        // CTAs per SM (128 registers, <= 112 KB shared memory)
 constexpr int WD_SW = 4;                          // warps that own a star in the sort (threads 0..127)
-static_assert(SPLIT_LEN % WD_CHUNK == 0, "segments are whole chunks");
+static_assert(SPLIT_LEN % WD_CHUNK == 0 && WIDE_SPLIT % WD_CHUNK == 0, "segments are whole chunks");
 static_assert(WD_CHUNK * 2 == TILE_THREADS, "two prep threads per star");
-
-template <int KB>
-struct WideGeom {
-  static constexpr int KS = 2 * KB - 1;           // strips an ROI of side <= MAXR spans
-  static constexpr int RS = KS <= 8 ? 8 : 16;     // strip ring
-  static constexpr int SYF = (KB | 1) * 16;       // floats per star: row profile (an odd number of 64-B slots)
-  static constexpr int SXF = RS * 8;              // floats per star: column profile ring
-  static constexpr int MAXR = 16 * (KB - 1) + 1;  // widest ROI side
-  // corner bins of the UNCLIPPED ROI origin (ly, lx), tile-relative: band key (ly >> 4) + KB - 1 (ly >= -(R - 1)),
-  // strip key (lx >> 3) + KS - 1, band-major
-  static constexpr int NBK = NBANDS + KB - 1;
-  static constexpr int NSK = NSTRIPS + KS - 1;
-  static constexpr int NBIN = NBK * NSK;          // 120 / 154 / 192
-  static constexpr int PER = NBIN / 32 + 1;       // bins per lane of the scanning warp (32 PER > NBIN: one lane
-                                                  // writes the total at bin NBIN)
-};
 
 template <int KB>
 struct WideSmem {
@@ -87,14 +72,12 @@ __global__ void __launch_bounds__(TILE_THREADS, WD_MINB) k_tile_wide(const uint3
                                                                      uint32_t* __restrict__ done, Header* hdr,
                                                                      float* __restrict__ seg_scratch) {
   using G = WideGeom<KB>;
-  constexpr uint32_t SYB = G::SYF * 4u, SXB = G::SXF * 4u;  // slot strides in bytes
   extern __shared__ __align__(16) unsigned char smem_raw[];
   WideSmem<KB>& S = *reinterpret_cast<WideSmem<KB>*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int sid = tid & (WD_CHUNK - 1);   // the chunk star this thread sorts and prepares
   const bool colhalf = tid >= WD_CHUNK;   // prep: false = row profile, true = column profile
   const uint32_t lt = (1u << lane) - 1u;
-  const float sk = fp.sk;
 
   const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
   const int Q = 8 * wx + q;
@@ -142,18 +125,10 @@ __global__ void __launch_bounds__(TILE_THREADS, WD_MINB) k_tile_wide(const uint3
         c1 = min(lx + fp.R - 1, TWe - 1);
         r0 = max(ly, 0);
         r1 = min(ly + fp.R - 1, THe - 1);
-        if (c0 <= c1 && r0 <= r1) key = (uint32_t)(((ly >> 4) + KB - 1) * G::NSK + (lx >> 3) + G::KS - 1);
+        key = wide_key<KB>(lx, ly, c0, c1, r0, r1);
       }
       // warps w and w + 4 hold the same stars in the same lanes: the same peers and ranks
-      // (the stars of the warp with the same key from 8 ballots: MATCH.ANY loops over the warp's distinct keys)
-      static_assert(G::NBIN < 256, "bin keys (and the no-bin key) fit 8 bits");
-      uint32_t peers = 0xffffffffu;
-#pragma unroll
-      for (int b = 0; b < 8; ++b) {
-        const uint32_t kb = (key >> b) & 1u;
-        const uint32_t m = __ballot_sync(0xffffffffu, kb);
-        peers &= kb ? m : ~m;
-      }
+      const uint32_t peers = key_peers(key);
       const uint32_t rank = __popc(peers & lt);
       if (warp < WD_SW) {
         // (the previous chunk's readers of hist -- warp 0's scan -- finished before its second barrier)
@@ -166,124 +141,18 @@ __global__ void __launch_bounds__(TILE_THREADS, WD_MINB) k_tile_wide(const uint3
       const uint32_t nb = base + WD_CHUNK;
       const uint32_t nid = nb + sid < j1 ? __ldg(&ids[nb + sid]) : 0u;
       __syncthreads();
-      if (warp == 0) {
-        uint32_t tot[G::PER], sum = 0;
-#pragma unroll
-        for (int h = 0; h < G::PER; ++h) {
-          const int bin = G::PER * lane + h;
-          uint32_t c[WD_SW];
-#pragma unroll
-          for (int w = 0; w < WD_SW; ++w) c[w] = bin < G::NBIN ? S.hist[w][bin] : 0u;
-          uint32_t run = 0;
-#pragma unroll
-          for (int w = 0; w < WD_SW; ++w) {
-            if (bin < G::NBIN) S.hist[w][bin] = run;
-            run += c[w];
-          }
-          tot[h] = run;
-          sum += run;
-        }
-        uint32_t incl = sum;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
-          if (lane >= o) incl += v;
-        }
-        uint32_t ex = incl - sum;
-#pragma unroll
-        for (int h = 0; h < G::PER; ++h) {
-          const int bin = G::PER * lane + h;
-          if (bin <= G::NBIN) S.binstart[bin] = ex;  // bin NBIN receives the total
-          ex += tot[h];
-        }
-      }
+      if (warp == 0) wide_scan<KB, WD_SW>(S.hist, S.binstart, lane);
       __syncthreads();
       // ======================= prep: the star's profiles at its sorted place j
       if (key < G::NBIN) {
         const uint32_t j = S.binstart[key] + S.hist[warp & (WD_SW - 1)][key] + rank;
-        const float2 sk2 = make_float2(sk, sk);
         // the unclipped ROI origin's band and strip (bands b0 .. b0 + KB - 1, strips q0 .. q0 + KS - 1 hold it)
         const int b0 = (int)(key / G::NSK) - (KB - 1), q0 = (int)(key % G::NSK) - (G::KS - 1);
         if (!colhalf) {
           if (CIRC) S.lo2[j] = lo2;
-          const float yr = r.y - (float)IY0;  // exact
-          const float2 s2 = make_float2(r.s, r.s);
-#pragma unroll
-          for (int k = 0; k < KB; ++k) {
-            const int bb = b0 + k;
-            if (bb < 0 || bb >= NBANDS) continue;  // never read
-            const int ra = r0 - 16 * bb, rb = r1 - 16 * bb;
-            const uint32_t m16 = (ra > 15 || rb < 0) ? 0u
-                                                     : (0xFFFFu >> (15 - min(rb, 15))) & (0xFFFFu << max(ra, 0)) & 0xFFFFu;
-            float4* dst = reinterpret_cast<float4*>(&S.gy[j * G::SYF + 16 * k]);
-#pragma unroll
-            for (int c = 0; c < 4; ++c) {
-              const int w = (c + lane) & 3;  // lane-rotated quad order (spreads the stores over the banks)
-              const uint32_t m = (m16 >> (4 * w)) & 0xFu;
-              float v[4] = {0.f, 0.f, 0.f, 0.f};
-              if (m) {
-                const float bf = (float)(16 * bb + 4 * w) - yr;  // exact
-                if (!INTEG) {
-                  const float2 bbv = make_float2(bf, bf);
-#pragma unroll
-                  for (int i = 0; i < 4; i += 2) {
-                    float2 d = __fadd2_rn(bbv, make_float2((float)i, (float)(i + 1)));
-                    d = __fmul2_rn(d, sk2);
-                    d = __fmul2_rn(d, make_float2(-d.x, -d.y));
-                    const float2 e = __fmul2_rn(make_float2(ex2_approx(d.x), ex2_approx(d.y)), s2);
-                    v[i] = (m >> i) & 1u ? e.x : 0.f;
-                    v[i + 1] = (m >> (i + 1)) & 1u ? e.y : 0.f;
-                  }
-                } else {
-                  float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
-#pragma unroll
-                  for (int i = 0; i < 4; ++i) {
-                    const float tn = (bf + (float)i + 0.5f) * fp.kint, en = edge_erfc(tn);
-                    v[i] = (m >> i) & 1u ? r.s * pix_mass(t, e, tn, en) : 0.f;
-                    t = tn;
-                    e = en;
-                  }
-                }
-              }
-              dst[w] = make_float4(v[0], v[1], v[2], v[3]);
-            }
-          }
+          wide_rows<KB, INTEG>(&S.gy[j * G::SYF], b0, r0, r1, r.y - (float)IY0, r.s, fp, lane);
         } else {
-          const float xr = r.x - (float)X0;  // exact
-#pragma unroll
-          for (int k = 0; k < G::KS; ++k) {
-            const int Qs = q0 + k;
-            if (Qs < 0 || Qs >= NSTRIPS) continue;  // never read
-            const int rel = 8 * Qs;
-            const int lo = max(c0 - rel, 0), hi = min(c1 - rel, 7);
-            const uint32_t m = hi >= lo ? ((0xFFu >> (7 - hi)) & (0xFFu << lo)) : 0u;
-            float v[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
-            if (m) {
-              const float bf = (float)rel - xr;  // exact
-              if (!INTEG) {
-#pragma unroll
-                for (int p = 0; p < 8; p += 2) {
-                  float2 d = __fmul2_rn(__fadd2_rn(make_float2(bf, bf), make_float2((float)p, (float)(p + 1))), sk2);
-                  d = __fmul2_rn(d, make_float2(-d.x, -d.y));
-                  v[p] = (m >> p) & 1u ? ex2_approx(d.x) : 0.f;
-                  v[p + 1] = (m >> (p + 1)) & 1u ? ex2_approx(d.y) : 0.f;
-                }
-              } else {
-                float t = (bf - 0.5f) * fp.kint, e = edge_erfc(t);
-#pragma unroll
-                for (int p = 0; p < 8; ++p) {
-                  const float tn = (bf + (float)p + 0.5f) * fp.kint, en = edge_erfc(tn);
-                  v[p] = (m >> p) & 1u ? pix_mass(t, e, tn, en) : 0.f;
-                  t = tn;
-                  e = en;
-                }
-              }
-            }
-            float* gs = &S.gx[j * G::SXF + (Qs & (G::RS - 1)) * 8];
-            const int sw = ((Qs >> 2) & 1) * 4;
-            *reinterpret_cast<float4*>(gs + sw) = make_float4(v[0], v[1], v[2], v[3]);
-            *reinterpret_cast<float4*>(gs + (sw ^ 4)) = make_float4(v[4], v[5], v[6], v[7]);
-          }
+          wide_cols<KB, INTEG>(&S.gx[j * G::SXF], q0, c0, c1, r.x - (float)X0, fp);
         }
       }
       const bool first = base == wi.jb, last = nb >= j1;
@@ -300,66 +169,9 @@ __global__ void __launch_bounds__(TILE_THREADS, WD_MINB) k_tile_wide(const uint3
       } else if (item_n < nitems && wn.jb + sid < wn.je) {
         nid0 = __ldg(&ids[wn.jb + sid]);
       }
-      // ======================= accumulate: lane group q walks its KB ranges (each padded with the zero slot)
-#pragma unroll 1
-      for (int k = 0; k < KB; ++k) {
-        // corner band B - k (band key B - k + KB - 1), corner strips Q - KS + 1 .. Q (strip keys Q .. Q + KS - 1)
-        const int bk = B - k + KB - 1;
-        const uint32_t s = S.binstart[bk * G::NSK + Q], e = S.binstart[bk * G::NSK + Q + G::KS];
-        const uint32_t len = e - s;
-        // sorted star j = s + t, band slot k; each lane group runs its own trip count (the warp's longest: the
-        // other groups' lanes idle), no padding reads
-        uint32_t ga = gy_base + s * SYB + 64u * (uint32_t)k, xa = gx_base + s * SXB;
-        uint32_t jj = s;
-        const uint32_t gend = ga + len * SYB;
-        // one step of look-ahead: the next star's operands are loaded before this one's FMAs (past the range end the
-        // loads read other shared-memory words, never used)
-        float4 gn, an, cn;
-        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(gn.x), "=f"(gn.y), "=f"(gn.z), "=f"(gn.w) : "r"(ga));
-        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(an.x), "=f"(an.y), "=f"(an.z), "=f"(an.w) : "r"(xa));
-        asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(cn.x), "=f"(cn.y), "=f"(cn.z), "=f"(cn.w) : "r"(xa + 16u));
-#pragma unroll 2
-        for (; ga < gend; ga += SYB, xa += SXB) {
-          const float4 g = gn, a = an, c = cn;
-          asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(gn.x), "=f"(gn.y), "=f"(gn.z), "=f"(gn.w) : "r"(ga + SYB));
-          asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(an.x), "=f"(an.y), "=f"(an.z), "=f"(an.w) : "r"(xa + SXB));
-          asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(cn.x), "=f"(cn.y), "=f"(cn.z), "=f"(cn.w) : "r"(xa + SXB + 16u));
-          const float gi[4] = {g.x, g.y, g.z, g.w};
-          if (!CIRC) {
-#pragma unroll
-            for (int i = 0; i < 4; ++i) {
-              const float2 gg = make_float2(gi[i], gi[i]);
-              acc[i][0] = __ffma2_rn(gg, make_float2(a.x, a.y), acc[i][0]);
-              acc[i][1] = __ffma2_rn(gg, make_float2(a.z, a.w), acc[i][1]);
-              acc[i][2] = __ffma2_rn(gg, make_float2(c.x, c.y), acc[i][2]);
-              acc[i][3] = __ffma2_rn(gg, make_float2(c.z, c.w), acc[i][3]);
-            }
-          } else {
-            // reading R21: the star's ROI origin from its slot, the per-pixel integer disc test (as k_tile_sb)
-            const uint32_t lo = S.lo2[jj++];
-            const int lx = (int)(int16_t)(lo & 0xFFFFu), ly = (int)(int16_t)(lo >> 16);
-            const float gx[8] = {a.x, a.y, a.z, a.w, c.x, c.y, c.z, c.w};  // columns 8 Q + ((p + 4 swz) & 7)
-            const int RR = fp.R * fp.R, R1 = fp.R - 1;
-#pragma unroll
-            for (int i = 0; i < 4; ++i) {
-              const int v = 2 * (16 * B + 4 * hq + i - ly) - R1;
-              const int thr = RR - v * v;
-              float gm[8];
-#pragma unroll
-              for (int p = 0; p < 8; ++p) {
-                const int u = 2 * (8 * Q + ((p + 4 * swz) & 7) - lx) - R1;
-                gm[p] = u * u <= thr ? gx[p] : 0.f;
-              }
-              const float2 gg = make_float2(gi[i], gi[i]);
-              acc[i][0] = __ffma2_rn(gg, make_float2(gm[0], gm[1]), acc[i][0]);
-              acc[i][1] = __ffma2_rn(gg, make_float2(gm[2], gm[3]), acc[i][1]);
-              acc[i][2] = __ffma2_rn(gg, make_float2(gm[4], gm[5]), acc[i][2]);
-              acc[i][3] = __ffma2_rn(gg, make_float2(gm[6], gm[7]), acc[i][3]);
-            }
-          }
-        }
-      }
-      if ((base + WD_CHUNK - wi.jb) % SPLIT_LEN == 0 && base + WD_CHUNK < j1) {
+      // ======================= accumulate: lane group q walks its KB ranges
+      wide_walk<KB, CIRC>(acc, S.binstart, gy_base, gx_base, S.lo2, B, Q, hq, swz, fp);
+      if ((base + WD_CHUNK - wi.jb) % (uint32_t)fp.split == 0 && base + WD_CHUNK < j1) {
         seg_flush(acc, seg_scratch, segs_done == 0);
         ++segs_done;
       }
@@ -396,6 +208,225 @@ __global__ void __launch_bounds__(TILE_THREADS, WD_MINB) k_tile_wide(const uint3
   }  // work loop
 }
 
+// ---------------------------------------------------------------------------------------------------------------
+// k_tile_wws: the same chunks, slots, ranges and per-pixel order as k_tile_wide (the two give bitwise-identical
+// images), warp-specialised as k_tile_ws is for R <= 17: 4 producer warps (one star per thread) sort each chunk and
+// write its profiles into stage s of an NS-deep ring, then arrive on full[s]; 8 consumer warps (the accumulators,
+// threads 0..255) wait on full[s], walk, arrive on empty[s] and write the tile after an item's last chunk.  At wide R
+// the walk dominates: the producers' sort, scan and profiles overlap it instead of sitting between CTA barriers, and
+// a consumer warp waits only for the producers or, NS - 1 chunks ahead, for the slowest consumer.  One CTA per SM,
+// work items in static round-robin order (parts of heavy tiles first).
+// ---------------------------------------------------------------------------------------------------------------
+namespace {
+constexpr int WW_CHUNK = 128;
+constexpr int WW_PROD = 4, WW_CONS = 8;
+constexpr int WW_THREADS = 32 * (WW_PROD + WW_CONS);
+constexpr uint32_t WW_LAST = 1u, WW_STOP = 2u, WW_SEGEND = 4u;
+static_assert(WW_CHUNK == 32 * WW_PROD && SPLIT_LEN % WW_CHUNK == 0, "one producer thread per star, whole segments");
+
+template <int KB>
+struct WwStage {
+  float gy[WW_CHUNK * WideGeom<KB>::SYF];
+  float gx[WW_CHUNK * WideGeom<KB>::SXF];
+  uint32_t binstart[(WideGeom<KB>::PER * 32 + 4) & ~3];
+  uint32_t lo2[WW_CHUNK];
+  uint32_t tile, aux, flags, pad;
+};
+template <int KB>
+__host__ __device__ constexpr int ww_ns() {
+  return 3 * sizeof(WwStage<KB>) + sizeof(uint32_t) * WW_PROD * WideGeom<KB>::NBIN + 128 <= 227 * 1024 ? 3 : 2;
+}
+template <int KB>
+struct WwSmem {
+  unsigned long long full[4], empty[4];
+  WwStage<KB> st[ww_ns<KB>()];
+  uint32_t hist[WW_PROD][WideGeom<KB>::NBIN];
+  int s_last;
+};
+static_assert(sizeof(WwSmem<5>) <= 227 * 1024 && sizeof(WwSmem<4>) <= 227 * 1024, "one CTA per SM fits");
+
+__device__ __forceinline__ uint32_t ww_smem(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void ww_mbar_init(unsigned long long* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(ww_smem(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void ww_arrive(unsigned long long* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(ww_smem(b)) : "memory");
+}
+__device__ __forceinline__ void ww_wait(unsigned long long* b, uint32_t parity) {
+  const uint32_t a = ww_smem(b);
+  uint32_t ok;
+  do {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(ok)
+        : "r"(a), "r"(parity)
+        : "memory");
+  } while (!ok);
+}
+__device__ __forceinline__ void ww_prod_barrier() { asm volatile("bar.sync 1, %0;" ::"n"(32 * WW_PROD) : "memory"); }
+}  // namespace
+
+template <int KB, bool INTEG, bool CIRC>
+__device__ __forceinline__ void wws_producer(WwSmem<KB>& S, const uint32_t* __restrict__ ids,
+                                             const StarRec* __restrict__ rec, const FrameParams& fp,
+                                             const WorkItem* __restrict__ items, uint32_t nitems) {
+  using G = WideGeom<KB>;
+  constexpr int NS = ww_ns<KB>();
+  const int pt = threadIdx.x - 32 * WW_CONS, lane = pt & 31, pw = pt >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  const uint32_t GS = gridDim.x;
+  const WorkItem none = {0u, 0u, 0u, 0u};
+  uint32_t it = blockIdx.x, c = 0;
+  WorkItem wi = it < nitems ? items[it] : none;
+  StarRec rcur = {};
+  if (wi.jb + (uint32_t)pt < wi.je) rcur = rec[__ldg(&ids[wi.jb + pt])];
+  while (it < nitems) {
+    const uint32_t nch = wi.je > wi.jb ? (wi.je - wi.jb + WW_CHUNK - 1) / WW_CHUNK : 1u;  // an empty item: 1 chunk
+    const bool more = it + GS < nitems;
+    const WorkItem wn = more ? items[it + GS] : none;
+    const int tx = (int)(wi.tile % (uint32_t)fp.ntx), ty = (int)(wi.tile / (uint32_t)fp.ntx);
+    const int X0 = tx * TILE_W, Y0 = ty * TILE_H, IY0 = fp.row0 + Y0;
+    const int TWe = min(TILE_W, fp.W - X0), THe = min(TILE_H, fp.rows - Y0);
+    for (uint32_t k = 0; k < nch; ++k, ++c) {
+      const uint32_t s = c % NS, ph = (c / NS) & 1u;
+      WwStage<KB>& T = S.st[s];
+      const uint32_t base = wi.jb + k * WW_CHUNK;
+      const StarRec r = rcur;
+      const bool valid = base + (uint32_t)pt < wi.je;
+      {  // the next chunk's record (this item's or the next item's first), one chunk ahead
+        const uint32_t nb = k + 1 < nch ? base + WW_CHUNK : wn.jb, ne = k + 1 < nch ? wi.je : wn.je;
+        rcur = StarRec{};
+        if (nb + (uint32_t)pt < ne) rcur = rec[__ldg(&ids[nb + pt])];
+      }
+      int c0 = 0, c1 = -1, r0 = 0, r1 = -1;
+      uint32_t key = G::NBIN, lo2 = 0u;
+      if (valid) {
+        const int lx = lo_x_of(r.lo) - X0, ly = lo_y_of(r.lo) - IY0;
+        lo2 = (uint32_t)(lx & 0xFFFF) | (uint32_t)ly << 16;
+        c0 = max(lx, 0);
+        c1 = min(lx + fp.R - 1, TWe - 1);
+        r0 = max(ly, 0);
+        r1 = min(ly + fp.R - 1, THe - 1);
+        key = wide_key<KB>(lx, ly, c0, c1, r0, r1);
+      }
+      const uint32_t peers = key_peers(key);
+      const uint32_t rank = __popc(peers & lt);
+      // (hist[pw] was last read by this warp's prep and by producer warp 0's scan, before the last producer barrier)
+#pragma unroll
+      for (int h = 0; h < G::PER; ++h)
+        if (lane + 32 * h < G::NBIN) S.hist[pw][lane + 32 * h] = 0u;
+      __syncwarp();
+      if (rank == 0 && key < G::NBIN) S.hist[pw][key] = __popc(peers);
+      ww_prod_barrier();
+      // stage s is free once every consumer thread has walked the chunk it held NS chunks ago
+      ww_wait(&S.empty[s], ph ^ 1u);
+      if (pw == 0) wide_scan<KB, WW_PROD>(S.hist, T.binstart, lane);
+      ww_prod_barrier();
+      if (key < G::NBIN) {
+        const uint32_t j = T.binstart[key] + S.hist[pw][key] + rank;
+        const int b0 = (int)(key / G::NSK) - (KB - 1), q0 = (int)(key % G::NSK) - (G::KS - 1);
+        if (CIRC) T.lo2[j] = lo2;
+        wide_rows<KB, INTEG>(&T.gy[j * G::SYF], b0, r0, r1, r.y - (float)IY0, r.s, fp, lane);
+        wide_cols<KB, INTEG>(&T.gx[j * G::SXF], q0, c0, c1, r.x - (float)X0, fp);
+      }
+      if (pt == 0) {
+        T.tile = wi.tile;
+        T.aux = wi.aux;
+        T.flags = k + 1 == nch ? WW_LAST : (((k + 1) % ((uint32_t)fp.split / WW_CHUNK)) == 0 ? WW_SEGEND : 0u);
+      }
+      ww_arrive(&S.full[s]);
+    }
+    it += GS;
+    wi = wn;
+  }
+  const uint32_t s = c % NS;  // the stop chunk releases the consumers
+  ww_wait(&S.empty[s], ((c / NS) & 1u) ^ 1u);
+  if (pt == 0) S.st[s].flags = WW_STOP;
+  ww_arrive(&S.full[s]);
+}
+
+template <int KB, bool CIRC>
+__device__ __forceinline__ void wws_consumer(WwSmem<KB>& S, const FrameParams& fp, void* __restrict__ out_,
+                                             const uint2* __restrict__ split_tab, float* __restrict__ part_buf,
+                                             uint32_t* __restrict__ done, float* __restrict__ seg_scratch) {
+  using G = WideGeom<KB>;
+  constexpr int NS = ww_ns<KB>();
+  constexpr uint32_t STB = sizeof(WwStage<KB>);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int q = lane >> 2, hq = lane & 3, wx = warp & 1, B = warp >> 1;
+  const int Q = 8 * wx + q;
+  const int swz = (Q >> 2) & 1;
+  const uint32_t gy_base0 = ww_smem(S.st[0].gy) + 16u * hq;
+  const uint32_t gx_base0 = ww_smem(S.st[0].gx) + 32u * (uint32_t)(Q & (G::RS - 1));
+  uint32_t segs_done = 0;
+  float2 acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
+  for (uint32_t c = 0;; ++c) {
+    const uint32_t s = c % NS, ph = (c / NS) & 1u;
+    const WwStage<KB>& T = S.st[s];
+    ww_wait(&S.full[s], ph);
+    const uint32_t flags = T.flags;
+    if (flags & WW_STOP) break;
+    const uint32_t tile = T.tile, aux = T.aux;
+    wide_walk<KB, CIRC>(acc, T.binstart, gy_base0 + s * STB, gx_base0 + s * STB, T.lo2, B, Q, hq, swz, fp);
+    ww_arrive(&S.empty[s]);
+    if (flags & WW_SEGEND) {
+      seg_flush(acc, seg_scratch, segs_done == 0);
+      ++segs_done;
+      continue;
+    }
+    if (!(flags & WW_LAST)) continue;
+    if (segs_done) {
+      seg_finish(acc, seg_scratch);
+      segs_done = 0;
+    }
+    if (swz) {
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const float2 t0 = acc[i][0], t1 = acc[i][1];
+        acc[i][0] = acc[i][2];
+        acc[i][1] = acc[i][3];
+        acc[i][2] = t0;
+        acc[i][3] = t1;
+      }
+    }
+    const WorkItem wi = {tile, 0u, 0u, aux};
+    const int tx = (int)(tile % (uint32_t)fp.ntx), ty = (int)(tile / (uint32_t)fp.ntx);
+    if (tile_reduce_parts<true, 32 * WW_CONS>(acc, wi, split_tab, part_buf, done, B, wx, q, hq, &S.s_last))
+      tile_store<true>(acc, fp, out_, ty * TILE_H, tx * TILE_W + 64 * wx + 8 * q, B, hq);
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int k = 0; k < 4; ++k) acc[i][k] = make_float2(0.f, 0.f);
+  }
+}
+
+template <int KB, bool INTEG, bool CIRC>
+__global__ void __launch_bounds__(WW_THREADS, 1) k_tile_wws(const uint32_t* __restrict__ ids,
+                                                            const StarRec* __restrict__ rec, FrameParams fp,
+                                                            void* __restrict__ out_, const WorkItem* __restrict__ items,
+                                                            const uint2* __restrict__ split_tab,
+                                                            float* __restrict__ part_buf, uint32_t* __restrict__ done,
+                                                            Header* hdr, float* __restrict__ seg_scratch) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  WwSmem<KB>& S = *reinterpret_cast<WwSmem<KB>*>(smem_raw);
+  const int tid = threadIdx.x;
+  if (tid < ww_ns<KB>()) {
+    ww_mbar_init(&S.full[tid], 32 * WW_PROD);  // every producer thread arrives once per chunk
+    ww_mbar_init(&S.empty[tid], 32 * WW_CONS);  // every consumer thread arrives once per chunk
+  }
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  __syncthreads();
+  const uint32_t nitems = __ldcg(&hdr->nitems);
+  if (tid >= 32 * WW_CONS)
+    wws_producer<KB, INTEG, CIRC>(S, ids, rec, fp, items, nitems);
+  else
+    wws_consumer<KB, CIRC>(S, fp, out_, split_tab, part_buf, done, seg_scratch);
+}
+
 namespace {
 using KW = void (*)(const uint32_t*, const StarRec*, FrameParams, void*, const WorkItem*, const uint2*, float*,
                     uint32_t*, Header*, float*);
@@ -403,6 +434,8 @@ template <int KB>
 struct WideTab {
   static constexpr KW k[2][2] = {{k_tile_wide<KB, false, false>, k_tile_wide<KB, false, true>},
                                  {k_tile_wide<KB, true, false>, k_tile_wide<KB, true, true>}};
+  static constexpr KW w[2][2] = {{k_tile_wws<KB, false, false>, k_tile_wws<KB, false, true>},
+                                 {k_tile_wws<KB, true, false>, k_tile_wws<KB, true, true>}};
 };
 static_assert(WideGeom<5>::MAXR == WIDE_MAXR, "KB = 5 covers the widest ROI");
 static_assert(2 * (sizeof(WideSmem<5>) + 1024 + 64) <= 228 * 1024, "two CTAs per SM fit");
@@ -419,6 +452,9 @@ bool wide_ok(int R) { return R >= WIDE_MINR_OPT && R > SB_MAXR && R <= WIDE_MAXR
 void init_tile_wide_kernel() {
   for (int a = 0; a < 2; ++a)
     for (int b = 0; b < 2; ++b) {
+      cudaFuncSetAttribute(WideTab<3>::w[a][b], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WwSmem<3>));
+      cudaFuncSetAttribute(WideTab<4>::w[a][b], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WwSmem<4>));
+      cudaFuncSetAttribute(WideTab<5>::w[a][b], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WwSmem<5>));
       cudaFuncSetAttribute(WideTab<3>::k[a][b], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WideSmem<3>));
       cudaFuncSetAttribute(WideTab<4>::k[a][b], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WideSmem<4>));
       cudaFuncSetAttribute(WideTab<5>::k[a][b], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(WideSmem<5>));
@@ -430,8 +466,15 @@ void launch_tile_wide(const uint32_t* ids, const StarRec* rec, const FrameParams
                       cudaStream_t st, float* seg_scratch) {
   const int64_t ntiles = (int64_t)fp.ntx * fp.nty;
   if (ntiles <= 0) return;
-  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)WD_MINB * num_sms);  // persistent CTAs
   const int kb = wide_kb(fp.R), a = fp.psf ? 1 : 0, b = fp.roi ? 1 : 0;
+  if (fp.tile_impl != 2) {  // every mode but STARSIM_TILE_SB: the warp-specialised kernel, one CTA per SM
+    const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)num_sms);
+    const KW k = kb == 3 ? WideTab<3>::w[a][b] : kb == 4 ? WideTab<4>::w[a][b] : WideTab<5>::w[a][b];
+    const size_t smem = kb == 3 ? sizeof(WwSmem<3>) : kb == 4 ? sizeof(WwSmem<4>) : sizeof(WwSmem<5>);
+    k<<<(unsigned)grid, WW_THREADS, smem, st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr, seg_scratch);
+    return;
+  }
+  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)WD_MINB * num_sms);  // persistent CTAs
   const KW k = kb == 3 ? WideTab<3>::k[a][b] : kb == 4 ? WideTab<4>::k[a][b] : WideTab<5>::k[a][b];
   const size_t smem = kb == 3 ? sizeof(WideSmem<3>) : kb == 4 ? sizeof(WideSmem<4>) : sizeof(WideSmem<5>);
   k<<<(unsigned)grid, TILE_THREADS, smem, st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr, seg_scratch);

@@ -483,6 +483,30 @@ def test_wide_roi_kernel(torch_dev, R, psf):
     assert float(np.abs(out["auto"] - out["lists"]).max()) <= 1e-5 * peak
 
 
+@pytest.mark.parametrize("psf", ["point", "integrated"])
+@pytest.mark.parametrize("W,H,n,R,seed,kind", [(537, 411, 4000, 33, 5, "adv"), (1000, 700, 20000, 47, 6, "uniform"),
+                                               (512, 384, 9000, 63, 7, "dense")])
+def test_wide_ws_equals_sync_bitwise(torch_dev, psf, W, H, n, R, seed, kind):
+    """k_tile_wws (warp-specialised, mode ws) and k_tile_wide (both roles in every warp, modes auto / sb) sum every
+    pixel in the same order: bitwise-identical images, incl. heavy tiles split into parts."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context
+    if kind == "dense":
+        f = _dense_field(n, W, H, 200.0, 150.0, 40.0, seed=seed)
+    elif kind == "adv":
+        f = synth.adversarial_field(n, W, H, R, seed=seed)
+    else:
+        f = synth.uniform_field(n, W, H, seed=seed, mag_hi=2.0)
+    args = to_dev(torch_dev, f)
+    out = {}
+    for mode in ("ws", "sb"):
+        with Context(0) as c:
+            c.set_tile_kernel(mode)
+            c.set_psf(psf)
+            out[mode] = c.render(*args, W, H, R / 6.0, R, 1.0)
+    assert torch.equal(out["ws"], out["sb"])
+
+
 @pytest.mark.parametrize("R", [31, 63])
 def test_wide_roi_heavy_tiles(torch_dev, ctx, R):
     """Clustered wide-ROI field with tiles of > 4 x SPLIT_LEN stars (split into parts): parity, determinism, bands
@@ -865,15 +889,15 @@ def test_set_star_count_semantics_and_einval(torch_dev, ctx):
 
 
 def test_unsplit_huge_tile_lists(torch_dev, ctx):
-    """More heavy-tile parts than the partial-buffer pool holds (PART_CAP = 512): the frame's heavy tiles are not
+    """More heavy-tile parts than the partial-buffer pool holds (PART_CAP = 2048): the frame's heavy tiles are not
     split and a work item carries a whole tile list of ~10^5 stars.  Every tile kernel then sums it in SPLIT_LEN
     segments exactly as it would sum the parts (reading R19; the segment partials go through a per-CTA scratch tile),
-    so the north-star tolerance holds (~37,000 fp32 additions per pixel, 600K stars in 60 x 60 px, each sequential
+    so the north-star tolerance holds (~120,000 fp32 additions per pixel, 2M stars in 60 x 60 px, each sequential
     chain <= 1,024 stars long) and the result is bitwise the same whether or not the planner split the tile: the
     bands below have fewer heavy tiles each, so they are split, and still equal the frame bit for bit."""
     torch, dev = torch_dev
     W, H, R, sigma = 256, 256, 15, 2.5
-    f = _dense_field(600000, W, H, 130.0, 130.0, 60.0, seed=5)
+    f = _dense_field(2000000, W, H, 130.0, 130.0, 60.0, seed=5)
     args = to_dev(torch_dev, f)
     a = ctx.render(*args, W, H, sigma, R, 1.0)
     tw, th, off, ids = ctx.get_bins()
@@ -883,6 +907,32 @@ def test_unsplit_huge_tile_lists(torch_dev, ctx):
     assert torch.equal(a, ctx.render(*args, W, H, sigma, R, 1.0))
     bands = [ctx.render_band(*args, W, H, g * 64, 64, sigma, R, 1.0) for g in range(H // 64)]
     assert torch.equal(torch.cat(bands, 0), a)
+
+
+@pytest.mark.parametrize("R", [33, 63])
+def test_wide_unsplit_huge_tile_lists(torch_dev, R):
+    """Wide ROIs (parts and segments of WIDE_SPLIT = 256 stars) with more parts than the pool holds: the frame's tiles
+    are walked whole in 256-star segments, the bands are split into parts -- bitwise the same; the warp-specialised
+    and the synchronous kernels agree bitwise; parity against the oracle."""
+    torch, dev = torch_dev
+    from paper_conf_ipps_lizzh12_b200 import Context
+    W, H, sigma = 256, 256, R / 6.0
+    f = _dense_field(400000, W, H, 130.0, 130.0, 60.0, seed=6)
+    args = to_dev(torch_dev, f)
+    ref = oracle.render(f.x, f.y, f.mag, W, H, sigma, R, 1.0, threads=_threads())
+    out = {}
+    for mode in ("ws", "sb"):
+        with Context(0) as c:
+            c.set_tile_kernel(mode)
+            a = c.render(*args, W, H, sigma, R, 1.0)
+            if mode == "ws":
+                tw, th, off, ids = c.get_bins()
+                assert int(np.sum(np.ceil(np.diff(off) / 256.0))) > 2048  # the pool overflows: nothing split
+            assert_parity(a.cpu().numpy(), ref, f"wide unsplit R={R} {mode}")
+            bands = [c.render_band(*args, W, H, g * 64, 64, sigma, R, 1.0) for g in range(H // 64)]
+            assert torch.equal(torch.cat(bands, 0), a)
+            out[mode] = a
+    assert torch.equal(out["ws"], out["sb"])
 
 
 def test_circle_roi_with_integrated_psf(torch_dev, ctx):
