@@ -183,8 +183,11 @@ struct DpSmem {
   uint16_t arr[DP_KEYS];          // the CTA's star indices grouped by tile (in arbitrary order inside a group)
   uint32_t s_w[DP_WARPS + 1];
   uint32_t bmap[DP_WARPS][DB_CTA / 32];  // per warp: a large group's members as a bitmap of star indices
+  uint32_t nbig;                         // the tiles of the large groups
+  uint16_t big[DP_KEYS / 32];
 };
 constexpr uint32_t DP_BIG = 32;  // groups of more pairs are placed through a bitmap, not the rank loop
+static_assert(DP_KEYS / (DP_BIG + 1) < DP_KEYS / 32, "the large-group list holds every large group");
 
 // tiles of a packed box (0 if the star is culled) and its e-th tile, e < box_n (row-major order inside the box)
 __device__ __forceinline__ int box_n(uint32_t code) {
@@ -263,6 +266,7 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
   const int tid = threadIdx.x, cta = blockIdx.x;
   const int64_t c0 = (int64_t)cta * DB_CTA;
   for (int t = tid; t <= ntiles; t += DP_THREADS) S.gstart[t] = 0u;
+  if (tid == 0) S.nbig = 0u;
   __syncthreads();
   // group sizes
 #pragma unroll
@@ -289,6 +293,7 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
       if (t < ntiles) {
         S.gstart[t] = run;
         S.cur[t] = run;
+        if (c[k] > DP_BIG) S.big[atomicAdd(&S.nbig, 1u)] = (uint16_t)t;
       }
       run += c[k];
     }
@@ -326,9 +331,9 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
   // counts) -- the same ascending-index list
   const int lane = tid & 31, warp = tid >> 5;
   uint32_t* bm = S.bmap[warp];
-  for (int t = warp; t < ntiles; t += DP_WARPS) {
+  for (uint32_t b = (uint32_t)warp; b < S.nbig; b += DP_WARPS) {
+    const int t = S.big[b];
     const uint32_t g0 = S.gstart[t], g1 = S.gstart[t + 1];
-    if (g1 - g0 <= DP_BIG) continue;  // warp-uniform
     constexpr int WPL = DB_CTA / 32 / 32;  // bitmap words per lane
 #pragma unroll
     for (int w = 0; w < WPL; ++w) bm[lane * WPL + w] = 0u;
@@ -338,12 +343,9 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
       atomicOr(&bm[v >> 5], 1u << (v & 31u));
     }
     __syncwarp();
-    uint32_t wv[WPL], cntl = 0;
+    uint32_t cntl = 0;
 #pragma unroll
-    for (int w = 0; w < WPL; ++w) {
-      wv[w] = bm[lane * WPL + w];
-      cntl += __popc(wv[w]);
-    }
+    for (int w = 0; w < WPL; ++w) cntl += __popc(bm[lane * WPL + w]);
     uint32_t incl = cntl;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -351,9 +353,9 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
       if (lane >= o) incl += q;
     }
     uint32_t pos = S.cur[t] + incl - cntl;
-#pragma unroll
+#pragma unroll 1
     for (int w = 0; w < WPL; ++w) {
-      uint32_t m = wv[w];
+      uint32_t m = bm[lane * WPL + w];
       while (m) {
         const int b = __ffs(m) - 1;
         m &= m - 1u;
