@@ -96,52 +96,48 @@ __global__ void __launch_bounds__(DC_THREADS, DC_MINB_OPT) k_dcount(const float*
 }
 
 // C is CTA-major: C[cta][t] (row stride ntiles), so k_dcount's and k_dplace's accesses to their own CTA's row are
-// coalesced.  k_dcolscan takes DCS_TILES tiles per CTA: it stages DCS_ROWS rows of the block in shared memory
-// (coalesced 128-B row reads), scans every tile's column there (lane l holds rows l + 32 k; one warp scan per 32 rows,
-// carried), and writes the exclusive prefixes back in place (coalesced), then the tile totals.
+// coalesced.  k_dcolscan takes DCS_TILES tiles per CTA, one per warp: lane l sums rows 8 l .. 8 l + 7 of its tile's
+// column in registers, one warp scan of the lane sums per DCS_ROWS rows (carried), the exclusive prefixes written back
+// in place, then the tile totals (round 1's one-warp-scan-per-32-rows chain was latency-bound: 10 us at T).
 constexpr int DCS_TILES = 8;   // one tile per warp
 constexpr int DCS_ROWS = 256;
+constexpr int DCS_RPL = DCS_ROWS / 32;  // rows per lane
 __global__ void __launch_bounds__(DCS_THREADS) k_dcolscan(uint32_t* __restrict__ C, int nCTA_cap, int ntiles,
                                                          uint32_t* __restrict__ cnt, int cstride, int64_t n,
                                                          const uint32_t* __restrict__ n_dev) {
   static_assert(DCS_THREADS == 32 * DCS_TILES, "one warp per tile");
-  __shared__ uint32_t sm[DCS_ROWS][DCS_TILES + 1];
+  static_assert(DCS_ROWS == 32 * DCS_RPL, "a lane holds DCS_RPL consecutive rows");
+  // warp w: tile t0 + w; lane l: rows 8 l .. 8 l + 7 of each DCS_ROWS-row block, summed serially in registers, then
+  // one warp scan of the lane sums (a single dependent scan per block instead of one per 32 rows)
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int t0 = blockIdx.x * DCS_TILES;
+  const int t = blockIdx.x * DCS_TILES + warp;
   const int nCTA = (n_dev && n > 0) ? dbin_live_ctas(n < (int64_t)*n_dev ? n : (int64_t)*n_dev) : nCTA_cap;
-  // staging map: thread -> (row tid / 8 + 32 i, tile tid % 8): 8 consecutive words (one sector) per row
-  const int sr = tid / DCS_TILES, st_ = tid % DCS_TILES;
-  const bool tin = t0 + st_ < ntiles;
-  uint32_t carry = 0;  // warp w: tile t0 + w (uniform across the warp)
+  if (t >= ntiles) return;  // warp-uniform (no block barrier below)
+  uint32_t carry = 0;
   for (int r0 = 0; r0 < nCTA; r0 += DCS_ROWS) {
-    const int rows = min(DCS_ROWS, nCTA - r0);
+    uint32_t v[DCS_RPL];
+    const int rb = r0 + DCS_RPL * lane;
 #pragma unroll
-    for (int i = 0; i < DCS_ROWS / 32; ++i) {
-      const int r = sr + 32 * i;
-      if (r < rows) sm[r][st_] = tin ? C[(int64_t)(r0 + r) * ntiles + t0 + st_] : 0u;
-    }
-    __syncthreads();
-    for (int k = 0; k < DCS_ROWS / 32 && 32 * k < rows; ++k) {
-      const int r = 32 * k + lane;
-      const uint32_t v = r < rows ? sm[r][warp] : 0u;
-      uint32_t incl = v;
+    for (int i = 0; i < DCS_RPL; ++i) v[i] = rb + i < nCTA ? C[(int64_t)(rb + i) * ntiles + t] : 0u;  // (L1: the
+    // 8 warps read the 8 words of one sector per row)
+    uint32_t sum = 0;
 #pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += u;
-      }
-      if (r < rows) sm[r][warp] = carry + incl - v;
-      carry += __shfl_sync(0xffffffffu, incl, 31);
-    }
-    __syncthreads();
+    for (int i = 0; i < DCS_RPL; ++i) sum += v[i];
+    uint32_t incl = sum;
 #pragma unroll
-    for (int i = 0; i < DCS_ROWS / 32; ++i) {
-      const int r = sr + 32 * i;
-      if (r < rows && tin) C[(int64_t)(r0 + r) * ntiles + t0 + st_] = sm[r][st_];
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += u;
     }
-    __syncthreads();
+    uint32_t run = carry + incl - sum;
+#pragma unroll
+    for (int i = 0; i < DCS_RPL; ++i) {
+      if (rb + i < nCTA) C[(int64_t)(rb + i) * ntiles + t] = run;
+      run += v[i];
+    }
+    carry += __shfl_sync(0xffffffffu, incl, 31);
   }
-  if (lane == 0 && t0 + warp < ntiles) cnt[(int64_t)(t0 + warp) * cstride] = carry;
+  if (lane == 0) cnt[(int64_t)t * cstride] = carry;
 }
 
 // block-wide exclusive scan of one value per thread (DP_THREADS); returns the prefix, *total the sum
