@@ -54,6 +54,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-strong", action="store_true", help="skip the strong_C5 record (C5 frame split over N bands)")
+    ap.add_argument("--no-wide", action="store_true", help="skip the wide-ROI record (C4 at R = 63)")
     return ap.parse_args()
 
 
@@ -253,6 +254,67 @@ def run_reference(args, world, rank):
 
 
 # ------------------------------------------------------------------------------------------------ strong scaling, C5
+def wide_roi_record(args, ctx, stream, flush, dev, sm_mhz, R=63):
+    """C4 at R = 63 (100K clustered stars, sigma = R/6): frame ms through AUTO (k_tile_wide), its tile kernel's live ms
+    and FP32/SFU roofline fraction, the list kernel (STARSIM_TILE_LISTS) and the atomic kernel on the same frame.  Each
+    frame timed like the headline (K steps, L2 flushed before each, CUDA events on the render stream)."""
+    import synth
+    import torch
+    cfg = synth.with_R(synth.CONFIGS["C4"], R)
+    f = cfg.field()
+    W, H, sig = cfg.W, cfg.H, cfg.sigma
+    A = synth.bench_gain(sig)
+    U, E = units_of(f, W, H, R)
+    x, y, m = (torch.from_numpy(a).to(dev) for a in (f.x, f.y, f.mag))
+    out = torch.empty((H, W), dtype=torch.float32, device=dev)
+
+    def frames(fn, profile=False):
+        for _ in range(max(3, args.warmup)):
+            fn()
+        torch.cuda.synchronize()
+        if profile:
+            ctx.profile(True)
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        for i in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.fill_(float(i))
+                ev[i][0].record(stream)
+                fn()
+                ev[i][1].record(stream)
+        torch.cuda.synchronize()
+        kt = None
+        if profile:
+            kt = ctx.kernel_times()
+            ctx.profile(False)
+        return sum(a.elapsed_time(b) for a, b in ev) / args.steps, kt
+
+    def tiled():
+        ctx.render(x, y, m, W, H, sig, R, A, out=out, stream=stream)
+
+    rec = {"workload": f"C4: {W}x{H}, {f.n} clustered stars, R={R}, sigma={sig:.2f}", "updates_per_frame": U,
+           "exps_per_frame": E}
+    ms, _ = frames(tiled)
+    _, kt = frames(tiled, profile=True)
+    tile_ms = kt["tile"][0] / max(1, kt["tile"][1])
+    peak_rate, t_star = fp32_sfu_peak_updates(sm_mhz, U, E)
+    rec["tiled"] = {"kernel": "k_tile_wide", "ms_per_frame": ms, "frames_per_s": 1e3 / ms, "updates_per_s": U / (ms * 1e-3),
+                    "tile_kernel_ms": tile_ms,
+                    "binning_ms": sum(kt[k][0] for k in ("prep", "sort", "csr") if k in kt) / args.steps}
+    rec["roofline"] = {"bound": "alu", "kernel": "k_tile_wide", "achieved": U / (tile_ms * 1e-3) / 1e9,
+                       "peak": peak_rate / 1e9, "unit": "Gupdates/s", "frac": t_star / (tile_ms * 1e-3),
+                       "t_star_us": t_star * 1e6}
+    ctx.set_tile_kernel("lists")
+    try:
+        ms_l, _ = frames(tiled)
+        _, kt_l = frames(tiled, profile=True)
+    finally:
+        ctx.set_tile_kernel(args.tile_kernel)
+    rec["lists"] = {"kernel": "k_tile", "ms_per_frame": ms_l, "tile_kernel_ms": kt_l["tile"][0] / max(1, kt_l["tile"][1])}
+    ms_a, _ = frames(lambda: ctx.render_atomic(x, y, m, W, H, sig, R, A, out=out, stream=stream))
+    rec["atomic"] = {"kernel": "k_atomic", "ms_per_frame": ms_a}
+    return rec
+
+
 def strong_c5(args, world, rank, ctx, stream, flush, dev):
     """The north star's strong-scaling target on the C5 frame (16384 x 16384, 10M uniform stars, R=15), measured in
     every run: t_1 = one GPU renders the whole frame (each rank does it alone, max over ranks); for N > 1 t_render =
@@ -611,6 +673,15 @@ def run_ours(args, world, rank, local_rank):
         torch.cuda.synchronize()
         ctx.set_psf("point")
         ctx.set_roi("square")
+    # the wide-ROI end of the C4 sweep (BASELINE configs[3]: 100K clustered stars, R = 63): the sorted-corner-bin wide
+    # kernel k_tile_wide (AUTO) against the list kernel k_tile and the paper's atomic design, with its own roofline
+    try:
+        if world == 1 and args.method == "tiled" and not args.no_wide:
+            variants["wide_roi_C4_R63"] = wide_roi_record(args, ctx, stream, flush, dev, sm_mhz)
+    except Exception as e:  # noqa: BLE001
+        variants["wide_roi_C4_R63"] = {"error": f"{type(e).__name__}: {e}"}
+        torch.cuda.synchronize()
+        ctx.set_tile_kernel(args.tile_kernel)
 
     # e2e: the same C-ABI call with host (pinned) catalogue in and image out, copies inside the timed region
     e2e = None
