@@ -123,8 +123,9 @@ int starsim_set_psf(starsim_ctx* ctx, int32_t mode);
  *     in the circle inscribed in it: ROI row / column offsets (i, j) with (2j - (R-1))^2 + (2i - (R-1))^2 <= R^2,
  *     an exact integer test, then clipped to the image.  Supported by every render: the star-centric ones (atomic,
  *     lookup table) and the tiled ones (render, render_band, render_band_to, render_gray), which mask the circle per
- *     pixel in the tile kernel's walk -- k_tile_sb's for roi <= 17 (whatever starsim_set_tile_kernel says) and
- *     k_tile's for wider ROIs -- with the same profiles and the same deterministic order.
+ *     pixel in the tile kernel's walk -- k_tile_sb's for R <= 17 and k_tile_wide's for 27 <= R <= 65 (whatever
+ *     starsim_set_tile_kernel says), k_tile's otherwise -- with the same profiles and the same
+ *     deterministic order.
  * EINVAL: ctx NULL or an unknown shape. */
 #define STARSIM_ROI_SQUARE 0
 #define STARSIM_ROI_CIRCLE 1
@@ -145,16 +146,22 @@ int starsim_set_binning(starsim_ctx* ctx, int32_t mode);
  * and write every pixel once; they differ in how a tile's star list is walked, hence in the (deterministic)
  * per-pixel summation order:
  *   STARSIM_TILE_AUTO (default): for R <= 17, STARSIM_TILE_WS on dense frames (expected list length per tile
- *     n (127 + R)(63 + R) / (width rows) >= 100, point PSF), else STARSIM_TILE_SB; for R > 17 the list kernel;
+ *     n (127 + R)(63 + R) / (width rows) >= 100, point PSF), else STARSIM_TILE_SB; for 27 <= R <= 65 k_tile_wide
+ *     (sorted corner bins of the unclipped ROI origin over <= 5 bands x 9 strips, both roles in every warp); else
+ *     the list kernel k_tile;
  *   STARSIM_TILE_LISTS: always the per-block entry-list kernel k_tile (the comparison / any R);
- *   STARSIM_TILE_SB: for R <= 17 k_tile_sb, sorted corner bins with both roles in every warp, else k_tile;
+ *   STARSIM_TILE_SB: for R <= 17 k_tile_sb, sorted corner bins with both roles in every warp; for 27 <= R <= 65
+ *     k_tile_wide; else k_tile;
  *   STARSIM_TILE_WS: for R <= 17 k_tile_ws, the warp-specialised sorted-corner-bin kernel (producer warps sort and
- *     evaluate profiles into a ring of shared-memory stages while consumer warps accumulate), else
- *     k_tile.  SB and WS sum every pixel in the same order: the same image bit for bit;
+ *     evaluate profiles into a ring of shared-memory stages while consumer warps accumulate); for
+ *     27 <= R <= 65 k_tile_wws, k_tile_wide's warp-specialised form; else k_tile.  SB and WS sum every pixel in the
+ *     same order: the same image bit for bit;
  *   STARSIM_TILE_T8: for R <= 17 k_t8sort (every list segment sorted by ROI corner bin into a record array) then
- *     k_tile8 (8 x 8-pixel lane blocks, profile ring in shared memory, warp-specialised), else k_tile.
- * Every kernel sums a tile list longer than 1024 stars in 1024-star segments, each segment's sum added in list order
- * (reading R19), so a tile gives the same bits whether or not it was split across CTAs.
+ *     k_tile8 (8 x 8-pixel lane blocks, profile ring in shared memory, warp-specialised); for
+ *     27 <= R <= 65 k_tile_wws; else k_tile.
+ * Every kernel sums a tile list longer than L stars in L-star segments, each segment's sum added in list order
+ * (reading R19), so a tile gives the same bits whether or not it was split across CTAs; L = 1024, and
+ * L = 256 for 27 <= R <= 65 (a star there costs up to R^2 FMAs: heavy tiles spread over more CTAs).
  * EINVAL: ctx NULL or an unknown mode. */
 #define STARSIM_TILE_AUTO 0
 #define STARSIM_TILE_LISTS 1
@@ -232,7 +239,7 @@ int starsim_get_bins(starsim_ctx* ctx, int32_t* tile_w, int32_t* tile_h,
  * elapsed milliseconds and launch counts since the last reset.  Classes (index into the arrays):
  *   0 "prep": per-star prep + tile counts (k_dcount, k_prep); 1 "sort": list placement / sorting (k_dplace,
  *   k_sortlists, k_t8sort); 2 "csr": tile scans + scatter (k_dcolscan, k_scan*, k_scatter); 3 "tile": the tile
- *   kernel (k_tile, k_tile_sb, k_tile_ws, k_tile8); 4 "atomic": the star-centric renders (k_atomic, k_lut);
+ *   kernel (k_tile, k_tile_sb, k_tile_ws, k_tile8, k_tile_wide, k_tile_wws); 4 "atomic": the star-centric renders (k_atomic, k_lut);
  *   5 memsets; 6 k_quantize; 7 k_split_aos; 8 "route": k_route_count + k_route_place.
  * While profiling is enabled, renders are launched directly (not through the captured CUDA graph) so that every
  * kernel can be bracketed; kernel durations are unaffected, only the launch gaps differ.

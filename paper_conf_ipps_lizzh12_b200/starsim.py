@@ -356,7 +356,8 @@ class Context:
 
     def set_roi(self, shape="square"):
         """"square" (the R x R ROI, reading R5) or "circle" (the pixel circle inscribed in it, NEXT-3, reading R21: every
-        render; the tiled ones mask it in k_tile_sb's walk for R <= 17 and in k_tile's above)."""
+        render; the tiled ones mask it in the tile kernel's walk: k_tile_sb for R <= 17, k_tile_wide for 27 <= R <= 65,
+        k_tile otherwise)."""
         starsim_set_roi(self.h, shape)
 
     def set_binning(self, mode="auto"):
@@ -364,8 +365,9 @@ class Context:
         starsim_set_binning(self.h, mode)
 
     def set_tile_kernel(self, mode="auto"):
-        """"auto" (R <= 17: "ws" on dense frames, else "sb"; R > 17: "lists"), "lists" (k_tile, any R), "sb" (k_tile_sb),
-        "ws" (k_tile_ws) or "t8" (k_t8sort + k_tile8); include/starsim.h, starsim_set_tile_kernel."""
+        """"auto" (R <= 17: "ws" on dense frames, else "sb"; 27 <= R <= 65: k_tile_wide; else "lists"), "lists" (k_tile,
+        any R), "sb" (k_tile_sb; k_tile_wide for 27 <= R <= 65), "ws" (k_tile_ws; k_tile_wws) or "t8" (k_t8sort + k_tile8;
+        k_tile_wws); include/starsim.h, starsim_set_tile_kernel."""
         starsim_set_tile_kernel(self.h, mode)
 
     def render_band(self, x, y, mag, width, height, row0, rows, sigma, roi, gain, out=None, stream=None):
