@@ -12,6 +12,8 @@ timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
   python tools/profile_frame.py --reps 3 > /dev/null 2>&1
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:k_ -s 8 -c 4 -f -o gpurun_out/${TAG}_full \
   python tools/profile_frame.py --reps 1 > gpurun_out/ncu_full.log 2>&1
+timeout 300 ncu --set full --import-source on --clock-control none -k regex:k_tile_wide -s 2 -c 1 -f \
+  -o gpurun_out/${TAG}_wide_R63 python tools/profile_frame.py --config C4 --R 63 --reps 1 > gpurun_out/ncu_wide.log 2>&1
 timeout 900 python tools/sweep.py --sweep all > gpurun_out/${TAG}_sweep.jsonl 2> gpurun_out/sweep.err
 for c in "C1 0" "fig2 0" "C2 0" "C3 1000" "C3 16000" "C3 100000" "C4 0" "T 0"; do
   set -- $c; timeout 120 python tools/frame_time.py --config $1 --n $2

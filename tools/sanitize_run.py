@@ -4,7 +4,8 @@ initcheck):  compute-sanitizer --tool racecheck python tools/sanitize_run.py
 C1 (1024^2, 1000 stars, R=5) and a heavy-tile field (256^2, 30K stars in a 40-px disc: split tiles, partial buffers,
 1024-star segments) through every tile kernel (lists, sb, ws, t8; both binning pipelines), a band, the gray epilogue,
 the integrated PSF, the circle ROI, the star-centric kernels, quantize, upload_aos and the band routing; a sparse 4096 x 2048
-frame (2,000 stars) for k_tile_lite; k_tile_ws fed by k_chsort."""
+frame (2,000 stars) for k_tile_lite; k_tile_ws fed by k_chsort; a heavy wide-ROI field (R = 47: k_tile_wide, k_tile_wws,
+256-star segments and parts)."""
 import os
 import sys
 
@@ -32,7 +33,8 @@ def main():
     dev = torch.device("cuda:0")
     c1 = synth.CONFIGS["C1"]
     cases = [("C1", c1.field(), c1.W, c1.H, c1.R, c1.sigma), ("heavy", heavy(30000, 256, 256, 3), 256, 256, 15, 2.5),
-             ("sparse", synth.uniform_field(2000, 4096, 2048, seed=5), 4096, 2048, 15, 2.5)]  # k_tile_lite
+             ("sparse", synth.uniform_field(2000, 4096, 2048, seed=5), 4096, 2048, 15, 2.5),  # k_tile_lite
+             ("wide", heavy(6000, 256, 256, 4), 256, 256, 47, 7.8)]  # k_tile_wide (sb/auto), k_tile_wws (ws/t8)
     with Context(0) as ctx:
         for name, f, W, H, R, sigma in cases:
             x, y, m = (torch.from_numpy(a).to(dev) for a in (f.x, f.y, f.mag))
