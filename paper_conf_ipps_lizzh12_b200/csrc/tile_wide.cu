@@ -218,8 +218,15 @@ __global__ void __launch_bounds__(TILE_THREADS, WD_MINB) k_tile_wide(const uint3
 // work items in static round-robin order (parts of heavy tiles first).
 // ---------------------------------------------------------------------------------------------------------------
 namespace {
-constexpr int WW_CHUNK = 128;
-constexpr int WW_PROD = 4, WW_CONS = 8;
+#ifndef WW_PROD_OPT
+#define WW_PROD_OPT 4
+#endif
+#ifndef WW_MINB_OPT
+#define WW_MINB_OPT 1
+#endif
+constexpr int WW_PROD = WW_PROD_OPT, WW_CONS = 8;  // producer warps (one star per thread), consumer warps
+constexpr int WW_CHUNK = 32 * WW_PROD;
+constexpr int WW_MINB = WW_MINB_OPT;               // CTAs per SM
 constexpr int WW_THREADS = 32 * (WW_PROD + WW_CONS);
 constexpr uint32_t WW_LAST = 1u, WW_STOP = 2u, WW_SEGEND = 4u;
 static_assert(WW_CHUNK == 32 * WW_PROD && SPLIT_LEN % WW_CHUNK == 0, "one producer thread per star, whole segments");
@@ -234,7 +241,8 @@ struct WwStage {
 };
 template <int KB>
 __host__ __device__ constexpr int ww_ns() {
-  return 3 * sizeof(WwStage<KB>) + sizeof(uint32_t) * WW_PROD * WideGeom<KB>::NBIN + 128 <= 227 * 1024 ? 3 : 2;
+  return WW_MINB * (3 * sizeof(WwStage<KB>) + sizeof(uint32_t) * WW_PROD * WideGeom<KB>::NBIN + 1200) <= 228 * 1024
+             ? 3 : 2;
 }
 template <int KB>
 struct WwSmem {
@@ -243,7 +251,7 @@ struct WwSmem {
   uint32_t hist[WW_PROD][WideGeom<KB>::NBIN];
   int s_last;
 };
-static_assert(sizeof(WwSmem<5>) <= 227 * 1024 && sizeof(WwSmem<4>) <= 227 * 1024, "one CTA per SM fits");
+static_assert(WW_MINB * (sizeof(WwSmem<5>) + 1024) <= 228 * 1024, "WW_MINB CTAs per SM fit");
 
 __device__ __forceinline__ uint32_t ww_smem(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void ww_mbar_init(unsigned long long* b, uint32_t count) {
@@ -405,7 +413,7 @@ __device__ __forceinline__ void wws_consumer(WwSmem<KB>& S, const FrameParams& f
 }
 
 template <int KB, bool INTEG, bool CIRC>
-__global__ void __launch_bounds__(WW_THREADS, 1) k_tile_wws(const uint32_t* __restrict__ ids,
+__global__ void __launch_bounds__(WW_THREADS, WW_MINB) k_tile_wws(const uint32_t* __restrict__ ids,
                                                             const StarRec* __restrict__ rec, FrameParams fp,
                                                             void* __restrict__ out_, const WorkItem* __restrict__ items,
                                                             const uint2* __restrict__ split_tab,
@@ -468,7 +476,7 @@ void launch_tile_wide(const uint32_t* ids, const StarRec* rec, const FrameParams
   if (ntiles <= 0) return;
   const int kb = wide_kb(fp.R), a = fp.psf ? 1 : 0, b = fp.roi ? 1 : 0;
   if (fp.tile_impl != 2) {  // every mode but STARSIM_TILE_SB: the warp-specialised kernel, one CTA per SM
-    const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)num_sms);
+    const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)WW_MINB * num_sms);
     const KW k = kb == 3 ? WideTab<3>::w[a][b] : kb == 4 ? WideTab<4>::w[a][b] : WideTab<5>::w[a][b];
     const size_t smem = kb == 3 ? sizeof(WwSmem<3>) : kb == 4 ? sizeof(WwSmem<4>) : sizeof(WwSmem<5>);
     k<<<(unsigned)grid, WW_THREADS, smem, st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr, seg_scratch);
