@@ -6,6 +6,19 @@
 
 namespace starsim {
 
+// Debug builds (-DSTARSIM_CHECKS, e.g. STARSIM_NVCC_EXTRA=-DSTARSIM_CHECKS): device-side bounds and invariant checks
+// that trap, standing in for compute-sanitizer where it is unavailable; compiled out otherwise.
+#ifdef STARSIM_CHECKS
+#define SS_CHECK(c) \
+  do {              \
+    if (!(c)) __trap(); \
+  } while (0)
+#else
+#define SS_CHECK(c) \
+  do {              \
+  } while (0)
+#endif
+
 // ---------------------------------------------------------------- tile geometry (DESIGN.md §Data layout)
 // A tile is the unit of binning and of one k_tile CTA: TILE_W x TILE_H pixels.  Inside it, warp (wx, wy) owns the
 // 64 x 16 block at columns 64*wx, rows 16*wy; the block is 8 strips of STRIP_W = 8 columns, one per group of 4 lanes.

@@ -289,7 +289,11 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
       if (t < ntiles) {
         S.gstart[t] = run;
         S.cur[t] = run;
-        if (c[k] > DP_BIG) S.big[atomicAdd(&S.nbig, 1u)] = (uint16_t)t;
+        if (c[k] > DP_BIG) {
+          const uint32_t bi = atomicAdd(&S.nbig, 1u);
+          SS_CHECK(bi < (uint32_t)(DP_KEYS / 32));
+          S.big[bi] = (uint16_t)t;
+        }
       }
       run += c[k];
     }
@@ -349,6 +353,7 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
       if (lane >= o) incl += q;
     }
     uint32_t pos = S.cur[t] + incl - cntl;
+    SS_CHECK(__shfl_sync(0xffffffffu, incl, 31) == g1 - g0);  // every member's bit set once
 #pragma unroll 1
     for (int w = 0; w < WPL; ++w) {
       uint32_t m = bm[lane * WPL + w];

@@ -34,6 +34,7 @@ __device__ __forceinline__ bool tile_reduce_parts(float2 (&acc)[4][4], const Wor
   if (wi.aux == ITEM_WHOLE) return true;
   const int tid = threadIdx.x;
   const uint2 sp = split_tab[wi.aux >> 12];
+  SS_CHECK((wi.aux & 0xFFFu) < sp.y && sp.x + sp.y <= (uint32_t)PART_CAP);
   float* pbuf = part_buf + (size_t)(sp.x + (wi.aux & 0xFFFu)) * (TILE_W * TILE_H);
 #pragma unroll
   for (int i = 0; i < 4; ++i) {

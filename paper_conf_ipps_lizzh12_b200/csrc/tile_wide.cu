@@ -146,6 +146,7 @@ __global__ void __launch_bounds__(TILE_THREADS, WD_MINB) k_tile_wide(const uint3
       // ======================= prep: the star's profiles at its sorted place j
       if (key < G::NBIN) {
         const uint32_t j = S.binstart[key] + S.hist[warp & (WD_SW - 1)][key] + rank;
+        SS_CHECK(j < S.binstart[G::NBIN] && S.binstart[G::NBIN] <= (uint32_t)nvalid);
         // the unclipped ROI origin's band and strip (bands b0 .. b0 + KB - 1, strips q0 .. q0 + KS - 1 hold it)
         const int b0 = (int)(key / G::NSK) - (KB - 1), q0 = (int)(key % G::NSK) - (G::KS - 1);
         if (!colhalf) {
@@ -332,6 +333,7 @@ __device__ __forceinline__ void wws_producer(WwSmem<KB>& S, const uint32_t* __re
       ww_prod_barrier();
       if (key < G::NBIN) {
         const uint32_t j = T.binstart[key] + S.hist[pw][key] + rank;
+        SS_CHECK(j < (uint32_t)WW_CHUNK && j < T.binstart[G::NBIN]);
         const int b0 = (int)(key / G::NSK) - (KB - 1), q0 = (int)(key % G::NSK) - (G::KS - 1);
         if (CIRC) T.lo2[j] = lo2;
         wide_rows<KB, INTEG>(&T.gy[j * G::SYF], b0, r0, r1, r.y - (float)IY0, r.s, fp, lane);

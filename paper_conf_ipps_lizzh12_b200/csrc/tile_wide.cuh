@@ -1,5 +1,5 @@
-// Pieces of the wide-ROI sorted-corner-bin tile kernels (tile_wide.cu: k_tile_wide, both roles in every warp;
-// tile_wws.cu: k_tile_wws, warp-specialised): geometry, corner-bin key, the bin scan, the profile preparation of one
+// Pieces of the wide-ROI sorted-corner-bin tile kernels (tile_wide.cu: k_tile_wide, both roles in every warp, and
+// k_tile_wws, warp-specialised): geometry, corner-bin key, the bin scan, the profile preparation of one
 // star and the walk of one chunk.  The design is described at the top of tile_wide.cu.
 #pragma once
 #include "common.cuh"
@@ -162,6 +162,7 @@ __device__ __forceinline__ void wide_cols(float* gxj, int q0, int c0, int c1, fl
         }
       }
     }
+    SS_CHECK(k < G::RS);  // the KS strips of a star have distinct ring positions
     float* gs = gxj + (Qs & (G::RS - 1)) * 8;
     const int sw = ((Qs >> 2) & 1) * 4;
     *reinterpret_cast<float4*>(gs + sw) = make_float4(v[0], v[1], v[2], v[3]);
@@ -184,6 +185,7 @@ __device__ __forceinline__ void wide_walk(float2 (&acc)[4][4], const uint32_t* b
     // corner band B - k (band key B - k + KB - 1), corner strips Q - KS + 1 .. Q (strip keys Q .. Q + KS - 1)
     const int bk = B - k + KB - 1;
     const uint32_t s = binstart[bk * G::NSK + Q], e = binstart[bk * G::NSK + Q + G::KS];
+    SS_CHECK(s <= e && e <= binstart[G::NBIN] && bk >= 0 && bk < G::NBK);
     uint32_t ga = gy_base + s * SYB + 64u * (uint32_t)k, xa = gx_base + s * SXB;
     uint32_t jj = s;
     const uint32_t gend = ga + (e - s) * SYB;
