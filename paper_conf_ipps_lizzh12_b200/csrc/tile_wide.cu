@@ -44,7 +44,14 @@ namespace starsim {
 namespace {
 
 constexpr int WD_CHUNK = 128;                     // stars per chunk (two prep threads per star)
-constexpr int WD_MINB = 2;                        // CTAs per SM (128 registers, <= 112 KB shared memory)
+#ifndef WD_MINB_SMALL_OPT
+#define WD_MINB_SMALL_OPT 2
+#endif
+// CTAs per SM: 2 for KB = 5 (128 registers, <= 112 KB shared memory); KB = 3, 4 (R <= 49) fit WD_MINB_SMALL_OPT
+template <int KB>
+struct WdMinB {
+  static constexpr int value = KB >= 5 ? 2 : WD_MINB_SMALL_OPT;
+};
 constexpr int WD_SW = 4;                          // warps that own a star in the sort (threads 0..127)
 static_assert(SPLIT_LEN % WD_CHUNK == 0 && WIDE_SPLIT % WD_CHUNK == 0, "segments are whole chunks");
 static_assert(WD_CHUNK * 2 == TILE_THREADS, "two prep threads per star");
@@ -63,7 +70,7 @@ struct WideSmem {
 }  // namespace
 
 template <int KB, bool INTEG, bool CIRC>
-__global__ void __launch_bounds__(TILE_THREADS, WD_MINB) k_tile_wide(const uint32_t* __restrict__ ids,
+__global__ void __launch_bounds__(TILE_THREADS, WdMinB<KB>::value) k_tile_wide(const uint32_t* __restrict__ ids,
                                                                      const StarRec* __restrict__ rec, FrameParams fp,
                                                                      void* __restrict__ out_,
                                                                      const WorkItem* __restrict__ items,
@@ -87,7 +94,7 @@ __global__ void __launch_bounds__(TILE_THREADS, WD_MINB) k_tile_wide(const uint3
   __shared__ int s_last;
   __shared__ uint32_t s_next;
 
-  // persistent CTAs (WD_MINB per SM): item blockIdx.x first, then items from the counter the planner zeroed (the
+  // persistent CTAs (WdMinB per SM): item blockIdx.x first, then items from the counter the planner zeroed (the
   // parts of heavy tiles come first); the next item's records are fetched while this one is walked (as k_tile_sb)
   const uint32_t nitems = __ldcg(&hdr->nitems);
   uint32_t item = blockIdx.x;
@@ -484,7 +491,8 @@ void launch_tile_wide(const uint32_t* ids, const StarRec* rec, const FrameParams
     k<<<(unsigned)grid, WW_THREADS, smem, st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr, seg_scratch);
     return;
   }
-  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)WD_MINB * num_sms);  // persistent CTAs
+  const int minb = kb >= 5 ? WdMinB<5>::value : WdMinB<3>::value;
+  const int64_t grid = std::min<int64_t>(ntiles + part_cap, (int64_t)minb * num_sms);  // persistent CTAs
   const KW k = kb == 3 ? WideTab<3>::k[a][b] : kb == 4 ? WideTab<4>::k[a][b] : WideTab<5>::k[a][b];
   const size_t smem = kb == 3 ? sizeof(WideSmem<3>) : kb == 4 ? sizeof(WideSmem<4>) : sizeof(WideSmem<5>);
   k<<<(unsigned)grid, TILE_THREADS, smem, st>>>(ids, rec, fp, out, items, split_tab, part_buf, done, hdr, seg_scratch);
