@@ -1,6 +1,6 @@
-// k_tile_wide: tile accumulation with sorted corner bins for wide ROIs, SB_MAXR < R <= WIDE_MAXR (17 < R <= 65:
-// the wide end of the C4 ROI sweep, BASELINE configs[3]; Table III's ROI-side axis) -- SURVEY.md
-// §8a step a5, Eqs. 2-3.
+// k_tile_wide: tile accumulation with sorted corner bins for wide ROIs, WIDE_MINR <= R <= WIDE_MAXR (27 <= R <= 65,
+// wide_ok(): the wide end of the C4 ROI sweep, BASELINE configs[3]; Table III's ROI-side axis) --
+// SURVEY.md §8a step a5, Eqs. 2-3.  Measured and discussed in DESIGN.md §9b.
 //
 // The design of k_tile_sb (tile_sb.cu) generalised from "an ROI spans <= 2 bands x 3 strips" to <= KB bands x
 // KS = 2 KB - 1 strips (KB = 3, 4, 5 for R <= 33, 49, 65).  Same tile geometry, lane layout (warp (wx, B) owns the
@@ -29,7 +29,10 @@
 // the row slot of a star is an odd number of 64-B band slots, so the band slots of consecutive stars alternate 64-B
 // halves of the 128-B bank line.
 //
-// Summation order of a pixel: per chunk (in list order; lists longer than SPLIT_LEN in R19 segments), range k = 0 ..
+// Heavy tiles: parts and segments of FrameParams::split = WIDE_SPLIT (256) stars (reading R19), so a heavy tile's
+// R^2-FMA stars spread over several CTAs.
+//
+// Summation order of a pixel: per chunk (in list order; lists longer than fp.split in R19 segments), range k = 0 ..
 // KB-1, each in sorted order (corner bin, then list order): deterministic and a function of the tile's own list only,
 // so tile-aligned band renders are bitwise the frame's pixels (reading R12).  No atomics on the image.
 #include <algorithm>
