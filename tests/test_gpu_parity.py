@@ -171,12 +171,13 @@ def test_bands_concatenate_to_frame(torch_dev, ctx, G):
     assert torch.equal(torch.cat(bands, 0), full)
 
 
-def test_unaligned_band_matches_oracle(torch_dev, ctx):
+@pytest.mark.parametrize("R,sigma", [(11, 1.8), (41, 6.8), (65, 10.8)])
+def test_unaligned_band_matches_oracle(torch_dev, ctx, R, sigma):
     W, H = 200, 150
-    f = synth.adversarial_field(800, W, H, 11, seed=9)
-    ref = oracle.render_band(f.x, f.y, f.mag, W, H, 37, 61, 1.8, 11, 1.0)
-    got = ctx.render_band(*to_dev(torch_dev, f), W, H, 37, 61, 1.8, 11, 1.0).cpu().numpy()
-    assert_parity(got, ref, "band 37+61")
+    f = synth.adversarial_field(800, W, H, R, seed=9)
+    ref = oracle.render_band(f.x, f.y, f.mag, W, H, 37, 61, sigma, R, 1.0)
+    got = ctx.render_band(*to_dev(torch_dev, f), W, H, 37, 61, sigma, R, 1.0).cpu().numpy()
+    assert_parity(got, ref, f"band 37+61 R={R}")
 
 
 # ---------------------------------------------------------------- quantiser
@@ -826,7 +827,8 @@ def test_route_band_parity(torch_dev, ctx, n, W, H, R, G, kind):
 
 
 @pytest.mark.parametrize("W,H,n,R,G", [(640, 1024, 40000, 15, 4),      # bands of <= 2048 tiles: dbin.cu binning
-                                       (16384, 2176, 200000, 15, 2)])  # 2176 tiles per band: bin.cu's pipeline
+                                       (16384, 2176, 200000, 15, 2),   # 2176 tiles per band: bin.cu's pipeline
+                                       (640, 1024, 20000, 47, 4)])     # wide ROIs: k_tile_wide (256-star parts)
 def test_band_from_routed_catalogue_is_bitwise_the_band(torch_dev, ctx, W, H, n, R, G):
     """A band rendered from the device-routed catalogue (starsim_route_band + starsim_set_star_count:
     Context.render_band_routed, what every rank does per frame for N > 1) equals the band rendered from the whole
