@@ -257,7 +257,7 @@ int enqueue_binning(starsim_ctx* c, const float* x, const float* y, const float*
                       (uint2*)c->split_tab.p, plan, done, ids, st);
       });
       if ((rc = check_launch(c, "k_dsmall"))) return rc;
-    } else if (n > 0 && c->dfused_grid > 0 && dbin_ctas(n) <= c->dfused_grid) {
+    } else if (n > 0 && c->dfused_grid > 0 && dfused_block_ok(n) && dbin_ctas(n) <= c->dfused_grid) {
       // every CTA of the catalogue resident: count, column scan and placement in one cooperative launch (k_dfused)
       cudaError_t le = cudaSuccess;
       timed(c, 0, st, [&] {

@@ -2,7 +2,8 @@
 // pairs by tile, with no global atomics and no per-tile sort.  Used when the frame (or band) has at most DB_MAXT
 // tiles and an ROI overlaps at most 2 x 2 tiles (R <= 65); bin.cu's atomic-slot pipeline covers the rest.
 //
-//   k_dcount     a1 + counts: CTA c takes stars [c*DB_CTA, (c+1)*DB_CTA); per star the record of step a1
+//   k_dcount     a1 + counts: CTA c takes stars [c*blk, (c+1)*blk) (blk = DB_CTA, or 1,024 for catalogues of at most
+//                DB_SMALL_N stars: dbin_block); per star the record of step a1
 //                (prep_star); per tile the number of pairs of the CTA (shared-memory atomics -- counts do not depend
 //                on order) -> row c of the block-major count matrix C[c][tile] (coalesced).
 //   k_dcolscan   per 8-tile column block: the rows staged in shared memory, exclusive scan of every tile's column
@@ -44,7 +45,16 @@ constexpr int DP_SPT = DB_CTA / DP_THREADS;      // stars per thread (strided by
 constexpr int DCS_THREADS = 256;
 
 // CTAs that hold stars (at least one: CTA 0 plans the tiles of an empty routed catalogue)
-__device__ __forceinline__ int dbin_live_ctas(int64_t n) { return n > 0 ? (int)((n + DB_CTA - 1) / DB_CTA) : 1; }
+// Stars per CTA (one row of the count matrix): DB_CTA, or DB_CTA_SMALL for catalogues of at most DB_SMALL_N stars
+// (4x the CTAs: a small catalogue's binning is the per-CTA latency of a few CTAs).  A function of
+// the catalogue capacity n only, the same for every kernel of a render.
+constexpr int DB_CTA_SMALL = DC_THREADS;
+#ifndef DB_SMALL_N_OPT
+#define DB_SMALL_N_OPT 262144
+#endif
+constexpr int64_t DB_SMALL_N = DB_SMALL_N_OPT;
+__host__ __device__ __forceinline__ int dbin_block(int64_t n) { return n <= DB_SMALL_N ? DB_CTA_SMALL : DB_CTA; }
+__device__ __forceinline__ int dbin_live_ctas(int64_t n, int blk) { return n > 0 ? (int)((n + blk - 1) / blk) : 1; }
 static_assert(DB_MAXT <= 65536 && DB_CTA <= 65536, "tile ids, slots and star indices are 16-bit in k_dplace");
 static_assert(DP_WARPS <= 32, "dp_block_scan scans the warp sums with one warp");
 
@@ -52,6 +62,7 @@ static_assert(DP_WARPS <= 32, "dp_block_scan scans the warp sums with one warp")
 // t0 + ntx + 1 if both); DP_NONE if the star is culled.  Written by k_dcount, read by k_dplace.
 constexpr uint32_t DP_NONE = 0xFFFFFFFFu;
 
+template <int SPT>  // stars per thread: the CTA's block is DC_THREADS * SPT stars
 __global__ void __launch_bounds__(DC_THREADS, DC_MINB_OPT) k_dcount(const float* __restrict__ X, const float* __restrict__ Y,
                                                        const float* __restrict__ M, int64_t n, FrameParams fp,
                                                        StarRec* __restrict__ rec, uint32_t* __restrict__ codes,
@@ -60,13 +71,13 @@ __global__ void __launch_bounds__(DC_THREADS, DC_MINB_OPT) k_dcount(const float*
   __shared__ uint32_t cnt[DB_MAXT];
   const int tid = threadIdx.x, cta = blockIdx.x;
   n = frame_n(n, fp);
-  if (cta >= dbin_live_ctas(n)) return;  // beyond a routed catalogue's device count: k_dcolscan skips the column
+  if (cta >= dbin_live_ctas(n, DC_THREADS * SPT)) return;  // beyond a routed catalogue's count: k_dcolscan skips it
   for (int t = tid; t < ntiles; t += DC_THREADS) cnt[t] = 0u;
   // all loads of the thread's stars first (one memory latency, not DC_PER)
-  const int64_t i0 = (int64_t)cta * DB_CTA + tid;
-  float xs[DC_PER], ys[DC_PER], ms[DC_PER];
+  const int64_t i0 = (int64_t)cta * (DC_THREADS * SPT) + tid;
+  float xs[SPT], ys[SPT], ms[SPT];
 #pragma unroll
-  for (int k = 0; k < DC_PER; ++k) {
+  for (int k = 0; k < SPT; ++k) {
     const int64_t i = i0 + (int64_t)k * DC_THREADS;
     const bool in = i < n;
     xs[k] = in ? __ldg(&X[i]) : 0.f;
@@ -75,7 +86,7 @@ __global__ void __launch_bounds__(DC_THREADS, DC_MINB_OPT) k_dcount(const float*
   }
   __syncthreads();
 #pragma unroll
-  for (int k = 0; k < DC_PER; ++k) {
+  for (int k = 0; k < SPT; ++k) {
     const int64_t i = i0 + (int64_t)k * DC_THREADS;
     if (i >= n) break;
     int cx0, cx1, cy0, cy1;
@@ -104,14 +115,14 @@ constexpr int DCS_ROWS = 256;
 constexpr int DCS_RPL = DCS_ROWS / 32;  // rows per lane
 __global__ void __launch_bounds__(DCS_THREADS) k_dcolscan(uint32_t* __restrict__ C, int nCTA_cap, int ntiles,
                                                          uint32_t* __restrict__ cnt, int cstride, int64_t n,
-                                                         const uint32_t* __restrict__ n_dev) {
+                                                         const uint32_t* __restrict__ n_dev, int blk) {
   static_assert(DCS_THREADS == 32 * DCS_TILES, "one warp per tile");
   static_assert(DCS_ROWS == 32 * DCS_RPL, "a lane holds DCS_RPL consecutive rows");
   // warp w: tile t0 + w; lane l: rows 8 l .. 8 l + 7 of each DCS_ROWS-row block, summed serially in registers, then
   // one warp scan of the lane sums (a single dependent scan per block instead of one per 32 rows)
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int t = blockIdx.x * DCS_TILES + warp;
-  const int nCTA = (n_dev && n > 0) ? dbin_live_ctas(n < (int64_t)*n_dev ? n : (int64_t)*n_dev) : nCTA_cap;
+  const int nCTA = (n_dev && n > 0) ? dbin_live_ctas(n < (int64_t)*n_dev ? n : (int64_t)*n_dev, blk) : nCTA_cap;
   if (t >= ntiles) return;  // warp-uniform (no block barrier below)
   uint32_t carry = 0;
   for (int r0 = 0; r0 < nCTA; r0 += DCS_ROWS) {
@@ -256,17 +267,18 @@ __device__ __forceinline__ void dp_scan_tiles(DpSmem& S, const uint32_t* __restr
 // Steps a3-a4 of k_dplace for the CTA's stars (codes in registers, star i = blockIdx.x DB_CTA + tid + k DP_THREADS):
 // group the pairs by tile in shared memory, rank each in its group by star index, write it to
 // tile_off[t] + C[t][cta] + rank (C == nullptr: a single CTA, every group starts at its tile's list start).
-__device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SPT], const FrameParams& fp,
+template <int SPT>
+__device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[SPT], const FrameParams& fp,
                                          const uint32_t* __restrict__ C, int nCTA, int ntiles,
                                          uint32_t* __restrict__ ids) {
   const int tid = threadIdx.x, cta = blockIdx.x;
-  const int64_t c0 = (int64_t)cta * DB_CTA;
+  const int64_t c0 = (int64_t)cta * (DP_THREADS * SPT);
   for (int t = tid; t <= ntiles; t += DP_THREADS) S.gstart[t] = 0u;
   if (tid == 0) S.nbig = 0u;
   __syncthreads();
   // group sizes
 #pragma unroll
-  for (int k = 0; k < DP_SPT; ++k) {
+  for (int k = 0; k < SPT; ++k) {
     const int nb = box_n(code[k]);
     for (int e = 0; e < nb; ++e) atomicAdd(&S.gstart[box_tile(code[k], e, fp.ntx)], 1u);
   }
@@ -302,7 +314,7 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
   __syncthreads();
   // group the star indices by tile (arbitrary order inside a group)
 #pragma unroll
-  for (int k = 0; k < DP_SPT; ++k) {
+  for (int k = 0; k < SPT; ++k) {
     const int nb = box_n(code[k]);
     for (int e = 0; e < nb; ++e)
       S.arr[atomicAdd(&S.cur[box_tile(code[k], e, fp.ntx)], 1u)] = (uint16_t)(tid + k * DP_THREADS);
@@ -314,7 +326,7 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
   // a pair's rank in its group = the group's stars with a smaller index (groups of at most DP_BIG pairs: the common
   // case of uniform fields)
 #pragma unroll
-  for (int k = 0; k < DP_SPT; ++k) {
+  for (int k = 0; k < SPT; ++k) {
     const uint32_t idx = (uint32_t)(tid + k * DP_THREADS);
     const int nb = box_n(code[k]);
     for (int e = 0; e < nb; ++e) {
@@ -367,6 +379,7 @@ __device__ __forceinline__ void dp_place(DpSmem& S, const uint32_t (&code)[DP_SP
   }
 }
 
+template <int SPT>
 __global__ void __launch_bounds__(DP_THREADS, DP_MINB) k_dplace(const uint32_t* __restrict__ codes, int64_t n, FrameParams fp,
                                                        const uint32_t* __restrict__ C, int nCTA, int ntiles,
                                                        const uint32_t* __restrict__ cnt, uint32_t* __restrict__ tile_off,
@@ -377,19 +390,19 @@ __global__ void __launch_bounds__(DP_THREADS, DP_MINB) k_dplace(const uint32_t* 
   extern __shared__ __align__(16) unsigned char dsm_raw[];
   DpSmem& S = *reinterpret_cast<DpSmem*>(dsm_raw);
   const int tid = threadIdx.x, cta = blockIdx.x;
-  const int64_t c0 = (int64_t)cta * DB_CTA;
+  const int64_t c0 = (int64_t)cta * (DP_THREADS * SPT);
   n = frame_n(n, fp);
   // step a2 is spread over every CTA of the grid (CTA c plans the tiles t = c mod gridDim.x; the grid has at least
   // ntiles / 256 CTAs, so a sparse frame's plan is not one CTA's serial work); only the CTAs that hold stars go on
   dp_scan_tiles(S, cnt, ntiles, (int)gridDim.x, tile_off, hdr, items, split_tab, part_cap, done);
-  if (cta >= dbin_live_ctas(n)) return;
-  uint32_t code[DP_SPT];
+  if (cta >= dbin_live_ctas(n, DP_THREADS * SPT)) return;
+  uint32_t code[SPT];
 #pragma unroll
-  for (int k = 0; k < DP_SPT; ++k) {
+  for (int k = 0; k < SPT; ++k) {
     const int64_t i = c0 + tid + k * DP_THREADS;
     code[k] = i < n ? __ldg(&codes[i]) : DP_NONE;
   }
-  dp_place(S, code, fp, C, nCTA, ntiles, ids);
+  dp_place<SPT>(S, code, fp, C, nCTA, ntiles, ids);
 }
 
 // k_dsmall: a catalogue of at most DB_CTA stars binned by ONE CTA in one launch -- k_dcount's step a1 and counts
@@ -439,7 +452,7 @@ __global__ void __launch_bounds__(DP_THREADS, 1) k_dsmall(const float* __restric
   }
   __syncthreads();
   dp_scan_tiles<true>(S, S.cur, ntiles, 1, tile_off, hdr, items, split_tab, part_cap, done);
-  dp_place(S, code, fp, nullptr, 1, ntiles, ids);
+  dp_place<DP_SPT>(S, code, fp, nullptr, 1, ntiles, ids);
 }
 
 
@@ -492,7 +505,7 @@ __global__ void __launch_bounds__(DP_THREADS, 2) k_dfused(const float* __restric
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, cta = blockIdx.x;
   const uint32_t nC = gridDim.x;
   n = frame_n(n, fp);
-  const int live = dbin_live_ctas(n);
+  const int live = dbin_live_ctas(n, DB_CTA);
   // ---- phase 1 (k_dcount)
   uint32_t code[DP_SPT];
 #pragma unroll
@@ -567,15 +580,17 @@ __global__ void __launch_bounds__(DP_THREADS, 2) k_dfused(const float* __restric
   // ---- phase 3 (k_dplace)
   dp_scan_tiles(F.dp, cntg, ntiles, (int)nC, tile_off, hdr, items, split_tab, part_cap, done);
   if (cta >= live) return;
-  dp_place(F.dp, code, fp, C, (int)nC, ntiles, ids);
+  dp_place<DP_SPT>(F.dp, code, fp, C, (int)nC, ntiles, ids);
 }
 
 size_t dbin_smem(int) { return sizeof(DpSmem); }
 
-int dbin_ctas(int64_t n) { return (int)((n + DB_CTA - 1) / DB_CTA); }
+int dbin_ctas(int64_t n) { return (int)((n + dbin_block(n) - 1) / dbin_block(n)); }
+bool dfused_block_ok(int64_t n) { return dbin_block(n) == DB_CTA; }  // k_dfused bins DB_CTA-star blocks only
 
 void init_dbin_kernels() {
-  cudaFuncSetAttribute(k_dplace, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DpSmem));
+  cudaFuncSetAttribute(k_dplace<DP_SPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DpSmem));
+  cudaFuncSetAttribute(k_dplace<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DpSmem));
   cudaFuncSetAttribute(k_dsmall, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DpSmem));
   cudaFuncSetAttribute(k_dfused, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DfSmem));
 }
@@ -599,7 +614,7 @@ cudaError_t launch_dfused(const float* x, const float* y, const float* m, int64_
                           uint32_t* bar, cudaStream_t st) {
   cudaMemsetAsync(bar, 0, sizeof(uint32_t), st);
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)dbin_ctas(n));
+  cfg.gridDim = dim3((unsigned)((n + DB_CTA - 1) / DB_CTA));
   cfg.blockDim = dim3(DP_THREADS);
   cfg.dynamicSmemBytes = sizeof(DfSmem);
   cfg.stream = st;
@@ -622,13 +637,17 @@ void launch_dsmall(const float* x, const float* y, const float* m, int64_t n, co
 void launch_dcount(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp, StarRec* rec,
                    uint32_t* codes, uint32_t* C, int ntiles, cudaStream_t st) {
   const int nc = dbin_ctas(n);
-  if (nc > 0) k_dcount<<<nc, DC_THREADS, 0, st>>>(x, y, m, n, fp, rec, codes, C, nc, ntiles);
+  if (nc <= 0) return;
+  if (dbin_block(n) == DB_CTA)
+    k_dcount<DC_PER><<<nc, DC_THREADS, 0, st>>>(x, y, m, n, fp, rec, codes, C, nc, ntiles);
+  else
+    k_dcount<1><<<nc, DC_THREADS, 0, st>>>(x, y, m, n, fp, rec, codes, C, nc, ntiles);
 }
 
 void launch_dcolscan(uint32_t* C, int64_t n, int ntiles, uint32_t* cnt, int cstride, const uint32_t* n_dev,
                      cudaStream_t st) {
   k_dcolscan<<<(ntiles + DCS_TILES - 1) / DCS_TILES, DCS_THREADS, 0, st>>>(C, dbin_ctas(n), ntiles, cnt, cstride, n,
-                                                                           n_dev);
+                                                                           n_dev, dbin_block(n));
 }
 
 void launch_dplace(const uint32_t* codes, int64_t n, const FrameParams& fp, const uint32_t* C, int ntiles,
@@ -636,9 +655,10 @@ void launch_dplace(const uint32_t* codes, int64_t n, const FrameParams& fp, cons
                    int part_cap, uint32_t* done, uint32_t* ids, cudaStream_t st) {
   const int nc = dbin_ctas(n);
   const int grid = std::max(nc, (ntiles + 255) / 256);  // planning CTAs (k_dplace)
-  if (nc > 0)
-    k_dplace<<<grid, DP_THREADS, sizeof(DpSmem), st>>>(codes, n, fp, C, nc, ntiles, cnt, tile_off, hdr, items,
-                                                        split_tab, part_cap, done, ids);
+  if (nc <= 0) return;
+  auto* k = dbin_block(n) == DB_CTA ? k_dplace<DP_SPT> : k_dplace<1>;
+  k<<<grid, DP_THREADS, sizeof(DpSmem), st>>>(codes, n, fp, C, nc, ntiles, cnt, tile_off, hdr, items, split_tab,
+                                              part_cap, done, ids);
 }
 
 }  // namespace starsim

@@ -17,7 +17,8 @@ void init_tile8_kernel();
 size_t tile8_scratch_floats(int num_sms);
 void init_dbin_kernels();
 size_t dbin_smem(int ntiles);
-int dbin_ctas(int64_t n);
+int dbin_ctas(int64_t n);          // rows of the count matrix (4,096-star blocks; 1,024-star blocks for small n)
+bool dfused_block_ok(int64_t n);  // k_dfused applies (it bins 4,096-star blocks only)
 bool dsmall_ok(int64_t n);  // k_dsmall applies (at most DB_CTA stars)
 int dfused_max_grid(int num_sms);
 cudaError_t launch_dfused(const float* x, const float* y, const float* m, int64_t n, const FrameParams& fp,
