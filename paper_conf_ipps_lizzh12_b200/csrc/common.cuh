@@ -86,7 +86,11 @@ constexpr int SPARSE_MAX = 32768;            // catalogues of at most this many 
 #define SPARSE_TESTS_OPT (8 << 20)
 #endif
 constexpr int64_t SPARSE_TESTS = SPARSE_TESTS_OPT;  // ... when stars x tiles (the tile CTAs' star tests) is at most this
-constexpr double LITE_AUTO_PER_TILE = 16.0;  // k_tile_lite is launched when the expected list per tile is <= this
+#ifndef LITE_AUTO_PER_TILE_OPT
+#define LITE_AUTO_PER_TILE_OPT 16.0
+#endif
+constexpr double LITE_AUTO_PER_TILE = LITE_AUTO_PER_TILE_OPT;  // k_tile_lite is launched when the expected list per
+                                                               // tile is <= this
 constexpr int64_t LITE_AUTO_TILES = 1024;    // ... and the frame / band has at least this many tiles
 constexpr int SPLIT_LEN = 1024;        // a tile list longer than this is split into parts of <= SPLIT_LEN stars
 constexpr int PART_CAP = 2048;         // partial-tile buffers (128 x 64 fp32 each, 64 MB) available per render
